@@ -1,0 +1,601 @@
+"""Planner oracle -- TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).
+
+Plain Python restatement of the paper's planning steps, written for checking by eye:
+
+  * operator graphs with static footprints (PAPER.md:345, :349 fn. 1): `Graph`
+  * the edge template graph of Fig. 1(b)/Fig. 3 and the CNN layers expanded as Fig. 7
+  * Table 1 accounting: total temporary data, I/O lower bound, per-operator baseline
+    
+  * operator splitting: per-operator memory requirement and split factors
+    (PAPER.md:359-365), Fig. 1(c) regimes
+  * halo back-propagation "from the leaves to the root"
+  * depth-first operator schedule and the "latest time of use" transfer
+    schedule with eager deletion (read as NEXT use, R10)
+  * brute force over all operator orders for tiny graphs (stands in for the PB model of
+    Fig. 5)
+  * the fused B200 chunk rule, which the library's planner must
+    reproduce bit-exactly (tests/test_plan_parity.py).
+"""
+from __future__ import annotations
+
+import itertools
+import math
+from dataclasses import dataclass, field
+
+
+# ============================================================================ graphs
+@dataclass
+class DS:
+    name: str
+    size: int               # floats (PAPER.md:741 counts floats)
+    kind: str = "temp"      # "input" | "param" | "temp" | "output"
+
+
+@dataclass
+class Op:
+    name: str
+    ins: list[int]
+    outs: list[int]
+
+
+@dataclass
+class Graph:
+    ds: list[DS] = field(default_factory=list)
+    ops: list[Op] = field(default_factory=list)
+
+    def add_ds(self, name, size, kind="temp") -> int:
+        self.ds.append(DS(name, int(size), kind))
+        return len(self.ds) - 1
+
+    def add_op(self, name, ins, outs) -> int:
+        self.ops.append(Op(name, list(ins), list(outs)))
+        return len(self.ops) - 1
+
+    # ---- accounting (Table 1)
+    def total_temp(self) -> int:
+        """'Total temporary data needed': sum of the sizes of all data structures."""
+        return sum(d.size for d in self.ds)
+
+    def io_lower_bound(self) -> int:
+        """'I/O transfers only (lower bound)': template inputs (data and parameters) plus
+        template outputs, each moved once."""
+        return sum(d.size for d in self.ds if d.kind in ("input", "param", "output"))
+
+    def baseline(self) -> int:
+        """Baseline of PAPER.md:613: 'For each operator, transfer input data to the GPU,
+        perform the operation and copy the results back to the CPU immediately.'"""
+        return sum(sum(self.ds[j].size for j in op.ins) + sum(self.ds[j].size for j in op.outs)
+                   for op in self.ops)
+
+    def req(self, op: Op) -> int:
+        """Memory requirement of an operator: 'sum of sizes of data structures associated
+        with each operator'."""
+        return sum(self.ds[j].size for j in set(op.ins) | set(op.outs))
+
+
+def edge_graph(H: int, W: int, ks: int = 16, orientations: int = 4, kernel_floats=True) -> Graph:
+    """Edge template: `orientations`/2 convolutions with precomputed rotated kernels, as many
+    remaps (negations), one max over all responses (Fig. 1(b), Fig. 3).
+    4 orientations: C1 C2 R1 R2 max; 8 orientations: C1-C4 R1-R4 max (Fig. 1(b))."""
+    g = Graph()
+    S = H * W
+    im = g.add_ds("Im", S, "input")
+    nconv = orientations // 2
+    ks_ = [g.add_ds(f"K{i+1}", ks * ks if kernel_floats else 0, "param") for i in range(nconv)]
+    conv_out, remap_out = [], []
+    for i in range(nconv):
+        e = g.add_ds(f"E{i+1}", S)
+        g.add_op(f"C{i+1}", [im, ks_[i]], [e])
+        conv_out.append(e)
+    for i in range(nconv):
+        e = g.add_ds(f"E{i+1+nconv}", S)
+        g.add_op(f"R{i+1}", [conv_out[i]], [e])
+        remap_out.append(e)
+    E = g.add_ds("E", S, "output")
+    g.add_op("max", conv_out + remap_out, [E])
+    return g
+
+
+def cnn_dims(H: int, W: int):
+    """Per-level plane sizes: VALID 5x5 convs and 2x2/2 subsampling
+    with floor((D-2)/2)+1."""
+    h1, w1 = H - 4, W - 4
+    h2, w2 = (h1 - 2) // 2 + 1, (w1 - 2) // 2 + 1
+    h3, w3 = h2 - 4, w2 - 4
+    h4, w4 = (h3 - 2) // 2 + 1, (w3 - 2) // 2 + 1
+    h5, w5 = h4 - 4, w4 - 4
+    return [(h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5)]
+
+
+def cnn_graph_fig7(H: int, W: int, n5: int) -> Graph:
+    """CNN template expanded operator by operator as Fig. 7: per layer
+    and output plane j, convolutions L_ij = In_i * K_ij, a chain of adds S_j1 = L_1j + L_2j,
+    S_jk = S_j(k-1) + L_(k+1)j, and O_j = S_last + B_j with a full-size bias plane B_j;
+    tanh: one op and one DS per plane; subsample: one op, a 4-float kernel and one output
+    per plane."""
+    g = Graph()
+    (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = cnn_dims(H, W)
+    planes = [g.add_ds("In1", H * W, "input")]
+
+    def conv(planes_in, n_out, k, ho, wo, tag, last=False):
+        outs = []
+        for j in range(n_out):
+            Ls = []
+            for i, p in enumerate(planes_in):
+                K = g.add_ds(f"{tag}.K{i+1}{j+1}", k * k, "param")
+                L = g.add_ds(f"{tag}.L{i+1}{j+1}", ho * wo)
+                g.add_op(f"{tag}.C{i+1}{j+1}", [p, K], [L])
+                Ls.append(L)
+            acc = Ls[0]
+            for i in range(1, len(Ls)):
+                S = g.add_ds(f"{tag}.S{j+1}{i}", ho * wo)
+                g.add_op(f"{tag}.A{j+1}{i}", [acc, Ls[i]], [S])
+                acc = S
+            B = g.add_ds(f"{tag}.B{j+1}", ho * wo, "param")
+            O = g.add_ds(f"{tag}.O{j+1}", ho * wo, "output" if last else "temp")
+            g.add_op(f"{tag}.AB{j+1}", [acc, B], [O])
+            outs.append(O)
+        return outs
+
+    def tanh(planes_in, size, tag):
+        outs = []
+        for i, p in enumerate(planes_in):
+            o = g.add_ds(f"{tag}.T{i+1}", size)
+            g.add_op(f"{tag}.tanh{i+1}", [p], [o])
+            outs.append(o)
+        return outs
+
+    def sub(planes_in, size, tag):
+        outs = []
+        for i, p in enumerate(planes_in):
+            P = g.add_ds(f"{tag}.P{i+1}", 4, "param")
+            o = g.add_ds(f"{tag}.O{i+1}", size)
+            g.add_op(f"{tag}.sub{i+1}", [p, P], [o])
+            outs.append(o)
+        return outs
+
+    x = conv(planes, 8, 5, h1, w1, "C1")
+    x = tanh(x, h1 * w1, "T1")
+    x = sub(x, h2 * w2, "S2")
+    x = tanh(x, h2 * w2, "T2")
+    x = conv(x, 20, 5, h3, w3, "C3")
+    x = tanh(x, h3 * w3, "T3")
+    x = sub(x, h4 * w4, "S4")
+    x = tanh(x, h4 * w4, "T4")
+    x = conv(x, n5, 5, h5, w5, "C5")
+    x = tanh(x, h5 * w5, "T5")
+    conv(x, 9, 1, h5, w5, "C6", last=True)
+    return g
+
+
+def cnn_conv_accumulate_baseline(H: int, W: int, n5: int) -> int:
+    """Layer-level baseline variant: every conv pair moves In_i + K_ij + the
+    accumulator in and the accumulator out; tanh moves in + out; subsample in + P + out.
+    Only the large-minus-small differences are pinned by Table 1."""
+    (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = cnn_dims(H, W)
+    A0, A1, A2, A3, A4, A5 = H * W, h1 * w1, h2 * w2, h3 * w3, h4 * w4, h5 * w5
+    t = 0
+    for n_in, n_out, k, a_in, a_out in [(1, 8, 5, A0, A1), (8, 20, 5, A2, A3),
+                                         (20, n5, 5, A4, A5), (n5, 9, 1, A5, A5)]:
+        t += n_in * n_out * (a_in + k * k + 2 * a_out)
+    t += 8 * 2 * A1 + 8 * (A1 + 4 + A2) + 8 * 2 * A2          # T1, S2, T2
+    t += 20 * 2 * A3 + 20 * (A3 + 4 + A4) + 20 * 2 * A4       # T3, S4, T4
+    t += n5 * 2 * A5                                          # T5
+    return t
+
+
+# ============================================================================ splitting
+def split_factors(g: Graph, M: int) -> dict[str, int]:
+    """Paper-mode operator splitting: an operator whose requirement
+    exceeds the GPU memory M is split into k = ceil(req/M) equal pieces."""
+    return {op.name: max(1, math.ceil(g.req(op) / M)) for op in g.ops}
+
+
+def fig1c_regime(S: float, M: float = 1500.0) -> str:
+    """Fig. 1(c) strategy for the 8-orientation edge graph at image size S on a GPU of
+    memory M, from req(C)=req(R)=2S, req(max)=9S, total=10S."""
+    g = edge_graph(1, 1, orientations=8, kernel_floats=False)
+    req = {op.name: g.req(op) * S for op in g.ops}
+    total = g.total_temp() * S
+    if S > M:
+        return "input_chunked"
+    if total <= M:
+        return "all_fit"
+    if req["max"] <= M:
+        return "max_separate"
+    if max(req[o] for o in req if o != "max") <= M:
+        return "max_split"
+    return "conv_remap_split"
+
+
+def back_propagate_rows(layers, r0: int, r1: int, H_in: int | None = None):
+    """Walk a chain of row-local operators from the output back to the input ('traversing
+    the split graph from the leaves to the root and inferring the sizes and offsets from
+    the kernel and output sizes'). layers: list of (kind, param) from input
+    to output, kind in {"valid", "same", "sub", "elem"}. Returns the row range needed at
+    every level, input first. SAME ranges are clipped to [0, H_in) (zeros outside)."""
+    ranges = [(r0, r1)]
+    a, b = r0, r1
+    for kind, p in reversed(layers):
+        if kind == "valid":
+            a, b = a, b + p - 1
+        elif kind == "same":
+            a, b = a - (p - 1) // 2, b + p // 2
+            if H_in is not None:
+                a, b = max(0, a), min(H_in, b)
+        elif kind == "sub":
+            a, b = p * a, p * b
+        elif kind == "elem":
+            pass
+        else:
+            raise ValueError(kind)
+        ranges.append((a, b))
+    return list(reversed(ranges))
+
+
+CNN_LAYERS = [("valid", 5), ("elem", 0), ("sub", 2), ("elem", 0), ("valid", 5), ("elem", 0),
+              ("sub", 2), ("elem", 0), ("valid", 5), ("elem", 0), ("valid", 1)]
+
+
+# ============================================================================ scheduling
+def dfs_order(g: Graph) -> list[int]:
+    """Depth-first operator schedule: schedule the entire sub-tree of a
+    child before its siblings; a node whose inputs are not ready is skipped (backtrack to
+    the parent and explore its other children). Children = consumers of an op's outputs in
+    graph-insertion order; start nodes in id order (R11)."""
+    producer = {}
+    for i, op in enumerate(g.ops):
+        for j in op.outs:
+            producer[j] = i
+    preds = [{producer[j] for j in op.ins if j in producer} for op in g.ops]
+    consumers = [[] for _ in g.ops]
+    for i, op in enumerate(g.ops):
+        for p in sorted(preds[i]):
+            pass
+    for c, op in enumerate(g.ops):
+        for j in op.ins:
+            if j in producer and c not in consumers[producer[j]]:
+                consumers[producer[j]].append(c)
+    for lst in consumers:
+        lst.sort()
+    done: list[int] = []
+    seen = set()
+
+    def visit(i):
+        done.append(i)
+        seen.add(i)
+        for c in consumers[i]:
+            if c not in seen and preds[c] <= seen:
+                visit(c)
+
+    for i in range(len(g.ops)):
+        if i not in seen and preds[i] <= seen:
+            visit(i)
+    assert len(done) == len(g.ops)
+    return done
+
+
+def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None) -> int:
+    """Transfer volume of an operator order under the 'latest time of use' policy
+    (read as next use -- DESIGN.md R10):
+      * the inputs and outputs of the running operator must be resident; a missing input is
+        copied to the GPU; outputs are allocated on the GPU;
+      * on shortage, move to the CPU the resident DS whose next use is furthest in the
+        future (no further use = infinitely far); ties: host-valid (clean) data first, then
+        lowest DS id; clean data is dropped for free, dirty data costs a copy to the CPU;
+      * data is deleted eagerly once no later operator uses it (template outputs are
+        instead copied to the CPU when evicted or at the end);
+      * initially everything is on the CPU, nothing on the GPU (PB constraints (11),(12)).
+    Returns the number of floats moved (H2D + D2H)."""
+    uses = {j: [] for j in range(len(g.ds))}
+    for t, i in enumerate(order):
+        for j in set(g.ops[i].ins) | set(g.ops[i].outs):
+            uses[j].append(t)
+    outputs = {j for j, d in enumerate(g.ds) if d.kind == "output"}
+    on_gpu: dict[int, bool] = {}          # DS -> dirty (GPU copy newer than host)
+    host_valid = {j for j, d in enumerate(g.ds) if d.kind in ("input", "param")}
+    moved = 0
+
+    def next_use(j, t):
+        for u in uses[j]:
+            if u > t:
+                return u
+        return math.inf
+
+    def used(t):
+        return sum(g.ds[j].size for j in on_gpu)
+
+    for t, i in enumerate(order):
+        op = g.ops[i]
+        need = list(dict.fromkeys(list(op.ins) + list(op.outs)))
+        pinned = set(need)
+        for j in need:
+            if j in on_gpu:
+                continue
+            sz = g.ds[j].size
+            while used(t) + sz > capacity:
+                cands = [k for k in on_gpu if k not in pinned]
+                if not cands:
+                    raise RuntimeError("operator does not fit")
+                cands.sort(key=lambda k: (-next_use(k, t), 0 if not on_gpu[k] else 1, k))
+                v = cands[0]
+                if on_gpu[v] and (next_use(v, t) != math.inf or v in outputs):
+                    moved += g.ds[v].size          # write back dirty data still needed
+                    host_valid.add(v)
+                    if trace is not None:
+                        trace.append(("d2h", g.ds[v].name))
+                del on_gpu[v]
+            if j in op.ins:
+                assert j in host_valid, g.ds[j].name
+                moved += sz
+                on_gpu[j] = False
+                if trace is not None:
+                    trace.append(("h2d", g.ds[j].name))
+            else:
+                on_gpu[j] = True
+                host_valid.discard(j)
+        if trace is not None:
+            trace.append(("run", op.name))
+        # eager deletion of data no later operator needs (outputs stay until copied back)
+        for j in list(on_gpu):
+            if next_use(j, t) == math.inf and j not in outputs:
+                del on_gpu[j]
+    for j in list(on_gpu):
+        if j in outputs and on_gpu[j]:
+            moved += g.ds[j].size
+            if trace is not None:
+                trace.append(("d2h", g.ds[j].name))
+    return moved
+
+
+def topological_orders(g: Graph):
+    """All operator orders that respect the data dependences (PB constraints (1)-(3))."""
+    producer = {}
+    for i, op in enumerate(g.ops):
+        for j in op.outs:
+            producer[j] = i
+    preds = [{producer[j] for j in op.ins if j in producer} for op in g.ops]
+    n = len(g.ops)
+
+    def rec(prefix, placed):
+        if len(prefix) == n:
+            yield list(prefix)
+            return
+        for i in range(n):
+            if i not in placed and preds[i] <= placed:
+                prefix.append(i)
+                placed.add(i)
+                yield from rec(prefix, placed)
+                placed.discard(i)
+                prefix.pop()
+
+    yield from rec([], set())
+
+
+def brute_force_min_transfers(g: Graph, capacity: int):
+    """Exhaustive minimum over all operator orders of the next-use transfer volume (a
+    tiny-graph stand-in for the PB optimum of Fig. 5/Fig. 6). Returns (min, n_orders,
+    n_optimal_orders)."""
+    best, n, nbest = math.inf, 0, 0
+    for order in topological_orders(g):
+        n += 1
+        v = simulate_transfers(g, order, capacity)
+        if v < best:
+            best, nbest = v, 1
+        elif v == best:
+            nbest += 1
+    return best, n, nbest
+
+
+def fig3_graph() -> tuple[Graph, dict[str, int]]:
+    """The split edge graph of Fig. 3 / Fig. 6: Im is 2 units, every
+    other DS 1 unit, convolution/remap/max split in two (kernels not drawn, size 0)."""
+    g = Graph()
+    im = g.add_ds("Im", 2, "input")
+    e = {}
+    for nm in ["E1'", "E1''", "E2'", "E2''", "E5'", "E5''", "E6'", "E6''"]:
+        e[nm] = g.add_ds(nm, 1)
+    e["E'"] = g.add_ds("E'", 1, "output")
+    e["E''"] = g.add_ds("E''", 1, "output")
+    ops = {}
+    ops["C1"] = g.add_op("C1", [im], [e["E1'"], e["E1''"]])
+    ops["C2"] = g.add_op("C2", [im], [e["E2'"], e["E2''"]])
+    ops["R1'"] = g.add_op("R1'", [e["E1'"]], [e["E5'"]])
+    ops["R1''"] = g.add_op("R1''", [e["E1''"]], [e["E5''"]])
+    ops["R2'"] = g.add_op("R2'", [e["E2'"]], [e["E6'"]])
+    ops["R2''"] = g.add_op("R2''", [e["E2''"]], [e["E6''"]])
+    ops["max1"] = g.add_op("max1", [e["E1'"], e["E2'"], e["E5'"], e["E6'"]], [e["E'"]])
+    ops["max2"] = g.add_op("max2", [e["E1''"], e["E2''"], e["E5''"], e["E6''"]], [e["E''"]])
+    return g, ops
+
+
+# ============================================================================ chunk rule
+DEPTH = 3                 # pipeline slots (H2D / compute / D2H in flight)
+MAX_CHUNK_PX = 1 << 24    # input pixels per chunk when memory does not bind
+F32 = 4
+
+
+def a256(x: int) -> int:
+    """Every arena buffer starts on a 256-byte boundary."""
+    return (int(x) + 255) // 256 * 256
+
+
+def _edge_rows(H: int, ks: int, r0: int, r1: int) -> dict:
+    rg = back_propagate_rows([("same", ks)], r0, r1, H_in=H)
+    return {"in": list(rg[0]), "out": list(rg[1])}
+
+
+def _cnn_rows(r0: int, r1: int) -> dict:
+    rg = back_propagate_rows(CNN_LAYERS, r0, r1)
+    # levels: 0 in, 1 C1, 2 T1, 3 S2, 4 T2, 5 C3, 6 T3, 7 S4, 8 T4, 9 C5, 10 T5, 11 C6
+    return {"in": list(rg[0]), "c1": list(rg[1]), "t2": list(rg[4]), "c3": list(rg[5]),
+            "t4": list(rg[8]), "out": list(rg[11])}
+
+
+def _span(r) -> int:
+    return r[1] - r[0]
+
+
+def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int = 20,
+               bias: str = "plane", budget: int = 0, max_chunk_px: int = MAX_CHUNK_PX,
+               depth: int = DEPTH, rank: int = 0, world: int = 1, device_io: bool = False) -> dict:
+    """Fused-mode plan, restated plainly; the library's
+    tg_plan_dump_json must produce the same dict (tests/test_plan_parity.py).
+
+    Offload units: the whole edge template is one unit (the paper's "best possible",
+    PAPER.md:727); the CNN is three units U1 = C1 T S2 T, U2 = C3 T S4 T, U3 = C5 T C6 whose
+    intermediates (T2, T4) stay in the chunk's device slot.
+
+    1. Batch mode (whole images per chunk) when an image has at most max_chunk_px pixels:
+       B = the largest b <= min(n, max_chunk_px // (H*W), ceil(n / (2*depth))) whose slot
+       fits. With device-resident I/O (no copies, depth 1): the largest b <= n that fits.
+    2. Otherwise row mode (split the image, never the kernel), one image per
+       chunk, R output rows: the largest R <= min(h_out, max(1, max_chunk_px // (W*f)))
+       whose widest slot fits, f = input rows per output row (edge 1, CNN 4). For CNN bias
+       planes two variants are sized -- all parameters resident, or bias rows streamed with
+       each chunk -- and the one with fewer predicted H2D bytes wins (tie: resident).
+    "fits" = param_bytes + depth * slot_bytes <= budget (budget 0 = uncapped).
+    Chunks are image-major, [i*R, min((i+1)*R, h_out)); rank g of world G executes chunks
+    [floor(C*g/G), floor(C*(g+1)/G)).
+    """
+    f = F32
+    if n <= 0 or H <= 0 or W <= 0:
+        raise ValueError("empty input")
+    if template == "edge":
+        h_out, w_out, in_per_out = H, W, 1
+        params = [ks * ks, ks * ks]
+        is_bias = [False, False]
+        rows = lambda r0, r1: _edge_rows(H, ks, r0, r1)          # noqa: E731
+        widest = lambda R: {"in": [0, min(H, R + ks - 1)], "out": [0, R]}  # noqa: E731
+    elif template == "cnn":
+        (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = cnn_dims(H, W)
+        if h5 <= 0 or w5 <= 0:
+            raise ValueError("image too small for the CNN")
+        h_out, w_out, in_per_out = h5, w5, 4
+        if bias == "plane":
+            bs = [8 * h1 * w1, 20 * h3 * w3, n5 * h5 * w5, 9 * h5 * w5]
+        else:
+            bs = [8, 20, n5, 9]
+        params = [8 * 25, bs[0], 8 * 4, 20 * 8 * 25, bs[1], 20 * 4, n5 * 20 * 25, bs[2], 9 * n5, bs[3]]
+        is_bias = [False, True, False, False, True, False, False, True, False, True]
+        rows = _cnn_rows
+        widest = lambda R: _cnn_rows(0, R)                        # noqa: E731
+    else:
+        raise ValueError(template)
+
+    def slot_bytes(B: int, R: int, rg: dict, streamed: bool) -> int:
+        s = 0
+        if not device_io:
+            s += a256(B * _span(rg["in"]) * W * f)
+        if template == "cnn":
+            s += a256(B * 8 * _span(rg["t2"]) * w2 * f)
+            s += a256(B * 20 * _span(rg["t4"]) * w4 * f)
+            if not device_io:
+                s += a256(B * 9 * R * w5 * f)
+            if streamed:
+                s += a256(8 * _span(rg["c1"]) * w1 * f)
+                s += a256(20 * _span(rg["c3"]) * w3 * f)
+                s += a256(n5 * R * w5 * f)
+                s += a256(9 * R * w5 * f)
+        elif not device_io:
+            s += a256(B * R * W * f)
+        return s
+
+    all_pb = sum(a256(p * f) for p in params)
+    nonbias_pb = sum(a256(p * f) for p, b in zip(params, is_bias) if not b)
+    if device_io:
+        depth = 1
+
+    def fits(pb: int, sb: int) -> bool:
+        return budget == 0 or pb + depth * sb <= budget
+
+    def chunk_list(split: str, B: int, R: int) -> list:
+        out = []
+        if split == "batch":
+            for b0 in range(0, n, B):
+                out.append({"img": b0, "nimg": min(B, n - b0), **rows(0, h_out)})
+        else:
+            for b0 in range(n):
+                for r0 in range(0, h_out, R):
+                    out.append({"img": b0, "nimg": 1, **rows(r0, min(h_out, r0 + R))})
+        return out
+
+    def h2d_of(chunks: list, pb: int, streamed: bool) -> int:
+        if device_io:
+            return 0
+        t = pb
+        for ch in chunks:
+            t += ch["nimg"] * _span(ch["in"]) * W * f
+            if streamed:
+                t += 8 * _span(ch["c1"]) * w1 * f + 20 * _span(ch["c3"]) * w3 * f
+                t += (n5 + 9) * _span(ch["out"]) * w5 * f
+        return t
+
+    base_bias = "none" if template == "edge" else ("resident" if bias == "plane" else "scalar")
+    choice = None
+    # 1. batch mode
+    if device_io:
+        bcap = n
+    elif H * W <= max_chunk_px:
+        bcap = min(n, max_chunk_px // (H * W), max(1, -(-n // (2 * depth))))
+    else:
+        bcap = 0
+    for b in range(bcap, 0, -1):
+        sb = slot_bytes(b, h_out, rows(0, h_out), False)
+        if fits(all_pb, sb):
+            choice = ("batch", b, h_out, base_bias, all_pb, sb)
+            break
+    # 2. row mode
+    if choice is None:
+        rcap = min(h_out, max(1, max_chunk_px // (W * in_per_out)))
+        cands = []
+        for bm in ([base_bias, "streamed"] if base_bias == "resident" else [base_bias]):
+            streamed = bm == "streamed"
+            pb = nonbias_pb if streamed else all_pb
+            lo, hi, best = 1, rcap, 0
+            while lo <= hi:                      # slot bytes grow monotonically with R
+                mid = (lo + hi) // 2
+                if fits(pb, slot_bytes(1, mid, widest(mid), streamed)):
+                    best, lo = mid, mid + 1
+                else:
+                    hi = mid - 1
+            if best:
+                sb = slot_bytes(1, best, widest(best), streamed)
+                cands.append((h2d_of(chunk_list("rows", 1, best), pb, streamed),
+                              ("rows", 1, best, bm, pb, sb)))
+        if not cands:
+            raise RuntimeError("infeasible: the budget cannot hold the smallest chunk")
+        cands.sort(key=lambda c: c[0])          # stable: resident wins ties
+        choice = cands[0][1]
+    split, B, R, bias_mode, pb, sb = choice
+    streamed = bias_mode == "streamed"
+    chunks = chunk_list(split, B, R)
+    C = len(chunks)
+    c0, c1 = (C * rank) // world, (C * (rank + 1)) // world
+    mine = chunks[c0:c1]
+    h2d = h2d_of(mine, pb, streamed)
+    d2h = 0
+    if not device_io:
+        planes_out = 9 if template == "cnn" else 1
+        d2h = sum(ch["nimg"] * planes_out * _span(ch["out"]) * w_out * f for ch in mine)
+
+    # Table 1 accounting (per template instance; images and per-image DS scale with n)
+    if template == "edge":
+        g = edge_graph(H, W, ks)
+    else:
+        g = cnn_graph_fig7(H, W, n5)
+    param_floats = sum(params)
+    per_img_floats = sum(d.size for d in g.ds if d.kind != "param")
+    out_floats = sum(d.size for d in g.ds if d.kind == "output")
+    io_lb = (n * (H * W + out_floats) + param_floats) * f
+    total = (n * per_img_floats + param_floats) * f
+    return {
+        "template": template, "n": n, "H": H, "W": W,
+        "ks": ks if template == "edge" else 0, "n5": n5 if template == "cnn" else 0,
+        "budget": budget, "depth": depth, "max_chunk_px": max_chunk_px,
+        "device_io": bool(device_io), "bias": bias_mode, "split": split, "B": B, "R": R,
+        "param_bytes": pb, "slot_bytes": sb, "arena_bytes": pb + depth * sb,
+        "n_chunks": C, "chunks": chunks, "shard": [rank, world, c0, c1],
+        "h2d_bytes": h2d, "d2h_bytes": d2h, "io_lower_bound_bytes": io_lb,
+        "total_temp_bytes": total, "n_ops_fig7": len(g.ops), "n_ds_fig7": len(g.ds),
+    }

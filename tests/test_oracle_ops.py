@@ -1,0 +1,147 @@
+"""Pins for the oracle's operators (oracle/oracle.c) against things other than itself:
+hand-computed worked examples (tests/golden/hand_examples.json), brute-force gathers with
+delta kernels (exact), torch.nn.functional in float64 (a library routine), and
+invariants that the paper's graph fixes (remap + max == max(|E1|, |E2|))."""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+import torch
+import torch.nn.functional as F
+
+from conftest import GOLDEN
+
+rng = np.random.default_rng(1234)
+
+
+def f32(a):
+    return np.asarray(a, dtype=np.float32)
+
+
+def hand():
+    with open(os.path.join(GOLDEN, "hand_examples.json")) as fh:
+        return json.load(fh)
+
+
+# ---------------------------------------------------------------- worked examples
+def test_hand_edge_4x4(orc):
+    ex = hand()["edge_4x4"]
+    img = f32(ex["image"])
+    E, E1, E2 = orc.edge(img, f32(ex["K1"]), f32(ex["K2"]), return_parts=True)
+    assert np.array_equal(E1, f32(ex["E1"]))
+    assert np.array_equal(E2, f32(ex["E2"]))
+    assert np.array_equal(E, f32(ex["E"]))
+
+
+def test_hand_subsample_5x5(orc):
+    ex = hand()["subsample_5x5"]
+    y = orc.subsample(f32(ex["x"]), f32(ex["P"]))
+    assert np.array_equal(y, f32(ex["y"]))
+
+
+def test_hand_valid_conv_3x3(orc):
+    ex = hand()["valid_3x4"]
+    y = orc.conv2d_valid(f32(ex["x"]), f32(ex["K"]))
+    assert np.array_equal(y, f32(ex["y"]))
+
+
+# ---------------------------------------------------------------- library routine pins
+def _torch_corr(x, K, padding):
+    xt = torch.from_numpy(np.asarray(x, np.float64))[None, None]
+    kt = torch.from_numpy(np.asarray(K, np.float64))[None, None]
+    return F.conv2d(xt, kt, padding=padding)[0, 0].numpy()
+
+
+def _ulp_close(a, b, ulps=1):
+    a, b = f32(a), f32(b)
+    d = np.abs(a.astype(np.float64) - b.astype(np.float64))
+    tol = ulps * np.spacing(np.maximum(np.abs(a), np.abs(b)).astype(np.float32)).astype(np.float64)
+    return bool(np.all(d <= tol + 1e-45))
+
+
+@pytest.mark.parametrize("H,W,k", [(7, 9, 3), (12, 10, 5), (20, 23, 16), (16, 16, 16), (5, 31, 4), (3, 3, 5)])
+def test_conv_same_vs_torch(orc, H, W, k):
+    x = f32(rng.standard_normal((H, W)))
+    K = f32(rng.standard_normal((k, k)))
+    y = orc.conv2d_same(x, K)
+    # torch 'same' pads (k-1)//2 top/left and k//2 bottom/right: the reading R2
+    ref = _torch_corr(x, K, "same").astype(np.float32)
+    assert y.shape == (H, W)
+    assert _ulp_close(y, ref)
+
+
+@pytest.mark.parametrize("H,W,k", [(9, 9, 5), (100, 100, 5), (13, 17, 1), (30, 11, 5)])
+def test_conv_valid_vs_torch(orc, H, W, k):
+    x = f32(rng.standard_normal((H, W)))
+    K = f32(rng.standard_normal((k, k)))
+    y = orc.conv2d_valid(x, K)
+    ref = _torch_corr(x, K, 0).astype(np.float32)
+    assert y.shape == (H - k + 1, W - k + 1)
+    assert _ulp_close(y, ref)
+
+
+def test_valid_conv_size_p367(orc):
+    """100x100 convolved with 5x5 gives 96x96."""
+    y = orc.conv2d_valid(np.zeros((100, 100), np.float32), np.ones((5, 5), np.float32))
+    assert y.shape == (96, 96)
+
+
+@pytest.mark.parametrize("H,W", [(6, 8), (7, 9), (483 // 10, 643 // 10), (2, 2)])
+def test_subsample_vs_torch(orc, H, W):
+    x = f32(rng.standard_normal((H, W)))
+    P = f32(rng.standard_normal((2, 2)))
+    y = orc.subsample(x, P)
+    ref = F.conv2d(torch.from_numpy(x.astype(np.float64))[None, None],
+                   torch.from_numpy(P.astype(np.float64))[None, None], stride=2)[0, 0].numpy()
+    assert y.shape == ((H - 2) // 2 + 1, (W - 2) // 2 + 1)
+    assert _ulp_close(y, ref.astype(np.float32))
+
+
+def test_tanh_add_neg(orc):
+    x = f32(rng.standard_normal(1000) * 3)
+    y = f32(rng.standard_normal(1000))
+    assert np.array_equal(orc.tanh(x), f32([math.tanh(float(v)) for v in x]))
+    assert np.array_equal(orc.add(x, y), x + y)   # one fp32 rounding == numpy fp32 add
+    assert np.array_equal(orc.neg(x), -x)
+
+
+def test_max_fold_order_and_ties(orc):
+    a = f32([1, -2, 0.0, 3, -0.0])
+    b = f32([2, -3, -0.0, 3, 0.0])
+    c = f32([0, -1, 0.0, 1, -1])
+    y = orc.max_fold(a, b, c)
+    assert np.array_equal(y, f32([2, -1, 0.0, 3, 0.0]))
+    # (a > b) ? a : b left fold keeps the FIRST of equal values: sign of zero from a
+    assert np.signbit(orc.max_fold(f32([-0.0]), f32([0.0]))[0])
+
+
+# ---------------------------------------------------------------- exact geometry pins
+def test_edge_delta_kernels_are_exact_gathers(orc):
+    """K1 = delta(i0,j0) turns C1 into a pure gather E1[r][c] = x~[r+i0-7][c+j0-7]; all 256
+    anchors on a 37x41 image (exact, no rounding)."""
+    H, W = 37, 41
+    x = f32(rng.random((H, W)))
+    xp = np.zeros((H + 15, W + 15), np.float32)
+    xp[7:7 + H, 7:7 + W] = x                     # zero padding 7 top/left, 8 bottom/right
+    for i0 in range(16):
+        for j0 in range(16):
+            K = np.zeros((16, 16), np.float32)
+            K[i0, j0] = 1.0
+            E, E1, E2 = orc.edge(x, K, K, return_parts=True)
+            ref = xp[i0:i0 + H, j0:j0 + W]
+            assert np.array_equal(E1, ref), (i0, j0)
+            assert np.array_equal(E, np.abs(ref))
+
+
+def test_edge_invariant_abs_max(orc):
+    """max(E1, E2, -E1, -E2) == max(|E1|, |E2|) (negation and max are exact)."""
+    from synth import edge_filter_np
+    K1, K2 = edge_filter_np()
+    x = f32(rng.random((50, 60)))
+    E, E1, E2 = orc.edge(x, K1, K2, return_parts=True)
+    assert np.array_equal(E, np.maximum(np.abs(E1), np.abs(E2)))
+    # K2 = rot90(K1) and C1, C2 are independent convolutions
+    assert np.array_equal(E1, orc.conv2d_same(x, K1))
+    assert np.array_equal(E2, orc.conv2d_same(x, K2))
