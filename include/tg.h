@@ -1,0 +1,209 @@
+/*
+ * tg.h -- C ABI of the B200-native out-of-core operator-graph executor.
+ *
+ * Method: N. Sundaram, A. Raghunathan, S. T. Chakradhar, "A framework for efficient and
+ * scalable execution of domain-specific templates on GPUs", IPDPS 2009. The
+ * user-facing contract of the paper is: templates are parametrized APIs (PAPER.md:51,
+ * :623 `edge_map = find_edges(Image, Kernel, num_orientations, Combine_op)`); a template
+ * is a graph of parallel operators with statically known footprints and splitting rules
+ * (PAPER.md:345, :349 fn. 1); the target GPU is described by parameters such as its
+ * memory capacity (Fig. 4, "Total GPU Memory" PAPER.md:409); the framework
+ * derives an execution plan and a run-time library executes it.
+ *
+ * Conventions for every function below:
+ *  - Return value: tg_status, TG_OK (0) on success, a negative TG_E_* code on failure.
+ *    No C++ exception or longjmp crosses this ABI. On failure tg_last_error() returns a
+ *    thread-local, NUL-terminated message describing the last failure of that thread.
+ *  - Data structures (DS) are dense fp32 arrays in [n][c][h][w] order (row-major, w
+ *    fastest), the paper's "floats". A DS is identified by a tg_id >= 0.
+ *  - Host buffers passed in are CALLER-OWNED; they must stay valid and unchanged (inputs,
+ *    parameters) or untouched (outputs) until tg_execute returns (or, for
+ *    tg_execute_async, until the compute stream reaches the end of the execution).
+ *    Pinned (page-locked) host memory is used as is; pageable memory is registered with
+ *    cudaHostRegister at the first execution and unregistered by tg_plan_destroy.
+ *  - Device memory is owned by the library: per device it obtains exactly ONE arena of
+ *    tg_plan_stats.peak_device_bytes bytes (never more than the device budget) through
+ *    tg_runtime.alloc (or cudaMalloc when no runtime is set) and returns it at
+ *    tg_plan_destroy. Device-resident inputs/outputs (tg_input_device/tg_output_device)
+ *    are caller-owned device buffers on the plan's device.
+ *  - Threading: a graph is not thread-safe while it is being built; a plan may be
+ *    executed repeatedly but by one thread at a time; independent plans may run
+ *    concurrently on disjoint devices.
+ */
+#ifndef TG_H
+#define TG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t tg_status;
+#define TG_OK 0
+#define TG_E_ARG (-1)          /* bad argument (NULL pointer, unknown id, bad enum)      */
+#define TG_E_SHAPE (-2)        /* shapes of the operands do not agree                    */
+#define TG_E_INFEASIBLE (-3)   /* the budget cannot hold even the smallest chunk of a unit
+                                  (unsplittable operators must fit)        */
+#define TG_E_CUDA (-4)         /* a CUDA runtime call failed (message has the CUDA error)*/
+#define TG_E_OOM (-5)          /* host or device allocation failed                       */
+#define TG_E_STATE (-6)        /* call not valid in the current state                    */
+#define TG_E_UNSUPPORTED (-7)  /* graph/mode combination not implemented                 */
+
+typedef struct tg_graph tg_graph;
+typedef struct tg_plan tg_plan;
+typedef int32_t tg_id;
+
+/* enums */
+#define TG_VALID 0        /* conv2d: output (H-k+1) x (W-k+1)                            */
+#define TG_SAME 1         /* conv2d: output H x W, zero padding (k-1)/2 top/left, k/2
+                             bottom/right (reading R2)                         */
+#define TG_ADD 0          /* elementwise y = x0 + x1 + ... (left to right)                */
+#define TG_NEG 1          /* elementwise y = -x0  (the edge template's "remap" R, R3)     */
+#define TG_AFFINE 2       /* elementwise y = a * x0 + b                                   */
+#define TG_ABS 3          /* elementwise y = |x0|                                         */
+#define TG_MAX 0          /* combine op of tg_find_edges                                  */
+#define TG_SUM 1          /* (not implemented in this round: TG_E_UNSUPPORTED)            */
+#define TG_MAXABS 2       /* (not implemented in this round: TG_E_UNSUPPORTED)            */
+#define TG_BIAS_PLANE 0   /* CNN bias: one full plane per output map (the paper's Fig. 7)
+                             shape [1][c][h][w], shared by every image of the batch       */
+#define TG_BIAS_SCALAR 1  /* CNN bias: one scalar per output map, shape [c]               */
+#define TG_FP32 0         /* all arithmetic in fp32 (FFMA); parity 1e-5 normwise          */
+#define TG_BF16_TC 1      /* CNN C3/C5/C6 on tcgen05 tensor cores, bf16 operands, fp32
+                             accumulation; parity 2e-2 normwise                           */
+#define TG_FUSED 0        /* offload units = fused templates (edge: 1 unit; CNN: 3)       */
+#define TG_PER_OP 1       /* paper mode: one operator per offload unit (not this round)   */
+#define TG_BASELINE 2     /* paper baseline of PAPER.md:613 (not this round)              */
+
+/* ------------------------------------------------------------------ graph building */
+tg_status tg_graph_create(tg_graph** g);
+void tg_graph_destroy(tg_graph* g);
+
+/* Template input (image batch) in HOST memory: [n][c][h][w] fp32, caller-owned. */
+tg_status tg_input(tg_graph* g, int64_t n, int64_t c, int64_t h, int64_t w, const float* host,
+                   tg_id* out);
+/* Template input already resident in DEVICE memory of the plan's device (in-core runs). */
+tg_status tg_input_device(tg_graph* g, int64_t n, int64_t c, int64_t h, int64_t w,
+                          const float* dev, tg_id* out);
+/* Parameter (kernel, bias, subsample weights) in HOST memory, shape [d0][d1][d2][d3]
+ * (unused leading dims = 1). Parameters are never split. */
+tg_status tg_param(tg_graph* g, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
+                   const float* host, tg_id* out);
+/* 2-D cross-correlation (reading R1) of every input plane with k[co][ci][kh][kw], summed
+ * over ci (a fully connected conv layer; Fig. 7 PAPER.md:641-713 is its per-pair
+ * expansion), plus an optional bias (-1 = none; [co] scalars or a plane [1][co][ho][wo]
+ * shared over n). pad = TG_VALID | TG_SAME. */
+tg_status tg_conv2d(tg_graph* g, tg_id x, tg_id k, tg_id bias, int32_t pad, tg_id* y);
+/* Elementwise op over same-shaped DS (op = TG_ADD | TG_NEG | TG_AFFINE | TG_ABS). */
+tg_status tg_elementwise(tg_graph* g, int32_t op, const tg_id* xs, int32_t nx, float a,
+                         float b, tg_id* y);
+tg_status tg_tanh(tg_graph* g, tg_id x, tg_id* y);
+/* n-ary max: y = left fold (x_k > m) ? x_k : m over xs in order (reading R5). */
+tg_status tg_max_combine(tg_graph* g, const tg_id* xs, int32_t nx, tg_id* y);
+/* Subsample: window s, stride s, kernel p[c][s][s] per plane (reading R8). */
+tg_status tg_subsample(tg_graph* g, tg_id x, tg_id p, int32_t s, tg_id* y);
+/* Bind template output y to caller-owned HOST memory sized by tg_shape(y). */
+tg_status tg_output(tg_graph* g, tg_id y, float* host_dst);
+/* Bind template output y to caller-owned DEVICE memory on the plan's device. */
+tg_status tg_output_device(tg_graph* g, tg_id y, float* dev_dst);
+/* dims = {n, c, h, w} of DS id. */
+tg_status tg_shape(const tg_graph* g, tg_id id, int64_t dims[4]);
+
+/* Template helpers (PAPER.md:623 find_edges; PAPER.md:635 the CNN built from torch5
+ * primitives). Both only append primitive nodes to the graph. */
+/* Edge detection: num_orientations/2 SAME convolutions of img with
+ * `kernel` ([1][1][k][k], k <= 16) and its rot90 rotations, as many remaps (negations)
+ * and one max combine. num_orientations = 4 (8: TG_E_UNSUPPORTED this round);
+ * combine_op = TG_MAX. */
+tg_status tg_find_edges(tg_graph* g, tg_id img, tg_id kernel, int32_t num_orientations,
+                        int32_t combine_op, tg_id* edge_map);
+/* CNN of SURVEY F2 (11 layers): C1(1->8,5x5) T S2 T C3(8->20,5x5) T S4 T C5(20->n5,5x5)
+ * T C6(n5->9,1x1); 1 <= n5 <= 128 (small net 20, large net 120). params order: K1[8][1][5][5],
+ * B1, P2[8][2][2], K3[20][8][5][5], B3, P4[20][2][2], K5[n5][20][5][5], B5, K6[9][n5][1][1],
+ * B6; Bk = plane [1][c][h][w] (TG_BIAS_PLANE) or [c] (TG_BIAS_SCALAR). */
+tg_status tg_cnn(tg_graph* g, tg_id img, int32_t n5, const tg_id params[10], int32_t bias_mode,
+                 tg_id* out);
+
+/* ------------------------------------------------------------------ target parameters */
+/* Devices the plan runs on (one host thread per device; chunks are split contiguously).
+ * Default: the current CUDA device. */
+tg_status tg_set_devices(tg_graph* g, const int32_t* ordinals, int32_t n);
+/* Device-memory budget per device in bytes ("Total GPU Memory"); 0 =
+ * uncapped. The plan's arena never exceeds it. */
+tg_status tg_set_device_budget(tg_graph* g, uint64_t bytes_per_device);
+tg_status tg_set_precision(tg_graph* g, int32_t prec);
+/* Input pixels per chunk when memory does not bind (default 1<<24) and pipeline depth
+ * (in-flight chunk slots, default 3, 1..8). */
+tg_status tg_set_chunking(tg_graph* g, int64_t max_chunk_px, int32_t depth);
+/* Multi-process sharding: this process executes chunk range [floor(C*rank/world),
+ * floor(C*(rank+1)/world)) of the global chunk list (no collective). */
+tg_status tg_set_shard(tg_graph* g, int32_t rank, int32_t world);
+
+/* Runtime hooks (PyTorch-backed in the Python binding). alloc returns device memory on
+ * `dev` (NULL on failure); stream returns a cudaStream_t for which = 0 (H2D), 1 (compute),
+ * 2 (D2H). Any member may be NULL (library default). The struct is copied. */
+typedef struct {
+    void* (*alloc)(size_t bytes, int32_t dev, void* ctx);
+    void (*free)(void* ptr, int32_t dev, void* ctx);
+    void* (*stream)(int32_t dev, int32_t which, void* ctx);
+    void* ctx;
+} tg_runtime;
+tg_status tg_set_runtime(tg_graph* g, const tg_runtime* rt);
+
+/* ------------------------------------------------------------------ plan / execute */
+/* Build the execution plan: recognise the template's offload units, split into chunks
+ * (PAPER.md:359-371), order them and size every transfer. Pure host
+ * code: works without a GPU. mode = TG_FUSED. The graph must outlive the plan. */
+tg_status tg_plan_create(const tg_graph* g, int32_t mode, tg_plan** plan);
+
+typedef struct {
+    uint64_t h2d_bytes;              /* predicted host->device bytes of this shard      */
+    uint64_t d2h_bytes;              /* predicted device->host bytes of this shard      */
+    uint64_t io_lower_bound_bytes;   /* template inputs + params + outputs, once        */
+    uint64_t total_temp_bytes;       /* sum of all DS at Fig. 7 granularity (Table 1)   */
+    uint64_t peak_device_bytes[8];   /* arena bytes per device of the plan              */
+    int64_t n_chunks;                /* global chunk count                              */
+    int64_t n_units;                 /* fused offload units per chunk                   */
+    int64_t n_ops_fig7;              /* operators of the template at Fig. 7 granularity */
+    int64_t n_ds_fig7;               /* data structures at Fig. 7 granularity           */
+    int64_t chunk_begin, chunk_end;  /* this shard's chunk range                        */
+    uint64_t host_registered_bytes;  /* pageable host bytes registered by the library   */
+} tg_plan_stats;
+tg_status tg_plan_stats_get(const tg_plan* plan, tg_plan_stats* out);
+
+/* Plan as JSON (chunks with halo row ranges, slot layout, byte counts); compared
+ * bit-exactly with the planner oracle. Writes at most cap bytes incl. NUL; *needed =
+ * required size incl. NUL. Returns TG_E_ARG when buf is too small (buf may be NULL). */
+tg_status tg_plan_dump_json(const tg_plan* plan, char* buf, size_t cap, size_t* needed);
+
+/* Execute the plan; blocks until outputs are valid in their destinations. */
+tg_status tg_execute(tg_plan* plan);
+/* Same, but returns once all work is enqueued; completion is ordered before any later work
+ * on the compute stream (which = 1) of every device of the plan. */
+tg_status tg_execute_async(tg_plan* plan);
+
+/* Per-launch timing of the fused kernels measured with CUDA events on the compute stream
+ * (enable before executing; tg_plan_timing_get synchronizes). Times are summed over all
+ * executions since enabling. */
+typedef struct {
+    int64_t launches;        /* kernel launches of the library                          */
+    int64_t executions;
+    double kernel_ms[4];     /* per unit kind: 0 edge, 1 CNN U1, 2 CNN U2, 3 CNN U3     */
+    int64_t unit_launches[4];
+    double h2d_ms, d2h_ms;   /* summed copy durations (copy streams)                    */
+} tg_timing;
+tg_status tg_plan_set_profiling(tg_plan* plan, int32_t on);
+tg_status tg_plan_timing_get(tg_plan* plan, tg_timing* out);
+/* Kernel launches issued by the library since plan creation (always counted). */
+int64_t tg_plan_launch_count(const tg_plan* plan);
+
+void tg_plan_destroy(tg_plan* plan);
+const char* tg_last_error(void);
+/* Library version string, e.g. "tg 0.1 sm_100a". */
+const char* tg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TG_H */

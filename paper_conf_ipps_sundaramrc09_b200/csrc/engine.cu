@@ -1,0 +1,597 @@
+// engine.cu -- the run-time library ("a simple run-time library to
+// orchestrate execution") that executes a plan on one or more B200s.
+//
+// Per device: ONE arena of exactly plan.arena_bytes (parameters + `depth` chunk slots;
+// a static layout, so the "fragmentation" margin of PAPER.md:409 is not needed), three
+// streams (H2D copy engine, compute, D2H copy engine) and per-slot events. The host thread
+// enqueues, for every chunk k of its shard, in slot s = k % depth:
+//     H2D   waits compute(k - depth)          copy input rows (+halo, +streamed bias rows)
+//     comp  waits H2D(k), D2H(k - depth)      fused offload-unit kernels
+//     D2H   waits comp(k)                     copy output rows into the caller's buffer
+// so copies of chunk k+1 / k-1 overlap the kernels of chunk k (the overlap the paper's
+// GPUs could not do). Everything is asynchronous; tg_execute synchronizes
+// once at the end. Several devices: one host thread per device over contiguous chunk
+// ranges; no collective.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "kernels/kernels.h"
+#include "tg_internal.h"
+
+using namespace tg;
+
+namespace {
+
+struct ProfRec {
+    int kind;  // 0 edge, 1 U1, 2 U2, 3 U3, 10 h2d, 11 d2h
+    cudaEvent_t a, b;
+};
+
+struct DevState {
+    int dev = 0;
+    cudaStream_t st[3] = {nullptr, nullptr, nullptr};
+    bool own_st[3] = {false, false, false};
+    char* arena = nullptr;
+    bool own_arena = false;
+    std::vector<cudaEvent_t> ev_h2d, ev_comp, ev_d2h;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_params = nullptr;
+    int64_t c0 = 0, c1 = 0;
+    std::vector<ProfRec> prof;
+    std::vector<cudaEvent_t> ev_pool;
+    int64_t launches = 0;
+};
+
+}  // namespace
+
+struct tg_exec {
+    std::vector<DevState> devs;
+    bool ready = false;
+    std::vector<void*> registered;
+    uint64_t registered_bytes = 0;
+    bool profiling = false;
+    tg_timing timing{};
+};
+
+namespace {
+
+#define CK(call)                                                                                   \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess) {                                                                   \
+            char m_[384];                                                                          \
+            std::snprintf(m_, sizeof m_, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_),   \
+                          __FILE__, __LINE__);                                                     \
+            return fail(TG_E_CUDA, m_);                                                            \
+        }                                                                                          \
+    } while (0)
+
+const Graph& graph_of(const tg_plan* p) { return p->graph->g; }
+
+cudaEvent_t pool_event(DevState& d) {
+    if (!d.ev_pool.empty()) {
+        cudaEvent_t e = d.ev_pool.back();
+        d.ev_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+    return e;
+}
+
+tg_status init_device(tg_plan* p, DevState& d) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    CK(cudaSetDevice(d.dev));
+    for (int w = 0; w < 3; ++w) {
+        void* s = (g.has_rt && g.rt.stream) ? g.rt.stream(d.dev, w, g.rt.ctx) : nullptr;
+        if (s) {
+            d.st[w] = (cudaStream_t)s;
+        } else {
+            CK(cudaStreamCreateWithFlags(&d.st[w], cudaStreamNonBlocking));
+            d.own_st[w] = true;
+        }
+    }
+    const size_t bytes = std::max<uint64_t>(c.arena_bytes, 256);
+    if (g.has_rt && g.rt.alloc) {
+        d.arena = (char*)g.rt.alloc(bytes, d.dev, g.rt.ctx);
+        if (!d.arena) return fail(TG_E_OOM, "runtime alloc of the device arena failed");
+    } else {
+        cudaError_t e = cudaMalloc((void**)&d.arena, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(TG_E_OOM, std::string("cudaMalloc of the device arena failed: ") + cudaGetErrorString(e));
+        }
+        d.own_arena = true;
+    }
+    const unsigned flags = cudaEventDisableTiming;
+    d.ev_h2d.resize(c.depth);
+    d.ev_comp.resize(c.depth);
+    d.ev_d2h.resize(c.depth);
+    for (int s = 0; s < c.depth; ++s) {
+        CK(cudaEventCreateWithFlags(&d.ev_h2d[s], flags));
+        CK(cudaEventCreateWithFlags(&d.ev_comp[s], flags));
+        CK(cudaEventCreateWithFlags(&d.ev_d2h[s], flags));
+    }
+    CK(cudaEventCreateWithFlags(&d.ev_fork, flags));
+    CK(cudaEventCreateWithFlags(&d.ev_join, flags));
+    CK(cudaEventCreateWithFlags(&d.ev_params, flags));
+    return TG_OK;
+}
+
+// Register caller-owned pageable host buffers once, so async copies run at full speed.
+tg_status register_host(tg_plan* p, tg_exec* x) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    if (c.device_io) return TG_OK;
+    std::vector<std::pair<void*, size_t>> bufs;
+    const Ds& X = g.ds[c.t.input];
+    const Ds& Y = g.ds[c.t.output];
+    bufs.push_back({(void*)X.src, (size_t)X.numel() * 4});
+    bufs.push_back({(void*)Y.dst, (size_t)Y.numel() * 4});
+    for (int id : c.param_ds) bufs.push_back({(void*)g.ds[id].src, (size_t)g.ds[id].numel() * 4});
+    for (auto& b : bufs) {
+        if (b.second < (1u << 20)) continue;  // small: pageable copies are fine
+        cudaPointerAttributes at{};
+        if (cudaPointerGetAttributes(&at, b.first) == cudaSuccess && at.type == cudaMemoryTypeHost) continue;
+        cudaGetLastError();
+        cudaError_t e = cudaHostRegister(b.first, b.second, cudaHostRegisterDefault);
+        if (e == cudaSuccess) {
+            x->registered.push_back(b.first);
+            x->registered_bytes += b.second;
+        } else {
+            cudaGetLastError();  // overlapping/foreign registration: fall back to pageable copies
+        }
+    }
+    return TG_OK;
+}
+
+inline char* slot_base(const PlanCore& c, DevState& d, int s) {
+    return d.arena + c.param_bytes + (uint64_t)s * c.slot_bytes;
+}
+
+// Copies of chunk inputs into slot s (H2D stream).
+tg_status enqueue_h2d(const tg_plan* p, DevState& d, const Chunk& ch, int s) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    const Template& t = c.t;
+    const Ds& X = g.ds[t.input];
+    char* base = slot_base(c, d, s);
+    const size_t W = (size_t)t.W;
+    const size_t rows = (size_t)ch.in.n();
+    // input rows [in.a, in.b) of nimg images: one strided copy
+    CK(cudaMemcpy2DAsync(base + c.slot.in, rows * W * 4, X.src + (size_t)ch.img * t.H * W + (size_t)ch.in.a * W,
+                         (size_t)t.H * W * 4, rows * W * 4, (size_t)ch.nimg, cudaMemcpyHostToDevice, d.st[0]));
+    if (t.kind == Tmpl::Cnn && c.bias == "streamed") {
+        // bias rows of every level this chunk's outputs depend on (planes strided)
+        struct B {
+            int prm;
+            uint64_t off;
+            int64_t planes, row0, rows, h, w;
+        } bs[4] = {{1, c.slot.b1, 8, ch.c1.a, ch.c1.n(), t.h[1], t.w[1]},
+                   {4, c.slot.b3, 20, ch.c3.a, ch.c3.n(), t.h[3], t.w[3]},
+                   {7, c.slot.b5, t.n5, ch.out.a, ch.out.n(), t.h[5], t.w[5]},
+                   {9, c.slot.b6, 9, ch.out.a, ch.out.n(), t.h[5], t.w[5]}};
+        for (const B& b : bs) {
+            const float* src = g.ds[t.prm[b.prm]].src + (size_t)b.row0 * b.w;
+            CK(cudaMemcpy2DAsync(base + b.off, (size_t)b.rows * b.w * 4, src, (size_t)b.h * b.w * 4,
+                                 (size_t)b.rows * b.w * 4, (size_t)b.planes, cudaMemcpyHostToDevice, d.st[0]));
+        }
+    }
+    return TG_OK;
+}
+
+tg_status enqueue_d2h(const tg_plan* p, DevState& d, const Chunk& ch, int s) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    const Template& t = c.t;
+    const Ds& Y = g.ds[t.output];
+    char* base = slot_base(c, d, s);
+    if (t.kind == Tmpl::Edge) {
+        const size_t W = (size_t)t.W, rows = (size_t)ch.out.n();
+        CK(cudaMemcpy2DAsync(Y.dst + (size_t)ch.img * t.H * W + (size_t)ch.out.a * W, (size_t)t.H * W * 4,
+                             base + c.slot.out, rows * W * 4, rows * W * 4, (size_t)ch.nimg, cudaMemcpyDeviceToHost,
+                             d.st[2]));
+    } else {
+        const size_t w5 = (size_t)t.w[5], h5 = (size_t)t.h[5], rows = (size_t)ch.out.n();
+        CK(cudaMemcpy2DAsync(Y.dst + (size_t)ch.img * 9 * h5 * w5 + (size_t)ch.out.a * w5, h5 * w5 * 4,
+                             base + c.slot.out, rows * w5 * 4, rows * w5 * 4, (size_t)ch.nimg * 9,
+                             cudaMemcpyDeviceToHost, d.st[2]));
+    }
+    return TG_OK;
+}
+
+struct KernelTimer {
+    tg_exec* x;
+    DevState& d;
+    int kind;
+    cudaEvent_t a = nullptr, b = nullptr;
+    KernelTimer(tg_exec* x_, DevState& d_, int kind_, cudaStream_t s) : x(x_), d(d_), kind(kind_) {
+        if (x->profiling) {
+            a = pool_event(d);
+            b = pool_event(d);
+            if (a) cudaEventRecord(a, s);
+        }
+    }
+    void done(cudaStream_t s) {
+        if (x->profiling && a && b) {
+            cudaEventRecord(b, s);
+            d.prof.push_back({kind, a, b});
+        }
+    }
+};
+
+tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int s) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    const Template& t = c.t;
+    char* base = slot_base(c, d, s);
+    cudaStream_t cs = d.st[1];
+    auto param = [&](int i) -> const float* {
+        return c.param_off[i] == UINT64_MAX ? nullptr : (const float*)(d.arena + c.param_off[i]);
+    };
+    const Ds& X = g.ds[t.input];
+    const Ds& Y = g.ds[t.output];
+    if (t.kind == Tmpl::Edge) {
+        EdgeArgs a{};
+        if (c.device_io) {
+            a.in = X.src + (size_t)ch.img * t.H * t.W;
+            a.in_img_stride = t.H * t.W;
+            a.in_row0 = 0;
+            a.in_rows = t.H;
+            a.out = Y.dst + (size_t)ch.img * t.H * t.W + (size_t)ch.out.a * t.W;
+            a.out_img_stride = t.H * t.W;
+        } else {
+            a.in = (const float*)(base + c.slot.in);
+            a.in_img_stride = ch.in.n() * t.W;
+            a.in_row0 = ch.in.a;
+            a.in_rows = ch.in.n();
+            a.out = (float*)(base + c.slot.out);
+            a.out_img_stride = ch.out.n() * t.W;
+        }
+        a.out_row0 = ch.out.a;
+        a.out_rows = ch.out.n();
+        a.H = t.H;
+        a.W = t.W;
+        a.nimg = ch.nimg;
+        a.k1 = param(0);
+        a.k2 = param(1);
+        a.ks = t.ks;
+        KernelTimer kt(x, d, 0, cs);
+        CK(launch_edge(a, cs));
+        kt.done(cs);
+        ++d.launches;
+        return TG_OK;
+    }
+    // CNN: U1 -> U2 -> U3 on the compute stream; T2 and T4 stay in the slot
+    const bool strm = c.bias == "streamed";
+    const bool plane = c.bias != "scalar";
+    const int64_t w1 = t.w[1], w2 = t.w[2], w3 = t.w[3], w4 = t.w[4], w5 = t.w[5];
+    float* t2 = (float*)(base + c.slot.t2);
+    float* t4 = (float*)(base + c.slot.t4);
+    {
+        CnnU1Args a{};
+        if (c.device_io) {
+            a.in = X.src + (size_t)ch.img * t.H * t.W;
+            a.in_img_stride = t.H * t.W;
+            a.in_row0 = 0;
+        } else {
+            a.in = (const float*)(base + c.slot.in);
+            a.in_img_stride = ch.in.n() * t.W;
+            a.in_row0 = ch.in.a;
+        }
+        a.W = t.W;
+        a.k1 = param(0);
+        a.b1_plane = plane;
+        if (strm) {
+            a.b1 = (const float*)(base + c.slot.b1);
+            a.b1_row0 = ch.c1.a;
+            a.b1_rows = ch.c1.n();
+        } else {
+            a.b1 = param(1);
+            a.b1_row0 = 0;
+            a.b1_rows = t.h[1];
+        }
+        a.p2 = param(2);
+        a.t2 = t2;
+        a.t2_img_stride = 8 * ch.t2.n() * w2;
+        a.t2_row0 = ch.t2.a;
+        a.t2_rows = ch.t2.n();
+        a.w1 = w1;
+        a.w2 = w2;
+        a.nimg = ch.nimg;
+        KernelTimer kt(x, d, 1, cs);
+        CK(launch_cnn_u1(a, cs));
+        kt.done(cs);
+        ++d.launches;
+    }
+    {
+        CnnU2Args a{};
+        a.t2 = t2;
+        a.t2_img_stride = 8 * ch.t2.n() * w2;
+        a.t2_row0 = ch.t2.a;
+        a.t2_rows = ch.t2.n();
+        a.w2 = w2;
+        a.k3 = param(3);
+        a.b3_plane = plane;
+        if (strm) {
+            a.b3 = (const float*)(base + c.slot.b3);
+            a.b3_row0 = ch.c3.a;
+            a.b3_rows = ch.c3.n();
+        } else {
+            a.b3 = param(4);
+            a.b3_row0 = 0;
+            a.b3_rows = t.h[3];
+        }
+        a.p4 = param(5);
+        a.t4 = t4;
+        a.t4_img_stride = 20 * ch.t4.n() * w4;
+        a.t4_row0 = ch.t4.a;
+        a.t4_rows = ch.t4.n();
+        a.w3 = w3;
+        a.w4 = w4;
+        a.nimg = ch.nimg;
+        a.bf16_tc = c.precision == TG_BF16_TC;
+        KernelTimer kt(x, d, 2, cs);
+        CK(launch_cnn_u2(a, cs));
+        kt.done(cs);
+        ++d.launches;
+    }
+    {
+        CnnU3Args a{};
+        a.t4 = t4;
+        a.t4_img_stride = 20 * ch.t4.n() * w4;
+        a.t4_row0 = ch.t4.a;
+        a.t4_rows = ch.t4.n();
+        a.w4 = w4;
+        a.k5 = param(6);
+        a.k6 = param(8);
+        a.b5_plane = a.b6_plane = plane;
+        if (strm) {
+            a.b5 = (const float*)(base + c.slot.b5);
+            a.b6 = (const float*)(base + c.slot.b6);
+            a.b5_row0 = a.b6_row0 = ch.out.a;
+            a.b5_rows = a.b6_rows = ch.out.n();
+        } else {
+            a.b5 = param(7);
+            a.b6 = param(9);
+            a.b5_row0 = a.b6_row0 = 0;
+            a.b5_rows = a.b6_rows = t.h[5];
+        }
+        if (c.device_io) {
+            a.out = Y.dst + (size_t)ch.img * 9 * t.h[5] * w5 + (size_t)ch.out.a * w5;
+            a.out_img_stride = 9 * t.h[5] * w5;
+            a.out_plane_stride = t.h[5] * w5;
+        } else {
+            a.out = (float*)(base + c.slot.out);
+            a.out_img_stride = 9 * ch.out.n() * w5;
+            a.out_plane_stride = ch.out.n() * w5;
+        }
+        a.out_row0 = ch.out.a;
+        a.out_rows = ch.out.n();
+        a.w5 = w5;
+        a.n5 = t.n5;
+        a.nimg = ch.nimg;
+        a.bf16_tc = c.precision == TG_BF16_TC;
+        KernelTimer kt(x, d, 3, cs);
+        CK(launch_cnn_u3(a, cs));
+        kt.done(cs);
+        ++d.launches;
+    }
+    return TG_OK;
+}
+
+tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    CK(cudaSetDevice(d.dev));
+    cudaStream_t S0 = d.st[0], S1 = d.st[1], S2 = d.st[2];
+    // fork the copy streams off the compute stream (orders this execution after earlier
+    // work on the compute stream, including a previous execution's join)
+    CK(cudaEventRecord(d.ev_fork, S1));
+    CK(cudaStreamWaitEvent(S0, d.ev_fork, 0));
+    CK(cudaStreamWaitEvent(S2, d.ev_fork, 0));
+    // parameters: once per execution (never split)
+    {
+        ProfRec pr{10, nullptr, nullptr};
+        if (x->profiling) {
+            pr.a = pool_event(d);
+            pr.b = pool_event(d);
+            cudaEventRecord(pr.a, S0);
+        }
+        for (size_t i = 0; i < c.param_ds.size(); ++i) {
+            if (c.param_off[i] == UINT64_MAX) continue;
+            const Ds& P = g.ds[c.param_ds[i]];
+            CK(cudaMemcpyAsync(d.arena + c.param_off[i], P.src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
+        }
+        if (x->profiling) {
+            cudaEventRecord(pr.b, S0);
+            d.prof.push_back(pr);
+        }
+        CK(cudaEventRecord(d.ev_params, S0));
+        CK(cudaStreamWaitEvent(S1, d.ev_params, 0));
+    }
+    const int D = c.depth;
+    for (int64_t k = 0; k < d.c1 - d.c0; ++k) {
+        const Chunk& ch = c.chunks[d.c0 + k];
+        const int s = (int)(k % D);
+        if (!c.device_io) {
+            if (k >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
+            ProfRec pr{10, nullptr, nullptr};
+            if (x->profiling) {
+                pr.a = pool_event(d);
+                pr.b = pool_event(d);
+                cudaEventRecord(pr.a, S0);
+            }
+            tg_status st = enqueue_h2d(p, d, ch, s);
+            if (st != TG_OK) return st;
+            if (x->profiling) {
+                cudaEventRecord(pr.b, S0);
+                d.prof.push_back(pr);
+            }
+            CK(cudaEventRecord(d.ev_h2d[s], S0));
+            CK(cudaStreamWaitEvent(S1, d.ev_h2d[s], 0));
+            if (k >= D) CK(cudaStreamWaitEvent(S1, d.ev_d2h[s], 0));
+        }
+        tg_status st = launch_units(p, x, d, ch, s);
+        if (st != TG_OK) return st;
+        CK(cudaEventRecord(d.ev_comp[s], S1));
+        if (!c.device_io) {
+            CK(cudaStreamWaitEvent(S2, d.ev_comp[s], 0));
+            ProfRec pr{11, nullptr, nullptr};
+            if (x->profiling) {
+                pr.a = pool_event(d);
+                pr.b = pool_event(d);
+                cudaEventRecord(pr.a, S2);
+            }
+            st = enqueue_d2h(p, d, ch, s);
+            if (st != TG_OK) return st;
+            if (x->profiling) {
+                cudaEventRecord(pr.b, S2);
+                d.prof.push_back(pr);
+            }
+            CK(cudaEventRecord(d.ev_d2h[s], S2));
+        }
+    }
+    // join: the compute stream waits for the last D2H, so it marks the end of everything
+    CK(cudaEventRecord(d.ev_join, S2));
+    CK(cudaStreamWaitEvent(S1, d.ev_join, 0));
+    if (blocking) CK(cudaStreamSynchronize(S1));
+    return TG_OK;
+}
+
+}  // namespace
+
+namespace tg {
+
+tg_status exec_run(tg_plan* p, bool blocking) {
+    if (!p->exec) p->exec = new tg_exec();
+    tg_exec* x = p->exec;
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    if (!x->ready) {
+        std::vector<int32_t> devs = g.devices;
+        if (devs.empty()) {
+            int cur = 0;
+            CK(cudaGetDevice(&cur));
+            devs.push_back(cur);
+        }
+        x->devs.resize(devs.size());
+        const int64_t n = c.c1 - c.c0, nd = (int64_t)devs.size();
+        for (size_t i = 0; i < devs.size(); ++i) {
+            DevState& d = x->devs[i];
+            d.dev = devs[i];
+            d.c0 = c.c0 + n * (int64_t)i / nd;
+            d.c1 = c.c0 + n * (int64_t)(i + 1) / nd;
+            tg_status st = init_device(p, d);
+            if (st != TG_OK) return st;
+        }
+        tg_status st = register_host(p, x);
+        if (st != TG_OK) return st;
+        x->ready = true;
+    }
+    tg_status result = TG_OK;
+    if (x->devs.size() == 1) {
+        result = run_device(p, x, x->devs[0], blocking);
+    } else {
+        std::vector<tg_status> sts(x->devs.size(), TG_OK);
+        std::vector<std::string> errs(x->devs.size());
+        std::vector<std::thread> th;
+        for (size_t i = 0; i < x->devs.size(); ++i)
+            th.emplace_back([&, i] {
+                sts[i] = run_device(p, x, x->devs[i], blocking);
+                if (sts[i] != TG_OK) errs[i] = tg_last_error();
+            });
+        for (auto& t : th) t.join();
+        for (size_t i = 0; i < sts.size(); ++i)
+            if (sts[i] != TG_OK) {
+                result = fail(sts[i], errs[i]);
+                break;
+            }
+    }
+    int64_t l = 0;
+    for (auto& d : x->devs) l += d.launches;
+    p->launches = l;
+    ++x->timing.executions;
+    return result;
+}
+
+tg_status exec_set_profiling(tg_plan* p, bool on) {
+    if (!p->exec) p->exec = new tg_exec();
+    p->exec->profiling = on;
+    if (on) {
+        p->exec->timing = tg_timing{};
+    }
+    return TG_OK;
+}
+
+tg_status exec_timing(tg_plan* p, tg_timing* out) {
+    if (!p->exec) {
+        *out = tg_timing{};
+        return TG_OK;
+    }
+    tg_exec* x = p->exec;
+    for (auto& d : x->devs) {
+        CK(cudaSetDevice(d.dev));
+        for (auto& r : d.prof) {
+            CK(cudaEventSynchronize(r.b));
+            float ms = 0.f;
+            CK(cudaEventElapsedTime(&ms, r.a, r.b));
+            if (r.kind < 4) {
+                x->timing.kernel_ms[r.kind] += ms;
+                x->timing.unit_launches[r.kind] += 1;
+                x->timing.launches += 1;
+            } else if (r.kind == 10) {
+                x->timing.h2d_ms += ms;
+            } else {
+                x->timing.d2h_ms += ms;
+            }
+            d.ev_pool.push_back(r.a);
+            d.ev_pool.push_back(r.b);
+        }
+        d.prof.clear();
+    }
+    *out = x->timing;
+    return TG_OK;
+}
+
+void exec_destroy(tg_plan* p) {
+    tg_exec* x = p->exec;
+    if (!x) return;
+    const Graph& g = graph_of(p);
+    for (auto& d : x->devs) {
+        if (cudaSetDevice(d.dev) != cudaSuccess) continue;
+        if (d.st[1]) cudaStreamSynchronize(d.st[1]);
+        for (auto& r : d.prof) {
+            cudaEventDestroy(r.a);
+            cudaEventDestroy(r.b);
+        }
+        for (auto e : d.ev_pool) cudaEventDestroy(e);
+        for (auto* v : {&d.ev_h2d, &d.ev_comp, &d.ev_d2h})
+            for (auto e : *v)
+                if (e) cudaEventDestroy(e);
+        for (auto e : {d.ev_fork, d.ev_join, d.ev_params})
+            if (e) cudaEventDestroy(e);
+        if (d.arena) {
+            if (d.own_arena)
+                cudaFree(d.arena);
+            else if (g.has_rt && g.rt.free)
+                g.rt.free(d.arena, d.dev, g.rt.ctx);
+        }
+        for (int w = 0; w < 3; ++w)
+            if (d.own_st[w] && d.st[w]) cudaStreamDestroy(d.st[w]);
+    }
+    for (void* ptr : x->registered) cudaHostUnregister(ptr);
+    cudaGetLastError();
+    delete x;
+    p->exec = nullptr;
+}
+
+uint64_t exec_registered_bytes(const tg_plan* p) { return p->exec ? p->exec->registered_bytes : 0; }
+
+}  // namespace tg

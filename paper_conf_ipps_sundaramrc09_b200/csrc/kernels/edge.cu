@@ -1,0 +1,173 @@
+// edge.cu -- K1, the fused edge-detection offload unit for sm_100a.
+//
+// Computes the whole 4-orientation edge template of PAPER.md:629 (Fig. 3 graph:
+// C1: E1 = Im*K1, C2: E2 = Im*K2, R1: E5 = -E1, R2: E6 = -E2, max: E = max(E1,E2,E5,E6))
+// in ONE pass over a chunk, so E1, E2, E5, E6 never leave registers -- the paper's "best
+// possible" configuration. SAME zero padding with anchor (ks-1)/2
+// (R2); a ks x ks kernel (ks <= 16) is embedded in a 16 x 16 frame at offset
+// 7 - (ks-1)/2 so one code path serves every size.
+//
+// Roofline: 2 x 256 FMA per output pixel vs 8 HBM bytes -> FP32-ALU
+// bound (128 flop/B >> ridge ~11 flop/B). The kernel is therefore organised to issue
+// FFMA back to back: each thread owns a 1 x 16 strip of outputs for both filters
+// (32 accumulators), and for each of the 16 filter rows loads its 32-wide input window
+// with 8 conflict-free LDS.128 and both filter rows with 8 broadcast LDS.128, then issues
+// 512 FFMA -- 3% load overhead. Tiles of 64 x 64 outputs, 256 threads; lanes of a warp own
+// 32 consecutive rows (row pitch 84 floats = 21 x 16 B, odd, so the 8 lanes of each LDS.128
+// phase hit 8 distinct 16-byte bank groups). The input tile (79 x 80 floats incl. the
+// 15-row/col halo) is staged once per CTA with 128-bit coalesced loads; zero fill gives
+// the SAME padding at image borders.
+//
+// Bit-exactness under splitting: every output pixel is the same sequence of fmaf in the
+// same order (filter row i, then column j) whatever tile or chunk it falls in.
+#include <cuda_runtime.h>
+
+#include "kernels.h"
+
+namespace tg {
+namespace {
+
+constexpr int kTileR = 64;
+constexpr int kTileC = 64;
+constexpr int kSmR = kTileR + 15;  // 79 rows incl. halo
+constexpr int kSmC = kTileC + 16;  // 80 cols: [c0-8, c0+72)
+constexpr int kPitch = 84;         // floats; 84/4 = 21 (odd) -> conflict-free LDS.128 across rows
+constexpr int kThreads = 256;
+
+__global__ void __launch_bounds__(kThreads, 2) edge_fused_kernel(EdgeArgs a) {
+    __shared__ __align__(16) float xs[kSmR * kPitch];
+    __shared__ __align__(16) float w1s[256];
+    __shared__ __align__(16) float w2s[256];
+
+    const int tid = threadIdx.x;
+    const int64_t img = blockIdx.z;
+    const int64_t tile_r0 = a.out_row0 + (int64_t)blockIdx.y * kTileR;  // global output row
+    const int64_t tile_c0 = (int64_t)blockIdx.x * kTileC;
+
+    // filters embedded in a 16 x 16 frame (zeros outside the ks x ks kernel)
+    {
+        const int off = 7 - (a.ks - 1) / 2;
+        const int r = tid >> 4, c = tid & 15;
+        const int rr = r - off, cc = c - off;
+        const bool in = rr >= 0 && rr < a.ks && cc >= 0 && cc < a.ks;
+        w1s[tid] = in ? __ldg(a.k1 + rr * a.ks + cc) : 0.f;
+        w2s[tid] = in ? __ldg(a.k2 + rr * a.ks + cc) : 0.f;
+    }
+
+    // stage the input tile: smem (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)
+    const float* __restrict__ inb = a.in + img * a.in_img_stride;
+    const bool vec = (a.W & 3) == 0 && ((reinterpret_cast<uintptr_t>(a.in) & 15) == 0) &&
+                     (a.in_img_stride & 3) == 0;
+    for (int idx = tid; idx < kSmR * (kSmC / 4); idx += kThreads) {
+        const int sr = idx / (kSmC / 4);
+        const int q = idx - sr * (kSmC / 4);
+        const int64_t g = tile_r0 - 7 + sr;
+        const int64_t gc = tile_c0 - 8 + 4 * q;
+        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (g >= 0 && g < a.H && g >= a.in_row0 && g < a.in_row0 + a.in_rows) {
+            const float* row = inb + (g - a.in_row0) * a.W;
+            if (vec && gc >= 0 && gc + 3 < a.W) {
+                v = __ldg(reinterpret_cast<const float4*>(row + gc));
+            } else {
+                v.x = (gc + 0 >= 0 && gc + 0 < a.W) ? __ldg(row + gc + 0) : 0.f;
+                v.y = (gc + 1 >= 0 && gc + 1 < a.W) ? __ldg(row + gc + 1) : 0.f;
+                v.z = (gc + 2 >= 0 && gc + 2 < a.W) ? __ldg(row + gc + 2) : 0.f;
+                v.w = (gc + 3 >= 0 && gc + 3 < a.W) ? __ldg(row + gc + 3) : 0.f;
+            }
+        }
+        *reinterpret_cast<float4*>(&xs[sr * kPitch + 4 * q]) = v;
+    }
+    __syncthreads();
+
+    const int warp = tid >> 5, lane = tid & 31;
+    const int lr = (warp >> 2) * 32 + lane;  // local output row
+    const int cb = (warp & 3) * 16;          // local output column base
+
+    float acc1[16], acc2[16];
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+        acc1[q] = 0.f;
+        acc2[q] = 0.f;
+    }
+
+#pragma unroll 1
+    for (int i = 0; i < 16; ++i) {
+        // input window: smem cols [cb, cb+32) <-> image cols [c0+cb-8, c0+cb+24);
+        // output column c0+cb+q, tap j reads image col c0+cb+q+j-7 = smem col cb+q+j+1
+        float x[32];
+        const float4* xr = reinterpret_cast<const float4*>(&xs[(lr + i) * kPitch + cb]);
+#pragma unroll
+        for (int v = 0; v < 8; ++v) {
+            const float4 t = xr[v];
+            x[4 * v + 0] = t.x;
+            x[4 * v + 1] = t.y;
+            x[4 * v + 2] = t.z;
+            x[4 * v + 3] = t.w;
+        }
+        float w1[16], w2[16];
+        const float4* w1r = reinterpret_cast<const float4*>(&w1s[i * 16]);
+        const float4* w2r = reinterpret_cast<const float4*>(&w2s[i * 16]);
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const float4 t1 = w1r[v];
+            const float4 t2 = w2r[v];
+            w1[4 * v + 0] = t1.x;
+            w1[4 * v + 1] = t1.y;
+            w1[4 * v + 2] = t1.z;
+            w1[4 * v + 3] = t1.w;
+            w2[4 * v + 0] = t2.x;
+            w2[4 * v + 1] = t2.y;
+            w2[4 * v + 2] = t2.z;
+            w2[4 * v + 3] = t2.w;
+        }
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+#pragma unroll
+            for (int q = 0; q < 16; ++q) {
+                acc1[q] = fmaf(x[q + j + 1], w1[j], acc1[q]);
+                acc2[q] = fmaf(x[q + j + 1], w2[j], acc2[q]);
+            }
+        }
+    }
+
+    // epilogue: remaps and the 4-way max fold (x > m) ? x : m in order E1, E2, E5, E6
+    const int64_t row = tile_r0 + lr;
+    if (row >= a.out_row0 + a.out_rows) return;
+    float e[16];
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+        const float e1 = acc1[q], e2 = acc2[q], e5 = -e1, e6 = -e2;
+        float m = e1;
+        m = (e2 > m) ? e2 : m;
+        m = (e5 > m) ? e5 : m;
+        m = (e6 > m) ? e6 : m;
+        e[q] = m;
+    }
+    float* orow = a.out + img * a.out_img_stride + (row - a.out_row0) * a.W;
+    const int64_t c0 = tile_c0 + cb;
+    const bool ovec = (a.W & 3) == 0 && ((reinterpret_cast<uintptr_t>(a.out) & 15) == 0) &&
+                      (a.out_img_stride & 3) == 0;
+    if (ovec && c0 + 15 < a.W) {
+#pragma unroll
+        for (int v = 0; v < 4; ++v)
+            *reinterpret_cast<float4*>(orow + c0 + 4 * v) =
+                make_float4(e[4 * v], e[4 * v + 1], e[4 * v + 2], e[4 * v + 3]);
+    } else {
+#pragma unroll
+        for (int q = 0; q < 16; ++q)
+            if (c0 + q < a.W) orow[c0 + q] = e[q];
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
+    if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
+    dim3 grid((unsigned)((a.W + kTileC - 1) / kTileC), (unsigned)((a.out_rows + kTileR - 1) / kTileR),
+              (unsigned)a.nimg);
+    if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
+    edge_fused_kernel<<<grid, kThreads, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+}  // namespace tg

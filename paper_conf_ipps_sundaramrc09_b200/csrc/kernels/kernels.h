@@ -1,0 +1,63 @@
+// kernels.h -- launchers of the fused sm_100a offload-unit kernels (product code).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace tg {
+
+// K1: the whole edge template as one kernel per chunk (the paper's "best
+// possible" single kernel): E = max(Im*K1, Im*K2, -(Im*K1), -(Im*K2)),
+// SAME zero padding. Rows are in GLOBAL image coordinates; rows outside [0, H) are zero.
+struct EdgeArgs {
+    const float* in;        // image rows [in_row0, in_row0 + in_rows) of nimg images
+    int64_t in_img_stride;  // floats between consecutive images in `in`
+    int64_t in_row0, in_rows;
+    float* out;             // output rows [out_row0, out_row0 + out_rows) of nimg images
+    int64_t out_img_stride;
+    int64_t out_row0, out_rows;
+    int64_t H, W;           // full image size
+    int64_t nimg;
+    const float* k1;        // ks x ks (device)
+    const float* k2;
+    int ks;                 // 1..16
+};
+cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s);
+
+// CNN offload units (fp32 FFMA path). Row ranges are global level coordinates.
+struct CnnU1Args {          // C1(1->8, 5x5) + bias + tanh + S2 + tanh  -> T2
+    const float* in; int64_t in_img_stride; int64_t in_row0;   // rows of the input image
+    int64_t W;                                                 // input width
+    const float* k1;        // [8][25]
+    const float* b1;        // plane [8][b1_rows][w1] starting at global C1 row b1_row0, or scalar [8]
+    int64_t b1_row0, b1_rows; int b1_plane;
+    const float* p2;        // [8][4]
+    float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows;  // [8][t2_rows][w2]
+    int64_t w1, w2;
+    int64_t nimg;
+};
+struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
+    const float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows; int64_t w2;
+    const float* k3;        // [20][8][25]
+    const float* b3; int64_t b3_row0, b3_rows; int b3_plane;      // plane [20][b3_rows][w3]
+    const float* p4;        // [20][4]
+    float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w3, w4;
+    int64_t nimg;
+    int bf16_tc;            // 1: tcgen05 bf16 path
+};
+struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + bias -> out
+    const float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w4;
+    const float* k5;        // [n5][20][25]
+    const float* b5; int64_t b5_row0, b5_rows; int b5_plane;      // plane [n5][b5_rows][w5]
+    const float* k6;        // [9][n5]
+    const float* b6; int64_t b6_row0, b6_rows; int b6_plane;      // plane [9][b6_rows][w5]
+    float* out; int64_t out_img_stride; int64_t out_plane_stride; int64_t out_row0, out_rows; int64_t w5;
+    int n5;
+    int64_t nimg;
+    int bf16_tc;
+};
+cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s);
+cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s);
+cudaError_t launch_cnn_u3(const CnnU3Args& a, cudaStream_t s);
+
+}  // namespace tg

@@ -1,0 +1,467 @@
+"""Thin Python binding of include/tg.h (ctypes; argument marshalling only).
+
+Every step of the hot path runs inside libtg.so (planner in C++, copies and fused sm_100a
+kernels driven by its stream engine). This module only converts arrays to pointers,
+checks status codes and -- when asked -- hands the library PyTorch-owned device memory
+and streams through the tg_runtime hooks. There is no fallback: if libtg.so is missing or
+fails to load, importing this module raises.
+
+The functions keep the C names (tg_graph_create, tg_input, ..., tg_execute); `Graph` and
+`Plan` are small conveniences over them.
+"""
+from __future__ import annotations
+
+import ctypes
+import json
+import os
+from typing import Sequence
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libtg.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+                      "(the CUDA library is the only implementation; there is no CPU fallback)")
+_lib = ctypes.CDLL(LIB_PATH)
+
+# ---------------------------------------------------------------------------- constants
+TG_OK, TG_E_ARG, TG_E_SHAPE, TG_E_INFEASIBLE, TG_E_CUDA, TG_E_OOM, TG_E_STATE, TG_E_UNSUPPORTED = \
+    0, -1, -2, -3, -4, -5, -6, -7
+TG_VALID, TG_SAME = 0, 1
+TG_ADD, TG_NEG, TG_AFFINE, TG_ABS = 0, 1, 2, 3
+TG_MAX, TG_SUM, TG_MAXABS = 0, 1, 2
+TG_BIAS_PLANE, TG_BIAS_SCALAR = 0, 1
+TG_FP32, TG_BF16_TC = 0, 1
+TG_FUSED, TG_PER_OP, TG_BASELINE = 0, 1, 2
+
+_STATUS = {v: k for k, v in dict(TG_E_ARG=-1, TG_E_SHAPE=-2, TG_E_INFEASIBLE=-3, TG_E_CUDA=-4,
+                                   TG_E_OOM=-5, TG_E_STATE=-6, TG_E_UNSUPPORTED=-7).items()}
+
+
+class TGError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{_STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+# ---------------------------------------------------------------------------- prototypes
+c_i32, c_i64, c_u64, c_sz = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64, ctypes.c_size_t
+vp = ctypes.c_void_p
+P_id = ctypes.POINTER(c_i32)
+
+ALLOC_FN = ctypes.CFUNCTYPE(vp, c_sz, c_i32, vp)
+FREE_FN = ctypes.CFUNCTYPE(None, vp, c_i32, vp)
+STREAM_FN = ctypes.CFUNCTYPE(vp, c_i32, c_i32, vp)
+
+
+class tg_runtime(ctypes.Structure):
+    _fields_ = [("alloc", ALLOC_FN), ("free", FREE_FN), ("stream", STREAM_FN), ("ctx", vp)]
+
+
+class tg_plan_stats(ctypes.Structure):
+    _fields_ = [("h2d_bytes", c_u64), ("d2h_bytes", c_u64), ("io_lower_bound_bytes", c_u64),
+                ("total_temp_bytes", c_u64), ("peak_device_bytes", c_u64 * 8), ("n_chunks", c_i64),
+                ("n_units", c_i64), ("n_ops_fig7", c_i64), ("n_ds_fig7", c_i64),
+                ("chunk_begin", c_i64), ("chunk_end", c_i64), ("host_registered_bytes", c_u64)]
+
+
+class tg_timing(ctypes.Structure):
+    _fields_ = [("launches", c_i64), ("executions", c_i64), ("kernel_ms", ctypes.c_double * 4),
+                ("unit_launches", c_i64 * 4), ("h2d_ms", ctypes.c_double), ("d2h_ms", ctypes.c_double)]
+
+
+_PROTOS = {
+    "tg_graph_create": (c_i32, [ctypes.POINTER(vp)]),
+    "tg_graph_destroy": (None, [vp]),
+    "tg_input": (c_i32, [vp, c_i64, c_i64, c_i64, c_i64, vp, P_id]),
+    "tg_input_device": (c_i32, [vp, c_i64, c_i64, c_i64, c_i64, vp, P_id]),
+    "tg_param": (c_i32, [vp, c_i64, c_i64, c_i64, c_i64, vp, P_id]),
+    "tg_conv2d": (c_i32, [vp, c_i32, c_i32, c_i32, c_i32, P_id]),
+    "tg_elementwise": (c_i32, [vp, c_i32, P_id, c_i32, ctypes.c_float, ctypes.c_float, P_id]),
+    "tg_tanh": (c_i32, [vp, c_i32, P_id]),
+    "tg_max_combine": (c_i32, [vp, P_id, c_i32, P_id]),
+    "tg_subsample": (c_i32, [vp, c_i32, c_i32, c_i32, P_id]),
+    "tg_output": (c_i32, [vp, c_i32, vp]),
+    "tg_output_device": (c_i32, [vp, c_i32, vp]),
+    "tg_shape": (c_i32, [vp, c_i32, ctypes.POINTER(c_i64)]),
+    "tg_find_edges": (c_i32, [vp, c_i32, c_i32, c_i32, c_i32, P_id]),
+    "tg_cnn": (c_i32, [vp, c_i32, c_i32, P_id, c_i32, P_id]),
+    "tg_set_devices": (c_i32, [vp, P_id, c_i32]),
+    "tg_set_device_budget": (c_i32, [vp, c_u64]),
+    "tg_set_precision": (c_i32, [vp, c_i32]),
+    "tg_set_chunking": (c_i32, [vp, c_i64, c_i32]),
+    "tg_set_shard": (c_i32, [vp, c_i32, c_i32]),
+    "tg_set_runtime": (c_i32, [vp, ctypes.POINTER(tg_runtime)]),
+    "tg_plan_create": (c_i32, [vp, c_i32, ctypes.POINTER(vp)]),
+    "tg_plan_stats_get": (c_i32, [vp, ctypes.POINTER(tg_plan_stats)]),
+    "tg_plan_dump_json": (c_i32, [vp, ctypes.c_char_p, c_sz, ctypes.POINTER(c_sz)]),
+    "tg_execute": (c_i32, [vp]),
+    "tg_execute_async": (c_i32, [vp]),
+    "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
+    "tg_plan_timing_get": (c_i32, [vp, ctypes.POINTER(tg_timing)]),
+    "tg_plan_launch_count": (c_i64, [vp]),
+    "tg_plan_destroy": (None, [vp]),
+    "tg_last_error": (ctypes.c_char_p, []),
+    "tg_version": (ctypes.c_char_p, []),
+}
+for _name, (_res, _args) in _PROTOS.items():
+    _f = getattr(_lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+EXPORTED = tuple(_PROTOS)
+
+
+def last_error() -> str:
+    return (_lib.tg_last_error() or b"").decode()
+
+
+def _ck(st: int) -> None:
+    if st != TG_OK:
+        raise TGError(st, last_error())
+
+
+def _ptr(a) -> int:
+    """Address of a C-contiguous float32 numpy array or torch tensor (host or device)."""
+    if isinstance(a, np.ndarray):
+        if a.dtype != np.float32 or not a.flags["C_CONTIGUOUS"]:
+            raise TypeError("arrays must be C-contiguous float32")
+        return a.ctypes.data
+    import torch
+    if isinstance(a, torch.Tensor):
+        if a.dtype != torch.float32 or not a.is_contiguous():
+            raise TypeError("tensors must be contiguous float32")
+        return a.data_ptr()
+    raise TypeError(f"unsupported buffer type {type(a)}")
+
+
+def _dims4(shape) -> tuple[int, int, int, int]:
+    shape = tuple(int(s) for s in shape)
+    if len(shape) > 4:
+        raise ValueError("at most 4 dims")
+    return (1,) * (4 - len(shape)) + shape
+
+
+# ---------------------------------------------------------------------------- C-named API
+def tg_graph_create() -> int:
+    h = vp()
+    _ck(_lib.tg_graph_create(ctypes.byref(h)))
+    return h.value
+
+
+def tg_graph_destroy(g: int) -> None:
+    _lib.tg_graph_destroy(g)
+
+
+def _id_call(fn, *args) -> int:
+    out = c_i32()
+    _ck(fn(*args, ctypes.byref(out)))
+    return out.value
+
+
+def tg_input(g, n, c, h, w, host_ptr) -> int:
+    return _id_call(_lib.tg_input, g, n, c, h, w, host_ptr)
+
+
+def tg_input_device(g, n, c, h, w, dev_ptr) -> int:
+    return _id_call(_lib.tg_input_device, g, n, c, h, w, dev_ptr)
+
+
+def tg_param(g, d0, d1, d2, d3, host_ptr) -> int:
+    return _id_call(_lib.tg_param, g, d0, d1, d2, d3, host_ptr)
+
+
+def tg_conv2d(g, x, k, bias, pad) -> int:
+    return _id_call(_lib.tg_conv2d, g, x, k, bias, pad)
+
+
+def tg_elementwise(g, op, xs: Sequence[int], a=1.0, b=0.0) -> int:
+    arr = (c_i32 * len(xs))(*xs)
+    return _id_call(_lib.tg_elementwise, g, op, arr, len(xs), a, b)
+
+
+def tg_tanh(g, x) -> int:
+    return _id_call(_lib.tg_tanh, g, x)
+
+
+def tg_max_combine(g, xs: Sequence[int]) -> int:
+    arr = (c_i32 * len(xs))(*xs)
+    return _id_call(_lib.tg_max_combine, g, arr, len(xs))
+
+
+def tg_subsample(g, x, p, s=2) -> int:
+    return _id_call(_lib.tg_subsample, g, x, p, s)
+
+
+def tg_output(g, y, host_ptr) -> None:
+    _ck(_lib.tg_output(g, y, host_ptr))
+
+
+def tg_output_device(g, y, dev_ptr) -> None:
+    _ck(_lib.tg_output_device(g, y, dev_ptr))
+
+
+def tg_shape(g, y) -> tuple[int, int, int, int]:
+    d = (c_i64 * 4)()
+    _ck(_lib.tg_shape(g, y, d))
+    return tuple(d)
+
+
+def tg_find_edges(g, img, kernel, num_orientations=4, combine_op=TG_MAX) -> int:
+    return _id_call(_lib.tg_find_edges, g, img, kernel, num_orientations, combine_op)
+
+
+def tg_cnn(g, img, n5, params: Sequence[int], bias_mode=TG_BIAS_PLANE) -> int:
+    arr = (c_i32 * 10)(*params)
+    return _id_call(_lib.tg_cnn, g, img, n5, arr, bias_mode)
+
+
+def tg_set_devices(g, ordinals: Sequence[int]) -> None:
+    arr = (c_i32 * len(ordinals))(*ordinals)
+    _ck(_lib.tg_set_devices(g, arr, len(ordinals)))
+
+
+def tg_set_device_budget(g, nbytes: int) -> None:
+    _ck(_lib.tg_set_device_budget(g, int(nbytes)))
+
+
+def tg_set_precision(g, prec: int) -> None:
+    _ck(_lib.tg_set_precision(g, prec))
+
+
+def tg_set_chunking(g, max_chunk_px: int, depth: int) -> None:
+    _ck(_lib.tg_set_chunking(g, int(max_chunk_px), int(depth)))
+
+
+def tg_set_shard(g, rank: int, world: int) -> None:
+    _ck(_lib.tg_set_shard(g, rank, world))
+
+
+def tg_set_runtime(g, rt) -> None:
+    _ck(_lib.tg_set_runtime(g, ctypes.byref(rt) if rt is not None else None))
+
+
+def tg_plan_create(g, mode=TG_FUSED) -> int:
+    h = vp()
+    _ck(_lib.tg_plan_create(g, mode, ctypes.byref(h)))
+    return h.value
+
+
+def tg_plan_stats_get(p) -> dict:
+    s = tg_plan_stats()
+    _ck(_lib.tg_plan_stats_get(p, ctypes.byref(s)))
+    d = {k: getattr(s, k) for k, _ in tg_plan_stats._fields_}
+    d["peak_device_bytes"] = list(s.peak_device_bytes)
+    return d
+
+
+def tg_plan_dump_json(p) -> dict:
+    need = c_sz()
+    _lib.tg_plan_dump_json(p, None, 0, ctypes.byref(need))
+    buf = ctypes.create_string_buffer(need.value)
+    _ck(_lib.tg_plan_dump_json(p, buf, need.value, ctypes.byref(need)))
+    return json.loads(buf.value.decode())
+
+
+def tg_execute(p) -> None:
+    _ck(_lib.tg_execute(p))
+
+
+def tg_execute_async(p) -> None:
+    _ck(_lib.tg_execute_async(p))
+
+
+def tg_plan_set_profiling(p, on: bool) -> None:
+    _ck(_lib.tg_plan_set_profiling(p, 1 if on else 0))
+
+
+def tg_plan_timing_get(p) -> dict:
+    t = tg_timing()
+    _ck(_lib.tg_plan_timing_get(p, ctypes.byref(t)))
+    return {"launches": t.launches, "executions": t.executions, "kernel_ms": list(t.kernel_ms),
+            "unit_launches": list(t.unit_launches), "h2d_ms": t.h2d_ms, "d2h_ms": t.d2h_ms}
+
+
+def tg_plan_launch_count(p) -> int:
+    return int(_lib.tg_plan_launch_count(p))
+
+
+def tg_plan_destroy(p) -> None:
+    _lib.tg_plan_destroy(p)
+
+
+def tg_version() -> str:
+    return _lib.tg_version().decode()
+
+
+# ---------------------------------------------------------------------------- torch runtime
+class TorchRuntime:
+    """tg_runtime backed by PyTorch: the arena comes from the caching allocator
+    (torch.empty(uint8)), the three streams are torch.cuda.Stream objects (non-blocking),
+    so callers can order torch work / CUDA events against the library's compute stream."""
+
+    def __init__(self):
+        import torch
+        self._torch = torch
+        self._bufs: dict[int, object] = {}
+        self._streams: dict[tuple[int, int], object] = {}
+        self._alloc = ALLOC_FN(self._alloc_cb)
+        self._free = FREE_FN(self._free_cb)
+        self._stream = STREAM_FN(self._stream_cb)
+        self.struct = tg_runtime(self._alloc, self._free, self._stream, None)
+
+    def _alloc_cb(self, nbytes, dev, ctx):
+        try:
+            t = self._torch.empty(int(nbytes), dtype=self._torch.uint8, device=f"cuda:{dev}")
+        except Exception:  # noqa: BLE001 - reported to the library as NULL (TG_E_OOM)
+            return None
+        self._bufs[t.data_ptr()] = t
+        return t.data_ptr()
+
+    def _free_cb(self, ptr, dev, ctx):
+        self._bufs.pop(int(ptr or 0), None)
+
+    def _stream_cb(self, dev, which, ctx):
+        key = (int(dev), int(which))
+        if key not in self._streams:
+            self._streams[key] = self._torch.cuda.Stream(device=f"cuda:{dev}")
+        return self._streams[key].cuda_stream
+
+    def stream(self, dev: int = 0, which: int = 1):
+        """The torch.cuda.Stream the library uses for `which` (0 H2D, 1 compute, 2 D2H)."""
+        key = (int(dev), int(which))
+        if key not in self._streams:
+            self._streams[key] = self._torch.cuda.Stream(device=f"cuda:{dev}")
+        return self._streams[key]
+
+
+# ---------------------------------------------------------------------------- conveniences
+class Graph:
+    """Owns a tg_graph and keeps every buffer handed to the library alive."""
+
+    def __init__(self):
+        self.h = tg_graph_create()
+        self._keep = []
+        self.runtime = None
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            tg_graph_destroy(self.h)
+            self.h = None
+
+    def input(self, a, device: bool = False) -> int:
+        self._keep.append(a)
+        n, c, h, w = _dims4(a.shape)
+        return (tg_input_device if device else tg_input)(self.h, n, c, h, w, _ptr(a))
+
+    def param(self, a) -> int:
+        a = np.ascontiguousarray(a, dtype=np.float32) if isinstance(a, np.ndarray) else a
+        self._keep.append(a)
+        return tg_param(self.h, *_dims4(a.shape), _ptr(a))
+
+    def output(self, y: int, a, device: bool = False) -> None:
+        self._keep.append(a)
+        (tg_output_device if device else tg_output)(self.h, y, _ptr(a))
+
+    def shape(self, y: int):
+        return tg_shape(self.h, y)
+
+    def find_edges(self, img: int, kernel: int, num_orientations=4, combine_op=TG_MAX) -> int:
+        return tg_find_edges(self.h, img, kernel, num_orientations, combine_op)
+
+    def cnn(self, img: int, n5: int, params: Sequence[int], bias_mode=TG_BIAS_PLANE) -> int:
+        return tg_cnn(self.h, img, n5, params, bias_mode)
+
+    def conv2d(self, x, k, bias=-1, pad=TG_VALID):
+        return tg_conv2d(self.h, x, k, bias, pad)
+
+    def neg(self, x):
+        return tg_elementwise(self.h, TG_NEG, [x])
+
+    def max_combine(self, xs):
+        return tg_max_combine(self.h, xs)
+
+    def set(self, budget: int | None = None, precision: int | None = None, devices=None,
+            max_chunk_px: int | None = None, depth: int | None = None, shard=None,
+            torch_runtime: bool = False):
+        if budget is not None:
+            tg_set_device_budget(self.h, budget)
+        if precision is not None:
+            tg_set_precision(self.h, precision)
+        if devices is not None:
+            tg_set_devices(self.h, list(devices))
+        if max_chunk_px is not None or depth is not None:
+            tg_set_chunking(self.h, max_chunk_px or (1 << 24), depth or 3)
+        if shard is not None:
+            tg_set_shard(self.h, *shard)
+        if torch_runtime:
+            self.runtime = TorchRuntime()
+            tg_set_runtime(self.h, self.runtime.struct)
+        return self
+
+    def plan(self, mode=TG_FUSED) -> "Plan":
+        return Plan(self, tg_plan_create(self.h, mode))
+
+
+class Plan:
+    def __init__(self, graph: Graph, h: int):
+        self.graph = graph
+        self.h = h
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            tg_plan_destroy(self.h)
+            self.h = None
+
+    def stats(self) -> dict:
+        return tg_plan_stats_get(self.h)
+
+    def json(self) -> dict:
+        return tg_plan_dump_json(self.h)
+
+    def execute(self, blocking: bool = True) -> None:
+        (tg_execute if blocking else tg_execute_async)(self.h)
+
+    def profiling(self, on: bool = True) -> None:
+        tg_plan_set_profiling(self.h, on)
+
+    def timing(self) -> dict:
+        return tg_plan_timing_get(self.h)
+
+    def launches(self) -> int:
+        return tg_plan_launch_count(self.h)
+
+    def compute_stream(self, dev: int = 0):
+        if self.graph.runtime is None:
+            raise RuntimeError("compute_stream needs set(torch_runtime=True)")
+        return self.graph.runtime.stream(dev, 1)
+
+
+def edge_graph(img, K1, K2=None, out=None, device: bool = False) -> tuple[Graph, int]:
+    """Edge template graph. With K2=None it is find_edges(img, K1, 4, TG_MAX) (K2 = rot90
+    K1); otherwise the same graph built from primitives with two given kernels."""
+    g = Graph()
+    x = g.input(img, device=device)
+    k1 = g.param(np.asarray(K1, np.float32).reshape(1, 1, *np.shape(K1)[-2:]))
+    if K2 is None:
+        e = g.find_edges(x, k1)
+    else:
+        k2 = g.param(np.asarray(K2, np.float32).reshape(1, 1, *np.shape(K2)[-2:]))
+        e1 = g.conv2d(x, k1, -1, TG_SAME)
+        e2 = g.conv2d(x, k2, -1, TG_SAME)
+        e = g.max_combine([e1, e2, g.neg(e1), g.neg(e2)])
+    if out is not None:
+        g.output(e, out, device=device)
+    return g, e
+
+
+def cnn_graph(img, n5: int, params, out=None, bias_mode=TG_BIAS_PLANE, device: bool = False) -> tuple[Graph, int]:
+    g = Graph()
+    x = g.input(img, device=device)
+    ids = [g.param(p) for p in params]
+    y = g.cnn(x, n5, ids, bias_mode)
+    if out is not None:
+        g.output(y, out, device=device)
+    return g, y

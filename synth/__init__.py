@@ -168,7 +168,7 @@ def images_torch(seed: int, n: int, H: int, W: int, device, n0: int = 0, out=Non
 
     if out is None:
         out = torch.empty((n, 1, H, W), dtype=torch.float32, device=device)
-    rows_per = max(1, (1 << 24) // max(W, 1))
+    rows_per = max(1, (1 << 25) // max(W, 1))
     for i in range(n):
         key = stream_key(seed, DS_IMAGE, n0 + i)
         for r0 in range(0, H, rows_per):

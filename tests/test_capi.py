@@ -1,0 +1,97 @@
+"""The C-ABI library loads on a CPU-only box, exports every function include/tg.h declares,
+and its host-side calls (graph building, planning, error reporting) work without a GPU."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+from conftest import ROOT
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "tg.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    names = re.findall(r"^\s*(?:const\s+)?[\w]+\s*\*?\s*(tg_\w+)\s*\(", src, flags=re.M)
+    return sorted(set(names))
+
+
+def test_library_exports_every_header_symbol():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    lib = ctypes.CDLL(tg.LIB_PATH)
+    names = header_functions()
+    assert len(names) >= 30
+    for n in names:
+        assert hasattr(lib, n), n
+    assert set(names) == set(tg.EXPORTED)
+    assert tg.tg_version().startswith("tg ")
+
+
+def test_errors_are_reported():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    g = tg.Graph()
+    x = g.input(np.zeros((1, 1, 8, 8), np.float32))
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_conv2d(g.h, x, 99, -1, tg.TG_SAME)
+    assert e.value.code == tg.TG_E_ARG and "unknown DS id" in str(e.value)
+    k = g.param(np.zeros((1, 2, 3, 3), np.float32))
+    with pytest.raises(tg.TGError) as e:
+        g.conv2d(x, k, -1, tg.TG_SAME)
+    assert e.value.code == tg.TG_E_SHAPE
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_set_shard(g.h, 2, 2)
+    assert e.value.code == tg.TG_E_ARG
+    with pytest.raises(tg.TGError) as e:   # no output bound
+        g.plan()
+    assert e.value.code == tg.TG_E_STATE
+
+
+def test_unsupported_graph_and_infeasible_budget():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    img = np.zeros((1, 1, 64, 64), np.float32)
+    g = tg.Graph()
+    x = g.input(img)
+    y = tg.tg_tanh(g.h, x)
+    g.output(y, np.zeros_like(img))
+    with pytest.raises(tg.TGError) as e:
+        g.plan()
+    assert e.value.code == tg.TG_E_UNSUPPORTED
+    K = np.ones((16, 16), np.float32)
+    g, _ = tg.edge_graph(img, K, out=np.zeros_like(img))
+    g.set(budget=4096)
+    with pytest.raises(tg.TGError) as e:
+        g.plan()
+    assert e.value.code == tg.TG_E_INFEASIBLE
+
+
+def test_shapes_and_templates_build():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    import synth
+    H, W = 480, 640
+    img = np.zeros((2, 1, H, W), np.float32)
+    prm = synth.cnn_params_np(1, 120, H, W)
+    g, y = tg.cnn_graph(img, 120, prm)
+    assert g.shape(y) == (2, 9, 113, 153)
+    g2, e = tg.edge_graph(img[:1], np.ones((16, 16), np.float32))
+    assert g2.shape(e) == (1, 1, H, W)
+
+
+def test_plan_stats_match_table1_counts():
+    """Stats of a planned template reproduce Table 1 and the operator/DS
+    counts of PAPER.md:637 through the library's own accounting."""
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    import synth
+    img = np.zeros((1, 1, 1000, 1000), np.float32)
+    g, _ = tg.edge_graph(img, np.ones((16, 16), np.float32), out=np.zeros_like(img))
+    s = g.plan().stats()
+    assert s["io_lower_bound_bytes"] == 2000512 * 4 and s["total_temp_bytes"] == 6000512 * 4
+    assert s["n_ops_fig7"] == 5 and s["n_ds_fig7"] == 8
+    for n5, total, io, ops, ds in [(20, 59308709, 4870082, 1600, 2434), (120, 163093609, 6649882, 7500, 11334)]:
+        img = np.zeros((1, 1, 480, 640), np.float32)
+        prm = synth.cnn_params_np(1, n5, 480, 640)
+        out = np.zeros((1, 9, 113, 153), np.float32)
+        g, _ = tg.cnn_graph(img, n5, prm, out=out)
+        s = g.plan().stats()
+        assert (s["total_temp_bytes"], s["io_lower_bound_bytes"]) == (total * 4, io * 4)
+        assert (s["n_ops_fig7"], s["n_ds_fig7"]) == (ops, ds)
