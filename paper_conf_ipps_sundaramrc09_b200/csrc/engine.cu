@@ -259,8 +259,8 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.H = t.H;
         a.W = t.W;
         a.nimg = ch.nimg;
-        a.k1 = param(0);
-        a.k2 = param(1);
+        a.k1_host = g.ds[c.param_ds[0]].src;
+        a.k2_host = g.ds[c.param_ds[1]].src;
         a.ks = t.ks;
         KernelTimer kt(x, d, 0, cs);
         CK(launch_edge(a, cs));
@@ -286,7 +286,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
             a.in_row0 = ch.in.a;
         }
         a.W = t.W;
-        a.k1 = param(0);
+        a.k1_host = g.ds[t.prm[0]].src;
         a.b1_plane = plane;
         if (strm) {
             a.b1 = (const float*)(base + c.slot.b1);
@@ -297,7 +297,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
             a.b1_row0 = 0;
             a.b1_rows = t.h[1];
         }
-        a.p2 = param(2);
+        a.p2_host = g.ds[t.prm[2]].src;
         a.t2 = t2;
         a.t2_img_stride = 8 * ch.t2.n() * w2;
         a.t2_row0 = ch.t2.a;
@@ -317,7 +317,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.t2_row0 = ch.t2.a;
         a.t2_rows = ch.t2.n();
         a.w2 = w2;
-        a.k3 = param(3);
+        a.k3_host = g.ds[t.prm[3]].src;
         a.b3_plane = plane;
         if (strm) {
             a.b3 = (const float*)(base + c.slot.b3);
@@ -328,7 +328,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
             a.b3_row0 = 0;
             a.b3_rows = t.h[3];
         }
-        a.p4 = param(5);
+        a.p4_host = g.ds[t.prm[5]].src;
         a.t4 = t4;
         a.t4_img_stride = 20 * ch.t4.n() * w4;
         a.t4_row0 = ch.t4.a;

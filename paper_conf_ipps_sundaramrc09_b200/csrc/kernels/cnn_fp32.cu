@@ -1,8 +1,336 @@
-// cnn_fp32.cu -- CNN offload units U1, U2, U3 (placeholder until the FFMA kernels land).
+// cnn_fp32.cu -- the three fused CNN offload units on FP32 CUDA cores (sm_100a).
+//
+// CNN of PAPER.md:635 (reconstructed in SURVEY F2): C1(1->8,5x5) T S2 T C3(8->20,5x5) T S4 T
+// C5(20->n5,5x5) T C6(n5->9,1x1). The paper expands each conv layer into per-pair
+// convolutions, partial-sum adds and a bias-plane add (Fig. 7); here one
+// kernel per offload unit keeps all of those temporaries in registers:
+//   U1: C1 + bias + tanh + S2 + tanh   -> T2 (8 planes)
+//   U2: C3 + bias + tanh + S4 + tanh   -> T4 (20 planes)
+//   U3: C5 + bias + tanh + C6 + bias   -> output (9 planes); T5 never leaves registers
+// Row coordinates are global level rows; a chunk's buffers start at the row0 the planner
+// back-propagated. Every output pixel is computed by the same instruction
+// sequence in the same order wherever its tile or chunk starts, so split runs are
+// bit-identical to unsplit runs.
+//
+// tanh: 1 - 2/(1 + e^{2x}) with MUFU ex2/rcp (x clamped to +-15): absolute error < 3e-7,
+// well inside the normwise 1e-5 parity bound.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstring>
+
 #include "kernels.h"
 
 namespace tg {
-cudaError_t launch_cnn_u1(const CnnU1Args&, cudaStream_t) { return cudaErrorNotSupported; }
-cudaError_t launch_cnn_u2(const CnnU2Args&, cudaStream_t) { return cudaErrorNotSupported; }
-cudaError_t launch_cnn_u3(const CnnU3Args&, cudaStream_t) { return cudaErrorNotSupported; }
+namespace {
+
+__device__ __forceinline__ float tanh_f(float x) {
+    x = fminf(fmaxf(x, -15.f), 15.f);
+    const float e = __expf(2.f * x);
+    return 1.f - __fdividef(2.f, 1.f + e);
+}
+
+// ============================================================================ U1
+// One thread per T2 pixel and all 8 channels: the 2x2 C1 pixels under it (4 x 8 x 25 FFMA
+// from a 6x6 input window), bias, tanh, the 2x2 subsample, tanh. Weights travel in the
+// constant bank (kernel parameter) so FFMAs take them as uniform operands.
+struct U1W {
+    float k1[8][25];
+    float p2[8][4];
+};
+
+constexpr int U1_TR = 8, U1_TC = 16;                // T2 tile (rows x cols) = 128 threads
+constexpr int U1_IR = 2 * U1_TR + 4, U1_IC = 2 * U1_TC + 4;  // 20 x 36 input window
+
+__global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const __grid_constant__ U1W w) {
+    __shared__ __align__(16) float xs[U1_IR * U1_IC];
+    const int tid = threadIdx.x, ty = tid / U1_TC, tx = tid % U1_TC;
+    const int64_t img = blockIdx.z;
+    const int64_t r2_0 = a.t2_row0 + (int64_t)blockIdx.y * U1_TR;  // global T2 row of the tile
+    const int64_t c2_0 = (int64_t)blockIdx.x * U1_TC;
+    const int64_t ir0 = 2 * r2_0, ic0 = 2 * c2_0;                  // global input row/col
+    const float* inb = a.in + img * a.in_img_stride;
+    const int64_t in_rows_avail = a.in_img_stride / a.W;
+    for (int idx = tid; idx < U1_IR * U1_IC; idx += 128) {
+        const int r = idx / U1_IC, c = idx - r * U1_IC;
+        const int64_t br = ir0 + r - a.in_row0, gc = ic0 + c;
+        xs[idx] = (br >= 0 && br < in_rows_avail && gc < a.W) ? __ldg(inb + br * a.W + gc) : 0.f;
+    }
+    __syncthreads();
+    const int64_t R2 = r2_0 + ty, C2 = c2_0 + tx;
+    if (R2 >= a.t2_row0 + a.t2_rows || C2 >= a.w2) return;
+
+    float acc[8][4];
+#pragma unroll
+    for (int ch = 0; ch < 8; ++ch)
+#pragma unroll
+        for (int p = 0; p < 4; ++p) acc[ch][p] = 0.f;
+#pragma unroll
+    for (int i = 0; i < 6; ++i) {
+        float x[6];
+        const float2* xr = reinterpret_cast<const float2*>(&xs[(2 * ty + i) * U1_IC + 2 * tx]);
+#pragma unroll
+        for (int v = 0; v < 3; ++v) {
+            const float2 t = xr[v];
+            x[2 * v] = t.x;
+            x[2 * v + 1] = t.y;
+        }
+#pragma unroll
+        for (int ra = 0; ra < 2; ++ra) {
+            const int ki = i - ra;  // kernel row for C1 row 2*R2 + ra
+            if (ki < 0 || ki > 4) continue;
+#pragma unroll
+            for (int ch = 0; ch < 8; ++ch)
+#pragma unroll
+                for (int kj = 0; kj < 5; ++kj)
+#pragma unroll
+                    for (int cb = 0; cb < 2; ++cb)
+                        acc[ch][ra * 2 + cb] = fmaf(x[cb + kj], w.k1[ch][ki * 5 + kj], acc[ch][ra * 2 + cb]);
+        }
+    }
+    float* t2 = a.t2 + img * a.t2_img_stride;
+    const int64_t plane = a.t2_rows * a.w2;
+#pragma unroll
+    for (int ch = 0; ch < 8; ++ch) {
+        float s = 0.f;
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+            const int64_t r1 = 2 * R2 + (p >> 1), c1 = 2 * C2 + (p & 1);
+            const float b = a.b1_plane ? __ldg(a.b1 + ((int64_t)ch * a.b1_rows + (r1 - a.b1_row0)) * a.w1 + c1)
+                                       : __ldg(a.b1 + ch);
+            const float t = tanh_f(acc[ch][p] + b);
+            s = fmaf(w.p2[ch][p], t, s);
+        }
+        t2[ch * plane + (R2 - a.t2_row0) * a.w2 + C2] = tanh_f(s);
+    }
+}
+
+// ============================================================================ U2
+// One thread per T4 pixel and all 20 channels (the 2x2 C3 pixels under it: 80
+// accumulators). Loop over the 8 input planes; per plane a fully unrolled 6-row sweep of
+// the 6x6 window (2000 FFMA). The 20x8x25 weights are a kernel parameter (constant bank).
+struct U2W {
+    float k3[8][25][20];  // [ci][tap][co]: the 20 output channels of one tap are contiguous
+    float p4[20][4];
+};
+
+constexpr int U2_TR = 8, U2_TC = 16;
+constexpr int U2_IR = 2 * U2_TR + 4, U2_IC = 2 * U2_TC + 4;  // 20 x 36 per plane
+
+__global__ void __launch_bounds__(128, 3) cnn_u2_kernel(const CnnU2Args a, const __grid_constant__ U2W w) {
+    __shared__ __align__(16) float xs[8][U2_IR * U2_IC];
+    const int tid = threadIdx.x, ty = tid / U2_TC, tx = tid % U2_TC;
+    const int64_t img = blockIdx.z;
+    const int64_t r4_0 = a.t4_row0 + (int64_t)blockIdx.y * U2_TR;
+    const int64_t c4_0 = (int64_t)blockIdx.x * U2_TC;
+    const int64_t ir0 = 2 * r4_0, ic0 = 2 * c4_0;  // global T2 row/col of the window
+    const float* t2b = a.t2 + img * a.t2_img_stride;
+    const int64_t plane = a.t2_rows * a.w2;
+    for (int idx = tid; idx < 8 * U2_IR * U2_IC; idx += 128) {
+        const int ci = idx / (U2_IR * U2_IC);
+        const int rem = idx - ci * (U2_IR * U2_IC);
+        const int r = rem / U2_IC, c = rem - r * U2_IC;
+        const int64_t br = ir0 + r - a.t2_row0, gc = ic0 + c;
+        xs[ci][rem] = (br >= 0 && br < a.t2_rows && gc < a.w2) ? t2b[ci * plane + br * a.w2 + gc] : 0.f;
+    }
+    __syncthreads();
+    const int64_t R4 = r4_0 + ty, C4 = c4_0 + tx;
+    if (R4 >= a.t4_row0 + a.t4_rows || C4 >= a.w4) return;
+
+    float acc[20][4];
+#pragma unroll
+    for (int co = 0; co < 20; ++co)
+#pragma unroll
+        for (int p = 0; p < 4; ++p) acc[co][p] = 0.f;
+#pragma unroll 1
+    for (int ci = 0; ci < 8; ++ci) {
+#pragma unroll
+        for (int i = 0; i < 6; ++i) {
+            float x[6];
+            const float2* xr = reinterpret_cast<const float2*>(&xs[ci][(2 * ty + i) * U2_IC + 2 * tx]);
+#pragma unroll
+            for (int v = 0; v < 3; ++v) {
+                const float2 t = xr[v];
+                x[2 * v] = t.x;
+                x[2 * v + 1] = t.y;
+            }
+#pragma unroll
+            for (int ra = 0; ra < 2; ++ra) {
+                const int ki = i - ra;
+                if (ki < 0 || ki > 4) continue;
+#pragma unroll
+                for (int kj = 0; kj < 5; ++kj)
+#pragma unroll
+                    for (int co = 0; co < 20; ++co) {
+                        const float wv = w.k3[ci][ki * 5 + kj][co];
+                        acc[co][ra * 2 + 0] = fmaf(x[kj], wv, acc[co][ra * 2 + 0]);
+                        acc[co][ra * 2 + 1] = fmaf(x[kj + 1], wv, acc[co][ra * 2 + 1]);
+                    }
+            }
+        }
+    }
+    float* t4 = a.t4 + img * a.t4_img_stride;
+    const int64_t oplane = a.t4_rows * a.w4;
+#pragma unroll
+    for (int co = 0; co < 20; ++co) {
+        float s = 0.f;
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+            const int64_t r3 = 2 * R4 + (p >> 1), c3 = 2 * C4 + (p & 1);
+            const float b = a.b3_plane ? __ldg(a.b3 + ((int64_t)co * a.b3_rows + (r3 - a.b3_row0)) * a.w3 + c3)
+                                       : __ldg(a.b3 + co);
+            s = fmaf(w.p4[co][p], tanh_f(acc[co][p] + b), s);
+        }
+        t4[co * oplane + (R4 - a.t4_row0) * a.w4 + C4] = tanh_f(s);
+    }
+}
+
+// ============================================================================ U3
+// One thread per 4 consecutive output pixels of a row. C5 channels in groups of 8: per
+// group, 4 px x 8 ch accumulators over 20 planes x 25 taps (weights staged in shared
+// memory, broadcast LDS.128), then bias + tanh and the group's contribution to the 9 C6
+// accumulators per pixel (C6 is a 1x1 conv: a dot product over n5 channels).
+constexpr int U3_TR = 8, U3_TCG = 16, U3_P = 4, U3_G = 8;
+constexpr int U3_TC = U3_TCG * U3_P;              // 64 output cols per tile
+constexpr int U3_IR = U3_TR + 4, U3_IC = U3_TC + 4;  // 12 x 68 per plane
+constexpr int U3_ICP = 68;                         // pitch (floats), 16-byte aligned rows
+
+__global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
+    extern __shared__ __align__(16) float sm[];
+    float* xs = sm;                                  // [20][U3_IR][U3_ICP]
+    float* ws = xs + 20 * U3_IR * U3_ICP;            // [20][25][8] group weights
+    float* k6s = ws + 20 * 25 * U3_G;                // [9][n5p]
+    const int n5 = a.n5, n5p = (n5 + U3_G - 1) / U3_G * U3_G;
+    const int tid = threadIdx.x, ty = tid / U3_TCG, tg = tid % U3_TCG;
+    const int64_t img = blockIdx.z;
+    const int64_t r5_0 = a.out_row0 + (int64_t)blockIdx.y * U3_TR;
+    const int64_t c5_0 = (int64_t)blockIdx.x * U3_TC;
+    const float* t4b = a.t4 + img * a.t4_img_stride;
+    const int64_t plane = a.t4_rows * a.w4;
+    for (int idx = tid; idx < 20 * U3_IR * U3_IC; idx += 128) {
+        const int ci = idx / (U3_IR * U3_IC);
+        const int rem = idx - ci * (U3_IR * U3_IC);
+        const int r = rem / U3_IC, c = rem - r * U3_IC;
+        const int64_t br = r5_0 + r - a.t4_row0, gc = c5_0 + c;
+        xs[(ci * U3_IR + r) * U3_ICP + c] =
+            (br >= 0 && br < a.t4_rows && gc < a.w4) ? t4b[ci * plane + br * a.w4 + gc] : 0.f;
+    }
+    for (int idx = tid; idx < 9 * n5p; idx += 128) {
+        const int o = idx / n5p, ch = idx - o * n5p;
+        k6s[idx] = ch < n5 ? __ldg(a.k6 + o * n5 + ch) : 0.f;
+    }
+    const int64_t R5 = r5_0 + ty, C5 = c5_0 + tg * U3_P;
+    const bool row_ok = R5 < a.out_row0 + a.out_rows;
+
+    float c6[9][U3_P];
+#pragma unroll
+    for (int o = 0; o < 9; ++o)
+#pragma unroll
+        for (int p = 0; p < U3_P; ++p) c6[o][p] = 0.f;
+
+    for (int g0 = 0; g0 < n5p; g0 += U3_G) {
+        __syncthreads();  // previous group's weights fully consumed (and tile staged)
+        for (int idx = tid; idx < 20 * 25 * U3_G; idx += 128) {
+            const int k = idx / U3_G, ch = idx - k * U3_G;  // k = ci*25 + tap
+            ws[idx] = (g0 + ch < n5) ? __ldg(a.k5 + (int64_t)(g0 + ch) * 500 + k) : 0.f;
+        }
+        __syncthreads();
+        float acc[U3_G][U3_P];
+#pragma unroll
+        for (int c = 0; c < U3_G; ++c)
+#pragma unroll
+            for (int p = 0; p < U3_P; ++p) acc[c][p] = 0.f;
+#pragma unroll 1
+        for (int ci = 0; ci < 20; ++ci) {
+#pragma unroll
+            for (int i = 0; i < 5; ++i) {
+                float x[8];
+                const float4* xr = reinterpret_cast<const float4*>(&xs[(ci * U3_IR + ty + i) * U3_ICP + tg * U3_P]);
+                const float4 x0 = xr[0], x1 = xr[1];
+                x[0] = x0.x; x[1] = x0.y; x[2] = x0.z; x[3] = x0.w;
+                x[4] = x1.x; x[5] = x1.y; x[6] = x1.z; x[7] = x1.w;
+#pragma unroll
+                for (int kj = 0; kj < 5; ++kj) {
+                    const float4* wr = reinterpret_cast<const float4*>(&ws[((ci * 25) + i * 5 + kj) * U3_G]);
+                    const float4 wa = wr[0], wb = wr[1];
+                    const float wv[8] = {wa.x, wa.y, wa.z, wa.w, wb.x, wb.y, wb.z, wb.w};
+#pragma unroll
+                    for (int c = 0; c < U3_G; ++c)
+#pragma unroll
+                        for (int p = 0; p < U3_P; ++p) acc[c][p] = fmaf(x[p + kj], wv[c], acc[c][p]);
+                }
+            }
+        }
+        // bias + tanh, then this group's share of the 1x1 C6 dot products
+#pragma unroll
+        for (int c = 0; c < U3_G; ++c) {
+            const int ch = g0 + c;
+            if (ch >= n5) break;
+#pragma unroll
+            for (int p = 0; p < U3_P; ++p) {
+                float b = 0.f;
+                if (row_ok && C5 + p < a.w5)
+                    b = a.b5_plane ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (R5 - a.b5_row0)) * a.w5 + C5 + p)
+                                   : __ldg(a.b5 + ch);
+                const float t = tanh_f(acc[c][p] + b);
+#pragma unroll
+                for (int o = 0; o < 9; ++o) c6[o][p] = fmaf(k6s[o * n5p + ch], t, c6[o][p]);
+            }
+        }
+    }
+    if (!row_ok) return;
+    float* ob = a.out + img * a.out_img_stride + (R5 - a.out_row0) * a.w5;
+#pragma unroll
+    for (int o = 0; o < 9; ++o)
+#pragma unroll
+        for (int p = 0; p < U3_P; ++p) {
+            const int64_t c = C5 + p;
+            if (c >= a.w5) continue;
+            const float b = a.b6_plane ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (R5 - a.b6_row0)) * a.w5 + c)
+                                       : __ldg(a.b6 + o);
+            ob[o * a.out_plane_stride + c] = c6[o][p] + b;
+        }
+}
+
+}  // namespace
+
+cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s) {
+    if (a.t2_rows <= 0 || a.nimg <= 0) return cudaSuccess;
+    U1W w;
+    std::memcpy(w.k1, a.k1_host, sizeof w.k1);
+    std::memcpy(w.p2, a.p2_host, sizeof w.p2);
+    dim3 grid((unsigned)((a.w2 + U1_TC - 1) / U1_TC), (unsigned)((a.t2_rows + U1_TR - 1) / U1_TR), (unsigned)a.nimg);
+    cnn_u1_kernel<<<grid, 128, 0, s>>>(a, w);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s) {
+    if (a.t4_rows <= 0 || a.nimg <= 0) return cudaSuccess;
+    U2W w;
+    for (int co = 0; co < 20; ++co)
+        for (int ci = 0; ci < 8; ++ci)
+            for (int t = 0; t < 25; ++t) w.k3[ci][t][co] = a.k3_host[(co * 8 + ci) * 25 + t];
+    std::memcpy(w.p4, a.p4_host, sizeof w.p4);
+    dim3 grid((unsigned)((a.w4 + U2_TC - 1) / U2_TC), (unsigned)((a.t4_rows + U2_TR - 1) / U2_TR), (unsigned)a.nimg);
+    cnn_u2_kernel<<<grid, 128, 0, s>>>(a, w);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cnn_u3(const CnnU3Args& a, cudaStream_t s) {
+    if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
+    const int n5p = (a.n5 + U3_G - 1) / U3_G * U3_G;
+    const size_t smem = sizeof(float) * (20 * U3_IR * U3_ICP + 20 * 25 * U3_G + 9 * n5p);
+    static std::atomic<uint32_t> configured{0};  // one bit per device
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(configured.load() & (1u << (dev & 31)))) {
+        cudaError_t e = cudaFuncSetAttribute(cnn_u3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
+        if (e != cudaSuccess) return e;
+        configured.fetch_or(1u << (dev & 31));
+    }
+    dim3 grid((unsigned)((a.w5 + U3_TC - 1) / U3_TC), (unsigned)((a.out_rows + U3_TR - 1) / U3_TR), (unsigned)a.nimg);
+    cnn_u3_kernel<<<grid, 128, smem, s>>>(a);
+    return cudaGetLastError();
+}
+
 }  // namespace tg

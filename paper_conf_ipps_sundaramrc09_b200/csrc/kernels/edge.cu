@@ -5,14 +5,14 @@
 // in ONE pass over a chunk, so E1, E2, E5, E6 never leave registers -- the paper's "best
 // possible" configuration. SAME zero padding with anchor (ks-1)/2
 // (R2); a ks x ks kernel (ks <= 16) is embedded in a 16 x 16 frame at offset
-// 7 - (ks-1)/2 so one code path serves every size.
+// 7 - (ks-1)/2 so one code path serves every size (zero taps add exact zeros).
 //
 // Roofline: 2 x 256 FMA per output pixel vs 8 HBM bytes -> FP32-ALU
 // bound (128 flop/B >> ridge ~11 flop/B). The kernel is therefore organised to issue
 // FFMA back to back: each thread owns a 1 x 16 strip of outputs for both filters
 // (32 accumulators), and for each of the 16 filter rows loads its 32-wide input window
-// with 8 conflict-free LDS.128 and both filter rows with 8 broadcast LDS.128, then issues
-// 512 FFMA -- 3% load overhead. Tiles of 64 x 64 outputs, 256 threads; lanes of a warp own
+// with 8 conflict-free LDS.128 and both filter rows from the constant bank (uniform
+// registers), then issues 512 FFMA -- under 3% load overhead. Tiles of 64 x 64 outputs, 256 threads; lanes of a warp own
 // 32 consecutive rows (row pitch 84 floats = 21 x 16 B, odd, so the 8 lanes of each LDS.128
 // phase hit 8 distinct 16-byte bank groups). The input tile (79 x 80 floats incl. the
 // 15-row/col halo) is staged once per CTA with 128-bit coalesced loads; zero fill gives
@@ -34,25 +34,23 @@ constexpr int kSmC = kTileC + 16;  // 80 cols: [c0-8, c0+72)
 constexpr int kPitch = 84;         // floats; 84/4 = 21 (odd) -> conflict-free LDS.128 across rows
 constexpr int kThreads = 256;
 
-__global__ void __launch_bounds__(kThreads, 2) edge_fused_kernel(EdgeArgs a) {
+// Both filters, embedded in 16 x 16 frames, travel as a __grid_constant__ kernel parameter:
+// the weights then sit in the constant bank and every FFMA reads them through a uniform
+// register (FFMA R, R, UR, R) -- only two vector-register operands per FFMA, which keeps
+// the register-file banks out of the way of the FMA pipe.
+struct EdgeWeights {
+    float w1[256];
+    float w2[256];
+};
+
+__global__ void __launch_bounds__(kThreads, 2)
+    edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
     __shared__ __align__(16) float xs[kSmR * kPitch];
-    __shared__ __align__(16) float w1s[256];
-    __shared__ __align__(16) float w2s[256];
 
     const int tid = threadIdx.x;
     const int64_t img = blockIdx.z;
     const int64_t tile_r0 = a.out_row0 + (int64_t)blockIdx.y * kTileR;  // global output row
     const int64_t tile_c0 = (int64_t)blockIdx.x * kTileC;
-
-    // filters embedded in a 16 x 16 frame (zeros outside the ks x ks kernel)
-    {
-        const int off = 7 - (a.ks - 1) / 2;
-        const int r = tid >> 4, c = tid & 15;
-        const int rr = r - off, cc = c - off;
-        const bool in = rr >= 0 && rr < a.ks && cc >= 0 && cc < a.ks;
-        w1s[tid] = in ? __ldg(a.k1 + rr * a.ks + cc) : 0.f;
-        w2s[tid] = in ? __ldg(a.k2 + rr * a.ks + cc) : 0.f;
-    }
 
     // stage the input tile: smem (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)
     const float* __restrict__ inb = a.in + img * a.in_img_stride;
@@ -104,22 +102,8 @@ __global__ void __launch_bounds__(kThreads, 2) edge_fused_kernel(EdgeArgs a) {
             x[4 * v + 2] = t.z;
             x[4 * v + 3] = t.w;
         }
-        float w1[16], w2[16];
-        const float4* w1r = reinterpret_cast<const float4*>(&w1s[i * 16]);
-        const float4* w2r = reinterpret_cast<const float4*>(&w2s[i * 16]);
-#pragma unroll
-        for (int v = 0; v < 4; ++v) {
-            const float4 t1 = w1r[v];
-            const float4 t2 = w2r[v];
-            w1[4 * v + 0] = t1.x;
-            w1[4 * v + 1] = t1.y;
-            w1[4 * v + 2] = t1.z;
-            w1[4 * v + 3] = t1.w;
-            w2[4 * v + 0] = t2.x;
-            w2[4 * v + 1] = t2.y;
-            w2[4 * v + 2] = t2.z;
-            w2[4 * v + 3] = t2.w;
-        }
+        const float* w1 = &wt.w1[i * 16];
+        const float* w2 = &wt.w2[i * 16];
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
 #pragma unroll
@@ -166,7 +150,15 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
     dim3 grid((unsigned)((a.W + kTileC - 1) / kTileC), (unsigned)((a.out_rows + kTileR - 1) / kTileR),
               (unsigned)a.nimg);
     if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
-    edge_fused_kernel<<<grid, kThreads, 0, s>>>(a);
+    // filters embedded in a 16 x 16 frame at offset 7 - (ks-1)/2 (zeros elsewhere)
+    EdgeWeights wt{};
+    const int off = 7 - (a.ks - 1) / 2;
+    for (int r = 0; r < a.ks; ++r)
+        for (int c = 0; c < a.ks; ++c) {
+            wt.w1[(r + off) * 16 + c + off] = a.k1_host[r * a.ks + c];
+            wt.w2[(r + off) * 16 + c + off] = a.k2_host[r * a.ks + c];
+        }
+    edge_fused_kernel<<<grid, kThreads, 0, s>>>(a, wt);
     return cudaGetLastError();
 }
 

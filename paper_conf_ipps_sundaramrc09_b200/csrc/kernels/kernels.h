@@ -18,8 +18,8 @@ struct EdgeArgs {
     int64_t out_row0, out_rows;
     int64_t H, W;           // full image size
     int64_t nimg;
-    const float* k1;        // ks x ks (device)
-    const float* k2;
+    const float* k1_host;   // ks x ks filters (host; passed to the kernel by value)
+    const float* k2_host;
     int ks;                 // 1..16
 };
 cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s);
@@ -28,19 +28,19 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s);
 struct CnnU1Args {          // C1(1->8, 5x5) + bias + tanh + S2 + tanh  -> T2
     const float* in; int64_t in_img_stride; int64_t in_row0;   // rows of the input image
     int64_t W;                                                 // input width
-    const float* k1;        // [8][25]
+    const float* k1_host;   // [8][25] (host; passed by value in the constant bank)
     const float* b1;        // plane [8][b1_rows][w1] starting at global C1 row b1_row0, or scalar [8]
     int64_t b1_row0, b1_rows; int b1_plane;
-    const float* p2;        // [8][4]
+    const float* p2_host;   // [8][4] (host)
     float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows;  // [8][t2_rows][w2]
     int64_t w1, w2;
     int64_t nimg;
 };
 struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
     const float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows; int64_t w2;
-    const float* k3;        // [20][8][25]
+    const float* k3_host;   // [20][8][25] (host; constant bank)
     const float* b3; int64_t b3_row0, b3_rows; int b3_plane;      // plane [20][b3_rows][w3]
-    const float* p4;        // [20][4]
+    const float* p4_host;   // [20][4] (host)
     float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w3, w4;
     int64_t nimg;
     int bf16_tc;            // 1: tcgen05 bf16 path

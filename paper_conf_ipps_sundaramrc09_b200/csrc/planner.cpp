@@ -99,10 +99,17 @@ static tg_status recognise_cnn(const Graph& g, int out, Template& t) {
     if (n5 < 1 || n5 > 128 || kd(c5, 1) != 20 || kd(c5, 2) != 5 || kd(c5, 3) != 5) return TG_E_UNSUPPORTED;
     if (kd(c6, 0) != 9 || kd(c6, 1) != n5 || kd(c6, 2) != 1 || kd(c6, 3) != 1) return TG_E_UNSUPPORTED;
     if (s2->s != 2 || s4->s != 2) return TG_E_UNSUPPORTED;
-    // bias kind must be uniform (all planes or all scalars)
-    int planes = 0;
-    for (const Node* c : {c1, c3, c5, c6}) planes += (g.ds[c->bias].numel() != g.ds[c->ins[1]].d[0]) ? 1 : 0;
-    if (planes != 0 && planes != 4) return TG_E_UNSUPPORTED;
+    // bias kind must be uniform: all planes [1][co][ho][wo] or all scalars [co] (a 1x1 plane
+    // is both)
+    int plane_ok = 0, scalar_ok = 0;
+    for (const Node* c : {c1, c3, c5, c6}) {
+        const Ds& B = g.ds[c->bias];
+        const Ds& O = g.ds[c->out];
+        plane_ok += (B.d[0] == 1 && B.d[1] == O.d[1] && B.d[2] == O.d[2] && B.d[3] == O.d[3]) ? 1 : 0;
+        scalar_ok += (B.numel() == O.d[1]) ? 1 : 0;
+    }
+    if (plane_ok != 4 && scalar_ok != 4) return TG_E_UNSUPPORTED;
+    const int planes = plane_ok == 4 ? 4 : 0;
     t.kind = Tmpl::Cnn;
     t.input = cur;
     t.output = out;

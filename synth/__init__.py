@@ -81,9 +81,14 @@ def image_np(seed: int, ds_id: int, n: int, shape, row0: int = 0, rows: int | No
 def uniform_np(seed: int, ds_id: int, shape, a: float, n: int = 0) -> np.ndarray:
     """float32 uniform(-a, a) tensor of `shape` (idx = C-order linear index)."""
     shape = tuple(int(s) for s in shape)
-    idx = np.arange(int(np.prod(shape)), dtype=np.uint64).reshape(shape)
-    u = (bits_np(seed, ds_id, n, idx) >> np.uint64(8)).astype(np.float64) * (2.0 ** -24)
-    return ((2.0 * u - 1.0) * float(a)).astype(np.float32)
+    total = int(np.prod(shape))
+    out = np.empty(total, dtype=np.float32)
+    step = 1 << 24
+    for s0 in range(0, total, step):      # bounded temporaries for multi-GB parameter sets
+        idx = np.arange(s0, min(total, s0 + step), dtype=np.uint64)
+        u = (bits_np(seed, ds_id, n, idx) >> np.uint64(8)).astype(np.float64) * (2.0 ** -24)
+        out[s0:s0 + idx.size] = ((2.0 * u - 1.0) * float(a)).astype(np.float32)
+    return out.reshape(shape)
 
 
 def images_np(seed: int, n: int, H: int, W: int, n0: int = 0) -> np.ndarray:

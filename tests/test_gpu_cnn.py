@@ -1,0 +1,176 @@
+"""GPU parity of the fused CNN units (U1, U2, U3; Fig. 7) against the CPU
+oracle: normwise 1e-5 per output plane on the fp32 path (R16), split == unsplit
+bit-exactly (rows with streamed bias rows, batches), device-resident == host-streamed, the
+delta-kernel geometry (every output is tanh^5 of one input pixel), and sampled rows of the
+paper-literal large CNN at 6400x4800 under the 1.5 GB budget."""
+import math
+
+import numpy as np
+import pytest
+
+import synth
+from gpu_util import need_gpu, normwise, pinned, torch
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def tg():
+    need_gpu()
+    from paper_conf_ipps_sundaramrc09_b200 import tg as t
+    torch.cuda.set_device(0)
+    return t
+
+
+def run_cnn(tg, img, n5, prm, bias="plane", budget=0, device=False, max_chunk_px=None, depth=None,
+            precision=None):
+    n, _, H, W = img.shape
+    h5, w5 = synth.cnn_dims(H, W)[4]
+    mode = tg.TG_BIAS_PLANE if bias == "plane" else tg.TG_BIAS_SCALAR
+    if device:
+        x = torch.from_numpy(img).cuda()
+        out = torch.zeros((n, 9, h5, w5), dtype=torch.float32, device="cuda")
+        g, _ = tg.cnn_graph(x, n5, prm, out=out, bias_mode=mode, device=True)
+    else:
+        out = np.zeros((n, 9, h5, w5), np.float32)
+        g, _ = tg.cnn_graph(img, n5, prm, out=out, bias_mode=mode)
+    g.set(budget=budget, torch_runtime=True, max_chunk_px=max_chunk_px, depth=depth, precision=precision)
+    p = g.plan()
+    p.execute()
+    return (out.cpu().numpy() if device else out), p
+
+
+@pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
+                                          (3, 67, 61, 20, "scalar"), (1, 97, 131, 120, "scalar"),
+                                          (1, 483 // 3, 643 // 3, 60, "plane"), (2, 32, 32, 7, "plane")])
+def test_cnn_parity(tg, orc, n, H, W, n5, bias):
+    seed = synth.seed_for_config(3)
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W, bias)
+    out, _ = run_cnn(tg, img, n5, prm, bias)
+    ref = orc.cnn(img, n5, prm, bias_plane=(bias == "plane"))
+    assert normwise(out, ref) <= 1e-5
+
+
+def test_cnn_vga_batch_both_nets(tg, orc):
+    """configs[2] shape (480x640 planes), a small batch of it, both nets."""
+    seed = synth.seed_for_config(3)
+    img = synth.images_np(seed, 2, 480, 640)
+    for n5 in (20, 120):
+        prm = synth.cnn_params_np(seed, n5, 480, 640)
+        out, p = run_cnn(tg, img, n5, prm)
+        assert p.stats()["n_ops_fig7"] == (1600 if n5 == 20 else 7500)
+        assert normwise(out, orc.cnn(img, n5, prm)) <= 1e-5
+
+
+@pytest.mark.parametrize("budget,mcp", [(0, 20000), (2_000_000, None), (1_200_000, None)])
+def test_cnn_split_equals_unsplit(tg, orc, budget, mcp):
+    seed = 77
+    n, H, W, n5 = 2, 200, 180, 40
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    full, p0 = run_cnn(tg, img, n5, prm)
+    split, p1 = run_cnn(tg, img, n5, prm, budget=budget, max_chunk_px=mcp)
+    j = p1.json()
+    assert j["n_chunks"] > p0.json()["n_chunks"]
+    if budget:
+        assert j["arena_bytes"] <= budget
+    assert np.array_equal(split, full), j["bias"]
+    assert normwise(full, orc.cnn(img, n5, prm)) <= 1e-5
+
+
+def test_cnn_streamed_bias_rows(tg, orc):
+    """A budget too small for the resident bias set forces bias rows to stream per chunk."""
+    seed = 78
+    img = synth.images_np(seed, 1, 300, 260)
+    prm = synth.cnn_params_np(seed, 120, 300, 260)
+    out, p = run_cnn(tg, img, 120, prm, budget=3_000_000)
+    assert p.json()["bias"] == "streamed"
+    full, _ = run_cnn(tg, img, 120, prm)
+    assert np.array_equal(out, full)
+    assert normwise(out, orc.cnn(img, 120, prm)) <= 1e-5
+
+
+def test_cnn_device_io_equals_streamed(tg):
+    seed = 79
+    img = synth.images_np(seed, 3, 100, 120)
+    prm = synth.cnn_params_np(seed, 20, 100, 120)
+    a, _ = run_cnn(tg, img, 20, prm, device=True)
+    b, _ = run_cnn(tg, img, 20, prm, budget=1_500_000)
+    assert np.array_equal(a, b)
+
+
+def _tanh32(v):
+    return np.float32(math.tanh(float(v)))
+
+
+def test_cnn_delta_geometry(tg):
+    rng = np.random.default_rng(17)
+    H, W, n5 = 83, 91, 20
+    (h1, w1), _, (h3, w3), _, (h5, w5) = synth.cnn_dims(H, W)
+    x = rng.random((1, 1, H, W)).astype(np.float32)
+    a1, p2 = rng.integers(0, 5, (8, 2)), rng.integers(0, 2, (8, 2))
+    a3, p4 = rng.integers(0, 5, (20, 2)), rng.integers(0, 2, (20, 2))
+    a5 = rng.integers(0, 5, (n5, 2))
+    K1 = np.zeros((8, 1, 5, 5), np.float32)
+    P2 = np.zeros((8, 2, 2), np.float32)
+    K3 = np.zeros((20, 8, 5, 5), np.float32)
+    P4 = np.zeros((20, 2, 2), np.float32)
+    K5 = np.zeros((n5, 20, 5, 5), np.float32)
+    K6 = np.zeros((9, n5, 1, 1), np.float32)
+    for j in range(8):
+        K1[j, 0, a1[j, 0], a1[j, 1]] = 1
+        P2[j, p2[j, 0], p2[j, 1]] = 1
+    for j in range(20):
+        K3[j, j % 8, a3[j, 0], a3[j, 1]] = 1
+        P4[j, p4[j, 0], p4[j, 1]] = 1
+    for j in range(n5):
+        K5[j, j % 20, a5[j, 0], a5[j, 1]] = 1
+    for j in range(9):
+        K6[j, j % n5, 0, 0] = 1
+    z = [np.zeros((1, c, h, w), np.float32) for c, (h, w) in [(8, (h1, w1)), (20, (h3, w3)), (n5, (h5, w5)), (9, (h5, w5))]]
+    prm = [K1, z[0], P2, K3, z[1], P4, K5, z[2], K6, z[3]]
+    out, _ = run_cnn(tg, x, n5, prm)
+    exp = np.empty((9, h5, w5), np.float32)
+    for j in range(9):
+        i = j % n5
+        m = i % 20
+        l = m % 8
+        for r in range(h5):
+            for c in range(w5):
+                R = 2 * (2 * (r + a5[i, 0]) + p4[m, 0] + a3[m, 0]) + p2[l, 0] + a1[l, 0]
+                C = 2 * (2 * (c + a5[i, 1]) + p4[m, 1] + a3[m, 1]) + p2[l, 1] + a1[l, 1]
+                v = x[0, 0, R, C]
+                for _ in range(5):
+                    v = _tanh32(v)
+                exp[j, r, c] = v
+    # exact gathers; only the five tanh evaluations round differently (|err| < 1e-6)
+    assert np.abs(out[0] - exp).max() < 1e-6
+
+
+def test_large_cnn_paper_size_sampled_rows(tg, orc):
+    """Paper-literal configs[3]: large CNN on one 6400x4800 image (17.66e9-float Fig. 7
+    footprint) under the 1.5 GB budget: bias rows stream; sampled output rows
+    at chunk boundaries match the oracle evaluated on each row's receptive band."""
+    H, W, n5 = 4800, 6400, 120
+    seed = synth.seed_for_config(4)
+    img = synth.images_np(seed, 1, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    h5, w5 = synth.cnn_dims(H, W)[4]
+    out, p = run_cnn(tg, img, n5, prm, budget=1536 << 20)
+    j = p.json()
+    assert j["bias"] == "streamed" and j["arena_bytes"] <= 1536 << 20
+    rows = {0, h5 - 1}
+    for ch in j["chunks"][:3]:
+        rows |= {ch["out"][0], ch["out"][1] - 1}
+    for r in sorted(rows):
+        band = np.ascontiguousarray(img[:, :, 4 * r:4 * r + 32])
+        bp = list(prm)
+        bp[1] = prm[1][:, :, 4 * r:4 * r + 28]
+        bp[4] = prm[4][:, :, 2 * r:2 * r + 10]
+        bp[7] = prm[7][:, :, r:r + 1]
+        bp[9] = prm[9][:, :, r:r + 1]
+        ref = orc.cnn(band, n5, bp)[0, :, 0]
+        got = out[0, :, r]
+        err = np.abs(got.astype(np.float64) - ref).max() / np.abs(ref).max()
+        assert err <= 1e-5, (r, err)
