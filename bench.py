@@ -137,19 +137,21 @@ def sum_over_ranks(x: float, world: int) -> float:
 
 
 # ------------------------------------------------------------------------------ workloads
-def edge_workload(rank: int):
-    """configs[1]: 15 images of 10000 x 10000 per GPU (6.0 GB fp32), weak scaling."""
+def workload(name: str, rank: int) -> dict:
+    """Per-GPU workloads (weak scaling: every rank processes its own images)."""
     import synth
-    return dict(template="edge", n=15, H=10000, W=10000, budget=768 << 20,
-                seed=synth.seed_for_config(2), n0=15 * rank)
-
-
-def cnn_workload(rank: int, net: str = "large"):
-    """configs[3]-style: the large CNN on 26 x 480x640 images per GPU (17 GB Fig. 7 footprint
-    in fp32), 1.5 GB budget."""
-    import synth
-    return dict(template="cnn", n=26, H=480, W=640, n5=120 if net == "large" else 20,
-                budget=1536 << 20, seed=synth.seed_for_config(4), n0=26 * rank)
+    if name == "edge":       # configs[1]: ~6 GB of large images, 768 MB budget
+        return dict(template="edge", n=15, H=10000, W=10000, budget=768 << 20, seed=synth.seed_for_config(2),
+                    n0=15 * rank, desc="edge-detection template (16x16 filter, 4 orientations, max)")
+    if name == "cnn4":       # configs[3] paper-literal: large CNN, one 6400x4800 image, 1.5 GB budget
+        return dict(template="cnn", n=1, H=4800, W=6400, n5=120, budget=1536 << 20, seed=synth.seed_for_config(4),
+                    n0=rank, desc="large CNN (n5=120, 7500 ops / 11334 DS at Fig. 7 granularity; 17.66e9-float "
+                                  "footprint, PAPER.md:745)")
+    if name in ("cnn3", "cnn3s"):  # configs[2]: CNN in-core on a batch
+        n5 = 120 if name == "cnn3" else 20
+        return dict(template="cnn", n=64, H=480, W=640, n5=n5, budget=0, seed=synth.seed_for_config(3),
+                    n0=64 * rank, desc=f"{'large' if n5 == 120 else 'small'} CNN (n5={n5}), batch of 64 x 480x640")
+    raise ValueError(name)
 
 
 def host_link_peak(dev: int) -> dict:
@@ -187,24 +189,58 @@ def host_link_peak(dev: int) -> dict:
     return best
 
 
-def run_edge(args, rank, world, local):
+def build_graph(tg, wl, x, out, device: bool, params):
+    if wl["template"] == "edge":
+        g, _ = tg.edge_graph(x, params[0], out=out, device=device)
+    else:
+        g, _ = tg.cnn_graph(x, wl["n5"], params, out=out, device=device)
+    return g
+
+
+def unit_flops_per_px(wl) -> dict:
+    """Algorithmic flops per pixel of each unit's OUTPUT level."""
+    if wl["template"] == "edge":
+        return {0: 2 * 2 * 256}
+    n5 = wl["n5"]
+    return {1: 4 * 8 * 25 * 2, 2: 4 * 20 * 200 * 2, 3: n5 * 500 * 2 + 9 * n5 * 2}
+
+
+def unit_out_px(wl) -> dict:
+    import synth
+    if wl["template"] == "edge":
+        return {0: wl["n"] * wl["H"] * wl["W"]}
+    (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = synth.cnn_dims(wl["H"], wl["W"])
+    return {1: wl["n"] * h2 * w2, 2: wl["n"] * h4 * w4, 3: wl["n"] * h5 * w5}
+
+
+KERNEL_NAMES = {0: "edge_fused_kernel (K1)", 1: "cnn_u1_kernel (U1: C1 T S2 T)", 2: "cnn_u2_kernel (U2: C3 T S4 T)",
+                3: "cnn_u3_kernel (U3: C5 T C6)"}
+
+
+def run(args, rank, world, local):
     import numpy as np
     import torch
 
     import synth
     from paper_conf_ipps_sundaramrc09_b200 import tg
 
-    wl = edge_workload(rank)
+    wl = workload(args.template, rank)
     n, H, W = wl["n"], wl["H"], wl["W"]
     px = n * H * W
     dev = torch.device(f"cuda:{local}")
-    K1, _ = synth.edge_filter_np()
-    # inputs generated on the device (counter-based, same bits as the host generator)
+    if wl["template"] == "edge":
+        params = [synth.edge_filter_np()[0]]
+        out_shape = (n, 1, H, W)
+    else:
+        params = synth.cnn_params_np(wl["seed"], wl["n5"], H, W)
+        h5, w5 = synth.cnn_dims(H, W)[4]
+        out_shape = (n, 9, h5, w5)
     x_dev = synth.images_torch(wl["seed"], n, H, W, dev, n0=wl["n0"])
-    y_dev = torch.empty_like(x_dev)
+    y_dev = torch.empty(out_shape, dtype=torch.float32, device=dev)
+
     # ---- value: device-resident, uncapped
-    g, _ = tg.edge_graph(x_dev, K1, out=y_dev, device=True)
-    g.set(torch_runtime=True)
+    g = build_graph(tg, wl, x_dev, y_dev, True, params)
+    g.set(torch_runtime=True, precision=args.precision_code)
     p = g.plan()
     cs = p.compute_stream(local)
     for _ in range(args.warmup):
@@ -222,38 +258,50 @@ def run_edge(args, rank, world, local):
     ms = e0.elapsed_time(e1) / args.steps
     launches = p.launches() - l0
     tim = p.timing()
-    kern_ms = tim["kernel_ms"][0] / max(1, tim["unit_launches"][0])
     ms_max = max_over_ranks(ms, world)
     value = world * px / (ms_max / 1e3) / 1e6
     clocks = clk.summary()
-    flops_per_launch = 2 * 2 * 256 * (px / max(1, tim["unit_launches"][0] / args.steps))
+    # dominant kernel: the unit with the largest summed time
+    fl, opx = unit_flops_per_px(wl), unit_out_px(wl)
+    k = max(fl, key=lambda u: tim["kernel_ms"][u])
+    nl = max(1, tim["unit_launches"][k])
+    kern_ms = tim["kernel_ms"][k] / nl
+    flops_per_launch = fl[k] * opx[k] * args.steps / nl
     achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
     peak_tf = fp32_peak_tflops(1965.0)
     traffic = None
-    tf_file = os.path.join(ROOT, "profiles", "k1_traffic.json")
+    tf_file = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf_file):
-        tr = json.load(open(tf_file))
-        # per launch, scaled to this launch's pixels (ncu capture: same kernel, same tiling)
-        traffic = tr["dram_bytes_per_px"] * (px / max(1, tim["unit_launches"][0] / args.steps))
-    del p, g
+        tr = json.load(open(tf_file)).get(f"{args.template}:{KERNEL_NAMES[k]}")
+        if tr:
+            traffic = tr["dram_bytes_per_out_px"] * opx[k] * args.steps / nl
+    roofline = {"bound": "alu", "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
+                "frac": achieved_tf / peak_tf, "traffic": traffic, "kernel": KERNEL_NAMES[k],
+                "kernel_ms_per_launch": kern_ms, "algorithmic_flop_per_launch": flops_per_launch,
+                "peak_basis": "FP32 FFMA: 148 SM x 128 lanes x 2 flop x 1965 MHz (clocks.max.sm)",
+                "kernel_share_of_step": tim["kernel_ms"][k] / args.steps / ms,
+                "units_ms_per_step": {KERNEL_NAMES[u]: tim["kernel_ms"][u] / args.steps for u in fl}}
+    y_ref = [y_dev[0].clone(), y_dev[-1].clone()]
+    del p, g, y_dev
 
     # ---- e2e: host pinned buffers through the C ABI, capped budget, streamed
     x_host = torch.empty((n, 1, H, W), dtype=torch.float32).pin_memory()
     x_host.copy_(x_dev)
-    y_host = torch.empty((n, 1, H, W), dtype=torch.float32).pin_memory()
     del x_dev
-    g2, _ = tg.edge_graph(x_host, K1, out=y_host)
-    g2.set(budget=wl["budget"], torch_runtime=True)
+    y_host = torch.empty(out_shape, dtype=torch.float32).pin_memory()
+    g2 = build_graph(tg, wl, x_host, y_host, False, params)
+    g2.set(budget=wl["budget"], torch_runtime=True, precision=args.precision_code)
     p2 = g2.plan()
     st = p2.stats()
+    js = p2.json()
     cs2 = p2.compute_stream(local)
     for _ in range(args.warmup):
         p2.execute()
     torch.cuda.synchronize()
-    # bit-exact check of the streamed result against the device-resident one (same kernels)
-    assert torch.equal(y_host[0, 0, :64].to(dev), y_dev[0, 0, :64]) and \
-        torch.equal(y_host[-1, 0, -64:].to(dev), y_dev[-1, 0, -64:]), "streamed != resident"
-    del y_dev
+    # the streamed result equals the device-resident one bit for bit (same kernels, same order)
+    assert torch.equal(y_host[0].to(dev), y_ref[0]) and torch.equal(y_host[-1].to(dev), y_ref[1]), \
+        "streamed != resident"
+    del y_ref
     p2.profiling(True)
     l2 = p2.launches()
     barrier(world)
@@ -270,85 +318,91 @@ def run_edge(args, rank, world, local):
     tim2 = p2.timing()
     ms2_max = max_over_ranks(ms2, world)
     e2e_value = world * px / (ms2_max / 1e3) / 1e6
-    link = host_link_peak(local) if rank == 0 else None
-    h2d, d2h = st["h2d_bytes"], st["d2h_bytes"]
-    out = {
-        "value": value, "ms_per_step": ms_max, "clocks": clocks, "gpu_launches": launches,
-        "roofline": {"bound": "alu", "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
-                     "frac": achieved_tf / peak_tf, "traffic": traffic,
-                     "kernel": "edge_fused_kernel (K1)", "kernel_ms_per_launch": kern_ms,
-                     "algorithmic_flop_per_px": 1024,
-                     "peak_basis": "148 SM x 128 FP32 lanes x 2 x 1965 MHz (clocks.max.sm)",
-                     "kernel_share_of_step": tim["kernel_ms"][0] / args.steps / ms},
-        "e2e": {"value": e2e_value, "unit": "Mpixels/s", "ms_per_step": ms2_max, "wall_ms_per_step": wall * 1e3,
-                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "io_lower_bound_bytes": st["io_lower_bound_bytes"],
-                "bytes_vs_lower_bound": (h2d + d2h) / st["io_lower_bound_bytes"],
-                "budget_bytes": wl["budget"], "arena_bytes": st["peak_device_bytes"][0],
-                "chunks": st["n_chunks"], "gpu_launches": launches2,
-                "kernel_ms_per_step": sum(tim2["kernel_ms"]) / args.steps,
-                "h2d_ms_per_step": tim2["h2d_ms"] / args.steps, "d2h_ms_per_step": tim2["d2h_ms"] / args.steps},
-        "config": {"workload": f"edge-detection template (16x16 filter, 4 orientations, max), {n} x {H}x{W} fp32 "
-                               f"images ({n * H * W * 4 / 1e9:.1f} GB) per GPU; value: device-resident, uncapped; "
-                               f"e2e: pinned host buffers, {wl['budget'] >> 20} MiB device budget, streamed",
-                   "template": "edge", "images_per_gpu": n, "H": H, "W": W, "budget_bytes_e2e": wl["budget"],
-                   "l2": "inputs 6.0 GB per step >> 126 MB L2 (no flush needed)", "precision": "fp32"},
-    }
-    if link:
-        achieved_link = (h2d / 1e9) / (ms2 / 1e3)
-        t_link = max(h2d / (link["bidir_each"] * 1e9), d2h / (link["bidir_each"] * 1e9))
-        out["e2e"]["host_link"] = {"peak_h2d_gbs": link["h2d"], "peak_d2h_gbs": link["d2h"],
-                                   "peak_bidir_each_gbs": link["bidir_each"],
-                                   "achieved_h2d_gbs": achieved_link,
-                                   "achieved_d2h_gbs": (d2h / 1e9) / (ms2 / 1e3),
-                                   "roofline_frac": t_link / (ms2 / 1e3)}
-    return out, px
+    # parameters stay resident after the first execution: a timed step moves the images,
+    # the streamed bias rows (if any) and the outputs
+    h2d, d2h = st["h2d_bytes_steady"], st["d2h_bytes"]
+    e2e = {"value": e2e_value, "unit": "Mpixels/s", "ms_per_step": ms2_max, "wall_ms_per_step": wall * 1e3,
+           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+           "io_lower_bound_bytes": st["io_lower_bound_bytes"],
+           "bytes_vs_lower_bound": (h2d + d2h) / st["io_lower_bound_bytes"],
+           "budget_bytes": wl["budget"], "arena_bytes": st["peak_device_bytes"][0], "chunks": st["n_chunks"],
+           "split": js["split"], "bias": js["bias"], "gpu_launches": launches2,
+           "kernel_ms_per_step": sum(tim2["kernel_ms"]) / args.steps,
+           "h2d_ms_per_step": tim2["h2d_ms"] / args.steps, "d2h_ms_per_step": tim2["d2h_ms"] / args.steps}
+    if rank == 0:
+        link = host_link_peak(local)
+        # link roofline: each direction at its solo peak, both together at the measured
+        # concurrent (bidirectional) rate
+        t_link = max(h2d / (link["h2d"] * 1e9), d2h / (link["d2h"] * 1e9),
+                     (h2d + d2h) / (2 * link["bidir_each"] * 1e9))
+        e2e["host_link"] = {"peak_h2d_gbs": link["h2d"], "peak_d2h_gbs": link["d2h"],
+                            "peak_bidir_each_gbs": link["bidir_each"],
+                            "achieved_h2d_gbs": (h2d / 1e9) / (ms2 / 1e3),
+                            "achieved_d2h_gbs": (d2h / 1e9) / (ms2 / 1e3),
+                            "roofline_time_ms": t_link * 1e3, "roofline_frac": t_link / (ms2 / 1e3)}
+    desc = (f"{wl['desc']}, {n} x {H}x{W} fp32 images ({px * 4 / 1e9:.2f} GB) per GPU; value: device-resident, "
+            f"uncapped; e2e: pinned host buffers, "
+            f"{'uncapped' if not wl['budget'] else str(wl['budget'] >> 20) + ' MiB device budget'}, streamed")
+    config = {"workload": desc, "template": wl["template"], "images_per_gpu": n, "H": H, "W": W,
+              "n5": wl.get("n5"), "budget_bytes_e2e": wl["budget"], "precision": args.precision,
+              "l2": f"inputs {px * 4 / 1e9:.2f} GB per step" + (" >> 126 MB L2 (no flush needed)" if px * 4 > 1e9
+                                                               else " (L2 not flushed)")}
+    return {"value": value, "ms_per_step": ms_max, "clocks": clocks, "gpu_launches": launches,
+            "roofline": roofline, "e2e": e2e, "config": config}
 
 
 # ------------------------------------------------------------------------------ CPU leg
-def cpu_oracle_sample(target_s: float = 12.0) -> dict:
-    """The CPU oracle (as it stands) on a bounded sample of the edge workload: a band of rows
-    of one 10000-wide image (the same per-pixel work as every row of the workload)."""
-    import numpy as np
-
+def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0) -> dict:
+    """The CPU oracle (as it stands) on a bounded sample of the workload: for the edge
+    template whole 10000x10000 images of configs[1] (plus a band of rows if one image is
+    too fast); for the CNN a band of rows of the workload's image. Reports input Mpx/s."""
     import oracle
     import synth
     oracle.build()
-    W = 10000
-    seed = synth.seed_for_config(2)
-    K1, K2 = synth.edge_filter_np()
-    rows = 16
-    while True:
-        band = synth.image_np(seed, synth.DS_IMAGE, 0, (10000, W), row0=0, rows=rows)
+    if template == "edge":
+        W = 10000
+        seed = synth.seed_for_config(2)
+        K1, K2 = synth.edge_filter_np()
+        done_px, t_tot, imgs = 0, 0.0, 0
+        while t_tot < target_s and imgs < 15:
+            img = synth.image_np(seed, synth.DS_IMAGE, imgs, (10000, W))
+            t0 = time.perf_counter()
+            oracle.edge(img, K1, K2)
+            t_tot += time.perf_counter() - t0
+            done_px += img.size
+            imgs += 1
+        sample = f"oracle.edge on {imgs} whole 10000x10000 images of configs[1] ({t_tot:.1f} s)"
+    else:
+        wl = workload(template, 0)
+        H, W, n5 = wl["H"], wl["W"], wl["n5"]
+        prm = synth.cnn_params_np(wl["seed"], n5, H, W)
+        img = synth.image_np(wl["seed"], synth.DS_IMAGE, 0, (H, W))
         t0 = time.perf_counter()
-        oracle.edge(band, K1, K2)
-        dt = time.perf_counter() - t0
-        if dt * 4 >= target_s or rows >= 10000:
-            break
-        rows = min(10000, int(rows * max(2.0, target_s / max(dt, 1e-3) / 2)))
-    return {"value": rows * W / dt / 1e6, "unit": "Mpixels/s", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"oracle.edge on a {rows}x{W} band of image 0 (config 2 inputs), {dt:.1f} s"}
+        oracle.cnn(img, n5, prm)
+        t_tot = time.perf_counter() - t0
+        done_px = H * W
+        sample = f"oracle.cnn on one {H}x{W} image of the workload ({t_tot:.1f} s)"
+    return {"value": done_px / t_tot / 1e6, "unit": "Mpixels/s", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": sample}
 
 
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    import oracle
-    oracle.build()
-    wl = edge_workload(0)
-    vals = []
-    for _ in range(args.warmup):
-        cpu_oracle_sample(2.0)
-    for _ in range(args.steps):
-        vals.append(cpu_oracle_sample(8.0))
+    wl = workload(args.template, 0)
+    for _ in range(min(args.warmup, 1)):
+        cpu_oracle_sample(args.template, 1.0)
+    vals = [cpu_oracle_sample(args.template, 8.0) for _ in range(args.steps)]
     v = statistics.median([x["value"] for x in vals])
+    px = wl["n"] * wl["H"] * wl["W"]
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "Mpixels/s",
             "n_gpus": int(args.gpus), "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": wl["H"] * wl["W"] * wl["n"] / (v * 1e6) * 1e3, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64-accumulate/f32", "data": "synthetic",
-            "config": {"workload": "edge-detection template, 10000-wide images (configs[1]); CPU oracle on row "
-                                   "bands of the same images", "template": "edge"},
+            "ms_per_step": px / (v * 1e6) * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32 (fp64 accumulation)", "data": "synthetic",
+            "config": {"workload": f"{wl['desc']}, {wl['n']} x {wl['H']}x{wl['W']} per GPU; the CPU oracle "
+                                   f"(oracle/oracle.c, OpenMP) timed on a bounded sample of it",
+                       "template": wl["template"]},
             "cpu_baseline": {"kind": "oracle", "cores": vals[0]["cores"], "sample": vals[-1]["sample"], "value": v},
             "e2e": {"value": v, "unit": "Mpixels/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -360,27 +414,31 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--template", default="edge", choices=["edge"])
+    ap.add_argument("--template", default="edge", choices=["edge", "cnn4", "cnn3", "cnn3s"])
+    ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16_tc"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
-    if args.warmup < 3:
-        args.warmup = 3
+    args.warmup = max(3, args.warmup)
     if args.impl == "reference":
         run_reference(args)
         return
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    args.precision_code = tg.TG_FP32 if args.precision == "fp32" else tg.TG_BF16_TC
     rank, world, local = dist_setup(args)
-    res, px = run_edge(args, rank, world, local)
+    res = run(args, rank, world, local)
     if rank == 0:
         line = {"metric": METRIC, "value": res["value"], "unit": "Mpixels/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms_per_step"],
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-                "data": "synthetic (counter-based generator, seed 0x5EED0002; 8-bit levels k/255)",
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "f32" if args.precision == "fp32" else "bf16 (fp32 accumulate)",
+                "data": "synthetic (counter-based generator synth/, 8-bit levels k/255)",
                 "config": res["config"], "roofline": res["roofline"], "e2e": res["e2e"], "clocks": res["clocks"],
-                "gpu_launches": res["gpu_launches"],
-                "paper_context": {"mpx_s": 24.3, "what": "edge 10000x10000, Tesla C870, host-to-host, no overlap "
-                                  "(PAPER.md:753); 25.5 on 8800 GTX"}}
+                "gpu_launches": res["gpu_launches"]}
+        if args.template == "edge":
+            line["paper_context"] = {"mpx_s": 24.3, "what": "edge 10000x10000, Tesla C870, host-to-host, no overlap "
+                                                            "(PAPER.md:753); 25.5 on 8800 GTX"}
         if world == 1 and not args.no_cpu:
-            line["cpu_baseline"] = cpu_oracle_sample()
+            line["cpu_baseline"] = cpu_oracle_sample(args.template)
         print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist

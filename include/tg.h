@@ -169,6 +169,8 @@ typedef struct {
     int64_t n_ds_fig7;               /* data structures at Fig. 7 granularity           */
     int64_t chunk_begin, chunk_end;  /* this shard's chunk range                        */
     uint64_t host_registered_bytes;  /* pageable host bytes registered by the library   */
+    uint64_t h2d_bytes_steady;       /* H2D bytes of a later execution: parameters stay
+                                        resident in the arena after the first one        */
 } tg_plan_stats;
 tg_status tg_plan_stats_get(const tg_plan* plan, tg_plan_stats* out);
 
@@ -195,6 +197,10 @@ typedef struct {
 } tg_timing;
 tg_status tg_plan_set_profiling(tg_plan* plan, int32_t on);
 tg_status tg_plan_timing_get(tg_plan* plan, tg_timing* out);
+/* Parameters are copied to the device by the first execution of a plan and stay resident
+ * in its arena; call this after changing parameter host data to re-upload them at the next
+ * execution. */
+tg_status tg_plan_invalidate_params(tg_plan* plan);
 /* Kernel launches issued by the library since plan creation (always counted). */
 int64_t tg_plan_launch_count(const tg_plan* plan);
 

@@ -377,6 +377,8 @@ tg_status tg_plan_stats_get(const tg_plan* p, tg_plan_stats* out) {
     out->chunk_begin = c.c0;
     out->chunk_end = c.c1;
     out->host_registered_bytes = exec_registered_bytes(p);
+    // steady state: parameters stay resident after the first execution
+    out->h2d_bytes_steady = c.device_io ? 0 : c.h2d - c.param_bytes;
     return TG_OK;
 }
 
@@ -420,6 +422,12 @@ tg_status tg_plan_timing_get(tg_plan* p, tg_timing* out) {
 }
 
 int64_t tg_plan_launch_count(const tg_plan* p) { return p ? p->launches : 0; }
+
+tg_status tg_plan_invalidate_params(tg_plan* p) {
+    if (!p) return fail(TG_E_ARG, "tg_plan_invalidate_params: NULL plan");
+    exec_invalidate_params(p);
+    return TG_OK;
+}
 
 void tg_plan_destroy(tg_plan* p) {
     if (!p) return;

@@ -45,6 +45,7 @@ struct DevState {
     std::vector<ProfRec> prof;
     std::vector<cudaEvent_t> ev_pool;
     int64_t launches = 0;
+    bool params_resident = false;  // parameters uploaded by an earlier execution
 };
 
 }  // namespace
@@ -56,6 +57,7 @@ struct tg_exec {
     uint64_t registered_bytes = 0;
     bool profiling = false;
     tg_timing timing{};
+    int64_t param_uploads = 0;
 };
 
 namespace {
@@ -396,8 +398,9 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
     CK(cudaEventRecord(d.ev_fork, S1));
     CK(cudaStreamWaitEvent(S0, d.ev_fork, 0));
     CK(cudaStreamWaitEvent(S2, d.ev_fork, 0));
-    // parameters: once per execution (never split)
-    {
+    // parameters (never split): uploaded by the first execution and kept
+    // resident in the arena for later ones (tg_plan_invalidate_params forces a re-upload)
+    if (!d.params_resident) {
         ProfRec pr{10, nullptr, nullptr};
         if (x->profiling) {
             pr.a = pool_event(d);
@@ -415,6 +418,8 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
         }
         CK(cudaEventRecord(d.ev_params, S0));
         CK(cudaStreamWaitEvent(S1, d.ev_params, 0));
+        d.params_resident = true;
+        x->param_uploads += 1;
     }
     const int D = c.depth;
     for (int64_t k = 0; k < d.c1 - d.c0; ++k) {
@@ -593,5 +598,10 @@ void exec_destroy(tg_plan* p) {
 }
 
 uint64_t exec_registered_bytes(const tg_plan* p) { return p->exec ? p->exec->registered_bytes : 0; }
+
+void exec_invalidate_params(tg_plan* p) {
+    if (!p->exec) return;
+    for (auto& d : p->exec->devs) d.params_resident = false;
+}
 
 }  // namespace tg

@@ -142,4 +142,5 @@ tg_status exec_set_profiling(tg_plan* p, bool on);
 tg_status exec_timing(tg_plan* p, tg_timing* out);
 void exec_destroy(tg_plan* p);
 uint64_t exec_registered_bytes(const tg_plan* p);
+void exec_invalidate_params(tg_plan* p);
 }  // namespace tg

@@ -64,7 +64,8 @@ class tg_plan_stats(ctypes.Structure):
     _fields_ = [("h2d_bytes", c_u64), ("d2h_bytes", c_u64), ("io_lower_bound_bytes", c_u64),
                 ("total_temp_bytes", c_u64), ("peak_device_bytes", c_u64 * 8), ("n_chunks", c_i64),
                 ("n_units", c_i64), ("n_ops_fig7", c_i64), ("n_ds_fig7", c_i64),
-                ("chunk_begin", c_i64), ("chunk_end", c_i64), ("host_registered_bytes", c_u64)]
+                ("chunk_begin", c_i64), ("chunk_end", c_i64), ("host_registered_bytes", c_u64),
+                ("h2d_bytes_steady", c_u64)]
 
 
 class tg_timing(ctypes.Structure):
@@ -102,6 +103,7 @@ _PROTOS = {
     "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
     "tg_plan_timing_get": (c_i32, [vp, ctypes.POINTER(tg_timing)]),
     "tg_plan_launch_count": (c_i64, [vp]),
+    "tg_plan_invalidate_params": (c_i32, [vp]),
     "tg_plan_destroy": (None, [vp]),
     "tg_last_error": (ctypes.c_char_p, []),
     "tg_version": (ctypes.c_char_p, []),
@@ -286,6 +288,10 @@ def tg_plan_timing_get(p) -> dict:
 
 def tg_plan_launch_count(p) -> int:
     return int(_lib.tg_plan_launch_count(p))
+
+
+def tg_plan_invalidate_params(p) -> None:
+    _ck(_lib.tg_plan_invalidate_params(p))
 
 
 def tg_plan_destroy(p) -> None:
