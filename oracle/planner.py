@@ -438,7 +438,8 @@ def _span(r) -> int:
 
 def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int = 20,
                bias: str = "plane", budget: int = 0, max_chunk_px: int = MAX_CHUNK_PX,
-               depth: int = DEPTH, rank: int = 0, world: int = 1, device_io: bool = False) -> dict:
+               depth: int = DEPTH, rank: int = 0, world: int = 1, device_io: bool = False,
+               precision: str = "fp32") -> dict:
     """Fused-mode plan, restated plainly; the library's
     tg_plan_dump_json must produce the same dict (tests/test_plan_parity.py).
 
@@ -503,6 +504,12 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
 
     all_pb = sum(a256(p * f) for p in params)
     nonbias_pb = sum(a256(p * f) for p, b in zip(params, is_bias) if not b)
+    if template == "cnn" and precision == "bf16_tc":
+        # bf16 B operands of the tensor-core C3 (15 K-steps x 2 halves x 32 maps x 8) and
+        # C5 (40 K-steps x 2 x n5 rounded up to 16 x 8), kept with the parameters
+        tc = a256(15 * 2 * 32 * 8 * 2) + a256(40 * 2 * ((n5 + 15) // 16 * 16) * 8 * 2)
+        all_pb += tc
+        nonbias_pb += tc
     if device_io:
         depth = 1
 
@@ -593,7 +600,7 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
         "template": template, "n": n, "H": H, "W": W,
         "ks": ks if template == "edge" else 0, "n5": n5 if template == "cnn" else 0,
         "budget": budget, "depth": depth, "max_chunk_px": max_chunk_px,
-        "device_io": bool(device_io), "bias": bias_mode, "split": split, "B": B, "R": R,
+        "device_io": bool(device_io), "precision": precision if template == "cnn" else "fp32", "bias": bias_mode, "split": split, "B": B, "R": R,
         "param_bytes": pb, "slot_bytes": sb, "arena_bytes": pb + depth * sb,
         "n_chunks": C, "chunks": chunks, "shard": [rank, world, c0, c1],
         "h2d_bytes": h2d, "d2h_bytes": d2h, "io_lower_bound_bytes": io_lb,

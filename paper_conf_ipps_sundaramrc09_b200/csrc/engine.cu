@@ -58,6 +58,7 @@ struct tg_exec {
     bool profiling = false;
     tg_timing timing{};
     int64_t param_uploads = 0;
+    std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
 };
 
 namespace {
@@ -339,8 +340,10 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.w4 = w4;
         a.nimg = ch.nimg;
         a.bf16_tc = c.precision == TG_BF16_TC;
+        a.k3_tc = c.k3tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k3tc_off);
+        a.p4_dev = param(5);
         KernelTimer kt(x, d, 2, cs);
-        CK(launch_cnn_u2(a, cs));
+        CK(a.bf16_tc ? launch_cnn_u2_tc(a, cs) : launch_cnn_u2(a, cs));
         kt.done(cs);
         ++d.launches;
     }
@@ -380,8 +383,10 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.n5 = t.n5;
         a.nimg = ch.nimg;
         a.bf16_tc = c.precision == TG_BF16_TC;
+        a.k5_tc = c.k5tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k5tc_off);
+        a.n_pad = cnn_n5_pad(t.n5);
         KernelTimer kt(x, d, 3, cs);
-        CK(launch_cnn_u3(a, cs));
+        CK(a.bf16_tc ? launch_cnn_u3_tc(a, cs) : launch_cnn_u3(a, cs));
         kt.done(cs);
         ++d.launches;
     }
@@ -411,6 +416,17 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
             if (c.param_off[i] == UINT64_MAX) continue;
             const Ds& P = g.ds[c.param_ds[i]];
             CK(cudaMemcpyAsync(d.arena + c.param_off[i], P.src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
+        }
+        if (c.k3tc_off != UINT64_MAX) {
+            // bf16 B operands of the tensor-core C3/C5 (prepared on the host once per plan)
+            if (x->k3tc.empty()) {
+                x->k3tc.resize(cnn_k3_tc_bytes() / 2);
+                x->k5tc.resize(cnn_k5_tc_bytes(c.t.n5) / 2);
+                cnn_prepare_k3_tc(g.ds[c.t.prm[3]].src, x->k3tc.data());
+                cnn_prepare_k5_tc(g.ds[c.t.prm[6]].src, c.t.n5, x->k5tc.data());
+            }
+            CK(cudaMemcpyAsync(d.arena + c.k3tc_off, x->k3tc.data(), x->k3tc.size() * 2, cudaMemcpyHostToDevice, S0));
+            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5tc.data(), x->k5tc.size() * 2, cudaMemcpyHostToDevice, S0));
         }
         if (x->profiling) {
             cudaEventRecord(pr.b, S0);

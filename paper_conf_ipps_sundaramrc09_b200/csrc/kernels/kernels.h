@@ -44,6 +44,8 @@ struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
     float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w3, w4;
     int64_t nimg;
     int bf16_tc;            // 1: tcgen05 bf16 path
+    const uint16_t* k3_tc;  // bf16 B operand prepared by cnn_prepare_k3_tc (device)
+    const float* p4_dev;    // [20][4] (device)
 };
 struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + bias -> out
     const float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w4;
@@ -55,9 +57,20 @@ struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + 
     int n5;
     int64_t nimg;
     int bf16_tc;
+    const uint16_t* k5_tc;  // bf16 B operand prepared by cnn_prepare_k5_tc (device)
+    int n_pad;              // n5 rounded up to a multiple of 16
 };
 cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3(const CnnU3Args& a, cudaStream_t s);
+
+// tcgen05 (bf16 operands, fp32 accumulation in TMEM) variants of U2 and U3 (cnn_tc.cu)
+cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s);
+cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s);
+size_t cnn_k3_tc_bytes();
+void cnn_prepare_k3_tc(const float* k3, uint16_t* dst);
+int cnn_n5_pad(int n5);
+size_t cnn_k5_tc_bytes(int n5);
+void cnn_prepare_k5_tc(const float* k5, int n5, uint16_t* dst);
 
 }  // namespace tg

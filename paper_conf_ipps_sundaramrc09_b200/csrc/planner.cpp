@@ -17,6 +17,7 @@
 #include <cstdio>
 #include <sstream>
 
+#include "kernels/kernels.h"
 #include "tg_internal.h"
 
 namespace tg {
@@ -269,8 +270,6 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     p.device_io = X.src_loc == Loc::Device && Y.dst_loc == Loc::Device;
     if ((X.src_loc == Loc::Device) != (Y.dst_loc == Loc::Device))
         return fail(TG_E_UNSUPPORTED, "plan: input and output must both be host or both be device resident");
-    if (t.kind == Tmpl::Cnn && g.precision == TG_BF16_TC && t.n5 % 4 != 0)
-        return fail(TG_E_UNSUPPORTED, "plan: TG_BF16_TC needs n5 % 4 == 0");
     const uint64_t f = 4;
     const int64_t H = t.H, W = t.W, n = t.n;
     const int64_t h_out = t.kind == Tmpl::Edge ? H : t.h[5];
@@ -292,6 +291,13 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         const uint64_t b = a256((uint64_t)g.ds[prm[i]].numel() * f);
         all_pb += b;
         if (!is_bias[i]) nonbias_pb += b;
+    }
+    // tensor-core path: bf16 B operands of C3 and C5 prepared once and kept with the params
+    uint64_t tc_bytes = 0;
+    if (t.kind == Tmpl::Cnn && g.precision == TG_BF16_TC) {
+        tc_bytes = a256(cnn_k3_tc_bytes()) + a256(cnn_k5_tc_bytes(t.n5));
+        all_pb += tc_bytes;
+        nonbias_pb += tc_bytes;
     }
     int32_t depth = p.device_io ? 1 : g.depth;
     p.depth = depth;
@@ -414,6 +420,13 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         p.param_off[i] = off;
         off += a256((uint64_t)g.ds[prm[i]].numel() * f);
     }
+    p.k3tc_off = p.k5tc_off = UINT64_MAX;
+    if (tc_bytes) {
+        p.k3tc_off = off;
+        off += a256(cnn_k3_tc_bytes());
+        p.k5tc_off = off;
+        off += a256(cnn_k5_tc_bytes(t.n5));
+    }
     p.chunks = chunk_list(batch, B, R);
     const int64_t C = (int64_t)p.chunks.size();
     p.rank = g.rank;
@@ -475,6 +488,8 @@ std::string plan_json(const PlanCore& p) {
     o << "\"ks\": " << (t.kind == Tmpl::Edge ? t.ks : 0) << ", \"n5\": " << (t.kind == Tmpl::Cnn ? t.n5 : 0) << ", ";
     o << "\"budget\": " << p.budget << ", \"depth\": " << p.depth << ", \"max_chunk_px\": " << p.max_chunk_px << ", ";
     o << "\"device_io\": " << (p.device_io ? "true" : "false") << ", ";
+    o << "\"precision\": \"" << (t.kind == Tmpl::Cnn && p.precision == TG_BF16_TC ? "bf16_tc" : "fp32") << "\", ";
+    o << "\"precision\": \"" << (p.precision == TG_BF16_TC ? "bf16_tc" : "fp32") << "\", ";
     o << "\"bias\": \"" << p.bias << "\", \"split\": \"" << p.split << "\", ";
     o << "\"B\": " << p.B << ", \"R\": " << p.R << ", ";
     o << "\"param_bytes\": " << p.param_bytes << ", \"slot_bytes\": " << p.slot_bytes

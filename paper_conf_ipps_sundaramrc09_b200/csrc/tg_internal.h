@@ -107,6 +107,7 @@ struct PlanCore {
     std::vector<uint64_t> param_off;  // offset of each param (template order) in param region
     std::vector<int> param_ds;        // DS ids in template order
     std::vector<bool> param_streamed; // true: bias rows streamed per chunk
+    uint64_t k3tc_off = UINT64_MAX, k5tc_off = UINT64_MAX;  // bf16 tensor-core B operands
     SlotLayout slot;
     std::vector<Chunk> chunks;        // global chunk list
     int64_t c0 = 0, c1 = 0;           // this process's shard

@@ -174,3 +174,35 @@ def test_large_cnn_paper_size_sampled_rows(tg, orc):
         got = out[0, :, r]
         err = np.abs(got.astype(np.float64) - ref).max() / np.abs(ref).max()
         assert err <= 1e-5, (r, err)
+
+
+# ------------------------------------------------------------------ tcgen05 bf16 path
+@pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
+                                          (2, 480, 640, 120, "plane"), (1, 480, 640, 20, "scalar"),
+                                          (1, 97, 1003, 120, "plane"), (1, 61, 67, 7, "plane"),
+                                          (1, 140, 1400, 33, "scalar")])
+def test_cnn_bf16_tc_parity(tg, orc, n, H, W, n5, bias):
+    """C3, C5 on tcgen05 (bf16 operands, fp32 accumulation): normwise <= 2e-2 (north_star);
+    covers the flattened (narrow) and column-window (wide) band modes of U3."""
+    seed = synth.seed_for_config(3) + 17
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W, bias)
+    out, p = run_cnn(tg, img, n5, prm, bias, precision=tg.TG_BF16_TC)
+    assert p.json()["precision"] == "bf16_tc"
+    ref = orc.cnn(img, n5, prm, bias_plane=(bias == "plane"))
+    err = normwise(out, ref)
+    assert err <= 2e-2, err
+    # and it really is the reduced-precision path (not the fp32 kernels)
+    out32, _ = run_cnn(tg, img, n5, prm, bias)
+    assert not np.array_equal(out, out32)
+
+
+def test_cnn_bf16_tc_split_equals_unsplit(tg):
+    seed = 91
+    n, H, W, n5 = 2, 200, 180, 120
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    full, p0 = run_cnn(tg, img, n5, prm, precision=tg.TG_BF16_TC)
+    split, p1 = run_cnn(tg, img, n5, prm, budget=2_000_000, precision=tg.TG_BF16_TC)
+    assert p1.json()["n_chunks"] > p0.json()["n_chunks"]
+    assert np.array_equal(split, full)

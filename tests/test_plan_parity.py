@@ -30,6 +30,9 @@ CASES = [
     ("cnn", 2, 480, 6400, dict(n5=20, device_io=True)),
     ("cnn", 64, 480, 640, dict(n5=120, device_io=True, budget=2 << 30)),
     ("cnn", 1, 4800, 6400, dict(n5=120, budget=1536 << 20, rank=1, world=2)),
+    ("cnn", 64, 480, 640, dict(n5=120, precision="bf16_tc")),
+    ("cnn", 1, 4800, 6400, dict(n5=120, budget=1536 << 20, precision="bf16_tc")),
+    ("cnn", 3, 200, 180, dict(n5=37, budget=2_000_000, precision="bf16_tc")),
 ]
 
 
@@ -73,7 +76,8 @@ def library_plan(tmpl, n, H, W, kw):
         g._keep.append(out)
         tg.tg_output(g.h, y, out.ctypes.data)
     g.set(budget=kw.get("budget", 0), max_chunk_px=kw.get("max_chunk_px", 1 << 24), depth=kw.get("depth", 3),
-          shard=(kw.get("rank", 0), kw.get("world", 1)))
+          shard=(kw.get("rank", 0), kw.get("world", 1)),
+          precision=tg.TG_BF16_TC if kw.get("precision") == "bf16_tc" else tg.TG_FP32)
     return g.plan().json()
 
 
