@@ -274,17 +274,31 @@ def run(args, rank, world, local):
     kern_ms = tim["kernel_ms"][k] / nl
     flops_per_launch = fl[k] * opx[k] * args.steps / nl
     achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
-    peak_tf = fp32_peak_tflops(1965.0)
+    tensor = args.precision == "bf16_tc" and k in (2, 3)
+    if tensor:
+        # C3 / C5 on tcgen05: bf16 dense peak MEASURED on this pool (MEASURED_PEAKS.json, burst:
+        # the kernel is timed on its own launches); algorithmic flops exclude K/N padding
+        peaks = json.load(open(PEAKS_FILE)) if os.path.exists(PEAKS_FILE) else {}
+        peak_tf = float(peaks.get("bf16_tflops", 1590.0))
+        peak_basis = ("bf16 dense, measured cuBLAS burst (MEASURED_PEAKS.json)" if "bf16_tflops" in peaks
+                      else "bf16 dense fallback 1.59 PFLOP/s (B200_PROFILING.md)")
+        fl = dict(fl)
+        fl[2], fl[3] = 4 * 20 * 200 * 2, wl["n5"] * 500 * 2   # the tensor-core part of each unit
+        flops_per_launch = fl[k] * opx[k] * args.steps / nl
+        achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
+    else:
+        peak_tf = fp32_peak_tflops(1965.0)
+        peak_basis = "FP32 FFMA: 148 SM x 128 lanes x 2 flop x 1965 MHz (clocks.max.sm)"
     traffic = None
     tf_file = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf_file):
         tr = json.load(open(tf_file)).get(f"{args.template}:{KERNEL_NAMES[k]}")
         if tr:
             traffic = tr["dram_bytes_per_out_px"] * opx[k] * args.steps / nl
-    roofline = {"bound": "alu", "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
+    roofline = {"bound": "tensor" if tensor else "alu", "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
                 "frac": achieved_tf / peak_tf, "traffic": traffic, "kernel": KERNEL_NAMES[k],
                 "kernel_ms_per_launch": kern_ms, "algorithmic_flop_per_launch": flops_per_launch,
-                "peak_basis": "FP32 FFMA: 148 SM x 128 lanes x 2 flop x 1965 MHz (clocks.max.sm)",
+                "peak_basis": peak_basis,
                 "kernel_share_of_step": tim["kernel_ms"][k] / args.steps / ms,
                 "units_ms_per_step": {KERNEL_NAMES[u]: tim["kernel_ms"][u] / args.steps for u in fl}}
     y_ref = [y_dev[0].clone(), y_dev[-1].clone()]

@@ -308,6 +308,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.w1 = w1;
         a.w2 = w2;
         a.nimg = ch.nimg;
+        a.bf16_out = c.precision == TG_BF16_TC;
         KernelTimer kt(x, d, 1, cs);
         CK(launch_cnn_u1(a, cs));
         kt.done(cs);

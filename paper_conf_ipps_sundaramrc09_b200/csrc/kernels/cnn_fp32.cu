@@ -90,6 +90,7 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
     }
     float* t2 = a.t2 + img * a.t2_img_stride;
     const int64_t plane = a.t2_rows * a.w2;
+    float tv[8];
 #pragma unroll
     for (int ch = 0; ch < 8; ++ch) {
         float s = 0.f;
@@ -101,7 +102,19 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
             const float t = tanh_f(acc[ch][p] + b);
             s = fmaf(w.p2[ch][p], t, s);
         }
-        t2[ch * plane + (R2 - a.t2_row0) * a.w2 + C2] = tanh_f(s);
+        tv[ch] = tanh_f(s);
+    }
+    if (a.bf16_out) {  // one 16-byte pixel of 8 bf16 channels (the tensor-core U2's operand rows)
+        uint4* d = reinterpret_cast<uint4*>(a.t2) + (img * a.t2_rows + (R2 - a.t2_row0)) * a.w2 + C2;
+        uint32_t p[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            asm("cvt.rn.bf16x2.f32 %0, %1, %2;\n" : "=r"(p[k]) : "f"(tv[2 * k + 1]), "f"(tv[2 * k]));
+        }
+        *d = make_uint4(p[0], p[1], p[2], p[3]);
+    } else {
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch) t2[ch * plane + (R2 - a.t2_row0) * a.w2 + C2] = tv[ch];
     }
 }
 

@@ -69,18 +69,13 @@ __global__ void __launch_bounds__(kThreads) cnn_u2_tc_kernel(const CnnU2Args a) 
         tc::mbar_init(&S.mbar, 1);
         tc::mbar_fence_init();
     }
-    // stage the T2 window as bf16 [row][col][ci]
-    const float* t2b = a.t2 + img * a.t2_img_stride;
-    const int64_t plane = a.t2_rows * a.w2;
+    // stage the T2 window: U1 wrote T2 as bf16 pixels [row][col][8 ch] = one 16-byte load each
+    const uint4* t2b = reinterpret_cast<const uint4*>(a.t2) + img * a.t2_rows * a.w2;
     for (int idx = tid; idx < U2_WR * U2_WP; idx += kThreads) {
         const int r = idx / U2_WP, c = idx - r * U2_WP;
         const int64_t br = 2 * R + r - a.t2_row0, gc = c0 + c;
-        float v[8];
         const bool ok = br >= 0 && br < a.t2_rows && gc < a.w2;
-#pragma unroll
-        for (int ci = 0; ci < 8; ++ci) v[ci] = ok ? t2b[ci * plane + br * a.w2 + gc] : 0.f;
-        S.a[idx] = make_uint4(tc::pack_bf16(v[0], v[1]), tc::pack_bf16(v[2], v[3]), tc::pack_bf16(v[4], v[5]),
-                              tc::pack_bf16(v[6], v[7]));
+        S.a[idx] = ok ? __ldg(t2b + br * a.w2 + gc) : make_uint4(0u, 0u, 0u, 0u);
     }
     const uint4* kb = reinterpret_cast<const uint4*>(a.k3_tc);
     for (int idx = tid; idx < U2_KS * 2 * U2_N; idx += kThreads) S.b[idx] = __ldg(kb + idx);
@@ -117,8 +112,7 @@ __global__ void __launch_bounds__(kThreads) cnn_u2_tc_kernel(const CnnU2Args a) 
     const int64_t C = c >> 1;                 // T4 column
     const bool row_ok = R < a.t4_row0 + a.t4_rows;
     const bool col_ok = c < a.w3;
-    float* t4 = a.t4 + img * a.t4_img_stride;
-    const int64_t oplane = a.t4_rows * a.w4;
+    float tv[20];
 #pragma unroll
     for (int co = 0; co < 20; ++co) {
         float t0 = 0.f, t1 = 0.f;
@@ -141,8 +135,18 @@ __global__ void __launch_bounds__(kThreads) cnn_u2_tc_kernel(const CnnU2Args a) 
             s = fmaf(S.p4[co][1], t01, s);
             s = fmaf(S.p4[co][2], t1, s);
             s = fmaf(S.p4[co][3], t11, s);
-            t4[co * oplane + (R - a.t4_row0) * a.w4 + C] = tanh_f(s);
+            tv[co] = tanh_f(s);
         }
+    }
+    if (row_ok && !(lane & 1) && C < a.w4) {
+        // T4 as bf16 channel blocks [3][rows][w4][8] (U3's tensor-core operand rows)
+        const int64_t bplane = a.t4_rows * a.w4;
+        uint4* t4 = reinterpret_cast<uint4*>(a.t4) + img * 3 * bplane + (R - a.t4_row0) * a.w4 + C;
+        t4[0] = make_uint4(tc::pack_bf16(tv[0], tv[1]), tc::pack_bf16(tv[2], tv[3]), tc::pack_bf16(tv[4], tv[5]),
+                           tc::pack_bf16(tv[6], tv[7]));
+        t4[bplane] = make_uint4(tc::pack_bf16(tv[8], tv[9]), tc::pack_bf16(tv[10], tv[11]),
+                                tc::pack_bf16(tv[12], tv[13]), tc::pack_bf16(tv[14], tv[15]));
+        t4[2 * bplane] = make_uint4(tc::pack_bf16(tv[16], tv[17]), tc::pack_bf16(tv[18], tv[19]), 0u, 0u);
     }
     tc::fence_before_sync();
     __syncthreads();
@@ -169,7 +173,9 @@ struct U3TcShared {
     uint32_t tmem;
 };
 
-__global__ void __launch_bounds__(kThreads, 2) cnn_u3_tc_kernel(const CnnU3Args a) {
+constexpr int kThreadsU3 = 256;  // 8 warps: warps 0-3 drain tile 0, warps 4-7 tile 1
+
+__global__ void __launch_bounds__(kThreadsU3, 2) cnn_u3_tc_kernel(const CnnU3Args a) {
     extern __shared__ __align__(128) uint8_t smraw[];
     U3TcShared& S = *reinterpret_cast<U3TcShared*>(smraw);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -204,29 +210,27 @@ __global__ void __launch_bounds__(kThreads, 2) cnn_u3_tc_kernel(const CnnU3Args 
         tc::mbar_fence_init();
     }
     // ---- stage the T4 window as bf16 [block][row][col][8]
-    const float* t4b = a.t4 + img * a.t4_img_stride;
-    const int64_t plane = a.t4_rows * a.w4;
+    // U2 wrote T4 as bf16 channel blocks [3][rows][w4][8]: three 16-byte loads per pixel
+    const int64_t bplane = a.t4_rows * a.w4;
+    const uint4* t4b = reinterpret_cast<const uint4*>(a.t4) + img * 3 * bplane;
     const int64_t wc0 = flat ? 0 : q0;
-    for (int idx = tid; idx < plane_px; idx += kThreads) {
+    for (int idx = tid; idx < plane_px; idx += kThreadsU3) {
         const int r = idx / WP, c = idx - r * WP;
         const int64_t br = wr0 + r - a.t4_row0, gc = wc0 + c;
         const bool ok = idx < WR * WP && br >= 0 && br < a.t4_rows && gc < a.w4;
-        float v[20];
-#pragma unroll
-        for (int ci = 0; ci < 20; ++ci) v[ci] = ok ? t4b[ci * plane + br * a.w4 + gc] : 0.f;
-        S.a[0][idx] = make_uint4(tc::pack_bf16(v[0], v[1]), tc::pack_bf16(v[2], v[3]), tc::pack_bf16(v[4], v[5]),
-                                 tc::pack_bf16(v[6], v[7]));
-        S.a[1][idx] = make_uint4(tc::pack_bf16(v[8], v[9]), tc::pack_bf16(v[10], v[11]),
-                                 tc::pack_bf16(v[12], v[13]), tc::pack_bf16(v[14], v[15]));
-        S.a[2][idx] = make_uint4(tc::pack_bf16(v[16], v[17]), tc::pack_bf16(v[18], v[19]), 0u, 0u);
+        const int64_t o = br * a.w4 + gc;
+        const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+        S.a[0][idx] = ok ? __ldg(t4b + o) : z;
+        S.a[1][idx] = ok ? __ldg(t4b + bplane + o) : z;
+        S.a[2][idx] = ok ? __ldg(t4b + 2 * bplane + o) : z;
     }
-    for (int idx = tid; idx < U3_NMAX * 9; idx += kThreads) {
+    for (int idx = tid; idx < U3_NMAX * 9; idx += kThreadsU3) {
         const int ch = idx / 9, o = idx - ch * 9;
         S.k6[ch][o] = ch < a.n5 ? __ldg(a.k6 + o * a.n5 + ch) : 0.f;
     }
     const uint4* kb = reinterpret_cast<const uint4*>(a.k5_tc);
     const int stage_vec = U3_KS_STAGE * 2 * NP;  // uint4 per stage
-    for (int idx = tid; idx < stage_vec; idx += kThreads) S.b[0][idx] = __ldg(kb + idx);
+    for (int idx = tid; idx < stage_vec; idx += kThreadsU3) S.b[0][idx] = __ldg(kb + idx);
     tc::fence_proxy_async();
     tc::fence_before_sync();
     __syncthreads();
@@ -265,7 +269,7 @@ __global__ void __launch_bounds__(kThreads, 2) cnn_u3_tc_kernel(const CnnU3Args 
             // buffer (st+1)&1 was read by stage st-1: wait for its MMAs before overwriting
             if (st >= 1) tc::mbar_wait(&S.mbar[(st + 1) & 1], (uint32_t)(((st - 1) >> 1) & 1));
             const uint4* src = kb + (size_t)(st + 1) * stage_vec;
-            for (int idx = tid; idx < stage_vec; idx += kThreads) S.b[(st + 1) & 1][idx] = __ldg(src + idx);
+            for (int idx = tid; idx < stage_vec; idx += kThreadsU3) S.b[(st + 1) & 1][idx] = __ldg(src + idx);
             tc::fence_proxy_async();
             tc::fence_before_sync();
             __syncthreads();
@@ -275,10 +279,11 @@ __global__ void __launch_bounds__(kThreads, 2) cnn_u3_tc_kernel(const CnnU3Args 
     tc::mbar_wait(&S.mbar[(kStages - 1) & 1], (uint32_t)(((kStages - 1) >> 1) & 1));
     tc::fence_after_sync();
 
-    // ---- epilogue: thread = position 32*warp + lane of tile t
-    const uint32_t lane_base = (uint32_t)(32 * warp) << 16;
-    for (int t = 0; t < 2; ++t) {
-        const int m = t * kTileM + 32 * warp + lane;
+    // ---- epilogue: warp w drains tile w/4, TMEM lanes 32*(w%4).. (its lane quarter)
+    const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
+    {
+        const int t = warp >> 2;
+        const int m = t * kTileM + 32 * (warp & 3) + lane;
         int64_t orow, ocol;
         if (flat) {
             const int64_t q = q0 + m;
@@ -408,7 +413,7 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     else
         bands = (unsigned)(a.out_rows * ((a.w5 + 2 * kTileM - 1) / (2 * kTileM)));
     dim3 grid(bands, 1, (unsigned)a.nimg);
-    cnn_u3_tc_kernel<<<grid, kThreads, smem, s>>>(a);
+    cnn_u3_tc_kernel<<<grid, kThreadsU3, smem, s>>>(a);
     return cudaGetLastError();
 }
 

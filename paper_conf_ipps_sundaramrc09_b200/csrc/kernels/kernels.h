@@ -35,6 +35,7 @@ struct CnnU1Args {          // C1(1->8, 5x5) + bias + tanh + S2 + tanh  -> T2
     float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows;  // [8][t2_rows][w2]
     int64_t w1, w2;
     int64_t nimg;
+    int bf16_out;           // 1: write T2 as bf16 [rows][w2][8] (operand layout of U2 on tcgen05)
 };
 struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
     const float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows; int64_t w2;
@@ -43,7 +44,8 @@ struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
     const float* p4_host;   // [20][4] (host)
     float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w3, w4;
     int64_t nimg;
-    int bf16_tc;            // 1: tcgen05 bf16 path
+    int bf16_tc;            // 1: tcgen05 bf16 path: T2 read as bf16 [rows][w2][8], T4 written
+                            //    as bf16 [3][rows][w4][8] (channel blocks 0-7, 8-15, 16-19+pad)
     const uint16_t* k3_tc;  // bf16 B operand prepared by cnn_prepare_k3_tc (device)
     const float* p4_dev;    // [20][4] (device)
 };
@@ -56,7 +58,7 @@ struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + 
     float* out; int64_t out_img_stride; int64_t out_plane_stride; int64_t out_row0, out_rows; int64_t w5;
     int n5;
     int64_t nimg;
-    int bf16_tc;
+    int bf16_tc;            // 1: tcgen05 path, T4 read as bf16 [3][rows][w4][8]
     const uint16_t* k5_tc;  // bf16 B operand prepared by cnn_prepare_k5_tc (device)
     int n_pad;              // n5 rounded up to a multiple of 16
 };
