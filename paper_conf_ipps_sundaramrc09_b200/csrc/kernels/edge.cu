@@ -12,15 +12,25 @@
 // FFMA back to back: each thread owns a 1 x 16 strip of outputs for both filters
 // (32 accumulators), and for each of the 16 filter rows loads its 32-wide input window
 // with 8 conflict-free LDS.128 and both filter rows from the constant bank (uniform
-// registers), then issues 512 FFMA -- under 3% load overhead. Tiles of 64 x 64 outputs, 256 threads; lanes of a warp own
-// 32 consecutive rows (row pitch 84 floats = 21 x 16 B, odd, so the 8 lanes of each LDS.128
-// phase hit 8 distinct 16-byte bank groups). The input tile (79 x 80 floats incl. the
-// 15-row/col halo) is staged once per CTA with 128-bit coalesced loads; zero fill gives
-// the SAME padding at image borders.
+// registers), then issues 512 FFMA -- under 3% load overhead. Tiles of 64 x 64 outputs,
+// 256 threads; lanes of a warp own 32 consecutive rows (row pitch 84 floats = 21 x 16 B,
+// odd, so the 8 lanes of each LDS.128 phase hit 8 distinct 16-byte bank groups).
+//
+// Tile staging. Main path (W % 4 == 0): a persistent grid (2 CTAs per SM) walks the tiles;
+// one thread issues a 3-D TMA load (cp.async.bulk.tensor, box 84 x 79 x 1) of the NEXT
+// tile into the other shared-memory buffer while the CTA computes the current one, and the
+// TMA's out-of-bounds zero fill is exactly the SAME padding at image borders. Fallback
+// (any W): each CTA stages its tile with bounds-checked 128-bit loads.
 //
 // Bit-exactness under splitting: every output pixel is the same sequence of fmaf in the
 // same order (filter row i, then column j) whatever tile or chunk it falls in.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <mutex>
 
 #include "kernels.h"
 
@@ -30,9 +40,11 @@ namespace {
 constexpr int kTileR = 64;
 constexpr int kTileC = 64;
 constexpr int kSmR = kTileR + 15;  // 79 rows incl. halo
-constexpr int kSmC = kTileC + 16;  // 80 cols: [c0-8, c0+72)
+constexpr int kSmC = kTileC + 16;  // 80 cols used: [c0-8, c0+72)
 constexpr int kPitch = 84;         // floats; 84/4 = 21 (odd) -> conflict-free LDS.128 across rows
 constexpr int kThreads = 256;
+constexpr int kTileBytes = kSmR * kPitch * 4;  // one TMA box (84 x 79 floats)
+constexpr int kBufStride = (kTileBytes + 127) / 128 * 128;
 
 // Both filters, embedded in 16 x 16 frames, travel as a __grid_constant__ kernel parameter:
 // the weights then sit in the constant bank and every FFMA reads them through a uniform
@@ -43,40 +55,11 @@ struct EdgeWeights {
     float w2[256];
 };
 
-__global__ void __launch_bounds__(kThreads, 2)
-    edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
-    __shared__ __align__(16) float xs[kSmR * kPitch];
-
+// Compute the 64 x 64 output tile whose input (+halo) is staged at xs (pitch kPitch, smem
+// (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)) and store it.
+__device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const EdgeArgs& a, const EdgeWeights& wt,
+                                          int64_t img, int64_t tile_r0, int64_t tile_c0) {
     const int tid = threadIdx.x;
-    const int64_t img = blockIdx.z;
-    const int64_t tile_r0 = a.out_row0 + (int64_t)blockIdx.y * kTileR;  // global output row
-    const int64_t tile_c0 = (int64_t)blockIdx.x * kTileC;
-
-    // stage the input tile: smem (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)
-    const float* __restrict__ inb = a.in + img * a.in_img_stride;
-    const bool vec = (a.W & 3) == 0 && ((reinterpret_cast<uintptr_t>(a.in) & 15) == 0) &&
-                     (a.in_img_stride & 3) == 0;
-    for (int idx = tid; idx < kSmR * (kSmC / 4); idx += kThreads) {
-        const int sr = idx / (kSmC / 4);
-        const int q = idx - sr * (kSmC / 4);
-        const int64_t g = tile_r0 - 7 + sr;
-        const int64_t gc = tile_c0 - 8 + 4 * q;
-        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (g >= 0 && g < a.H && g >= a.in_row0 && g < a.in_row0 + a.in_rows) {
-            const float* row = inb + (g - a.in_row0) * a.W;
-            if (vec && gc >= 0 && gc + 3 < a.W) {
-                v = __ldg(reinterpret_cast<const float4*>(row + gc));
-            } else {
-                v.x = (gc + 0 >= 0 && gc + 0 < a.W) ? __ldg(row + gc + 0) : 0.f;
-                v.y = (gc + 1 >= 0 && gc + 1 < a.W) ? __ldg(row + gc + 1) : 0.f;
-                v.z = (gc + 2 >= 0 && gc + 2 < a.W) ? __ldg(row + gc + 2) : 0.f;
-                v.w = (gc + 3 >= 0 && gc + 3 < a.W) ? __ldg(row + gc + 3) : 0.f;
-            }
-        }
-        *reinterpret_cast<float4*>(&xs[sr * kPitch + 4 * q]) = v;
-    }
-    __syncthreads();
-
     const int warp = tid >> 5, lane = tid & 31;
     const int lr = (warp >> 2) * 32 + lane;  // local output row
     const int cb = (warp & 3) * 16;          // local output column base
@@ -143,13 +126,123 @@ __global__ void __launch_bounds__(kThreads, 2)
     }
 }
 
+// ---------------------------------------------------------------------------- fallback
+__global__ void __launch_bounds__(kThreads, 2)
+    edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
+    __shared__ __align__(16) float xs[kSmR * kPitch];
+    const int tid = threadIdx.x;
+    const int64_t img = blockIdx.z;
+    const int64_t tile_r0 = a.out_row0 + (int64_t)blockIdx.y * kTileR;  // global output row
+    const int64_t tile_c0 = (int64_t)blockIdx.x * kTileC;
+    const float* __restrict__ inb = a.in + img * a.in_img_stride;
+    const bool vec = (a.W & 3) == 0 && ((reinterpret_cast<uintptr_t>(a.in) & 15) == 0) &&
+                     (a.in_img_stride & 3) == 0;
+    for (int idx = tid; idx < kSmR * (kSmC / 4); idx += kThreads) {
+        const int sr = idx / (kSmC / 4);
+        const int q = idx - sr * (kSmC / 4);
+        const int64_t g = tile_r0 - 7 + sr;
+        const int64_t gc = tile_c0 - 8 + 4 * q;
+        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (g >= 0 && g < a.H && g >= a.in_row0 && g < a.in_row0 + a.in_rows) {
+            const float* row = inb + (g - a.in_row0) * a.W;
+            if (vec && gc >= 0 && gc + 3 < a.W) {
+                v = __ldg(reinterpret_cast<const float4*>(row + gc));
+            } else {
+                v.x = (gc + 0 >= 0 && gc + 0 < a.W) ? __ldg(row + gc + 0) : 0.f;
+                v.y = (gc + 1 >= 0 && gc + 1 < a.W) ? __ldg(row + gc + 1) : 0.f;
+                v.z = (gc + 2 >= 0 && gc + 2 < a.W) ? __ldg(row + gc + 2) : 0.f;
+                v.w = (gc + 3 >= 0 && gc + 3 < a.W) ? __ldg(row + gc + 3) : 0.f;
+            }
+        }
+        *reinterpret_cast<float4*>(&xs[sr * kPitch + 4 * q]) = v;
+    }
+    __syncthreads();
+    edge_tile(xs, a, wt, img, tile_r0, tile_c0);
+}
+
+// ---------------------------------------------------------------------------- TMA path
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__global__ void __launch_bounds__(kThreads, 2)
+    edge_fused_tma_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt,
+                          const __grid_constant__ CUtensorMap tmap, const int tiles_c, const int tiles_r,
+                          const int64_t ntiles) {
+    extern __shared__ __align__(128) uint8_t smraw[];
+    // two tile buffers at 128-byte aligned shared-memory addresses
+    uint8_t* base = smraw + ((128 - (smem_u32(smraw) & 127)) & 127);
+    float* buf0 = reinterpret_cast<float*>(base);
+    float* buf1 = reinterpret_cast<float*>(base + kBufStride);
+    __shared__ __align__(8) uint64_t full[2];
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(&full[0])) : "memory");
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(&full[1])) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+    auto coords = [&](int64_t t, int64_t& img, int64_t& tr0, int64_t& tc0) {
+        const int64_t per_img = (int64_t)tiles_c * tiles_r;
+        img = t / per_img;
+        const int64_t rem = t - img * per_img;
+        const int64_t ty = rem / tiles_c;
+        tr0 = a.out_row0 + ty * kTileR;
+        tc0 = (rem - ty * tiles_c) * kTileC;
+    };
+    auto issue = [&](int64_t t, int b) {
+        int64_t img, tr0, tc0;
+        coords(t, img, tr0, tc0);
+        // box origin: image col tc0 - 8, buffer row (tr0 - 7) - in_row0 (out-of-range -> zeros)
+        const int x = (int)(tc0 - 8), y = (int)(tr0 - 7 - a.in_row0), z = (int)img;
+        float* dst = b ? buf1 : buf0;
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(&full[b])),
+                     "r"(kTileBytes)
+                     : "memory");
+        asm volatile(
+            "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+            "[%5];\n" ::"r"(smem_u32(dst)),
+            "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(x), "r"(y), "r"(z), "r"(smem_u32(&full[b]))
+            : "memory");
+    };
+    int64_t t = blockIdx.x;
+    if (tid == 0 && t < ntiles) issue(t, 0);
+    for (int k = 0; t < ntiles; ++k, t += gridDim.x) {
+        const int b = k & 1;
+        if (tid == 0 && t + gridDim.x < ntiles) issue(t + gridDim.x, b ^ 1);  // prefetch the next tile
+        const uint32_t parity = (uint32_t)((k >> 1) & 1);
+        asm volatile(
+            "{\n\t.reg .pred done;\n\t"
+            "WAIT_%=:\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 done, [%0], %1;\n\t"
+            "@!done bra WAIT_%=;\n\t}\n" ::"r"(smem_u32(&full[b])),
+            "r"(parity)
+            : "memory");
+        int64_t img, tr0, tc0;
+        coords(t, img, tr0, tc0);
+        edge_tile(b ? buf1 : buf0, a, wt, img, tr0, tc0);
+        __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
+    }
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    });
+    return fn;
+}
+
 }  // namespace
 
 cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
-    dim3 grid((unsigned)((a.W + kTileC - 1) / kTileC), (unsigned)((a.out_rows + kTileR - 1) / kTileR),
-              (unsigned)a.nimg);
-    if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
     // filters embedded in a 16 x 16 frame at offset 7 - (ks-1)/2 (zeros elsewhere)
     EdgeWeights wt{};
     const int off = 7 - (a.ks - 1) / 2;
@@ -158,6 +251,40 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
             wt.w1[(r + off) * 16 + c + off] = a.k1_host[r * a.ks + c];
             wt.w2[(r + off) * 16 + c + off] = a.k2_host[r * a.ks + c];
         }
+    const int tiles_c = (int)((a.W + kTileC - 1) / kTileC);
+    const int tiles_r = (int)((a.out_rows + kTileR - 1) / kTileR);
+    PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
+    const bool tma_ok = enc && (a.W & 3) == 0 && (reinterpret_cast<uintptr_t>(a.in) & 15) == 0 &&
+                        a.in_img_stride == a.in_rows * a.W && a.in_rows < (1ll << 31) && a.W < (1ll << 31);
+    if (tma_ok) {
+        CUtensorMap tmap;
+        const cuuint64_t gdim[3] = {(cuuint64_t)a.W, (cuuint64_t)a.in_rows, (cuuint64_t)a.nimg};
+        const cuuint64_t gstride[2] = {(cuuint64_t)a.W * 4, (cuuint64_t)a.in_rows * a.W * 4};
+        const cuuint32_t box[3] = {(cuuint32_t)kPitch, (cuuint32_t)kSmR, 1};
+        const cuuint32_t estride[3] = {1, 1, 1};
+        CUresult r = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(a.in), gdim, gstride, box, estride,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r == CUDA_SUCCESS) {
+            static std::atomic<uint32_t> configured{0};
+            int dev = 0, sms = 148;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            const size_t smem = 2 * (size_t)kBufStride + 128;
+            if (!(configured.load() & (1u << (dev & 31)))) {
+                cudaError_t e =
+                    cudaFuncSetAttribute(edge_fused_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                if (e != cudaSuccess) return e;
+                configured.fetch_or(1u << (dev & 31));
+            }
+            const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
+            const int64_t grid = std::min<int64_t>(ntiles, 2 * (int64_t)sms);
+            edge_fused_tma_kernel<<<(unsigned)grid, kThreads, smem, s>>>(a, wt, tmap, tiles_c, tiles_r, ntiles);
+            return cudaGetLastError();
+        }
+    }
+    dim3 grid((unsigned)tiles_c, (unsigned)tiles_r, (unsigned)a.nimg);
+    if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
     edge_fused_kernel<<<grid, kThreads, 0, s>>>(a, wt);
     return cudaGetLastError();
 }
