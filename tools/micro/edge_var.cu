@@ -197,9 +197,8 @@ __global__ void __launch_bounds__(kThreads, 2)
     extern __shared__ __align__(128) uint8_t smraw[];
     // two tile buffers at 128-byte aligned shared-memory addresses
     uint8_t* base = smraw + ((128 - (smem_u32(smraw) & 127)) & 127);
-    float* buf0 = reinterpret_cast<float*>(base);                   // TMA stage 0
-    float* buf1 = reinterpret_cast<float*>(base + kBufStride);      // TMA stage 1
-    float* xs1 = reinterpret_cast<float*>(base + 2 * kBufStride);   // current tile shifted by one column
+    float* buf0 = reinterpret_cast<float*>(base);                   // stage 0: tile, shifted tile
+    float* buf1 = reinterpret_cast<float*>(base + 2 * kBufStride);  // stage 1
     __shared__ __align__(8) uint64_t full[2];
     const int tid = threadIdx.x;
     if (tid == 0) {
@@ -224,15 +223,13 @@ __global__ void __launch_bounds__(kThreads, 2)
         const int x = (int)(tc0 - 8), y = (int)(tr0 - 7 - a.in_row0), z = (int)img;
         float* dst = b ? buf1 : buf0;
         asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(&full[b])),
-                     "r"(kTileBytes)
+                     "r"(2 * kTileBytes)
                      : "memory");
-        // (TMA box origins must be 16-byte aligned, so the one-column shift for the FFMA2
-        // pairs is made in shared memory after the tile lands)
-        for (int h = 0; h < 1; ++h)
+        for (int h = 0; h < 2; ++h)  // the tile, and the tile one column to the right (xs1)
             asm volatile(
                 "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, "
                 "%4}], [%5];\n" ::"r"(smem_u32(dst) + (uint32_t)(h * kBufStride)),
-                "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(x), "r"(y), "r"(z), "r"(smem_u32(&full[b]))
+                "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(x + 4 * h), "r"(y), "r"(z), "r"(smem_u32(&full[b]))
                 : "memory");
     };
     int64_t t = blockIdx.x;
@@ -251,15 +248,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         int64_t img, tr0, tc0;
         coords(t, img, tr0, tc0);
         const float* tb = b ? buf1 : buf0;
-        // xs1[r][c] = tb[r][c+1] (128-bit loads/stores; column 79 of a row is never read)
-        for (int idx = threadIdx.x; idx < kSmR * (kSmC / 4); idx += kThreads) {
-            const int sr = idx / (kSmC / 4), q = idx - sr * (kSmC / 4);
-            const float4 lo = *reinterpret_cast<const float4*>(&tb[sr * kPitch + 4 * q]);
-            const float4 hi = *reinterpret_cast<const float4*>(&tb[sr * kPitch + 4 * q + 4]);
-            *reinterpret_cast<float4*>(&xs1[sr * kPitch + 4 * q]) = make_float4(lo.y, lo.z, lo.w, hi.x);
-        }
-        __syncthreads();
-        edge_tile(tb, xs1, a, wt, img, tr0, tc0);
+        edge_tile(tb, tb + kBufStride / 4, a, wt, img, tr0, tc0);
         __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
     }
 }
@@ -308,7 +297,7 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
             int dev = 0, sms = 148;
             cudaGetDevice(&dev);
             cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            const size_t smem = 3 * (size_t)kBufStride + 128;
+            const size_t smem = 4 * (size_t)kBufStride + 128;
             if (!(configured.load() & (1u << (dev & 31)))) {
                 cudaError_t e =
                     cudaFuncSetAttribute(edge_fused_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
