@@ -205,6 +205,33 @@ tg_status tg_plan_invalidate_params(tg_plan* plan);
 int64_t tg_plan_launch_count(const tg_plan* plan);
 
 void tg_plan_destroy(tg_plan* plan);
+
+/* ------------------------------------------------------------------ transfer scheduling */
+/* The paper's heuristic offload/transfer scheduler (Section 3.3.1) over an
+ * abstract operator graph whose data structures have sizes in any unit (floats, bytes, or
+ * the "units" of Fig. 3). Pure host code. */
+typedef struct tg_sched tg_sched;
+#define TG_DS_INPUT 0   /* template input: starts valid on the host                      */
+#define TG_DS_PARAM 1   /* parameter: starts valid on the host                           */
+#define TG_DS_TEMP 2    /* intermediate: produced by an operator                         */
+#define TG_DS_OUTPUT 3  /* template output: must end on the host (PB constraint (13))    */
+tg_status tg_sched_create(tg_sched** s);
+void tg_sched_destroy(tg_sched* s);
+tg_status tg_sched_add_ds(tg_sched* s, uint64_t size, int32_t kind, int32_t* id);
+/* An operator reading ins[0..nin) and writing outs[0..nout) (DS ids). */
+tg_status tg_sched_add_op(tg_sched* s, const int32_t* ins, int32_t nin, const int32_t* outs, int32_t nout,
+                          int32_t* id);
+/* Depth-first operator schedule: order[0..n_ops) receives operator ids.
+ * Children are consumers in insertion order, start nodes in id order (R11). */
+tg_status tg_sched_dfs_order(const tg_sched* s, int32_t* order);
+/* "Latest time of use" transfer schedule for a given operator order (read
+ * as next use, R10) within `capacity`: *moved = total size copied host<->GPU.
+ * If trace != NULL it receives (kind, id) pairs -- kind 0 = copy DS id to the GPU, 1 = run
+ * operator id, 2 = copy DS id to the host; trace_cap counts pairs; *trace_len = pairs used.
+ * TG_E_INFEASIBLE if an operator's inputs and outputs do not fit together. */
+tg_status tg_sched_transfers(const tg_sched* s, const int32_t* order, uint64_t capacity, uint64_t* moved,
+                             int32_t* trace, int64_t trace_cap, int64_t* trace_len);
+
 const char* tg_last_error(void);
 /* Library version string, e.g. "tg 0.1 sm_100a". */
 const char* tg_version(void);

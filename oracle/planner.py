@@ -340,7 +340,7 @@ def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None) ->
         for j in list(on_gpu):
             if next_use(j, t) == math.inf and j not in outputs:
                 del on_gpu[j]
-    for j in list(on_gpu):
+    for j in sorted(on_gpu):          # outputs still on the GPU go to the host, in id order
         if j in outputs and on_gpu[j]:
             moved += g.ds[j].size
             if trace is not None:

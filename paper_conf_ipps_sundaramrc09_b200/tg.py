@@ -105,6 +105,12 @@ _PROTOS = {
     "tg_plan_launch_count": (c_i64, [vp]),
     "tg_plan_invalidate_params": (c_i32, [vp]),
     "tg_plan_destroy": (None, [vp]),
+    "tg_sched_create": (c_i32, [ctypes.POINTER(vp)]),
+    "tg_sched_destroy": (None, [vp]),
+    "tg_sched_add_ds": (c_i32, [vp, c_u64, c_i32, P_id]),
+    "tg_sched_add_op": (c_i32, [vp, P_id, c_i32, P_id, c_i32, P_id]),
+    "tg_sched_dfs_order": (c_i32, [vp, P_id]),
+    "tg_sched_transfers": (c_i32, [vp, P_id, c_u64, ctypes.POINTER(c_u64), P_id, c_i64, ctypes.POINTER(c_i64)]),
     "tg_last_error": (ctypes.c_char_p, []),
     "tg_version": (ctypes.c_char_p, []),
 }
@@ -296,6 +302,49 @@ def tg_plan_invalidate_params(p) -> None:
 
 def tg_plan_destroy(p) -> None:
     _lib.tg_plan_destroy(p)
+
+
+TG_DS_INPUT, TG_DS_PARAM, TG_DS_TEMP, TG_DS_OUTPUT = 0, 1, 2, 3
+
+
+class Sched:
+    """The paper's DFS + latest-time-of-use scheduler (tg_sched_*) over an abstract graph."""
+
+    def __init__(self):
+        h = vp()
+        _ck(_lib.tg_sched_create(ctypes.byref(h)))
+        self.h = h.value
+        self.n_ops = 0
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            _lib.tg_sched_destroy(self.h)
+            self.h = None
+
+    def add_ds(self, size: int, kind: int) -> int:
+        return _id_call(_lib.tg_sched_add_ds, self.h, int(size), int(kind))
+
+    def add_op(self, ins: Sequence[int], outs: Sequence[int]) -> int:
+        a = (c_i32 * max(1, len(ins)))(*ins)
+        b = (c_i32 * max(1, len(outs)))(*outs)
+        self.n_ops += 1
+        return _id_call(_lib.tg_sched_add_op, self.h, a, len(ins), b, len(outs))
+
+    def dfs_order(self) -> list[int]:
+        o = (c_i32 * max(1, self.n_ops))()
+        _ck(_lib.tg_sched_dfs_order(self.h, o))
+        return list(o)[: self.n_ops]
+
+    def transfers(self, order: Sequence[int], capacity: int, trace: bool = False):
+        o = (c_i32 * max(1, len(order)))(*order)
+        moved = c_u64()
+        n = c_i64()
+        _ck(_lib.tg_sched_transfers(self.h, o, int(capacity), ctypes.byref(moved), None, 0, ctypes.byref(n)))
+        if not trace:
+            return moved.value
+        buf = (c_i32 * (2 * max(1, n.value)))()
+        _ck(_lib.tg_sched_transfers(self.h, o, int(capacity), ctypes.byref(moved), buf, n.value, ctypes.byref(n)))
+        return moved.value, [(buf[2 * i], buf[2 * i + 1]) for i in range(n.value)]
 
 
 def tg_version() -> str:

@@ -1,0 +1,89 @@
+"""The library's scheduler (csrc/sched.cpp, tg_sched_*) against the planner oracle
+(oracle/planner.py): Fig. 3 schedule (a) = 15 and (b) = 8 transfer units (PAPER.md:229,
+299), the Fig. 6 trace, the DFS order, and random DAGs
+(transfer volume and full trace bit-exact)."""
+import json
+import os
+import random
+
+import pytest
+
+from conftest import GOLDEN
+from oracle import planner as P
+
+KIND = {"input": 0, "param": 1, "temp": 2, "output": 3}
+
+
+def to_sched(g):
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    s = tg.Sched()
+    for d in g.ds:
+        s.add_ds(d.size, KIND[d.kind])
+    for op in g.ops:
+        s.add_op(op.ins, op.outs)
+    return s
+
+
+def oracle_trace(g, order, cap):
+    tr = []
+    moved = P.simulate_transfers(g, order, cap, tr)
+    names_ds = {d.name: i for i, d in enumerate(g.ds)}
+    names_op = {o.name: i for i, o in enumerate(g.ops)}
+    kind = {"h2d": 0, "run": 1, "d2h": 2}
+    return moved, [(kind[k], names_op[n] if k == "run" else names_ds[n]) for k, n in tr]
+
+
+def test_fig3_and_fig6():
+    gold = json.load(open(os.path.join(GOLDEN, "schedules.json")))
+    g, ops = P.fig3_graph()
+    s = to_sched(g)
+    for key in ("a", "b"):
+        order = [ops[n] for n in gold["fig3"][key]["order"]]
+        assert s.transfers(order, gold["fig3"]["capacity"]) == gold["fig3"][key]["units"]
+    order = [ops[n] for n in gold["fig3"]["b"]["order"]]
+    moved, tr = s.transfers(order, 5, trace=True)
+    assert (moved, tr) == oracle_trace(g, order, 5)
+    assert s.dfs_order() == P.dfs_order(g)
+
+
+def random_dag(rng, n_ops):
+    g = P.Graph()
+    inputs = [g.add_ds(f"in{i}", rng.randint(1, 4), "input") for i in range(rng.randint(1, 3))]
+    avail = list(inputs)
+    for i in range(n_ops):
+        ins = rng.sample(avail, min(len(avail), rng.randint(1, 3)))
+        outs = [g.add_ds(f"t{i}_{k}", rng.randint(1, 4)) for k in range(rng.randint(1, 2))]
+        g.add_op(f"op{i}", ins, outs)
+        avail.extend(outs)
+    # DS never read become outputs
+    read = {j for op in g.ops for j in op.ins}
+    for j, d in enumerate(g.ds):
+        if d.kind == "temp" and j not in read:
+            d.kind = "output"
+    return g
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_random_dags_bit_exact(seed):
+    rng = random.Random(seed)
+    g = random_dag(rng, rng.randint(3, 12))
+    s = to_sched(g)
+    order = P.dfs_order(g)
+    assert s.dfs_order() == order
+    need = max(P.Graph.req(g, op) for op in g.ops)
+    for cap in (need, need + 2, need + 5, 10 ** 6):
+        assert s.transfers(order, cap, trace=True) == oracle_trace(g, order, cap)
+    topo = list(P.topological_orders(g)) if len(g.ops) <= 7 else [order]
+    for o in topo[:20]:
+        assert s.transfers(o, need + 1) == P.simulate_transfers(g, o, need + 1)
+
+
+def test_infeasible_and_errors():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    g, ops = P.fig3_graph()
+    s = to_sched(g)
+    with pytest.raises(tg.TGError) as e:
+        s.transfers(P.dfs_order(g), 3)      # max needs 5 units at once
+    assert e.value.code == tg.TG_E_INFEASIBLE
+    with pytest.raises(tg.TGError):
+        s.transfers([0, 0, 1, 2, 3, 4, 5, 6], 5)
