@@ -73,8 +73,11 @@ typedef int32_t tg_id;
 #define TG_BF16_TC 1      /* CNN C3/C5/C6 on tcgen05 tensor cores, bf16 operands, fp32
                              accumulation; parity 2e-2 normwise                           */
 #define TG_FUSED 0        /* offload units = fused templates (edge: 1 unit; CNN: 3)       */
-#define TG_PER_OP 1       /* paper mode: one operator per offload unit (not this round)   */
-#define TG_BASELINE 2     /* paper baseline of PAPER.md:613 (not this round)              */
+#define TG_PER_OP 1       /* paper mode: one operator per offload unit, DFS
+                             order + latest-time-of-use transfers, one
+                             stream, generic per-operator kernels, no splitting           */
+#define TG_BASELINE 2     /* paper baseline: per operator copy inputs in,
+                             run, copy outputs out, keep nothing                          */
 
 /* ------------------------------------------------------------------ graph building */
 tg_status tg_graph_create(tg_graph** g);
@@ -154,7 +157,9 @@ tg_status tg_set_runtime(tg_graph* g, const tg_runtime* rt);
 /* ------------------------------------------------------------------ plan / execute */
 /* Build the execution plan: recognise the template's offload units, split into chunks
  * (PAPER.md:359-371), order them and size every transfer. Pure host
- * code: works without a GPU. mode = TG_FUSED. The graph must outlive the plan. */
+ * code: works without a GPU. mode = TG_FUSED (edge/CNN templates, split into chunks),
+ * TG_PER_OP or TG_BASELINE (any graph, host I/O, one device, operators run whole:
+ * TG_E_INFEASIBLE if one does not fit). The graph must outlive the plan. */
 tg_status tg_plan_create(const tg_graph* g, int32_t mode, tg_plan** plan);
 
 typedef struct {

@@ -346,11 +346,12 @@ tg_status tg_set_runtime(tg_graph* g, const tg_runtime* rt) {
 
 tg_status tg_plan_create(const tg_graph* g, int32_t mode, tg_plan** plan) {
     if (!g || !plan) return fail(TG_E_ARG, "tg_plan_create: NULL argument");
-    if (mode != TG_FUSED) return fail(TG_E_UNSUPPORTED, "tg_plan_create: only TG_FUSED in this round");
+    if (mode != TG_FUSED && mode != TG_PER_OP && mode != TG_BASELINE)
+        return fail(TG_E_ARG, "tg_plan_create: mode must be TG_FUSED, TG_PER_OP or TG_BASELINE");
     TG_GUARD_BEGIN
     auto* p = new tg_plan();
     p->graph = g;
-    tg_status st = make_plan(g->g, mode, p->core);
+    tg_status st = mode == TG_FUSED ? make_plan(g->g, mode, p->core) : make_plan_per_op(g->g, mode, p->core);
     if (st != TG_OK) {
         delete p;
         return st;
@@ -378,7 +379,7 @@ tg_status tg_plan_stats_get(const tg_plan* p, tg_plan_stats* out) {
     out->chunk_end = c.c1;
     out->host_registered_bytes = exec_registered_bytes(p);
     // steady state: parameters stay resident after the first execution
-    out->h2d_bytes_steady = c.device_io ? 0 : c.h2d - c.param_bytes;
+    out->h2d_bytes_steady = c.device_io ? 0 : (c.mode == TG_FUSED ? c.h2d - c.param_bytes : c.h2d);
     return TG_OK;
 }
 
@@ -396,6 +397,7 @@ tg_status tg_plan_dump_json(const tg_plan* p, char* buf, size_t cap, size_t* nee
 tg_status tg_execute(tg_plan* p) {
     if (!p) return fail(TG_E_ARG, "tg_execute: NULL plan");
     TG_GUARD_BEGIN
+    if (p->core.mode != TG_FUSED) return exec_run_per_op(p, true);
     return exec_run(p, true);
     TG_GUARD_END
 }
@@ -403,6 +405,7 @@ tg_status tg_execute(tg_plan* p) {
 tg_status tg_execute_async(tg_plan* p) {
     if (!p) return fail(TG_E_ARG, "tg_execute_async: NULL plan");
     TG_GUARD_BEGIN
+    if (p->core.mode != TG_FUSED) return exec_run_per_op(p, false);
     return exec_run(p, false);
     TG_GUARD_END
 }
@@ -410,6 +413,10 @@ tg_status tg_execute_async(tg_plan* p) {
 tg_status tg_plan_set_profiling(tg_plan* p, int32_t on) {
     if (!p) return fail(TG_E_ARG, "tg_plan_set_profiling: NULL plan");
     TG_GUARD_BEGIN
+    if (p->core.mode != TG_FUSED) {
+        exec_set_profiling_per_op(p, on != 0);
+        return TG_OK;
+    }
     return exec_set_profiling(p, on != 0);
     TG_GUARD_END
 }
@@ -417,6 +424,7 @@ tg_status tg_plan_set_profiling(tg_plan* p, int32_t on) {
 tg_status tg_plan_timing_get(tg_plan* p, tg_timing* out) {
     if (!p || !out) return fail(TG_E_ARG, "tg_plan_timing_get: NULL argument");
     TG_GUARD_BEGIN
+    if (p->core.mode != TG_FUSED) return exec_timing_per_op(p, out);
     return exec_timing(p, out);
     TG_GUARD_END
 }
@@ -432,6 +440,7 @@ tg_status tg_plan_invalidate_params(tg_plan* p) {
 void tg_plan_destroy(tg_plan* p) {
     if (!p) return;
     exec_destroy(p);
+    exec_destroy_per_op(p);
     delete p;
 }
 

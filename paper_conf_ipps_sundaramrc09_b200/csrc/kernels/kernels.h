@@ -66,6 +66,28 @@ cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3(const CnnU3Args& a, cudaStream_t s);
 
+// Generic per-operator kernels (generic.cu) for the TG_PER_OP / TG_BASELINE modes.
+struct GenConvArgs {
+    const float* x; const float* k; const float* bias; float* y;
+    int64_t n, ci, h, w, co, kh, kw, ho, wo;
+    int pt, pl;             // top/left padding (0 for VALID)
+    int bias_kind;          // 0 none, 1 scalar [co], 2 plane [co][ho][wo]
+};
+constexpr int kGenMaxInputs = 16;
+struct GenElemArgs {
+    const float* xs[kGenMaxInputs]; int nx;
+    float* y; int64_t numel;
+    int op;                 // 0 add, 1 neg, 2 affine, 3 abs, 4 tanh, 5 max
+    float a, b;
+};
+struct GenSubArgs {
+    const float* x; const float* p; float* y;
+    int64_t n, c, h, w, ho, wo; int s;
+};
+cudaError_t launch_gen_conv(const GenConvArgs& a, cudaStream_t s);
+cudaError_t launch_gen_elem(const GenElemArgs& a, cudaStream_t s);
+cudaError_t launch_gen_sub(const GenSubArgs& a, cudaStream_t s);
+
 // tcgen05 (bf16 operands, fp32 accumulation in TMEM) variants of U2 and U3 (cnn_tc.cu)
 cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s);

@@ -480,6 +480,7 @@ static void jrange(std::ostringstream& o, const char* k, const RowRange& r) {
 }
 
 std::string plan_json(const PlanCore& p) {
+    if (p.mode != TG_FUSED) return plan_json_per_op(p);
     const Template& t = p.t;
     std::ostringstream o;
     o << "{";

@@ -21,18 +21,6 @@
 
 #include "tg_internal.h"
 
-struct tg_sched {
-    struct D {
-        uint64_t size;
-        int32_t kind;
-    };
-    struct O {
-        std::vector<int32_t> ins, outs;
-    };
-    std::vector<D> ds;
-    std::vector<O> ops;
-};
-
 namespace tg {
 
 std::vector<int32_t> sched_dfs(const tg_sched& s) {
@@ -84,7 +72,7 @@ std::vector<int32_t> sched_dfs(const tg_sched& s) {
 // Returns the transfer volume; trace entries are (kind, id): 0 = H2D of DS id, 1 = run op id,
 // 2 = D2H of DS id. Returns UINT64_MAX if an operator does not fit at all.
 uint64_t sched_transfers(const tg_sched& s, const std::vector<int32_t>& order, uint64_t capacity,
-                         std::vector<std::pair<int32_t, int32_t>>* trace) {
+                         std::vector<std::pair<int32_t, int32_t>>* trace, bool frees) {
     const size_t nds = s.ds.size();
     std::vector<std::vector<size_t>> uses(nds);
     for (size_t t = 0; t < order.size(); ++t) {
@@ -139,6 +127,7 @@ uint64_t sched_transfers(const tg_sched& s, const std::vector<int32_t>& order, u
                 }
                 on_gpu[victim] = -1;
                 used -= s.ds[victim].size;
+                if (trace && frees) trace->push_back({3, victim});
             }
             const bool is_in = std::find(op.ins.begin(), op.ins.end(), j) != op.ins.end();
             if (is_in) {
@@ -157,6 +146,7 @@ uint64_t sched_transfers(const tg_sched& s, const std::vector<int32_t>& order, u
             if (on_gpu[k] >= 0 && next_use((int32_t)k, t) == INF && !is_output((int32_t)k)) {
                 on_gpu[k] = -1;
                 used -= s.ds[k].size;
+                if (trace && frees) trace->push_back({3, (int32_t)k});
             }
     }
     for (size_t k = 0; k < nds; ++k)
@@ -229,7 +219,7 @@ tg_status tg_sched_transfers(const tg_sched* s, const int32_t* order, uint64_t c
         placed[i] = 1;
     }
     std::vector<std::pair<int32_t, int32_t>> tr;
-    const uint64_t m = sched_transfers(*s, ord, capacity, &tr);
+    const uint64_t m = sched_transfers(*s, ord, capacity, &tr, false);
     if (m == UINT64_MAX)
         return fail(TG_E_INFEASIBLE, "tg_sched_transfers: an operator does not fit, or reads data not yet produced");
     *moved = m;

@@ -115,12 +115,43 @@ struct PlanCore {
     uint64_t h2d = 0, d2h = 0, io_lb = 0, total = 0;
     int64_t nops = 0, nds = 0;
     int64_t n_units = 1;
+    // per-operator modes (TG_PER_OP, TG_BASELINE): the abstract schedule over graph DS/nodes
+    std::vector<int> po_ds;       // sched DS id -> graph DS id
+    std::vector<uint64_t> po_size;
+    std::vector<int32_t> po_kind;
+    std::vector<int> po_ops;      // sched op id -> graph node id
+    std::vector<std::vector<int32_t>> po_ins, po_outs;
+    std::vector<int32_t> po_order;
+    std::vector<std::pair<int32_t, int32_t>> po_trace;  // (0 h2d | 1 run | 2 d2h | 3 free, id)
+    uint64_t po_capacity = 0;
 };
 
 tg_status recognise(const Graph& g, Template& t);
+tg_status make_plan_per_op(const Graph& g, int32_t mode, PlanCore& p);
 tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p);
 std::string plan_json(const PlanCore& p);
+std::string plan_json_per_op(const PlanCore& p);
 
+}  // namespace tg
+
+// abstract operator graph of the transfer scheduler (sched.cpp)
+struct tg_sched {
+    struct D {
+        uint64_t size;
+        int32_t kind;  // TG_DS_*
+    };
+    struct O {
+        std::vector<int32_t> ins, outs;
+    };
+    std::vector<D> ds;
+    std::vector<O> ops;
+};
+
+namespace tg {
+std::vector<int32_t> sched_dfs(const tg_sched& s);
+// trace kinds: 0 H2D ds, 1 run op, 2 D2H ds, 3 (frees only) ds leaves the GPU
+uint64_t sched_transfers(const tg_sched& s, const std::vector<int32_t>& order, uint64_t capacity,
+                         std::vector<std::pair<int32_t, int32_t>>* trace, bool frees);
 }  // namespace tg
 
 // opaque handles
@@ -128,12 +159,14 @@ struct tg_graph {
     tg::Graph g;
 };
 
-struct tg_exec;  // engine state (engine.cu)
+struct tg_exec;         // engine state (engine.cu)
+struct tg_perop_exec;   // per-operator executor state (engine_perop.cu)
 
 struct tg_plan {
     const tg_graph* graph = nullptr;
     tg::PlanCore core;
     tg_exec* exec = nullptr;
+    tg_perop_exec* perop = nullptr;
     int64_t launches = 0;
 };
 
@@ -144,4 +177,8 @@ tg_status exec_timing(tg_plan* p, tg_timing* out);
 void exec_destroy(tg_plan* p);
 uint64_t exec_registered_bytes(const tg_plan* p);
 void exec_invalidate_params(tg_plan* p);
+tg_status exec_run_per_op(tg_plan* p, bool blocking);
+tg_status exec_timing_per_op(tg_plan* p, tg_timing* out);
+void exec_set_profiling_per_op(tg_plan* p, bool on);
+void exec_destroy_per_op(tg_plan* p);
 }  // namespace tg
