@@ -154,8 +154,12 @@ tg_status make_plan_per_op(const Graph& g, int32_t mode, PlanCore& p) {
     p.d2h = d2h;
     p.param_bytes = 0;
     p.slot_bytes = 0;
-    // first-fit allocation inside the arena: the 1/8 margin absorbs fragmentation
-    p.arena_bytes = g.budget ? g.budget : a256(peak + peak / 8 + 256 * s.ds.size());
+    // first-fit allocation inside the arena; capped: the 1/8 margin between the scheduling
+    // capacity and the arena absorbs fragmentation; uncapped: room for every DS
+    uint64_t all = 0;
+    for (auto& d : s.ds) all += a256(d.size);
+    (void)peak;
+    p.arena_bytes = g.budget ? g.budget : all;
     p.split = "none";
     p.bias = "none";
     p.c0 = 0;
