@@ -206,3 +206,25 @@ def test_cnn_bf16_tc_split_equals_unsplit(tg):
     split, p1 = run_cnn(tg, img, n5, prm, budget=2_000_000, precision=tg.TG_BF16_TC)
     assert p1.json()["n_chunks"] > p0.json()["n_chunks"]
     assert np.array_equal(split, full)
+
+
+@pytest.mark.parametrize("n5,prec", [(20, "fp32"), (120, "fp32"), (120, "bf16_tc")])
+def test_cnn_config3_full_batch_sampled(tg, orc, n5, prec):
+    """BASELINE configs[2] at full size in the bench's launch configuration (64 x 480x640 images,
+    device-resident, uncapped): images 0, 31 and 63 match the oracle."""
+    n, H, W = 64, 480, 640
+    seed = synth.seed_for_config(3)
+    x = synth.images_torch(seed, n, H, W, "cuda")
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    h5, w5 = synth.cnn_dims(H, W)[4]
+    y = torch.zeros((n, 9, h5, w5), dtype=torch.float32, device="cuda")
+    g, _ = tg.cnn_graph(x, n5, prm, out=y, device=True)
+    g.set(torch_runtime=True, precision=tg.TG_BF16_TC if prec == "bf16_tc" else tg.TG_FP32)
+    p = g.plan()
+    p.execute()
+    out = y.cpu().numpy()
+    img = x.cpu().numpy()
+    tol = 2e-2 if prec == "bf16_tc" else 1e-5
+    for b in (0, 31, 63):
+        ref = orc.cnn(img[b:b + 1], n5, prm)
+        assert normwise(out[b:b + 1], ref) <= tol, b
