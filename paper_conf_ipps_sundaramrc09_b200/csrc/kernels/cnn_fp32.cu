@@ -35,7 +35,7 @@ __device__ __forceinline__ float tanh_f(float x) {
 // from a 6x6 input window), bias, tanh, the 2x2 subsample, tanh. Weights travel in the
 // constant bank (kernel parameter) so FFMAs take them as uniform operands.
 struct U1W {
-    float k1[8][25];
+    float k1[25][8];  // [tap][ch]: channel pairs are adjacent (one FFMA2 operand)
     float p2[8][4];
 };
 
@@ -60,11 +60,12 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
     const int64_t R2 = r2_0 + ty, C2 = c2_0 + tx;
     if (R2 >= a.t2_row0 + a.t2_rows || C2 >= a.w2) return;
 
-    float acc[8][4];
+    // FFMA2 over channel pairs (2c, 2c+1): each lane rounds exactly like fmaf
+    float2 acc2[4][4];
 #pragma unroll
-    for (int ch = 0; ch < 8; ++ch)
+    for (int cp = 0; cp < 4; ++cp)
 #pragma unroll
-        for (int p = 0; p < 4; ++p) acc[ch][p] = 0.f;
+        for (int p = 0; p < 4; ++p) acc2[cp][p] = make_float2(0.f, 0.f);
 #pragma unroll
     for (int i = 0; i < 6; ++i) {
         float x[6];
@@ -80,12 +81,14 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
             const int ki = i - ra;  // kernel row for C1 row 2*R2 + ra
             if (ki < 0 || ki > 4) continue;
 #pragma unroll
-            for (int ch = 0; ch < 8; ++ch)
+            for (int cp = 0; cp < 4; ++cp)
 #pragma unroll
-                for (int kj = 0; kj < 5; ++kj)
+                for (int kj = 0; kj < 5; ++kj) {
+                    const float2 wv = make_float2(w.k1[ki * 5 + kj][2 * cp], w.k1[ki * 5 + kj][2 * cp + 1]);
 #pragma unroll
                     for (int cb = 0; cb < 2; ++cb)
-                        acc[ch][ra * 2 + cb] = fmaf(x[cb + kj], w.k1[ch][ki * 5 + kj], acc[ch][ra * 2 + cb]);
+                        acc2[cp][ra * 2 + cb] = __ffma2_rn(make_float2(x[cb + kj], x[cb + kj]), wv, acc2[cp][ra * 2 + cb]);
+                }
         }
     }
     float* t2 = a.t2 + img * a.t2_img_stride;
@@ -99,7 +102,8 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
             const int64_t r1 = 2 * R2 + (p >> 1), c1 = 2 * C2 + (p & 1);
             const float b = a.b1_plane ? __ldg(a.b1 + ((int64_t)ch * a.b1_rows + (r1 - a.b1_row0)) * a.w1 + c1)
                                        : __ldg(a.b1 + ch);
-            const float t = tanh_f(acc[ch][p] + b);
+            const float av = (ch & 1) ? acc2[ch >> 1][p].y : acc2[ch >> 1][p].x;
+            const float t = tanh_f(av + b);
             s = fmaf(w.p2[ch][p], t, s);
         }
         tv[ch] = tanh_f(s);
@@ -130,7 +134,7 @@ struct U2W {
 constexpr int U2_TR = 8, U2_TC = 16;
 constexpr int U2_IR = 2 * U2_TR + 4, U2_IC = 2 * U2_TC + 4;  // 20 x 36 per plane
 
-__global__ void __launch_bounds__(128, 3) cnn_u2_kernel(const CnnU2Args a, const __grid_constant__ U2W w) {
+__global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const __grid_constant__ U2W w) {
     __shared__ __align__(16) float xs[8][U2_IR * U2_IC];
     const int tid = threadIdx.x, ty = tid / U2_TC, tx = tid % U2_TC;
     const int64_t img = blockIdx.z;
@@ -150,11 +154,11 @@ __global__ void __launch_bounds__(128, 3) cnn_u2_kernel(const CnnU2Args a, const
     const int64_t R4 = r4_0 + ty, C4 = c4_0 + tx;
     if (R4 >= a.t4_row0 + a.t4_rows || C4 >= a.w4) return;
 
-    float acc[20][4];
+    float2 acc2[10][4];  // channel pairs (2c, 2c+1), FFMA2
 #pragma unroll
-    for (int co = 0; co < 20; ++co)
+    for (int cp = 0; cp < 10; ++cp)
 #pragma unroll
-        for (int p = 0; p < 4; ++p) acc[co][p] = 0.f;
+        for (int p = 0; p < 4; ++p) acc2[cp][p] = make_float2(0.f, 0.f);
 #pragma unroll 1
     for (int ci = 0; ci < 8; ++ci) {
 #pragma unroll
@@ -174,10 +178,10 @@ __global__ void __launch_bounds__(128, 3) cnn_u2_kernel(const CnnU2Args a, const
 #pragma unroll
                 for (int kj = 0; kj < 5; ++kj)
 #pragma unroll
-                    for (int co = 0; co < 20; ++co) {
-                        const float wv = w.k3[ci][ki * 5 + kj][co];
-                        acc[co][ra * 2 + 0] = fmaf(x[kj], wv, acc[co][ra * 2 + 0]);
-                        acc[co][ra * 2 + 1] = fmaf(x[kj + 1], wv, acc[co][ra * 2 + 1]);
+                    for (int cp = 0; cp < 10; ++cp) {
+                        const float2 wv = make_float2(w.k3[ci][ki * 5 + kj][2 * cp], w.k3[ci][ki * 5 + kj][2 * cp + 1]);
+                        acc2[cp][ra * 2 + 0] = __ffma2_rn(make_float2(x[kj], x[kj]), wv, acc2[cp][ra * 2 + 0]);
+                        acc2[cp][ra * 2 + 1] = __ffma2_rn(make_float2(x[kj + 1], x[kj + 1]), wv, acc2[cp][ra * 2 + 1]);
                     }
             }
         }
@@ -192,7 +196,8 @@ __global__ void __launch_bounds__(128, 3) cnn_u2_kernel(const CnnU2Args a, const
             const int64_t r3 = 2 * R4 + (p >> 1), c3 = 2 * C4 + (p & 1);
             const float b = a.b3_plane ? __ldg(a.b3 + ((int64_t)co * a.b3_rows + (r3 - a.b3_row0)) * a.w3 + c3)
                                        : __ldg(a.b3 + co);
-            s = fmaf(w.p4[co][p], tanh_f(acc[co][p] + b), s);
+            const float av = (co & 1) ? acc2[co >> 1][p].y : acc2[co >> 1][p].x;
+            s = fmaf(w.p4[co][p], tanh_f(av + b), s);
         }
         t4[co * oplane + (R4 - a.t4_row0) * a.w4 + C4] = tanh_f(s);
     }
@@ -248,11 +253,11 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
             ws[idx] = (g0 + ch < n5) ? __ldg(a.k5 + (int64_t)(g0 + ch) * 500 + k) : 0.f;
         }
         __syncthreads();
-        float acc[U3_G][U3_P];
+        float2 acc2[U3_G / 2][U3_P];  // channel pairs, FFMA2
 #pragma unroll
-        for (int c = 0; c < U3_G; ++c)
+        for (int c = 0; c < U3_G / 2; ++c)
 #pragma unroll
-            for (int p = 0; p < U3_P; ++p) acc[c][p] = 0.f;
+            for (int p = 0; p < U3_P; ++p) acc2[c][p] = make_float2(0.f, 0.f);
 #pragma unroll 1
         for (int ci = 0; ci < 20; ++ci) {
 #pragma unroll
@@ -266,11 +271,13 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
                 for (int kj = 0; kj < 5; ++kj) {
                     const float4* wr = reinterpret_cast<const float4*>(&ws[((ci * 25) + i * 5 + kj) * U3_G]);
                     const float4 wa = wr[0], wb = wr[1];
-                    const float wv[8] = {wa.x, wa.y, wa.z, wa.w, wb.x, wb.y, wb.z, wb.w};
+                    const float2 wv[4] = {make_float2(wa.x, wa.y), make_float2(wa.z, wa.w), make_float2(wb.x, wb.y),
+                                          make_float2(wb.z, wb.w)};
 #pragma unroll
-                    for (int c = 0; c < U3_G; ++c)
+                    for (int c = 0; c < U3_G / 2; ++c)
 #pragma unroll
-                        for (int p = 0; p < U3_P; ++p) acc[c][p] = fmaf(x[p + kj], wv[c], acc[c][p]);
+                        for (int p = 0; p < U3_P; ++p)
+                            acc2[c][p] = __ffma2_rn(make_float2(x[p + kj], x[p + kj]), wv[c], acc2[c][p]);
                 }
             }
         }
@@ -285,7 +292,8 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
                 if (row_ok && C5 + p < a.w5)
                     b = a.b5_plane ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (R5 - a.b5_row0)) * a.w5 + C5 + p)
                                    : __ldg(a.b5 + ch);
-                const float t = tanh_f(acc[c][p] + b);
+                const float av = (c & 1) ? acc2[c >> 1][p].y : acc2[c >> 1][p].x;
+                const float t = tanh_f(av + b);
 #pragma unroll
                 for (int o = 0; o < 9; ++o) c6[o][p] = fmaf(k6s[o * n5p + ch], t, c6[o][p]);
             }
@@ -310,7 +318,8 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
 cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s) {
     if (a.t2_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     U1W w;
-    std::memcpy(w.k1, a.k1_host, sizeof w.k1);
+    for (int ch = 0; ch < 8; ++ch)
+        for (int t = 0; t < 25; ++t) w.k1[t][ch] = a.k1_host[ch * 25 + t];
     std::memcpy(w.p2, a.p2_host, sizeof w.p2);
     dim3 grid((unsigned)((a.w2 + U1_TC - 1) / U1_TC), (unsigned)((a.t2_rows + U1_TR - 1) / U1_TR), (unsigned)a.nimg);
     cnn_u1_kernel<<<grid, 128, 0, s>>>(a, w);
