@@ -143,3 +143,18 @@ def test_full_size_sampled_rows(tg, orc):
             got = out[b, 0, r]
             err = np.abs(got.astype(np.float64) - ref).max() / np.abs(ref).max()
             assert err <= 1e-5, (b, r, err)
+
+
+def test_two_host_threads_same_device(tg, orc):
+    """tg_set_devices([0, 0]): the one-host-thread-per-device dispatcher with both
+    shards on the one GPU of the box -- same chunk list, disjoint output rows, same bits."""
+    img = synth.images_np(21, 3, 300, 260)
+    K1, K2 = synth.random_edge_filters_np(21)
+    ref, _ = run_edge(tg, img, K1, K2, budget=400_000)
+    out = np.zeros_like(img)
+    g, _ = tg.edge_graph(img, K1, K2, out=out)
+    g.set(budget=400_000, devices=[0, 0], torch_runtime=True)
+    p = g.plan()
+    p.execute()
+    assert p.stats()["n_chunks"] >= 4
+    assert np.array_equal(out, ref)
