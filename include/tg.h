@@ -64,8 +64,8 @@ typedef int32_t tg_id;
 #define TG_AFFINE 2       /* elementwise y = a * x0 + b                                   */
 #define TG_ABS 3          /* elementwise y = |x0|                                         */
 #define TG_MAX 0          /* combine op of tg_find_edges                                  */
-#define TG_SUM 1          /* (not implemented in this round: TG_E_UNSUPPORTED)            */
-#define TG_MAXABS 2       /* (not implemented in this round: TG_E_UNSUPPORTED)            */
+#define TG_SUM 1          /* combine op: sum of the convolutions' responses              */
+#define TG_MAXABS 2       /* combine op: max of |response|                                */
 #define TG_BIAS_PLANE 0   /* CNN bias: one full plane per output map (the paper's Fig. 7)
                              shape [1][c][h][w], shared by every image of the batch       */
 #define TG_BIAS_SCALAR 1  /* CNN bias: one scalar per output map, shape [c]               */
@@ -115,10 +115,13 @@ tg_status tg_shape(const tg_graph* g, tg_id id, int64_t dims[4]);
 
 /* Template helpers (PAPER.md:623 find_edges; PAPER.md:635 the CNN built from torch5
  * primitives). Both only append primitive nodes to the graph. */
-/* Edge detection: num_orientations/2 SAME convolutions of img with
- * `kernel` ([1][1][k][k], k <= 16) and its rot90 rotations, as many remaps (negations)
- * and one max combine. num_orientations = 4 (8: TG_E_UNSUPPORTED this round);
- * combine_op = TG_MAX. */
+/* Edge detection: num_orientations (2, 4 or 8) orientations in steps of
+ * 360/num_orientations degrees; the first half are SAME convolutions of img with `kernel`
+ * ([1][1][k][k], k <= 16) rotated on the host (multiples of 90 degrees exactly, others by
+ * bilinear interpolation, R18), the second half their remaps (negations).
+ * combine_op: TG_MAX (max over all orientations), TG_MAXABS (max |response| of the
+ * convolutions), TG_SUM (sum of the convolutions; the remaps would cancel). TG_FUSED runs
+ * any of these as one kernel (up to 4 convolutions). */
 tg_status tg_find_edges(tg_graph* g, tg_id img, tg_id kernel, int32_t num_orientations,
                         int32_t combine_op, tg_id* edge_map);
 /* CNN of SURVEY F2 (11 layers): C1(1->8,5x5) T S2 T C3(8->20,5x5) T S4 T C5(20->n5,5x5)

@@ -146,6 +146,26 @@ def edge(img, K1, K2, return_parts: bool = False):
     return (E, E1, E2) if return_parts else E
 
 
+def edge_general(img, kernels, combine: str = "max") -> np.ndarray:
+    """Edge graph with explicit filters ('combining the results by doing a
+    reduction such as addition/max/max absolute value'), node by node: E_i = Im * K_i (SAME);
+    max: left fold over E_1..E_k, -E_1..-E_k; sum: left fold of fp32 adds; maxabs: fold over
+    |E_i|; maxplain: fold over E_i."""
+    E = [conv2d_same(img, K) for K in kernels]
+    if combine == "max":
+        return max_fold(*(E + [neg(e) for e in E]))
+    if combine == "sum":
+        s = E[0]
+        for e in E[1:]:
+            s = add(s, e)
+        return s
+    if combine == "maxabs":
+        return max_fold(*[np.abs(e) for e in E])
+    if combine == "maxplain":
+        return max_fold(*E)
+    raise ValueError(combine)
+
+
 def cnn(img, n5: int, params, bias_plane: bool = True) -> np.ndarray:
     """CNN template. img: [n][1][H][W] or [H][W]; params in the
     order K1,B1,P2,K3,B3,P4,K5,B5,K6,B6. Returns [n][9][H6][W6]."""

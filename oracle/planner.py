@@ -96,6 +96,33 @@ def edge_graph(H: int, W: int, ks: int = 16, orientations: int = 4, kernel_float
     return g
 
 
+def edge_graph_general(H: int, W: int, ks: int, nf: int, combine: str) -> Graph:
+    """Edge graph with nf convolutions combined by 'max' (responses and their remaps,
+    PAPER.md:627-629), 'sum' (addition), 'maxabs' (max absolute value) or 'maxplain' (max of
+    the responses) -- the reductions PAPER.md:621 lists."""
+    if combine == "max":
+        return edge_graph(H, W, ks, orientations=2 * nf)
+    g = Graph()
+    S = H * W
+    im = g.add_ds("Im", S, "input")
+    resp = []
+    for i in range(nf):
+        k = g.add_ds(f"K{i+1}", ks * ks, "param")
+        e = g.add_ds(f"E{i+1}", S)
+        g.add_op(f"C{i+1}", [im, k], [e])
+        resp.append(e)
+    if combine == "maxabs":
+        absd = []
+        for i, e in enumerate(resp):
+            a = g.add_ds(f"A{i+1}", S)
+            g.add_op(f"abs{i+1}", [e], [a])
+            absd.append(a)
+        resp = absd
+    E = g.add_ds("E", S, "output")
+    g.add_op("sum" if combine == "sum" else "max", resp, [E])
+    return g
+
+
 def cnn_dims(H: int, W: int):
     """Per-level plane sizes: VALID 5x5 convs and 2x2/2 subsampling
     with floor((D-2)/2)+1."""
@@ -439,7 +466,7 @@ def _span(r) -> int:
 def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int = 20,
                bias: str = "plane", budget: int = 0, max_chunk_px: int = MAX_CHUNK_PX,
                depth: int = DEPTH, rank: int = 0, world: int = 1, device_io: bool = False,
-               precision: str = "fp32") -> dict:
+               precision: str = "fp32", nf: int = 2, combine: str = "max") -> dict:
     """Fused-mode plan, restated plainly; the library's
     tg_plan_dump_json must produce the same dict (tests/test_plan_parity.py).
 
@@ -464,8 +491,8 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
         raise ValueError("empty input")
     if template == "edge":
         h_out, w_out, in_per_out = H, W, 1
-        params = [ks * ks, ks * ks]
-        is_bias = [False, False]
+        params = [ks * ks] * nf
+        is_bias = [False] * nf
         rows = lambda r0, r1: _edge_rows(H, ks, r0, r1)          # noqa: E731
         widest = lambda R: {"in": [0, min(H, R + ks - 1)], "out": [0, R]}  # noqa: E731
     elif template == "cnn":
@@ -588,7 +615,7 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
 
     # Table 1 accounting (per template instance; images and per-image DS scale with n)
     if template == "edge":
-        g = edge_graph(H, W, ks)
+        g = edge_graph_general(H, W, ks, nf, combine)
     else:
         g = cnn_graph_fig7(H, W, n5)
     param_floats = sum(params)
@@ -599,6 +626,7 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
     return {
         "template": template, "n": n, "H": H, "W": W,
         "ks": ks if template == "edge" else 0, "n5": n5 if template == "cnn" else 0,
+        "nf": nf if template == "edge" else 0, "combine": combine if template == "edge" else "none",
         "budget": budget, "depth": depth, "max_chunk_px": max_chunk_px,
         "device_io": bool(device_io), "precision": precision if template == "cnn" else "fp32", "bias": bias_mode, "split": split, "B": B, "R": R,
         "param_bytes": pb, "slot_bytes": sb, "arena_bytes": pb + depth * sb,

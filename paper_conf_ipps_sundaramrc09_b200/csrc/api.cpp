@@ -1,6 +1,7 @@
 // api.cpp -- the C ABI of include/tg.h: graph building, target parameters, plan handles.
 // Graph nodes follow the paper's operator graph (vertices are parallel
 // computations, edges data dependencies; footprints statically known).
+#include <cmath>
 #include <cstring>
 #include <new>
 #include <string>
@@ -232,13 +233,60 @@ tg_status tg_shape(const tg_graph* g, tg_id id, int64_t dims[4]) {
 // find_edges(Image, Kernel, num_orientations, Combine_op): orientations at
 // 0 and 90 degrees are convolutions with the kernel and its rot90 (precomputed host data,
 // the 2 x 256 kernel floats of Table 1), 180 and 270 degrees are remaps.
+// Kernel rotated counter-clockwise by `deg` about its centre: multiples of 90 degrees are exact
+// index permutations (90: R[i][j] = K[j][k-1-i], as numpy.rot90); other angles sample K
+// bilinearly at the rotated position (zero outside) -- DESIGN.md reading R18.
+static std::vector<float> rotate_kernel(const float* K, int64_t k, int deg) {
+    std::vector<float> r(k * k, 0.f);
+    deg = ((deg % 360) + 360) % 360;
+    if (deg % 90 == 0) {
+        for (int64_t i = 0; i < k; ++i)
+            for (int64_t j = 0; j < k; ++j) {
+                int64_t si = i, sj = j;
+                for (int q = 0; q < deg / 90; ++q) {  // apply rot90 q times
+                    const int64_t ti = sj, tj = k - 1 - si;
+                    si = ti;
+                    sj = tj;
+                }
+                r[i * k + j] = K[si * k + sj];
+            }
+        return r;
+    }
+    const double th = deg * 3.14159265358979323846 / 180.0, c0 = (k - 1) / 2.0;
+    const double cs = std::cos(th), sn = std::sin(th);
+    for (int64_t i = 0; i < k; ++i)
+        for (int64_t j = 0; j < k; ++j) {
+            const double y = i - c0, x = j - c0;
+            const double sr = c0 + y * cs + x * sn, sc = c0 - y * sn + x * cs;
+            const int64_t r0 = (int64_t)std::floor(sr), q0 = (int64_t)std::floor(sc);
+            const double fr = sr - r0, fc = sc - q0;
+            double v = 0.0;
+            for (int dr = 0; dr < 2; ++dr)
+                for (int dc = 0; dc < 2; ++dc) {
+                    const int64_t rr = r0 + dr, cc = q0 + dc;
+                    if (rr < 0 || rr >= k || cc < 0 || cc >= k) continue;
+                    v += (dr ? fr : 1 - fr) * (dc ? fc : 1 - fc) * K[rr * k + cc];
+                }
+            r[i * k + j] = (float)v;
+        }
+    return r;
+}
+
+// find_edges(Image, Kernel, num_orientations, Combine_op): orientations are
+// rotations of the filter in steps of 360/num_orientations degrees; the first half are
+// convolutions with the rotated kernel (precomputed host data, the kernel floats of Table 1),
+// the second half are remaps (negations) of the first. Combine: TG_MAX over
+// all orientations, TG_MAXABS = max |response| of the convolutions, TG_SUM = sum of the
+// convolutions' responses (adding the remaps would cancel them).
 tg_status tg_find_edges(tg_graph* g, tg_id img, tg_id kernel, int32_t num_orientations,
                         int32_t combine_op, tg_id* edge_map) {
     if (!g || !edge_map) return fail(TG_E_ARG, "tg_find_edges: NULL argument");
     Graph& G = g->g;
     if (!valid_id(G, img) || !valid_id(G, kernel)) return fail(TG_E_ARG, "tg_find_edges: unknown DS id");
-    if (num_orientations != 4) return fail(TG_E_UNSUPPORTED, "tg_find_edges: only 4 orientations in this round");
-    if (combine_op != TG_MAX) return fail(TG_E_UNSUPPORTED, "tg_find_edges: only TG_MAX combine in this round");
+    if (num_orientations != 2 && num_orientations != 4 && num_orientations != 8)
+        return fail(TG_E_ARG, "tg_find_edges: num_orientations must be 2, 4 or 8");
+    if (combine_op != TG_MAX && combine_op != TG_SUM && combine_op != TG_MAXABS)
+        return fail(TG_E_ARG, "tg_find_edges: combine_op must be TG_MAX, TG_SUM or TG_MAXABS");
     const Ds& K = G.ds[kernel];
     if (K.kind != DsKind::Param || K.d[0] != 1 || K.d[1] != 1 || K.d[2] != K.d[3])
         return fail(TG_E_SHAPE, "tg_find_edges: kernel must be a square [1][1][k][k] parameter");
@@ -246,24 +294,43 @@ tg_status tg_find_edges(tg_graph* g, tg_id img, tg_id kernel, int32_t num_orient
     if (K.src_loc != Loc::Host) return fail(TG_E_ARG, "tg_find_edges: kernel must be host data");
     TG_GUARD_BEGIN
     const int64_t k = K.d[2];
-    // K2 = rot90(K1) (counter-clockwise): K2[i][j] = K1[j][k-1-i]
-    std::vector<float> r(k * k);
-    for (int64_t i = 0; i < k; ++i)
-        for (int64_t j = 0; j < k; ++j) r[i * k + j] = K.src[j * k + (k - 1 - i)];
-    int64_t d[4] = {1, 1, k, k};
-    tg_id k2 = add_ds(G, d, DsKind::Param);
-    G.ds[k2].owned = std::move(r);
-    G.ds[k2].src = G.ds[k2].owned.data();
-    G.ds[k2].src_loc = Loc::Host;
-    tg_id e1, e2, e5, e6, e;
+    const int nconv = num_orientations / 2, step = 360 / num_orientations;
+    std::vector<tg_id> resp;
     tg_status st;
-    if ((st = tg_conv2d(g, img, kernel, -1, TG_SAME, &e1)) != TG_OK) return st;
-    if ((st = tg_conv2d(g, img, k2, -1, TG_SAME, &e2)) != TG_OK) return st;
-    if ((st = tg_elementwise(g, TG_NEG, &e1, 1, 0.f, 0.f, &e5)) != TG_OK) return st;
-    if ((st = tg_elementwise(g, TG_NEG, &e2, 1, 0.f, 0.f, &e6)) != TG_OK) return st;
-    tg_id xs[4] = {e1, e2, e5, e6};
-    if ((st = tg_max_combine(g, xs, 4, &e)) != TG_OK) return st;
-    *edge_map = e;
+    for (int f = 0; f < nconv; ++f) {
+        tg_id kid = kernel;
+        if (f > 0) {
+            int64_t d[4] = {1, 1, k, k};
+            kid = add_ds(G, d, DsKind::Param);
+            G.ds[kid].owned = rotate_kernel(G.ds[kernel].src, k, f * step);
+            G.ds[kid].src = G.ds[kid].owned.data();
+            G.ds[kid].src_loc = Loc::Host;
+        }
+        tg_id e;
+        if ((st = tg_conv2d(g, img, kid, -1, TG_SAME, &e)) != TG_OK) return st;
+        resp.push_back(e);
+    }
+    tg_id out;
+    if (combine_op == TG_SUM) {
+        if ((st = tg_elementwise(g, TG_ADD, resp.data(), (int32_t)resp.size(), 1.f, 0.f, &out)) != TG_OK) return st;
+    } else if (combine_op == TG_MAXABS) {
+        std::vector<tg_id> ab;
+        for (tg_id e : resp) {
+            tg_id a;
+            if ((st = tg_elementwise(g, TG_ABS, &e, 1, 0.f, 0.f, &a)) != TG_OK) return st;
+            ab.push_back(a);
+        }
+        if ((st = tg_max_combine(g, ab.data(), (int32_t)ab.size(), &out)) != TG_OK) return st;
+    } else {
+        std::vector<tg_id> all = resp;
+        for (tg_id e : resp) {
+            tg_id r;
+            if ((st = tg_elementwise(g, TG_NEG, &e, 1, 0.f, 0.f, &r)) != TG_OK) return st;
+            all.push_back(r);
+        }
+        if ((st = tg_max_combine(g, all.data(), (int32_t)all.size(), &out)) != TG_OK) return st;
+    }
+    *edge_map = out;
     return TG_OK;
     TG_GUARD_END
 }

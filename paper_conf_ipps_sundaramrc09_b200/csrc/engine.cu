@@ -262,8 +262,9 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.H = t.H;
         a.W = t.W;
         a.nimg = ch.nimg;
-        a.k1_host = g.ds[c.param_ds[0]].src;
-        a.k2_host = g.ds[c.param_ds[1]].src;
+        for (int f = 0; f < t.nf; ++f) a.k_host[f] = g.ds[c.param_ds[f]].src;
+        a.nf = t.nf;
+        a.combine = t.combine;
         a.ks = t.ks;
         KernelTimer kt(x, d, 0, cs);
         CK(launch_edge(a, cs));

@@ -3,7 +3,9 @@
 // Computes the whole 4-orientation edge template of PAPER.md:629 (Fig. 3 graph:
 // C1: E1 = Im*K1, C2: E2 = Im*K2, R1: E5 = -E1, R2: E6 = -E2, max: E = max(E1,E2,E5,E6))
 // in ONE pass over a chunk, so E1, E2, E5, E6 never leave registers -- the paper's "best
-// possible" configuration. SAME zero padding with anchor (ks-1)/2
+// possible" configuration. The same kernel takes up to 4 convolutions (the
+// 8-orientation graph of Fig. 1(b)) and the other combine ops of PAPER.md:621 (addition,
+// max absolute value). SAME zero padding with anchor (ks-1)/2
 // (R2); a ks x ks kernel (ks <= 16) is embedded in a 16 x 16 frame at offset
 // 7 - (ks-1)/2 so one code path serves every size (zero taps add exact zeros).
 //
@@ -51,8 +53,7 @@ constexpr int kBufStride = (kTileBytes + 127) / 128 * 128;
 // register (FFMA R, R, UR, R) -- only two vector-register operands per FFMA, which keeps
 // the register-file banks out of the way of the FMA pipe.
 struct EdgeWeights {
-    float w1[256];  // broadcast to both lanes of an FFMA2 (uniform-register operand .F32)
-    float w2[256];
+    float w[4][256];  // up to 4 filters, processed in pairs; broadcast to both lanes of an FFMA2
 };
 
 // Compute the 64 x 64 output tile whose input (+halo) is staged at xs (pitch kPitch, smem
@@ -69,64 +70,82 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const fl
     // adjacent output columns; each lane rounds exactly like fmaf, so results are bit-identical
     // to scalar FMAs in the same order. The pair (x[s], x[s+1]) for an odd s comes from the
     // second copy of the tile, staged one column to the left (xs1[c] = xs[c+1]).
-    float2 a1[8], a2[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-        a1[q] = make_float2(0.f, 0.f);
-        a2[q] = make_float2(0.f, 0.f);
-    }
-
-#pragma unroll 1
-    for (int i = 0; i < 16; ++i) {
-        // input window: smem cols [cb, cb+32) <-> image cols [c0+cb-8, c0+cb+24);
-        // output column c0+cb+q, tap j reads image col c0+cb+q+j-7 = smem col cb+q+j+1
-        float2 xe[16], xo[16];  // xe[k] = (x[2k], x[2k+1]), xo[k] = (x[2k+1], x[2k+2])
-        const float4* r0 = reinterpret_cast<const float4*>(&xs[(lr + i) * kPitch + cb]);
-        const float4* r1 = reinterpret_cast<const float4*>(&xs1[(lr + i) * kPitch + cb]);
-#pragma unroll
-        for (int v = 0; v < 8; ++v) {
-            const float4 t = r0[v];
-            const float4 u = r1[v];
-            xe[2 * v] = make_float2(t.x, t.y);
-            xe[2 * v + 1] = make_float2(t.z, t.w);
-            xo[2 * v] = make_float2(u.x, u.y);
-            xo[2 * v + 1] = make_float2(u.z, u.w);
-        }
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-            const float2 w1 = make_float2(wt.w1[i * 16 + j], wt.w1[i * 16 + j]);
-            const float2 w2 = make_float2(wt.w2[i * 16 + j], wt.w2[i * 16 + j]);
-#pragma unroll
-            for (int q = 0; q < 8; ++q) {
-                const int s = 2 * q + j + 1;  // x index of output column 2q for tap j
-                const float2 xp = (s & 1) ? xo[s >> 1] : xe[s >> 1];
-                a1[q] = __ffma2_rn(xp, w1, a1[q]);
-                a2[q] = __ffma2_rn(xp, w2, a2[q]);
-            }
-        }
-    }
-    float acc1[16], acc2[16];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-        acc1[2 * q] = a1[q].x;
-        acc1[2 * q + 1] = a1[q].y;
-        acc2[2 * q] = a2[q].x;
-        acc2[2 * q + 1] = a2[q].y;
-    }
-
-    // epilogue: remaps and the 4-way max fold (x > m) ? x : m in order E1, E2, E5, E6
-    const int64_t row = tile_r0 + lr;
-    if (row >= a.out_row0 + a.out_rows) return;
+    // Filters are processed two at a time; the combine op folds each pair's responses into e[]
+    // (8 orientations = 4 convolutions = 2 passes over the same staged tile).
     float e[16];
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
-        const float e1 = acc1[q], e2 = acc2[q], e5 = -e1, e6 = -e2;
-        float m = e1;
-        m = (e2 > m) ? e2 : m;
-        m = (e5 > m) ? e5 : m;
-        m = (e6 > m) ? e6 : m;
-        e[q] = m;
+    for (int q = 0; q < 16; ++q) e[q] = 0.f;
+#pragma unroll 1
+    for (int fp = 0; 2 * fp < a.nf; ++fp) {
+        float2 a1[8], a2[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            a1[q] = make_float2(0.f, 0.f);
+            a2[q] = make_float2(0.f, 0.f);
+        }
+        const float* wf1 = wt.w[2 * fp];
+        const float* wf2 = wt.w[2 * fp + 1];
+#pragma unroll 1
+        for (int i = 0; i < 16; ++i) {
+            // input window: smem cols [cb, cb+32) <-> image cols [c0+cb-8, c0+cb+24);
+            // output column c0+cb+q, tap j reads image col c0+cb+q+j-7 = smem col cb+q+j+1
+            float2 xe[16], xo[16];  // xe[k] = (x[2k], x[2k+1]), xo[k] = (x[2k+1], x[2k+2])
+            const float4* r0 = reinterpret_cast<const float4*>(&xs[(lr + i) * kPitch + cb]);
+            const float4* r1 = reinterpret_cast<const float4*>(&xs1[(lr + i) * kPitch + cb]);
+#pragma unroll
+            for (int v = 0; v < 8; ++v) {
+                const float4 t = r0[v];
+                const float4 u = r1[v];
+                xe[2 * v] = make_float2(t.x, t.y);
+                xe[2 * v + 1] = make_float2(t.z, t.w);
+                xo[2 * v] = make_float2(u.x, u.y);
+                xo[2 * v + 1] = make_float2(u.z, u.w);
+            }
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                const float2 w1 = make_float2(wf1[i * 16 + j], wf1[i * 16 + j]);
+                const float2 w2 = make_float2(wf2[i * 16 + j], wf2[i * 16 + j]);
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                    const int s = 2 * q + j + 1;  // x index of output column 2q for tap j
+                    const float2 xp = (s & 1) ? xo[s >> 1] : xe[s >> 1];
+                    a1[q] = __ffma2_rn(xp, w1, a1[q]);
+                    a2[q] = __ffma2_rn(xp, w2, a2[q]);
+                }
+            }
+        }
+        // combine (x > m) ? x : m folds; sum = left fold of fp32 adds
+        const bool has2 = 2 * fp + 1 < a.nf;
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+            const float e1 = (q & 1) ? a1[q >> 1].y : a1[q >> 1].x;
+            const float e2 = (q & 1) ? a2[q >> 1].y : a2[q >> 1].x;
+            float m = e[q];
+            switch (a.combine) {
+                case 1:  // SUM
+                    m = fp == 0 ? e1 : m + e1;
+                    if (has2) m = m + e2;
+                    break;
+                case 2:  // MAXABS
+                    m = fp == 0 ? fabsf(e1) : ((fabsf(e1) > m) ? fabsf(e1) : m);
+                    if (has2) m = (fabsf(e2) > m) ? fabsf(e2) : m;
+                    break;
+                case 3:  // plain max of the responses
+                    m = fp == 0 ? e1 : ((e1 > m) ? e1 : m);
+                    if (has2) m = (e2 > m) ? e2 : m;
+                    break;
+                default:  // MAX over the responses and their remaps (negations): E1, E2, -E1, -E2
+                    m = fp == 0 ? e1 : ((e1 > m) ? e1 : m);
+                    if (has2) m = (e2 > m) ? e2 : m;
+                    m = (-e1 > m) ? -e1 : m;
+                    if (has2) m = (-e2 > m) ? -e2 : m;
+            }
+            e[q] = m;
+        }
     }
+
+    const int64_t row = tile_r0 + lr;
+    if (row >= a.out_row0 + a.out_rows) return;
     float* orow = a.out + img * a.out_img_stride + (row - a.out_row0) * a.W;
     const int64_t c0 = tile_c0 + cb;
     const bool ovec = (a.W & 3) == 0 && ((reinterpret_cast<uintptr_t>(a.out) & 15) == 0) &&
@@ -282,13 +301,12 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     // filters embedded in a 16 x 16 frame at offset 7 - (ks-1)/2 (zeros elsewhere)
+    if (a.nf < 1 || a.nf > 4) return cudaErrorInvalidValue;
     EdgeWeights wt{};
     const int off = 7 - (a.ks - 1) / 2;
-    for (int r = 0; r < a.ks; ++r)
-        for (int c = 0; c < a.ks; ++c) {
-            wt.w1[(r + off) * 16 + c + off] = a.k1_host[r * a.ks + c];
-            wt.w2[(r + off) * 16 + c + off] = a.k2_host[r * a.ks + c];
-        }
+    for (int f = 0; f < a.nf; ++f)
+        for (int r = 0; r < a.ks; ++r)
+            for (int c = 0; c < a.ks; ++c) wt.w[f][(r + off) * 16 + c + off] = a.k_host[f][r * a.ks + c];
     const int tiles_c = (int)((a.W + kTileC - 1) / kTileC);
     const int tiles_r = (int)((a.out_rows + kTileR - 1) / kTileR);
     PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();

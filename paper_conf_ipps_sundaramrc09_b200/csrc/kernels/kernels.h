@@ -8,7 +8,8 @@ namespace tg {
 
 // K1: the whole edge template as one kernel per chunk (the paper's "best
 // possible" single kernel): E = max(Im*K1, Im*K2, -(Im*K1), -(Im*K2)),
-// SAME zero padding. Rows are in GLOBAL image coordinates; rows outside [0, H) are zero.
+// SAME zero padding; generally nf <= 4 convolutions combined by max (with remaps), sum,
+// max-abs or plain max. Rows are in GLOBAL image coordinates; rows outside [0, H) are zero.
 struct EdgeArgs {
     const float* in;        // image rows [in_row0, in_row0 + in_rows) of nimg images
     int64_t in_img_stride;  // floats between consecutive images in `in`
@@ -18,9 +19,10 @@ struct EdgeArgs {
     int64_t out_row0, out_rows;
     int64_t H, W;           // full image size
     int64_t nimg;
-    const float* k1_host;   // ks x ks filters (host; passed to the kernel by value)
-    const float* k2_host;
+    const float* k_host[4]; // nf ks x ks filters (host; passed to the kernel by value)
+    int nf;                 // 1..4 convolutions
     int ks;                 // 1..16
+    int combine;            // 0 max over responses and remaps, 1 sum, 2 max |.|, 3 max
 };
 cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s);
 

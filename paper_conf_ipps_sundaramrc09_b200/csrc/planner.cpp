@@ -36,43 +36,73 @@ static bool is_same_conv_1ch(const Graph& g, const Node* n) {
     return K.d[0] == 1 && K.d[1] == 1 && K.d[2] == K.d[3] && K.d[2] >= 1 && K.d[2] <= 16;
 }
 
+// Edge template (Fig. 1(b)): 1..4 SAME convolutions of one image combined by
+//   max over the responses and their remaps (negations)   [combine 0, the paper's template]
+//   sum of the responses                                   [combine 1, "addition"]
+//   max of |response|                                      [combine 2, "max absolute value"]
+//   max of the responses                                   [combine 3]
 static tg_status recognise_edge(const Graph& g, int out, Template& t) {
-    const Node* mx = producer(g, out);
-    if (!mx || mx->op != OpKind::Max || mx->ins.size() != 4) return TG_E_UNSUPPORTED;
+    const Node* top = producer(g, out);
+    if (!top) return TG_E_UNSUPPORTED;
+    const bool is_max = top->op == OpKind::Max;
+    const bool is_sum = top->op == OpKind::Elem && top->elem == TG_ADD;
+    if (!is_max && !is_sum) return TG_E_UNSUPPORTED;
     std::vector<const Node*> convs;
-    std::vector<int> conv_out;
-    std::vector<int> negated;
-    for (int x : mx->ins) {
+    std::vector<int> conv_out, negated, absed;
+    for (int x : top->ins) {
         const Node* p = producer(g, x);
-        if (p && p->op == OpKind::Elem && p->elem == TG_NEG) {
-            negated.push_back(p->ins[0]);
-        } else if (is_same_conv_1ch(g, p)) {
+        if (is_same_conv_1ch(g, p)) {
             convs.push_back(p);
             conv_out.push_back(x);
+        } else if (p && p->op == OpKind::Elem && p->elem == TG_NEG) {
+            negated.push_back(p->ins[0]);
+        } else if (p && p->op == OpKind::Elem && p->elem == TG_ABS) {
+            absed.push_back(p->ins[0]);
         } else {
             return TG_E_UNSUPPORTED;
         }
     }
-    if (convs.size() != 2 || negated.size() != 2) return TG_E_UNSUPPORTED;
-    // the remaps must negate exactly the two convolution outputs
-    if (!((negated[0] == conv_out[0] && negated[1] == conv_out[1]) ||
-          (negated[0] == conv_out[1] && negated[1] == conv_out[0])))
-        return TG_E_UNSUPPORTED;
-    if (convs[0]->ins[0] != convs[1]->ins[0]) return TG_E_UNSUPPORTED;
+    int combine;
+    if (is_sum) {
+        if (!negated.empty() || !absed.empty()) return TG_E_UNSUPPORTED;
+        combine = 1;
+    } else if (!absed.empty()) {
+        if (!convs.empty() || !negated.empty()) return TG_E_UNSUPPORTED;
+        for (int x : absed) {
+            const Node* p = producer(g, x);
+            if (!is_same_conv_1ch(g, p)) return TG_E_UNSUPPORTED;
+            convs.push_back(p);
+            conv_out.push_back(x);
+        }
+        combine = 2;
+    } else if (!negated.empty()) {
+        // the remaps must negate exactly the convolution outputs (each once)
+        std::vector<int> a = negated, b = conv_out;
+        std::sort(a.begin(), a.end());
+        std::sort(b.begin(), b.end());
+        if (a != b || std::adjacent_find(a.begin(), a.end()) != a.end()) return TG_E_UNSUPPORTED;
+        combine = 0;
+    } else {
+        combine = 3;
+    }
+    if (convs.empty() || convs.size() > 4) return TG_E_UNSUPPORTED;
     const int x = convs[0]->ins[0];
     const Ds& X = g.ds[x];
     if (X.kind != DsKind::Input || X.d[1] != 1) return TG_E_UNSUPPORTED;
-    const int ka = convs[0]->ins[1], kb = convs[1]->ins[1];
-    if (g.ds[ka].d[2] != g.ds[kb].d[2]) return TG_E_UNSUPPORTED;
+    for (const Node* c : convs)
+        if (c->ins[0] != x || g.ds[c->ins[1]].d[2] != g.ds[convs[0]->ins[1]].d[2]) return TG_E_UNSUPPORTED;
     t.kind = Tmpl::Edge;
     t.input = x;
     t.output = out;
     t.n = X.d[0];
     t.H = X.d[2];
     t.W = X.d[3];
-    t.ks = (int)g.ds[ka].d[2];
-    t.k1 = ka;
-    t.k2 = kb;
+    t.ks = (int)g.ds[convs[0]->ins[1]].d[2];
+    t.nf = (int)convs.size();
+    t.combine = combine;
+    for (int f = 0; f < t.nf; ++f) t.kk[f] = convs[f]->ins[1];
+    t.k1 = t.kk[0];
+    t.k2 = t.nf > 1 ? t.kk[1] : -1;
     return TG_OK;
 }
 
@@ -280,8 +310,8 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     std::vector<int> prm;
     std::vector<bool> is_bias;
     if (t.kind == Tmpl::Edge) {
-        prm = {t.k1, t.k2};
-        is_bias = {false, false};
+        prm.assign(t.kk, t.kk + t.nf);
+        is_bias.assign(t.nf, false);
     } else {
         prm.assign(t.prm, t.prm + 10);
         is_bias = {false, true, false, false, true, false, false, true, false, true};
@@ -446,11 +476,13 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     uint64_t param_floats = 0;
     for (int id : prm) param_floats += (uint64_t)g.ds[id].numel();
     if (t.kind == Tmpl::Edge) {
-        const uint64_t S = (uint64_t)H * W;
+        const uint64_t S = (uint64_t)H * W, k = (uint64_t)t.nf;
+        // per image: Im, the k responses, k remaps / abs (combine 0, 2), the combined output
+        const uint64_t planes = (t.combine == 0 || t.combine == 2) ? 2 * k + 2 : k + 2;
         p.io_lb = ((uint64_t)n * 2 * S + param_floats) * f;
-        p.total = ((uint64_t)n * 6 * S + param_floats) * f;  // Im, E1, E2, E5, E6, E
-        p.nops = 5;                                          // C1 C2 R1 R2 max
-        p.nds = 8;                                           // Im K1 K2 E1 E2 E5 E6 E
+        p.total = ((uint64_t)n * planes * S + param_floats) * f;  // 4 orientations: Im E1 E2 E5 E6 E
+        p.nops = (int64_t)(planes - 1);                            // convolutions (+remaps) + combine
+        p.nds = (int64_t)(planes + k);                             // + the k kernels
         p.n_units = 1;
     } else {
         const uint64_t A0 = (uint64_t)H * W, A1 = (uint64_t)t.h[1] * t.w[1], A2 = (uint64_t)t.h[2] * t.w[2],
@@ -487,6 +519,8 @@ std::string plan_json(const PlanCore& p) {
     o << "\"template\": \"" << (t.kind == Tmpl::Edge ? "edge" : "cnn") << "\", ";
     o << "\"n\": " << t.n << ", \"H\": " << t.H << ", \"W\": " << t.W << ", ";
     o << "\"ks\": " << (t.kind == Tmpl::Edge ? t.ks : 0) << ", \"n5\": " << (t.kind == Tmpl::Cnn ? t.n5 : 0) << ", ";
+    static const char* kComb[4] = {"max", "sum", "maxabs", "maxplain"};
+    o << "\"nf\": " << (t.kind == Tmpl::Edge ? t.nf : 0) << ", \"combine\": \"" << (t.kind == Tmpl::Edge ? kComb[t.combine] : "none") << "\", ";
     o << "\"budget\": " << p.budget << ", \"depth\": " << p.depth << ", \"max_chunk_px\": " << p.max_chunk_px << ", ";
     o << "\"device_io\": " << (p.device_io ? "true" : "false") << ", ";
     o << "\"precision\": \"" << (t.kind == Tmpl::Cnn && p.precision == TG_BF16_TC ? "bf16_tc" : "fp32") << "\", ";

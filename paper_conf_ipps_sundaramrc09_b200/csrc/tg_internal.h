@@ -79,6 +79,9 @@ struct Template {
     // edge
     int ks = 16;
     int k1 = -1, k2 = -1;  // kernel DS ids (fold order E1, E2, -E1, -E2)
+    int nf = 2;            // convolutions (orientations with remaps = 2 nf)
+    int kk[4] = {-1, -1, -1, -1};
+    int combine = 0;       // 0 max with remaps, 1 sum, 2 max |.|, 3 max
     // cnn
     int n5 = 0;
     bool bias_plane = true;

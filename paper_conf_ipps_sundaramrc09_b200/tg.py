@@ -512,6 +512,42 @@ def edge_graph(img, K1, K2=None, out=None, device: bool = False) -> tuple[Graph,
     return g, e
 
 
+def edge_graph_general(img, kernels, combine: str = "max", out=None, device: bool = False) -> tuple[Graph, int]:
+    """Edge graph from primitives with explicit filters: len(kernels) SAME convolutions combined
+    by 'max' (responses and their remaps), 'sum', 'maxabs' or 'maxplain'."""
+    g = Graph()
+    x = g.input(img, device=device)
+    resp = []
+    for K in kernels:
+        k = g.param(np.asarray(K, np.float32).reshape(1, 1, *np.shape(K)[-2:]))
+        resp.append(g.conv2d(x, k, -1, TG_SAME))
+    if combine == "max":
+        e = g.max_combine(resp + [g.neg(r) for r in resp])
+    elif combine == "sum":
+        e = tg_elementwise(g.h, TG_ADD, resp)
+    elif combine == "maxabs":
+        e = g.max_combine([tg_elementwise(g.h, TG_ABS, [r]) for r in resp])
+    elif combine == "maxplain":
+        e = g.max_combine(resp)
+    else:
+        raise ValueError(combine)
+    if out is not None:
+        g.output(e, out, device=device)
+    return g, e
+
+
+def find_edges_graph(img, kernel, num_orientations: int = 4, combine_op: int = TG_MAX, out=None,
+                     device: bool = False) -> tuple[Graph, int]:
+    """find_edges(Image, Kernel, num_orientations, Combine_op) (PAPER.md:623)."""
+    g = Graph()
+    x = g.input(img, device=device)
+    k = g.param(np.asarray(kernel, np.float32).reshape(1, 1, *np.shape(kernel)[-2:]))
+    e = g.find_edges(x, k, num_orientations, combine_op)
+    if out is not None:
+        g.output(e, out, device=device)
+    return g, e
+
+
 def cnn_graph(img, n5: int, params, out=None, bias_mode=TG_BIAS_PLANE, device: bool = False) -> tuple[Graph, int]:
     g = Graph()
     x = g.input(img, device=device)

@@ -158,3 +158,61 @@ def test_two_host_threads_same_device(tg, orc):
     p.execute()
     assert p.stats()["n_chunks"] >= 4
     assert np.array_equal(out, ref)
+
+
+@pytest.mark.parametrize("nf", [1, 2, 3, 4])
+@pytest.mark.parametrize("combine", ["max", "sum", "maxabs", "maxplain"])
+def test_edge_general_combines(tg, orc, nf, combine):
+    """Up to 4 convolutions (8 orientations, Fig. 1(b)) and the reductions of PAPER.md:621 in one
+    fused K1 launch, split into chunks by a budget."""
+    img = synth.images_np(31, 2, 150, 132)
+    rs = np.random.default_rng(nf)
+    K = [(rs.standard_normal((16, 16)) / 16).astype(np.float32) for _ in range(nf)]
+    out = np.zeros_like(img)
+    g, _ = tg.edge_graph_general(img, K, combine, out=out)
+    g.set(budget=250_000, torch_runtime=True)
+    p = g.plan()
+    assert p.json()["nf"] == nf and p.json()["combine"] == combine and p.json()["n_chunks"] > 2
+    p.execute()
+    ref = np.stack([orc.edge_general(img[b, 0], K, combine) for b in range(2)])[:, None]
+    assert normwise(out, ref) <= 1e-5
+
+
+def _rot(K, deg):
+    """Test-side restatement of reading R18 (kernel rotation about its centre)."""
+    k = K.shape[0]
+    if deg % 90 == 0:
+        return np.ascontiguousarray(np.rot90(K, deg // 90))
+    th = np.deg2rad(deg)
+    c0 = (k - 1) / 2.0
+    R = np.zeros_like(K)
+    for i in range(k):
+        for j in range(k):
+            y, x = i - c0, j - c0
+            sr, sc = c0 + y * np.cos(th) + x * np.sin(th), c0 - y * np.sin(th) + x * np.cos(th)
+            r0, q0 = int(np.floor(sr)), int(np.floor(sc))
+            fr, fc = sr - r0, sc - q0
+            v = 0.0
+            for dr in (0, 1):
+                for dc in (0, 1):
+                    rr, cc = r0 + dr, q0 + dc
+                    if 0 <= rr < k and 0 <= cc < k:
+                        v += (fr if dr else 1 - fr) * (fc if dc else 1 - fc) * float(K[rr, cc])
+            R[i, j] = np.float32(v)
+    return R
+
+
+@pytest.mark.parametrize("n_or,comb", [(8, "max"), (8, "sum"), (4, "maxabs"), (2, "max")])
+def test_find_edges_orientations(tg, orc, n_or, comb):
+    """find_edges(Image, Kernel, num_orientations, Combine_op) with the rotations
+    of reading R18 (8 orientations: 0, 45, 90, 135 degrees + remaps)."""
+    img = synth.images_np(41, 1, 200, 180)
+    K1, _ = synth.edge_filter_np()
+    code = {"max": tg.TG_MAX, "sum": tg.TG_SUM, "maxabs": tg.TG_MAXABS}[comb]
+    out = np.zeros_like(img)
+    g, _ = tg.find_edges_graph(img, K1, n_or, code, out=out)
+    g.set(torch_runtime=True)
+    g.plan().execute()
+    Ks = [_rot(K1, i * 360 // n_or) for i in range(n_or // 2)]
+    ref = orc.edge_general(img[0, 0], Ks, comb)
+    assert normwise(out[0], ref[None]) <= 1e-5

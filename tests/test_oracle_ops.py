@@ -145,3 +145,17 @@ def test_edge_invariant_abs_max(orc):
     # K2 = rot90(K1) and C1, C2 are independent convolutions
     assert np.array_equal(E1, orc.conv2d_same(x, K1))
     assert np.array_equal(E2, orc.conv2d_same(x, K2))
+
+
+def test_edge_general_reduces_to_pinned_template(orc):
+    """edge_general composes pinned operators; with 2 filters and 'max' it IS the 4-orientation
+    template, and the other reductions obey their definitions exactly."""
+    x = f32(rng.random((40, 52)))
+    K = [f32(rng.standard_normal((16, 16))) for _ in range(4)]
+    assert np.array_equal(orc.edge_general(x, K[:2], "max"), orc.edge(x, K[0], K[1]))
+    E = [orc.conv2d_same(x, k) for k in K]
+    assert np.array_equal(orc.edge_general(x, K, "maxabs"), np.max(np.abs(np.stack(E)), axis=0))
+    assert np.array_equal(orc.edge_general(x, K, "maxplain"), np.max(np.stack(E), axis=0))
+    s = ((E[0] + E[1]) + E[2]) + E[3]          # fp32 left fold
+    assert np.array_equal(orc.edge_general(x, K, "sum"), s)
+    assert np.array_equal(orc.edge_general(x, K, "max"), np.max(np.abs(np.stack(E)), axis=0))

@@ -31,6 +31,10 @@ CASES = [
     ("cnn", 64, 480, 640, dict(n5=120, device_io=True, budget=2 << 30)),
     ("cnn", 1, 4800, 6400, dict(n5=120, budget=1536 << 20, rank=1, world=2)),
     ("cnn", 64, 480, 640, dict(n5=120, precision="bf16_tc")),
+    ("edge", 2, 500, 400, dict(orient=8, comb="max", budget=2_000_000)),
+    ("edge", 1, 300, 200, dict(orient=8, comb="sum")),
+    ("edge", 3, 100, 64, dict(orient=2, comb="maxabs", budget=90_000)),
+    ("edge", 1, 64, 64, dict(orient=4, comb="maxabs")),
     ("cnn", 1, 4800, 6400, dict(n5=120, budget=1536 << 20, precision="bf16_tc")),
     ("cnn", 3, 200, 180, dict(n5=37, budget=2_000_000, precision="bf16_tc")),
 ]
@@ -51,7 +55,8 @@ def library_plan(tmpl, n, H, W, kw):
     if tmpl == "edge":
         ks = kw.get("ks", 16)
         k1 = g.param(np.ones((1, 1, ks, ks), np.float32))
-        y = g.find_edges(x, k1)
+        comb = {"max": tg.TG_MAX, "sum": tg.TG_SUM, "maxabs": tg.TG_MAXABS}[kw.get("comb", "max")]
+        y = g.find_edges(x, k1, kw.get("orient", 4), comb)
     else:
         n5 = kw["n5"]
         bias = kw.get("bias", "plane")
@@ -85,7 +90,10 @@ def library_plan(tmpl, n, H, W, kw):
 def test_plan_matches_oracle(case):
     tmpl, n, H, W, kw = case
     got = library_plan(tmpl, n, H, W, kw)
-    okw = {k: v for k, v in kw.items()}
+    okw = {k: v for k, v in kw.items() if k not in ("orient", "comb")}
+    if tmpl == "edge":
+        okw["nf"] = kw.get("orient", 4) // 2
+        okw["combine"] = kw.get("comb", "max")
     want = P.fused_plan(tmpl, n, H, W, **okw)
     assert set(got) == set(want)
     for k in want:
