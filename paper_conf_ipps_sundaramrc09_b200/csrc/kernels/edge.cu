@@ -58,6 +58,7 @@ struct EdgeWeights {
 
 // Compute the 64 x 64 output tile whose input (+halo) is staged at xs (pitch kPitch, smem
 // (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)) and store it.
+template <int kComb, int kPairs>
 __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const float* __restrict__ xs1,
                                           const EdgeArgs& a, const EdgeWeights& wt, int64_t img, int64_t tile_r0,
                                           int64_t tile_c0) {
@@ -75,8 +76,8 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const fl
     float e[16];
 #pragma unroll
     for (int q = 0; q < 16; ++q) e[q] = 0.f;
-#pragma unroll 1
-    for (int fp = 0; 2 * fp < a.nf; ++fp) {
+#pragma unroll
+    for (int fp = 0; fp < kPairs; ++fp) {  // compile-time: constant-bank weight offsets
         float2 a1[8], a2[8];
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
@@ -121,7 +122,7 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const fl
             const float e1 = (q & 1) ? a1[q >> 1].y : a1[q >> 1].x;
             const float e2 = (q & 1) ? a2[q >> 1].y : a2[q >> 1].x;
             float m = e[q];
-            switch (a.combine) {
+            switch (kComb) {
                 case 1:  // SUM
                     m = fp == 0 ? e1 : m + e1;
                     if (has2) m = m + e2;
@@ -163,6 +164,7 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const fl
 }
 
 // ---------------------------------------------------------------------------- fallback
+template <int kComb, int kPairs>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
     extern __shared__ __align__(16) float smf[];
@@ -200,7 +202,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         xs1[sr * kPitch + sc] = sc + 1 < kSmC ? xs[sr * kPitch + sc + 1] : 0.f;
     }
     __syncthreads();
-    edge_tile(xs, xs1, a, wt, img, tile_r0, tile_c0);
+    edge_tile<kComb, kPairs>(xs, xs1, a, wt, img, tile_r0, tile_c0);
 }
 
 // ---------------------------------------------------------------------------- TMA path
@@ -208,6 +210,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+template <int kComb, int kPairs>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_tma_kernel(const __grid_constant__ CUtensorMap tmap, const EdgeArgs a,
                           const __grid_constant__ EdgeWeights wt, const int tiles_c, const int tiles_r,
@@ -278,7 +281,7 @@ __global__ void __launch_bounds__(kThreads, 2)
             *reinterpret_cast<float4*>(&xs1[sr * kPitch + 4 * q]) = make_float4(lo.y, lo.z, lo.w, hi.x);
         }
         __syncthreads();
-        edge_tile(tb, xs1, a, wt, img, tr0, tc0);
+        edge_tile<kComb, kPairs>(tb, xs1, a, wt, img, tr0, tc0);
         __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
     }
 }
@@ -298,7 +301,27 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 
 }  // namespace
 
+template <int kComb, int kPairs>
+cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s);
+
+template <int kPairs>
+cudaError_t launch_edge_p(const EdgeArgs& a, cudaStream_t s) {
+    switch (a.combine) {
+        case 0: return launch_edge_t<0, kPairs>(a, s);
+        case 1: return launch_edge_t<1, kPairs>(a, s);
+        case 2: return launch_edge_t<2, kPairs>(a, s);
+        case 3: return launch_edge_t<3, kPairs>(a, s);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
 cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
+    if (a.nf < 1 || a.nf > 4) return cudaErrorInvalidValue;
+    return a.nf <= 2 ? launch_edge_p<1>(a, s) : launch_edge_p<2>(a, s);
+}
+
+template <int kComb, int kPairs>
+cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     // filters embedded in a 16 x 16 frame at offset 7 - (ks-1)/2 (zeros elsewhere)
     if (a.nf < 1 || a.nf > 4) return cudaErrorInvalidValue;
@@ -329,13 +352,13 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
             const size_t smem = 3 * (size_t)kBufStride + 128;
             if (!(configured.load() & (1u << (dev & 31)))) {
                 cudaError_t e =
-                    cudaFuncSetAttribute(edge_fused_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                    cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
                 if (e != cudaSuccess) return e;
                 configured.fetch_or(1u << (dev & 31));
             }
             const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
             const int64_t grid = std::min<int64_t>(ntiles, 2 * (int64_t)sms);
-            edge_fused_tma_kernel<<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
+            edge_fused_tma_kernel<kComb, kPairs><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
             return cudaGetLastError();
         }
     }
@@ -346,11 +369,11 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
     cudaGetDevice(&dev);
     const size_t fsmem = 2 * (size_t)kSmR * kPitch * 4;
     if (!(fb_configured.load() & (1u << (dev & 31)))) {
-        cudaError_t e = cudaFuncSetAttribute(edge_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem);
+        cudaError_t e = cudaFuncSetAttribute(edge_fused_kernel<kComb, kPairs>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem);
         if (e != cudaSuccess) return e;
         fb_configured.fetch_or(1u << (dev & 31));
     }
-    edge_fused_kernel<<<grid, kThreads, fsmem, s>>>(a, wt);
+    edge_fused_kernel<kComb, kPairs><<<grid, kThreads, fsmem, s>>>(a, wt);
     return cudaGetLastError();
 }
 
