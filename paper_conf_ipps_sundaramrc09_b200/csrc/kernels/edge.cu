@@ -10,13 +10,14 @@
 // 7 - (ks-1)/2 so one code path serves every size (zero taps add exact zeros).
 //
 // Roofline: 2 x 256 FMA per output pixel vs 8 HBM bytes -> FP32-ALU
-// bound (128 flop/B >> ridge ~11 flop/B). The kernel is therefore organised to issue
-// FFMA back to back: each thread owns a 1 x 16 strip of outputs for both filters
-// (32 accumulators), and for each of the 16 filter rows loads its 32-wide input window
-// with 8 conflict-free LDS.128 and both filter rows from the constant bank (uniform
-// registers), then issues 512 FFMA -- under 3% load overhead. Tiles of 64 x 64 outputs,
-// 256 threads; lanes of a warp own 32 consecutive rows (row pitch 84 floats = 21 x 16 B,
-// odd, so the 8 lanes of each LDS.128 phase hit 8 distinct 16-byte bank groups).
+// bound (128 flop/B >> ridge ~11 flop/B). The kernel is organised to keep the FMA pipe busy:
+// each thread owns a 1 x 16 strip of outputs; per filter row it loads its 32-wide input
+// window with 8 conflict-free LDS.128 and issues 256 FFMA2 (paired FP32 FMA, sm_100) that
+// update BOTH filters' accumulators at once: (E1[q], E2[q]) += x[q+j+1] * (K1[i][j], K2[i][j]),
+// the x operand broadcast from one register and the weight pair a uniform register loaded
+// from the constant bank (__grid_constant__ parameter). Tiles of 64 x 64 outputs, 256
+// threads; lanes of a warp own 32 consecutive rows (row pitch 84 floats = 21 x 16 B, odd,
+// so the 8 lanes of each LDS.128 phase hit 8 distinct 16-byte bank groups).
 //
 // Tile staging. Main path (W % 4 == 0): a persistent grid (2 CTAs per SM) walks the tiles;
 // one thread issues a 3-D TMA load (cp.async.bulk.tensor, box 84 x 79 x 1) of the NEXT
@@ -53,74 +54,59 @@ constexpr int kBufStride = (kTileBytes + 127) / 128 * 128;
 // register (FFMA R, R, UR, R) -- only two vector-register operands per FFMA, which keeps
 // the register-file banks out of the way of the FMA pipe.
 struct EdgeWeights {
-    float w[4][256];  // up to 4 filters, processed in pairs; broadcast to both lanes of an FFMA2
+    float2 w[2][256];  // filter pairs (2p, 2p+1) interleaved per tap: one FFMA2 weight operand
 };
 
 // Compute the 64 x 64 output tile whose input (+halo) is staged at xs (pitch kPitch, smem
 // (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)) and store it.
 template <int kComb, int kPairs>
-__device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const float* __restrict__ xs1,
-                                          const EdgeArgs& a, const EdgeWeights& wt, int64_t img, int64_t tile_r0,
-                                          int64_t tile_c0) {
+__device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const EdgeArgs& a, const EdgeWeights& wt,
+                                          int64_t img, int64_t tile_r0, int64_t tile_c0) {
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
     const int lr = (warp >> 2) * 32 + lane;  // local output row
     const int cb = (warp & 3) * 16;          // local output column base
 
-    // Paired FP32 FMA (FFMA2, sm_100): one instruction updates the accumulators of two
-    // adjacent output columns; each lane rounds exactly like fmaf, so results are bit-identical
-    // to scalar FMAs in the same order. The pair (x[s], x[s+1]) for an odd s comes from the
-    // second copy of the tile, staged one column to the left (xs1[c] = xs[c+1]).
-    // Filters are processed two at a time; the combine op folds each pair's responses into e[]
-    // (8 orientations = 4 convolutions = 2 passes over the same staged tile).
+    // Paired FP32 FMA (FFMA2, sm_100) over a PAIR OF FILTERS: acc[q] = (E_2p[q], E_2p+1[q]) +=
+    // x[q+j+1] (register, broadcast to both lanes) * (K_2p[i][j], K_2p+1[i][j]) (uniform-register
+    // pair from the constant bank). Each lane rounds exactly like fmaf, in the same (i, j) order
+    // as a scalar loop. Filter pairs run one after the other over the same staged tile, and the
+    // combine op folds each pair into e[] (8 orientations = 4 convolutions = 2 pairs).
     float e[16];
 #pragma unroll
     for (int q = 0; q < 16; ++q) e[q] = 0.f;
 #pragma unroll
     for (int fp = 0; fp < kPairs; ++fp) {  // compile-time: constant-bank weight offsets
-        float2 a1[8], a2[8];
+        float2 acc[16];
 #pragma unroll
-        for (int q = 0; q < 8; ++q) {
-            a1[q] = make_float2(0.f, 0.f);
-            a2[q] = make_float2(0.f, 0.f);
-        }
-        const float* wf1 = wt.w[2 * fp];
-        const float* wf2 = wt.w[2 * fp + 1];
+        for (int q = 0; q < 16; ++q) acc[q] = make_float2(0.f, 0.f);
 #pragma unroll 1
         for (int i = 0; i < 16; ++i) {
             // input window: smem cols [cb, cb+32) <-> image cols [c0+cb-8, c0+cb+24);
             // output column c0+cb+q, tap j reads image col c0+cb+q+j-7 = smem col cb+q+j+1
-            float2 xe[16], xo[16];  // xe[k] = (x[2k], x[2k+1]), xo[k] = (x[2k+1], x[2k+2])
-            const float4* r0 = reinterpret_cast<const float4*>(&xs[(lr + i) * kPitch + cb]);
-            const float4* r1 = reinterpret_cast<const float4*>(&xs1[(lr + i) * kPitch + cb]);
+            float x[32];
+            const float4* xr = reinterpret_cast<const float4*>(&xs[(lr + i) * kPitch + cb]);
 #pragma unroll
             for (int v = 0; v < 8; ++v) {
-                const float4 t = r0[v];
-                const float4 u = r1[v];
-                xe[2 * v] = make_float2(t.x, t.y);
-                xe[2 * v + 1] = make_float2(t.z, t.w);
-                xo[2 * v] = make_float2(u.x, u.y);
-                xo[2 * v + 1] = make_float2(u.z, u.w);
+                const float4 t = xr[v];
+                x[4 * v + 0] = t.x;
+                x[4 * v + 1] = t.y;
+                x[4 * v + 2] = t.z;
+                x[4 * v + 3] = t.w;
             }
 #pragma unroll
             for (int j = 0; j < 16; ++j) {
-                const float2 w1 = make_float2(wf1[i * 16 + j], wf1[i * 16 + j]);
-                const float2 w2 = make_float2(wf2[i * 16 + j], wf2[i * 16 + j]);
+                const float2 w = wt.w[fp][i * 16 + j];
 #pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                    const int s = 2 * q + j + 1;  // x index of output column 2q for tap j
-                    const float2 xp = (s & 1) ? xo[s >> 1] : xe[s >> 1];
-                    a1[q] = __ffma2_rn(xp, w1, a1[q]);
-                    a2[q] = __ffma2_rn(xp, w2, a2[q]);
-                }
+                for (int q = 0; q < 16; ++q)
+                    acc[q] = __ffma2_rn(make_float2(x[q + j + 1], x[q + j + 1]), w, acc[q]);
             }
         }
         // combine (x > m) ? x : m folds; sum = left fold of fp32 adds
         const bool has2 = 2 * fp + 1 < a.nf;
 #pragma unroll
         for (int q = 0; q < 16; ++q) {
-            const float e1 = (q & 1) ? a1[q >> 1].y : a1[q >> 1].x;
-            const float e2 = (q & 1) ? a2[q >> 1].y : a2[q >> 1].x;
+            const float e1 = acc[q].x, e2 = acc[q].y;
             float m = e[q];
             switch (kComb) {
                 case 1:  // SUM
@@ -167,9 +153,7 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const fl
 template <int kComb, int kPairs>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
-    extern __shared__ __align__(16) float smf[];
-    float* xs = smf;
-    float* xs1 = smf + kSmR * kPitch;  // the same tile shifted left by one column
+    __shared__ __align__(16) float xs[kSmR * kPitch];
     const int tid = threadIdx.x;
     const int64_t img = blockIdx.z;
     const int64_t tile_r0 = a.out_row0 + (int64_t)blockIdx.y * kTileR;  // global output row
@@ -197,12 +181,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         *reinterpret_cast<float4*>(&xs[sr * kPitch + 4 * q]) = v;
     }
     __syncthreads();
-    for (int idx = tid; idx < kSmR * kSmC; idx += kThreads) {
-        const int sr = idx / kSmC, sc = idx - sr * kSmC;
-        xs1[sr * kPitch + sc] = sc + 1 < kSmC ? xs[sr * kPitch + sc + 1] : 0.f;
-    }
-    __syncthreads();
-    edge_tile<kComb, kPairs>(xs, xs1, a, wt, img, tile_r0, tile_c0);
+    edge_tile<kComb, kPairs>(xs, a, wt, img, tile_r0, tile_c0);
 }
 
 // ---------------------------------------------------------------------------- TMA path
@@ -221,7 +200,6 @@ __global__ void __launch_bounds__(kThreads, 2)
     uint8_t* base = smraw + ((128 - (smem_u32(smraw) & 127)) & 127);
     float* buf0 = reinterpret_cast<float*>(base);                   // TMA stage 0
     float* buf1 = reinterpret_cast<float*>(base + kBufStride);      // TMA stage 1
-    float* xs1 = reinterpret_cast<float*>(base + 2 * kBufStride);   // current tile shifted by one column
     __shared__ __align__(8) uint64_t full[2];
     const int tid = threadIdx.x;
     if (tid == 0) {
@@ -273,15 +251,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         int64_t img, tr0, tc0;
         coords(t, img, tr0, tc0);
         const float* tb = b ? buf1 : buf0;
-        // xs1[r][c] = tb[r][c+1] (128-bit loads/stores; column 79 of a row is never read)
-        for (int idx = threadIdx.x; idx < kSmR * (kSmC / 4); idx += kThreads) {
-            const int sr = idx / (kSmC / 4), q = idx - sr * (kSmC / 4);
-            const float4 lo = *reinterpret_cast<const float4*>(&tb[sr * kPitch + 4 * q]);
-            const float4 hi = *reinterpret_cast<const float4*>(&tb[sr * kPitch + 4 * q + 4]);
-            *reinterpret_cast<float4*>(&xs1[sr * kPitch + 4 * q]) = make_float4(lo.y, lo.z, lo.w, hi.x);
-        }
-        __syncthreads();
-        edge_tile<kComb, kPairs>(tb, xs1, a, wt, img, tr0, tc0);
+        edge_tile<kComb, kPairs>(tb, a, wt, img, tr0, tc0);
         __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
     }
 }
@@ -329,7 +299,10 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
     const int off = 7 - (a.ks - 1) / 2;
     for (int f = 0; f < a.nf; ++f)
         for (int r = 0; r < a.ks; ++r)
-            for (int c = 0; c < a.ks; ++c) wt.w[f][(r + off) * 16 + c + off] = a.k_host[f][r * a.ks + c];
+            for (int c = 0; c < a.ks; ++c) {
+                float2& w = wt.w[f >> 1][(r + off) * 16 + c + off];
+                (f & 1 ? w.y : w.x) = a.k_host[f][r * a.ks + c];
+            }
     const int tiles_c = (int)((a.W + kTileC - 1) / kTileC);
     const int tiles_r = (int)((a.out_rows + kTileR - 1) / kTileR);
     PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
@@ -349,7 +322,7 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
             int dev = 0, sms = 148;
             cudaGetDevice(&dev);
             cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            const size_t smem = 3 * (size_t)kBufStride + 128;
+            const size_t smem = 2 * (size_t)kBufStride + 128;
             if (!(configured.load() & (1u << (dev & 31)))) {
                 cudaError_t e =
                     cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -364,16 +337,7 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
     }
     dim3 grid((unsigned)tiles_c, (unsigned)tiles_r, (unsigned)a.nimg);
     if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
-    static std::atomic<uint32_t> fb_configured{0};
-    int dev = 0;
-    cudaGetDevice(&dev);
-    const size_t fsmem = 2 * (size_t)kSmR * kPitch * 4;
-    if (!(fb_configured.load() & (1u << (dev & 31)))) {
-        cudaError_t e = cudaFuncSetAttribute(edge_fused_kernel<kComb, kPairs>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem);
-        if (e != cudaSuccess) return e;
-        fb_configured.fetch_or(1u << (dev & 31));
-    }
-    edge_fused_kernel<kComb, kPairs><<<grid, kThreads, fsmem, s>>>(a, wt);
+    edge_fused_kernel<kComb, kPairs><<<grid, kThreads, 0, s>>>(a, wt);
     return cudaGetLastError();
 }
 
