@@ -387,6 +387,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.bf16_tc = c.precision == TG_BF16_TC;
         a.k5_tc = c.k5tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k5tc_off);
         a.n_pad = cnn_n5_pad(t.n5);
+        a.k6_host = g.ds[t.prm[8]].src;
         KernelTimer kt(x, d, 3, cs);
         CK(a.bf16_tc ? launch_cnn_u3_tc(a, cs) : launch_cnn_u3(a, cs));
         kt.done(cs);

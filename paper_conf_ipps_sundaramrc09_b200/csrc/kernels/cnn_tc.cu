@@ -20,6 +20,7 @@
 // Precision: bf16 operands, fp32 accumulation; parity bound 2e-2 normwise (R16).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstring>
 #include <vector>
@@ -154,180 +155,253 @@ __global__ void __launch_bounds__(kThreads) cnn_u2_tc_kernel(const CnnU2Args a) 
 }
 
 // ============================================================================ U3 (C5 + C6)
-// Band = 256 output positions (two M=128 tiles). Narrow images (w4 <= kFlatMax): positions are
-// the flattened (row, col) index over rows of pitch w4 (columns >= w5 are discarded); wide
-// images: one output row, columns [c0, c0+256), window pitch 262.
+// Warp-specialised and persistent (one CTA per SM, 9 warps):
+//   warp 8, one thread   producer + MMA issuer: per band, 1-D bulk copies (TMA engine) of the
+//                        input window into one of two A buffers; the 40 K-steps of the C5 B
+//                        operand stream through a 4-slot ring of bulk copies (the weights are the
+//                        same for every band); tcgen05.mma into one of two TMEM accumulators
+//                        (2 tiles x NP columns each); tcgen05.commit releases the ring slot, the
+//                        A buffer and hands the accumulator to the epilogue
+//   warps 0-7            epilogue: TMEM -> registers, bias plane + tanh, the 1x1 C6 layer as a
+//                        dot product over n5 (weights in the constant bank), + bias -> output
+// so the epilogue of band k overlaps the MMAs of band k+1 and the copies of band k+2.
+// Bands are 256 output positions (two M=128 tiles): narrow images (w4 <= kFlatMax) use the
+// flattened (row, col) index with the window pitch = w4 (columns >= w5 discarded; a window is
+// a run of whole T4 rows = one contiguous copy per channel block); wide images use 256-column
+// segments of one output row (window pitch 262, 5 row copies per block).
 constexpr int kFlatMax = 180;
-constexpr int U3_WR_COL = 5, U3_WP_COL = 2 * kTileM + 6;
-constexpr int U3_KS = 40, U3_KS_STAGE = 4;    // 40 K-steps streamed in stages of 4
+constexpr int U3_KS = 40, U3_KS_STAGE = 4, U3_STAGES = U3_KS / U3_KS_STAGE, U3_BRING = 4;
 constexpr int U3_NMAX = 128;
-// window pixels per channel block: flat mode <= (256 + 6 * w4) + 8, column mode 5 * 262 + 8
-constexpr int U3_APLANE_MAX = 1416;
-static_assert(2 * kTileM + 6 * kFlatMax + 8 <= U3_APLANE_MAX && U3_WR_COL * U3_WP_COL + 8 <= U3_APLANE_MAX, "window");
+constexpr int U3_WP_COL = 2 * kTileM + 6;
+constexpr int U3_APX = 1320;  // window pixels per block: flat <= 7*180+8, column 5*262+8
+constexpr int kEpiWarps = 8;
+constexpr int kThreadsU3 = (kEpiWarps + 1) * 32;
 
-struct U3TcShared {
-    uint4 a[3][U3_APLANE_MAX];                      // channel blocks 0-7, 8-15, 16-19(+4 zero)
-    uint4 b[2][U3_KS_STAGE * 2 * U3_NMAX];          // double-buffered B stages
-    float k6[U3_NMAX][12];                          // [ch][o] (9 used)
-    uint64_t mbar[2];
+struct U3K6 {
+    float k6[U3_NMAX][12];  // [ch][o] (9 used): C6 weights, broadcast from the constant bank
+};
+
+struct U3Smem {
+    uint4 a[2][3][U3_APX];                         // double-buffered window, 3 channel blocks
+    uint4 b[U3_BRING][U3_KS_STAGE * 2 * U3_NMAX];  // B ring (4 K-steps per slot)
+    uint64_t a_full[2], a_empty[2], b_full[U3_BRING], b_empty[U3_BRING], t_full[2], t_empty[2];
     uint32_t tmem;
 };
 
-constexpr int kThreadsU3 = 256;  // 8 warps: warps 0-3 drain tile 0, warps 4-7 tile 1
-
-__global__ void __launch_bounds__(kThreadsU3, 2) cnn_u3_tc_kernel(const CnnU3Args a) {
-    extern __shared__ __align__(128) uint8_t smraw[];
-    U3TcShared& S = *reinterpret_cast<U3TcShared*>(smraw);
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int NP = a.n_pad;                 // n5 padded to a multiple of 16 (<= 128)
-    const int64_t img = blockIdx.z;
-    const bool flat = a.w4 <= kFlatMax;
-    // ---- band geometry
-    int64_t q0, wr0;  // first position; first window row (global T4 row)
+struct U3Band {
+    int64_t img, q0, wr0, wc0;
     int WP, WR, base;
-    if (flat) {
-        q0 = (int64_t)blockIdx.x * 2 * kTileM;         // flattened over rows [out_row0, +out_rows)
-        const int64_t r_first = q0 / a.w4;
-        wr0 = a.out_row0 + r_first;
-        WP = (int)a.w4;
-        base = (int)(q0 - r_first * a.w4);
-        WR = (base + 2 * kTileM - 1) / WP + 1 + 4;  // rows the band spans + the 4-row halo
-    } else {
-        const int64_t bands_per_row = (a.w5 + 2 * kTileM - 1) / (2 * kTileM);
-        const int64_t row = blockIdx.x / bands_per_row;
-        q0 = (blockIdx.x - row * bands_per_row) * 2 * kTileM;  // column of position 0
-        wr0 = a.out_row0 + row;
-        WP = U3_WP_COL;
-        WR = U3_WR_COL;
-        base = 0;
-    }
-    const int plane_px = WR * WP + 8;  // + spare pixels (read by the zero-weight half of tap pair (4,5))
+};
 
-    if (warp == 0) tc::tmem_alloc<256>(&S.tmem);
+__device__ __forceinline__ U3Band u3_band(const CnnU3Args& a, int64_t band, int64_t per_img, bool flat) {
+    U3Band g;
+    g.img = band / per_img;
+    const int64_t bi = band - g.img * per_img;
+    if (flat) {
+        g.q0 = bi * 2 * kTileM;
+        const int64_t r_first = g.q0 / a.w4;
+        g.wr0 = a.out_row0 + r_first;
+        g.wc0 = 0;
+        g.WP = (int)a.w4;
+        g.base = (int)(g.q0 - r_first * a.w4);
+        g.WR = (g.base + 2 * kTileM - 1) / g.WP + 1 + 4;
+    } else {
+        const int64_t bpr = (a.w5 + 2 * kTileM - 1) / (2 * kTileM);
+        const int64_t row = bi / bpr;
+        g.q0 = (bi - row * bpr) * 2 * kTileM;
+        g.wr0 = a.out_row0 + row;
+        g.wc0 = g.q0;
+        g.WP = U3_WP_COL;
+        g.WR = 5;
+        g.base = 0;
+    }
+    return g;
+}
+
+__global__ void __launch_bounds__(kThreadsU3, 1)
+    cnn_u3_tc_kernel(const CnnU3Args a, const __grid_constant__ U3K6 k6w, const int64_t nbands) {
+    extern __shared__ __align__(128) uint8_t smraw[];
+    U3Smem& S = *reinterpret_cast<U3Smem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int NP = a.n_pad;
+    const bool flat = a.w4 <= kFlatMax;
+    const int64_t per_img = flat ? (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM)
+                                 : a.out_rows * ((a.w5 + 2 * kTileM - 1) / (2 * kTileM));
+    const int64_t bplane = a.t4_rows * a.w4;
+
+    if (warp == 0) tc::tmem_alloc<512>(&S.tmem);
     if (tid == 0) {
-        tc::mbar_init(&S.mbar[0], 1);
-        tc::mbar_init(&S.mbar[1], 1);
+        for (int i = 0; i < 2; ++i) {
+            tc::mbar_init(&S.a_full[i], 1);
+            tc::mbar_init(&S.a_empty[i], 1);
+            tc::mbar_init(&S.t_full[i], 1);
+            tc::mbar_init(&S.t_empty[i], kEpiWarps);
+        }
+        for (int i = 0; i < U3_BRING; ++i) {
+            tc::mbar_init(&S.b_full[i], 1);
+            tc::mbar_init(&S.b_empty[i], 1);
+        }
         tc::mbar_fence_init();
     }
-    // ---- stage the T4 window as bf16 [block][row][col][8]
-    // U2 wrote T4 as bf16 channel blocks [3][rows][w4][8]: three 16-byte loads per pixel
-    const int64_t bplane = a.t4_rows * a.w4;
-    const uint4* t4b = reinterpret_cast<const uint4*>(a.t4) + img * 3 * bplane;
-    const int64_t wc0 = flat ? 0 : q0;
-    for (int idx = tid; idx < plane_px; idx += kThreadsU3) {
-        const int r = idx / WP, c = idx - r * WP;
-        const int64_t br = wr0 + r - a.t4_row0, gc = wc0 + c;
-        const bool ok = idx < WR * WP && br >= 0 && br < a.t4_rows && gc < a.w4;
-        const int64_t o = br * a.w4 + gc;
-        const uint4 z = make_uint4(0u, 0u, 0u, 0u);
-        S.a[0][idx] = ok ? __ldg(t4b + o) : z;
-        S.a[1][idx] = ok ? __ldg(t4b + bplane + o) : z;
-        S.a[2][idx] = ok ? __ldg(t4b + 2 * bplane + o) : z;
-    }
-    for (int idx = tid; idx < U3_NMAX * 9; idx += kThreadsU3) {
-        const int ch = idx / 9, o = idx - ch * 9;
-        S.k6[ch][o] = ch < a.n5 ? __ldg(a.k6 + o * a.n5 + ch) : 0.f;
-    }
-    const uint4* kb = reinterpret_cast<const uint4*>(a.k5_tc);
-    const int stage_vec = U3_KS_STAGE * 2 * NP;  // uint4 per stage
-    for (int idx = tid; idx < stage_vec; idx += kThreadsU3) S.b[0][idx] = __ldg(kb + idx);
+    // windows start zeroed: pixels a copy does not cover (beyond the image, the spare pixels of
+    // tap pair (4,5)) then only ever hold finite T4 values
+    for (int idx = tid; idx < 2 * 3 * U3_APX; idx += kThreadsU3) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
     tc::fence_proxy_async();
     tc::fence_before_sync();
     __syncthreads();
     tc::fence_after_sync();
     const uint32_t tmem = S.tmem;
-    const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);
-    const uint32_t plane_bytes = (uint32_t)(U3_APLANE_MAX * 16);
-    const uint32_t a_base = tc::smem_u32(S.a[0]);
 
-    constexpr int kStages = U3_KS / U3_KS_STAGE;
-    for (int st = 0; st < kStages; ++st) {
-        if (tid == 0) {
-            tc::fence_after_sync();
-            const uint32_t b_base = tc::smem_u32(S.b[st & 1]);
-            for (int u = 0; u < U3_KS_STAGE; ++u) {
-                const int ks = st * U3_KS_STAGE + u;
-                const int i = ks / 8, r8 = ks % 8;
-                uint32_t a_addr, lbo;
-                if (r8 < 5) {  // channels 0-15 of tap (i, r8): blocks 0 and 1
-                    a_addr = a_base + (uint32_t)((base + i * WP + r8) * 16);
-                    lbo = plane_bytes;
-                } else {       // channels 16-19 of taps (i, j) and (i, j+1): block 2, next pixel
-                    const int j = 2 * (r8 - 5);
-                    a_addr = a_base + 2 * plane_bytes + (uint32_t)((base + i * WP + j) * 16);
-                    lbo = 16;
+    if (warp == kEpiWarps) {
+        if (lane == 0) {
+            // ------------------------------------------------------------ producer + MMA
+            const uint4* t4b_all = reinterpret_cast<const uint4*>(a.t4);
+            const uint4* kb = reinterpret_cast<const uint4*>(a.k5_tc);
+            const uint32_t stage_bytes = (uint32_t)(U3_KS_STAGE * 2 * NP * 16);
+            const int64_t my_bands = nbands > blockIdx.x ? (nbands - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+            const int64_t total_stages = my_bands * U3_STAGES;
+            auto load_b = [&](int64_t gs) {
+                const int slot = (int)(gs % U3_BRING);
+                tc::mbar_expect_tx(&S.b_full[slot], stage_bytes);
+                tc::bulk_g2s(S.b[slot], kb + (size_t)(gs % U3_STAGES) * (stage_bytes / 16), stage_bytes, &S.b_full[slot]);
+            };
+            auto load_a = [&](int64_t band, int buf) {
+                const U3Band g = u3_band(a, band, per_img, flat);
+                const uint4* t4b = t4b_all + g.img * 3 * bplane;
+                const int64_t r0 = g.wr0 - a.t4_row0;
+                uint32_t bytes = 0;
+                if (flat) {
+                    const int64_t rows = min((int64_t)g.WR, a.t4_rows - r0);
+                    bytes = (uint32_t)(3 * rows * a.w4 * 16);
+                    tc::mbar_expect_tx(&S.a_full[buf], bytes);
+                    for (int blk = 0; blk < 3; ++blk)
+                        tc::bulk_g2s(S.a[buf][blk], t4b + blk * bplane + r0 * a.w4, (uint32_t)(rows * a.w4 * 16),
+                                     &S.a_full[buf]);
+                } else {
+                    const int64_t cols = min((int64_t)U3_WP_COL, a.w4 - g.wc0);
+                    bytes = (uint32_t)(3 * 5 * cols * 16);
+                    tc::mbar_expect_tx(&S.a_full[buf], bytes);
+                    for (int blk = 0; blk < 3; ++blk)
+                        for (int r = 0; r < 5; ++r)
+                            tc::bulk_g2s(&S.a[buf][blk][r * U3_WP_COL], t4b + blk * bplane + (r0 + r) * a.w4 + g.wc0,
+                                         (uint32_t)(cols * 16), &S.a_full[buf]);
                 }
-                const uint64_t bd = tc::make_desc(b_base + (uint32_t)(u * 2 * NP * 16), (uint32_t)(NP * 16), 128);
-                for (int t = 0; t < 2; ++t) {
-                    const uint64_t ad = tc::make_desc(a_addr + (uint32_t)(t * kTileM * 16), lbo, 128);
-                    tc::mma_bf16(tmem + (uint32_t)(t * NP), ad, bd, idesc, ks > 0 ? 1u : 0u);
+            };
+            const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);
+            for (int64_t gs = 0; gs < (int64_t)(U3_BRING - 1) && gs < total_stages; ++gs) load_b(gs);
+            if (my_bands > 0) load_a(blockIdx.x, 0);
+            int64_t gs = 0;
+            for (int64_t k = 0; k < my_bands; ++k) {
+                const int buf = (int)(k & 1);
+                const U3Band g = u3_band(a, blockIdx.x + k * gridDim.x, per_img, flat);
+                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k >> 1) & 1));
+                if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+                tc::fence_after_sync();
+                const uint32_t a_base = tc::smem_u32(S.a[buf][0]);
+                const uint32_t plane_bytes = (uint32_t)(U3_APX * 16);
+                const uint32_t d_base = tmem + (uint32_t)(buf * 256);
+                for (int st = 0; st < U3_STAGES; ++st, ++gs) {
+                    const int slot = (int)(gs % U3_BRING);
+                    tc::mbar_wait(&S.b_full[slot], (uint32_t)((gs / U3_BRING) & 1));
+                    tc::fence_after_sync();
+                    const uint32_t b_base = tc::smem_u32(S.b[slot]);
+                    for (int u = 0; u < U3_KS_STAGE; ++u) {
+                        const int ks = st * U3_KS_STAGE + u;
+                        const int i = ks / 8, r8 = ks % 8;
+                        uint32_t a_addr, lbo;
+                        if (r8 < 5) {  // channels 0-15 of tap (i, r8): blocks 0 and 1
+                            a_addr = a_base + (uint32_t)((g.base + i * g.WP + r8) * 16);
+                            lbo = plane_bytes;
+                        } else {       // channels 16-19 of taps (i, j), (i, j+1): block 2, next pixel
+                            a_addr = a_base + 2 * plane_bytes + (uint32_t)((g.base + i * g.WP + 2 * (r8 - 5)) * 16);
+                            lbo = 16;
+                        }
+                        const uint64_t bd = tc::make_desc(b_base + (uint32_t)(u * 2 * NP * 16), (uint32_t)(NP * 16), 128);
+                        for (int t = 0; t < 2; ++t) {
+                            const uint64_t ad = tc::make_desc(a_addr + (uint32_t)(t * kTileM * 16), lbo, 128);
+                            tc::mma_bf16(d_base + (uint32_t)(t * NP), ad, bd, idesc, ks > 0 ? 1u : 0u);
+                        }
+                    }
+                    tc::commit(&S.b_empty[slot]);
+                    // refill the slot of stage gs-1 with stage gs+BRING-1 (it has BRING-1 stages to land)
+                    if (gs + U3_BRING - 1 < total_stages) {
+                        if (gs >= 1) tc::mbar_wait(&S.b_empty[(gs - 1) % U3_BRING], (uint32_t)(((gs - 1) / U3_BRING) & 1));
+                        load_b(gs + U3_BRING - 1);
+                    }
+                }
+                tc::commit(&S.a_empty[buf]);
+                tc::commit(&S.t_full[buf]);
+                // prefetch the next band's window into the other buffer (freed by band k-1's MMAs)
+                if (k + 1 < my_bands) {
+                    if (k >= 1) tc::mbar_wait(&S.a_empty[buf ^ 1], (uint32_t)(((k - 1) >> 1) & 1));
+                    load_a(blockIdx.x + (k + 1) * gridDim.x, buf ^ 1);
                 }
             }
-            tc::commit(&S.mbar[st & 1]);
         }
-        if (st + 1 < kStages) {
-            // buffer (st+1)&1 was read by stage st-1: wait for its MMAs before overwriting
-            if (st >= 1) tc::mbar_wait(&S.mbar[(st + 1) & 1], (uint32_t)(((st - 1) >> 1) & 1));
-            const uint4* src = kb + (size_t)(st + 1) * stage_vec;
-            for (int idx = tid; idx < stage_vec; idx += kThreadsU3) S.b[(st + 1) & 1][idx] = __ldg(src + idx);
-            tc::fence_proxy_async();
-            tc::fence_before_sync();
-            __syncthreads();
-        }
-    }
-    // the last stage's commit covers every MMA issued before it
-    tc::mbar_wait(&S.mbar[(kStages - 1) & 1], (uint32_t)(((kStages - 1) >> 1) & 1));
-    tc::fence_after_sync();
-
-    // ---- epilogue: warp w drains tile w/4, TMEM lanes 32*(w%4).. (its lane quarter)
-    const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
-    {
-        const int t = warp >> 2;
-        const int m = t * kTileM + 32 * (warp & 3) + lane;
-        int64_t orow, ocol;
-        if (flat) {
-            const int64_t q = q0 + m;
-            orow = a.out_row0 + q / a.w4;
-            ocol = q - (q / a.w4) * a.w4;
-        } else {
-            orow = wr0;
-            ocol = q0 + m;
-        }
-        const bool ok = orow < a.out_row0 + a.out_rows && ocol < a.w5;
-        float c6[9];
+    } else {
+        // ---------------------------------------------------------------- epilogue warps
+        const int t = warp >> 2;  // tile
+        const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
+        int64_t k = 0;
+        for (int64_t band = blockIdx.x; band < nbands; band += gridDim.x, ++k) {
+            const int buf = (int)(k & 1);
+            const U3Band g = u3_band(a, band, per_img, flat);
+            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
+            tc::fence_after_sync();
+            const int m = t * kTileM + 32 * (warp & 3) + lane;
+            int64_t orow, ocol;
+            if (flat) {
+                const int64_t q = g.q0 + m;
+                orow = a.out_row0 + q / a.w4;
+                ocol = q - (q / a.w4) * a.w4;
+            } else {
+                orow = g.wr0;
+                ocol = g.q0 + m;
+            }
+            const bool ok = orow < a.out_row0 + a.out_rows && ocol < a.w5;
+            float c6[9];
 #pragma unroll
-        for (int o = 0; o < 9; ++o) c6[o] = 0.f;
-        for (int cb = 0; cb < NP; cb += 32) {
-            float v[32];
-            tc::tmem_ld32(tmem + lane_base + (uint32_t)(t * NP + cb), v);  // warp-uniform
-            if (ok) {
+            for (int o = 0; o < 9; ++o) c6[o] = 0.f;
+            for (int cb = 0; cb < NP; cb += 32) {
+                float v[32];
+                tc::tmem_ld32(tmem + lane_base + (uint32_t)(buf * 256 + t * NP + cb), v);  // warp-uniform
+                if (ok) {
+                    float bv[32];
 #pragma unroll
-                for (int u = 0; u < 32; ++u) {
-                    const int ch = cb + u;
-                    if (ch < a.n5) {
-                        const float b = a.b5_plane
-                                            ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (orow - a.b5_row0)) * a.w5 + ocol)
-                                            : __ldg(a.b5 + ch);
-                        const float th = tanh_f(v[u] + b);
+                    for (int u = 0; u < 32; ++u) {  // all 32 bias loads in flight first
+                        const int ch = min(cb + u, a.n5 - 1);
+                        bv[u] = a.b5_plane ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (orow - a.b5_row0)) * a.w5 + ocol)
+                                           : __ldg(a.b5 + ch);
+                    }
 #pragma unroll
-                        for (int o = 0; o < 9; ++o) c6[o] = fmaf(S.k6[ch][o], th, c6[o]);
+                    for (int u = 0; u < 32; ++u) {
+                        const int ch = cb + u;
+                        if (ch < a.n5) {
+                            const float th = tanh_f(v[u] + bv[u]);
+#pragma unroll
+                            for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], th, c6[o]);
+                        }
                     }
                 }
             }
-        }
-        if (ok) {
-            float* ob = a.out + img * a.out_img_stride + (orow - a.out_row0) * a.w5 + ocol;
+            tc::fence_before_sync();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);  // the accumulator can be reused
+            if (ok) {
+                float* ob = a.out + g.img * a.out_img_stride + (orow - a.out_row0) * a.w5 + ocol;
 #pragma unroll
-            for (int o = 0; o < 9; ++o) {
-                const float b = a.b6_plane ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (orow - a.b6_row0)) * a.w5 + ocol)
-                                           : __ldg(a.b6 + o);
-                ob[o * a.out_plane_stride] = c6[o] + b;
+                for (int o = 0; o < 9; ++o) {
+                    const float b = a.b6_plane
+                                        ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (orow - a.b6_row0)) * a.w5 + ocol)
+                                        : __ldg(a.b6 + o);
+                    ob[o * a.out_plane_stride] = c6[o] + b;
+                }
             }
         }
     }
     tc::fence_before_sync();
     __syncthreads();
-    if (warp == 0) tc::tmem_dealloc<256>(tmem);
+    if (warp == 0) tc::tmem_dealloc<512>(tmem);
 }
 
 uint16_t to_bf16(float f) {  // round to nearest even (host)
@@ -403,17 +477,22 @@ cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s) {
 
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
-    if (a.n_pad > U3_NMAX || a.n_pad % 16) return cudaErrorInvalidValue;
+    if (a.n_pad > U3_NMAX || a.n_pad % 16 || a.n5 > U3_NMAX) return cudaErrorInvalidValue;
     static std::atomic<uint32_t> flags{0};
-    const size_t smem = sizeof(U3TcShared);
+    const size_t smem = sizeof(U3Smem) + 128;
     if (!set_smem_attr((const void*)cnn_u3_tc_kernel, smem, flags)) return cudaErrorInvalidValue;
-    unsigned bands;
-    if (a.w4 <= kFlatMax)
-        bands = (unsigned)((a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM));
-    else
-        bands = (unsigned)(a.out_rows * ((a.w5 + 2 * kTileM - 1) / (2 * kTileM)));
-    dim3 grid(bands, 1, (unsigned)a.nimg);
-    cnn_u3_tc_kernel<<<grid, kThreadsU3, smem, s>>>(a);
+    const bool flat = a.w4 <= kFlatMax;
+    const int64_t per_img = flat ? (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM)
+                                 : a.out_rows * ((a.w5 + 2 * kTileM - 1) / (2 * kTileM));
+    U3K6 k6w{};
+    for (int ch = 0; ch < a.n5; ++ch)
+        for (int o = 0; o < 9; ++o) k6w.k6[ch][o] = a.k6_host[o * a.n5 + ch];
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t nbands = per_img * a.nimg;
+    const unsigned grid = (unsigned)std::min<int64_t>(nbands, sms);
+    cnn_u3_tc_kernel<<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands);
     return cudaGetLastError();
 }
 

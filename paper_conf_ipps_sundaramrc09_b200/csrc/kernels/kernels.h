@@ -62,6 +62,7 @@ struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + 
     int64_t nimg;
     int bf16_tc;            // 1: tcgen05 path, T4 read as bf16 [3][rows][w4][8]
     const uint16_t* k5_tc;  // bf16 B operand prepared by cnn_prepare_k5_tc (device)
+    const float* k6_host;   // [9][n5] (host; passed by value to the tensor-core kernel)
     int n_pad;              // n5 rounded up to a multiple of 16
 };
 cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s);
