@@ -190,7 +190,9 @@ tg_status tg_plan_dump_json(const tg_plan* plan, char* buf, size_t cap, size_t* 
 /* Execute the plan; blocks until outputs are valid in their destinations. */
 tg_status tg_execute(tg_plan* plan);
 /* Same, but returns once all work is enqueued; completion is ordered before any later work
- * on the compute stream (which = 1) of every device of the plan. */
+ * on the compute stream (which = 1) of every device of the plan. Back-to-back executions
+ * of one host-I/O plan pipeline: the next execution's first H2D copies may run while the
+ * previous one's last chunks compute and download (each copy waits only for its slot). */
 tg_status tg_execute_async(tg_plan* plan);
 
 /* Per-launch timing of the fused kernels measured with CUDA events on the compute stream

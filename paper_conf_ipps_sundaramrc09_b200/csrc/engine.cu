@@ -46,6 +46,7 @@ struct DevState {
     std::vector<cudaEvent_t> ev_pool;
     int64_t launches = 0;
     bool params_resident = false;  // parameters uploaded by an earlier execution
+    int64_t seq = 0;               // chunks enqueued on this device over all executions (slot ring)
 };
 
 }  // namespace
@@ -401,11 +402,17 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
     const PlanCore& c = p->core;
     CK(cudaSetDevice(d.dev));
     cudaStream_t S0 = d.st[0], S1 = d.st[1], S2 = d.st[2];
-    // fork the copy streams off the compute stream (orders this execution after earlier
-    // work on the compute stream, including a previous execution's join)
+    // Fork: the copy streams are ordered after earlier work on the compute stream only where
+    // they need to be -- device-resident I/O (inputs may come from earlier kernels) and a
+    // parameter (re-)upload (earlier kernels may still read the old parameters). Otherwise a
+    // new execution's H2D copies only wait for their slot to be free (the slot ring and its
+    // events persist across executions), so back-to-back executions of one plan pipeline:
+    // the next batch uploads while the previous one's last chunks compute and download.
     CK(cudaEventRecord(d.ev_fork, S1));
-    CK(cudaStreamWaitEvent(S0, d.ev_fork, 0));
-    CK(cudaStreamWaitEvent(S2, d.ev_fork, 0));
+    if (c.device_io || !d.params_resident) {
+        CK(cudaStreamWaitEvent(S0, d.ev_fork, 0));
+        CK(cudaStreamWaitEvent(S2, d.ev_fork, 0));
+    }
     // parameters (never split): uploaded by the first execution and kept
     // resident in the arena for later ones (tg_plan_invalidate_params forces a re-upload)
     if (!d.params_resident) {
@@ -441,11 +448,11 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
         x->param_uploads += 1;
     }
     const int D = c.depth;
-    for (int64_t k = 0; k < d.c1 - d.c0; ++k) {
+    for (int64_t k = 0; k < d.c1 - d.c0; ++k, ++d.seq) {
         const Chunk& ch = c.chunks[d.c0 + k];
-        const int s = (int)(k % D);
+        const int s = (int)(d.seq % D);
         if (!c.device_io) {
-            if (k >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
+            if (d.seq >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
             ProfRec pr{10, nullptr, nullptr};
             if (x->profiling) {
                 pr.a = pool_event(d);
@@ -460,7 +467,7 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
             }
             CK(cudaEventRecord(d.ev_h2d[s], S0));
             CK(cudaStreamWaitEvent(S1, d.ev_h2d[s], 0));
-            if (k >= D) CK(cudaStreamWaitEvent(S1, d.ev_d2h[s], 0));
+            if (d.seq >= D) CK(cudaStreamWaitEvent(S1, d.ev_d2h[s], 0));
         }
         tg_status st = launch_units(p, x, d, ch, s);
         if (st != TG_OK) return st;
@@ -621,6 +628,8 @@ uint64_t exec_registered_bytes(const tg_plan* p) { return p->exec ? p->exec->reg
 void exec_invalidate_params(tg_plan* p) {
     if (!p->exec) return;
     for (auto& d : p->exec->devs) d.params_resident = false;
+    p->exec->k3tc.clear();  // the bf16 tensor-core operands are re-derived from the new values
+    p->exec->k5tc.clear();
 }
 
 }  // namespace tg

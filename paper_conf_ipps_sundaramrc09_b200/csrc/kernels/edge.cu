@@ -7,7 +7,10 @@
 // 8-orientation graph of Fig. 1(b)) and the other combine ops of PAPER.md:621 (addition,
 // max absolute value). SAME zero padding with anchor (ks-1)/2
 // (R2); a ks x ks kernel (ks <= 16) is embedded in a 16 x 16 frame at offset
-// 7 - (ks-1)/2 so one code path serves every size (zero taps add exact zeros).
+// 7 - (ks-1)/2 so one code path serves every size. The tap loops are specialised on the
+// frame kF in {4, 8, 16}: a ks <= kF kernel has all its nonzero taps inside the centred
+// kF x kF window [8 - kF/2, 8 + kF/2) of the 16 x 16 frame, so only those taps are issued
+// (Fig. 2's small kernels cost (kF/16)^2 of the 16 x 16 work instead of all of it).
 //
 // Roofline: 2 x 256 FMA per output pixel vs 8 HBM bytes -> FP32-ALU
 // bound (128 flop/B >> ridge ~11 flop/B). The kernel is organised to keep the FMA pipe busy:
@@ -59,7 +62,7 @@ struct EdgeWeights {
 
 // Compute the 64 x 64 output tile whose input (+halo) is staged at xs (pitch kPitch, smem
 // (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)) and store it.
-template <int kComb, int kPairs>
+template <int kComb, int kPairs, int kF>
 __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const EdgeArgs& a, const EdgeWeights& wt,
                                           int64_t img, int64_t tile_r0, int64_t tile_c0) {
     const int tid = threadIdx.x;
@@ -80,8 +83,9 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const Ed
         float2 acc[16];
 #pragma unroll
         for (int q = 0; q < 16; ++q) acc[q] = make_float2(0.f, 0.f);
+        constexpr int kOff = 8 - kF / 2;  // first tap row/column of the kF x kF window
 #pragma unroll 1
-        for (int i = 0; i < 16; ++i) {
+        for (int i = kOff; i < kOff + kF; ++i) {
             // input window: smem cols [cb, cb+32) <-> image cols [c0+cb-8, c0+cb+24);
             // output column c0+cb+q, tap j reads image col c0+cb+q+j-7 = smem col cb+q+j+1
             float x[32];
@@ -95,7 +99,7 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const Ed
                 x[4 * v + 3] = t.w;
             }
 #pragma unroll
-            for (int j = 0; j < 16; ++j) {
+            for (int j = kOff; j < kOff + kF; ++j) {
                 const float2 w = wt.w[fp][i * 16 + j];
 #pragma unroll
                 for (int q = 0; q < 16; ++q)
@@ -150,7 +154,7 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const Ed
 }
 
 // ---------------------------------------------------------------------------- fallback
-template <int kComb, int kPairs>
+template <int kComb, int kPairs, int kF>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
     __shared__ __align__(16) float xs[kSmR * kPitch];
@@ -181,7 +185,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         *reinterpret_cast<float4*>(&xs[sr * kPitch + 4 * q]) = v;
     }
     __syncthreads();
-    edge_tile<kComb, kPairs>(xs, a, wt, img, tile_r0, tile_c0);
+    edge_tile<kComb, kPairs, kF>(xs, a, wt, img, tile_r0, tile_c0);
 }
 
 // ---------------------------------------------------------------------------- TMA path
@@ -189,7 +193,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-template <int kComb, int kPairs>
+template <int kComb, int kPairs, int kF>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_tma_kernel(const __grid_constant__ CUtensorMap tmap, const EdgeArgs a,
                           const __grid_constant__ EdgeWeights wt, const int tiles_c, const int tiles_r,
@@ -251,7 +255,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         int64_t img, tr0, tc0;
         coords(t, img, tr0, tc0);
         const float* tb = b ? buf1 : buf0;
-        edge_tile<kComb, kPairs>(tb, a, wt, img, tr0, tc0);
+        edge_tile<kComb, kPairs, kF>(tb, a, wt, img, tr0, tc0);
         __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
     }
 }
@@ -271,26 +275,33 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 
 }  // namespace
 
-template <int kComb, int kPairs>
+template <int kComb, int kPairs, int kF>
 cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s);
 
-template <int kPairs>
+template <int kPairs, int kF>
 cudaError_t launch_edge_p(const EdgeArgs& a, cudaStream_t s) {
     switch (a.combine) {
-        case 0: return launch_edge_t<0, kPairs>(a, s);
-        case 1: return launch_edge_t<1, kPairs>(a, s);
-        case 2: return launch_edge_t<2, kPairs>(a, s);
-        case 3: return launch_edge_t<3, kPairs>(a, s);
+        case 0: return launch_edge_t<0, kPairs, kF>(a, s);
+        case 1: return launch_edge_t<1, kPairs, kF>(a, s);
+        case 2: return launch_edge_t<2, kPairs, kF>(a, s);
+        case 3: return launch_edge_t<3, kPairs, kF>(a, s);
         default: return cudaErrorInvalidValue;
     }
 }
 
-cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
-    if (a.nf < 1 || a.nf > 4) return cudaErrorInvalidValue;
-    return a.nf <= 2 ? launch_edge_p<1>(a, s) : launch_edge_p<2>(a, s);
+template <int kF>
+cudaError_t launch_edge_f(const EdgeArgs& a, cudaStream_t s) {
+    return a.nf <= 2 ? launch_edge_p<1, kF>(a, s) : launch_edge_p<2, kF>(a, s);
 }
 
-template <int kComb, int kPairs>
+cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
+    if (a.nf < 1 || a.nf > 4 || a.ks < 1 || a.ks > 16) return cudaErrorInvalidValue;
+    if (a.ks <= 4) return launch_edge_f<4>(a, s);
+    if (a.ks <= 8) return launch_edge_f<8>(a, s);
+    return launch_edge_f<16>(a, s);
+}
+
+template <int kComb, int kPairs, int kF>
 cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     // filters embedded in a 16 x 16 frame at offset 7 - (ks-1)/2 (zeros elsewhere)
@@ -325,19 +336,19 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
             const size_t smem = 2 * (size_t)kBufStride + 128;
             if (!(configured.load() & (1u << (dev & 31)))) {
                 cudaError_t e =
-                    cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                    cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs, kF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
                 if (e != cudaSuccess) return e;
                 configured.fetch_or(1u << (dev & 31));
             }
             const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
             const int64_t grid = std::min<int64_t>(ntiles, 2 * (int64_t)sms);
-            edge_fused_tma_kernel<kComb, kPairs><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
+            edge_fused_tma_kernel<kComb, kPairs, kF><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
             return cudaGetLastError();
         }
     }
     dim3 grid((unsigned)tiles_c, (unsigned)tiles_r, (unsigned)a.nimg);
     if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
-    edge_fused_kernel<kComb, kPairs><<<grid, kThreads, 0, s>>>(a, wt);
+    edge_fused_kernel<kComb, kPairs, kF><<<grid, kThreads, 0, s>>>(a, wt);
     return cudaGetLastError();
 }
 

@@ -488,6 +488,9 @@ class Plan:
     def launches(self) -> int:
         return tg_plan_launch_count(self.h)
 
+    def invalidate_params(self) -> None:
+        tg_plan_invalidate_params(self.h)
+
     def compute_stream(self, dev: int = 0):
         if self.graph.runtime is None:
             raise RuntimeError("compute_stream needs set(torch_runtime=True)")

@@ -228,3 +228,58 @@ def test_cnn_config3_full_batch_sampled(tg, orc, n5, prec):
     for b in (0, 31, 63):
         ref = orc.cnn(img[b:b + 1], n5, prm)
         assert normwise(out[b:b + 1], ref) <= tol, b
+
+
+@pytest.mark.parametrize("prec", ["fp32", "bf16_tc"])
+def test_cnn_invalidate_params(tg, orc, prec):
+    """Parameters stay resident in the arena after the first execution; after the caller
+    changes them in place, tg_plan_invalidate_params makes the next execution re-upload them
+    (and re-derive the bf16 tensor-core operands). Without it the old values are used."""
+    seed = 77
+    n, H, W, n5 = 2, 100, 120, 20
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    out = np.zeros((n, 9) + synth.cnn_dims(H, W)[4], np.float32)
+    g, _ = tg.cnn_graph(img, n5, prm, out=out)
+    g.set(torch_runtime=True, precision=tg.TG_BF16_TC if prec == "bf16_tc" else tg.TG_FP32)
+    p = g.plan()
+    p.execute()
+    first = out.copy()
+    tol = 2e-2 if prec == "bf16_tc" else 1e-5
+    assert normwise(first, orc.cnn(img, n5, prm)) <= tol
+    for i in (1, 4, 6, 7, 9):          # arena-resident: B1, B3, K5, B5, B6 (K1, K3, P2, P4
+        # travel by value with every launch and take effect at once)
+        prm[i] *= np.float32(-0.5)
+    p.execute()                        # still the resident (old) parameters
+    if prec == "fp32":
+        assert np.array_equal(out, first)
+    p.invalidate_params()
+    p.execute()
+    assert normwise(out, orc.cnn(img, n5, prm)) <= tol
+    assert not np.allclose(out, first)
+
+
+@pytest.mark.parametrize("bias", ["resident", "streamed"])
+def test_cnn_pipelined_async_executions(tg, bias):
+    """Back-to-back tg_execute_async calls of one host-I/O plan overlap (the slot ring persists
+    across executions); every execution still produces the blocking result bit for bit."""
+    seed = 78
+    n, H, W, n5 = 3, 160, 150, 20
+    img_t = pinned((n, 1, H, W))
+    img_t.copy_(torch.from_numpy(synth.images_np(seed, n, H, W)))
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    out_t = pinned((n, 9) + synth.cnn_dims(H, W)[4])
+    g, _ = tg.cnn_graph(img_t, n5, prm, out=out_t)
+    # a budget small enough for row chunks (streamed bias rows) or only batch chunks
+    g.set(torch_runtime=True, budget=1_000_000 if bias == "streamed" else 0, max_chunk_px=H * W, depth=2)
+    p = g.plan()
+    assert p.json()["bias"] == bias and p.json()["n_chunks"] >= 3
+    p.execute()
+    ref = out_t.clone()
+    for _ in range(4):
+        out_t.zero_()
+        torch.cuda.synchronize()
+        for _ in range(3):
+            p.execute(blocking=False)
+        torch.cuda.synchronize()
+        assert torch.equal(out_t, ref)

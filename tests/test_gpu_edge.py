@@ -178,6 +178,24 @@ def test_edge_general_combines(tg, orc, nf, combine):
     assert normwise(out, ref) <= 1e-5
 
 
+@pytest.mark.parametrize("ks", list(range(1, 17)))
+def test_edge_every_kernel_size(tg, orc, ks):
+    """Every ks in 1..16 (the kernel issues only the taps of the smallest 4/8/16 frame that
+    holds the SAME-anchored ks x ks kernel): odd/even anchors and both sides of each frame edge,
+    on a ragged image split into chunks."""
+    img = synth.images_np(40 + ks, 1, 97, 76)
+    rs = np.random.default_rng(100 + ks)
+    K = [(rs.standard_normal((ks, ks)) / ks).astype(np.float32) for _ in range(3)]
+    out = np.zeros_like(img)
+    g, _ = tg.edge_graph_general(img, K, "max", out=out)
+    g.set(budget=40_000, torch_runtime=True)
+    p = g.plan()
+    assert p.json()["n_chunks"] > 1
+    p.execute()
+    ref = orc.edge_general(img[0, 0], K, "max")[None, None]
+    assert normwise(out, ref) <= 1e-5
+
+
 def _rot(K, deg):
     """Test-side restatement of reading R18 (kernel rotation about its centre)."""
     k = K.shape[0]
@@ -216,3 +234,26 @@ def test_find_edges_orientations(tg, orc, n_or, comb):
     Ks = [_rot(K1, i * 360 // n_or) for i in range(n_or // 2)]
     ref = orc.edge_general(img[0, 0], Ks, comb)
     assert normwise(out[0], ref[None]) <= 1e-5
+
+
+def test_pipelined_async_executions(tg):
+    """Back-to-back async executions of one plan overlap across the persistent slot ring
+    (depth 2, many chunks); the results equal the blocking execution bit for bit."""
+    n, H, W = 3, 300, 256
+    img_t = pinned((n, 1, H, W))
+    img_t.copy_(torch.from_numpy(synth.images_np(12, n, H, W)))
+    out_t = pinned((n, 1, H, W))
+    K1, _ = synth.edge_filter_np()
+    g, _ = tg.edge_graph(img_t, K1, out=out_t)
+    g.set(budget=400_000, depth=2, torch_runtime=True)
+    p = g.plan()
+    assert p.stats()["n_chunks"] >= 8
+    p.execute()
+    ref = out_t.clone()
+    for _ in range(3):
+        out_t.zero_()
+        torch.cuda.synchronize()
+        for _ in range(4):
+            p.execute(blocking=False)
+        torch.cuda.synchronize()
+        assert torch.equal(out_t, ref)

@@ -1,0 +1,83 @@
+"""Figures 2 and 8 of the paper re-run on one B200 (host pinned input -> host output, fp32).
+
+Fig. 2: one 8000x8000 image convolved with a k x k kernel, k = 2..16 (K1 with
+one filter and the plain-max combine = a single SAME convolution), time split into H2D / kernel /
+D2H: "without overlap" = the three summed as the paper's GPUs had to run them, "with
+overlap" = the streamed plan's wall time. (The paper's C870: transfers 30-75 % of the time.)
+
+Fig. 8: edge template (16x16, 4 orientations) time vs image side at the
+768 MiB budget and uncapped, against the "best possible" single fused kernel on device-resident
+data (the paper was within 20 % of it; its baseline failed before 8000^2).
+Prints one JSON line per point."""
+import json
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+from paper_conf_ipps_sundaramrc09_b200 import tg  # noqa: E402
+
+
+def timed(p, reps=3):
+    p.execute()
+    torch.cuda.synchronize()
+    best = 1e9
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        p.execute()
+        torch.cuda.synchronize()
+        best = min(best, time.perf_counter() - t0)
+    return best
+
+
+def fig2():
+    H = W = 8000
+    img = torch.empty((1, 1, H, W), dtype=torch.float32).pin_memory()
+    img.copy_(synth.images_torch(7, 1, H, W, "cuda").cpu())
+    out = torch.empty_like(img).pin_memory()
+    for k in (2, 4, 6, 8, 10, 12, 14, 16):
+        K = synth.uniform_np(7, synth.DS_EDGE_K1, (k, k), 1.0 / k)
+        g, _ = tg.edge_graph_general(img, [K], "maxplain", out=out)
+        g.set(torch_runtime=True, budget=768 << 20)
+        p = g.plan()
+        wall = timed(p)
+        p.profiling(True)
+        p.execute()
+        t = p.timing()
+        h2d, ker, d2h = t["h2d_ms"], sum(t["kernel_ms"]), t["d2h_ms"]
+        serial = h2d + ker + d2h
+        print(json.dumps({"fig": 2, "k": k, "h2d_ms": h2d, "kernel_ms": ker, "d2h_ms": d2h,
+                          "transfer_share_no_overlap": (h2d + d2h) / serial, "serial_ms": serial,
+                          "overlapped_wall_ms": wall * 1e3}), flush=True)
+
+
+def fig8():
+    K1, _ = synth.edge_filter_np()
+    for side in (1000, 2000, 4000, 8000, 12000, 16000, 24000):
+        H = W = side
+        x = synth.images_torch(8, 1, H, W, "cuda")
+        img = torch.empty((1, 1, H, W), dtype=torch.float32).pin_memory()
+        img.copy_(x.cpu())
+        out = torch.empty_like(img).pin_memory()
+        res = {"fig": 8, "side": side}
+        for name, budget in (("capped_768MiB", 768 << 20), ("uncapped", 0)):
+            g, _ = tg.edge_graph(img, K1, out=out)
+            g.set(torch_runtime=True, budget=budget)
+            res[name + "_s"] = timed(g.plan())
+        y = torch.empty_like(x)
+        g, _ = tg.edge_graph(x, K1, out=y, device=True)
+        g.set(torch_runtime=True)
+        res["best_possible_kernel_s"] = timed(g.plan())
+        res["capped_vs_uncapped"] = res["capped_768MiB_s"] / res["uncapped_s"]
+        print(json.dumps(res), flush=True)
+        del x, y, img, out
+
+
+if __name__ == "__main__":
+    torch.cuda.set_device(0)
+    fig2()
+    fig8()
