@@ -207,6 +207,19 @@ typedef struct {
 } tg_timing;
 tg_status tg_plan_set_profiling(tg_plan* plan, int32_t on);
 tg_status tg_plan_timing_get(tg_plan* plan, tg_timing* out);
+
+/* Timeline of the profiled copies and launches (fused mode): one record per H2D chunk copy,
+ * kernel launch and D2H chunk copy, in enqueue order, with start/end in ms relative to the
+ * first profiled record of its device in the batch collected. Collected (and appended) by
+ * tg_plan_timing_get / this call, which synchronize; cleared by tg_plan_set_profiling(1).
+ * Writes min(cap, total) records to out (out may be NULL when cap == 0); *n = total. */
+typedef struct {
+    int32_t device;
+    int32_t kind;            /* 0 edge, 1..3 CNN U1..U3, 10 H2D copy, 11 D2H copy        */
+    int64_t chunk;           /* chunk index within the plan (-1: parameter upload)       */
+    double t0_ms, t1_ms;
+} tg_trace_rec;
+tg_status tg_plan_trace_get(tg_plan* plan, tg_trace_rec* out, size_t cap, size_t* n);
 /* Parameters are copied to the device by the first execution of a plan and stay resident
  * in its arena; call this after changing parameter host data to re-upload them at the next
  * execution. */

@@ -20,6 +20,10 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O2", "-Xptxas", "-v",
          f"-I{os.path.join(ROOT, 'include')}", f"-I{CSRC}", "--expt-relaxed-constexpr"]
+# experiments only (tools/): extra -D flags build into their own object directory and always relink
+EXTRA = os.environ.get("TG_NVCC_DEFS", "").split()
+if EXTRA:
+    BUILD = BUILD + "_" + "_".join(d.strip("-").replace("=", "") for d in EXTRA)
 
 
 def sources():
@@ -28,7 +32,8 @@ def sources():
 
 
 def _headers_mtime():
-    hs = glob.glob(os.path.join(CSRC, "**", "*.h"), recursive=True) + [os.path.join(ROOT, "include", "tg.h")]
+    hs = (glob.glob(os.path.join(CSRC, "**", "*.h"), recursive=True)
+          + glob.glob(os.path.join(CSRC, "**", "*.cuh"), recursive=True) + [os.path.join(ROOT, "include", "tg.h")])
     return max(os.path.getmtime(h) for h in hs)
 
 
@@ -37,9 +42,9 @@ def _compile(src: str, verbose: bool) -> str:
     obj = os.path.join(BUILD, rel + ".o")
     if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(src), _headers_mtime()):
         return obj
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
+    cmd = [NVCC, *ARCH, *FLAGS, *EXTRA, "-c", src, "-o", obj]
     if src.endswith(".cpp"):
-        cmd = [NVCC, *ARCH, *FLAGS, "-x", "cu", "-c", src, "-o", obj]
+        cmd = [NVCC, *ARCH, *FLAGS, *EXTRA, "-x", "cu", "-c", src, "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")
@@ -55,11 +60,16 @@ def build(verbose: bool = False) -> str:
     srcs = sources()
     with ThreadPoolExecutor(max_workers=min(8, len(srcs))) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), srcs))
-    if not os.path.exists(LIB) or os.path.getmtime(LIB) < max(os.path.getmtime(o) for o in objs):
+    stamp = LIB + ".flags"  # which -D flags the current libtg.so was linked from
+    old = open(stamp).read() if os.path.exists(stamp) else ""
+    if (EXTRA or old != " ".join(EXTRA) or not os.path.exists(LIB)
+            or os.path.getmtime(LIB) < max(os.path.getmtime(o) for o in objs)):
         cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-lpthread"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
+        with open(stamp, "w") as f:
+            f.write(" ".join(EXTRA))
     return LIB
 
 

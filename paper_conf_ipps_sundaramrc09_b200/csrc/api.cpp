@@ -496,6 +496,14 @@ tg_status tg_plan_timing_get(tg_plan* p, tg_timing* out) {
     TG_GUARD_END
 }
 
+tg_status tg_plan_trace_get(tg_plan* p, tg_trace_rec* out, size_t cap, size_t* n) {
+    if (!p || !n || (cap && !out)) return fail(TG_E_ARG, "tg_plan_trace_get: NULL argument");
+    TG_GUARD_BEGIN
+    if (p->core.mode != TG_FUSED) return fail(TG_E_UNSUPPORTED, "tg_plan_trace_get: fused plans only");
+    return exec_trace(p, out, cap, n);
+    TG_GUARD_END
+}
+
 int64_t tg_plan_launch_count(const tg_plan* p) { return p ? p->launches : 0; }
 
 tg_status tg_plan_invalidate_params(tg_plan* p) {

@@ -31,6 +31,7 @@ namespace {
 struct ProfRec {
     int kind;  // 0 edge, 1 U1, 2 U2, 3 U3, 10 h2d, 11 d2h
     cudaEvent_t a, b;
+    int64_t chunk = -1;
 };
 
 struct DevState {
@@ -58,6 +59,7 @@ struct tg_exec {
     uint64_t registered_bytes = 0;
     bool profiling = false;
     tg_timing timing{};
+    std::vector<tg_trace_rec> trace;  // timeline collected from the profiling events
     int64_t param_uploads = 0;
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
 };
@@ -214,8 +216,10 @@ struct KernelTimer {
     tg_exec* x;
     DevState& d;
     int kind;
+    int64_t chunk;
     cudaEvent_t a = nullptr, b = nullptr;
-    KernelTimer(tg_exec* x_, DevState& d_, int kind_, cudaStream_t s) : x(x_), d(d_), kind(kind_) {
+    KernelTimer(tg_exec* x_, DevState& d_, int kind_, int64_t chunk_, cudaStream_t s)
+        : x(x_), d(d_), kind(kind_), chunk(chunk_) {
         if (x->profiling) {
             a = pool_event(d);
             b = pool_event(d);
@@ -225,7 +229,7 @@ struct KernelTimer {
     void done(cudaStream_t s) {
         if (x->profiling && a && b) {
             cudaEventRecord(b, s);
-            d.prof.push_back({kind, a, b});
+            d.prof.push_back({kind, a, b, chunk});
         }
     }
 };
@@ -236,6 +240,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
     const Template& t = c.t;
     char* base = slot_base(c, d, s);
     cudaStream_t cs = d.st[1];
+    const int64_t ci = &ch - c.chunks.data();  // chunk index (trace records)
     auto param = [&](int i) -> const float* {
         return c.param_off[i] == UINT64_MAX ? nullptr : (const float*)(d.arena + c.param_off[i]);
     };
@@ -267,7 +272,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.nf = t.nf;
         a.combine = t.combine;
         a.ks = t.ks;
-        KernelTimer kt(x, d, 0, cs);
+        KernelTimer kt(x, d, 0, ci, cs);
         CK(launch_edge(a, cs));
         kt.done(cs);
         ++d.launches;
@@ -311,7 +316,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.w2 = w2;
         a.nimg = ch.nimg;
         a.bf16_out = c.precision == TG_BF16_TC;
-        KernelTimer kt(x, d, 1, cs);
+        KernelTimer kt(x, d, 1, ci, cs);
         CK(launch_cnn_u1(a, cs));
         kt.done(cs);
         ++d.launches;
@@ -345,7 +350,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.bf16_tc = c.precision == TG_BF16_TC;
         a.k3_tc = c.k3tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k3tc_off);
         a.p4_dev = param(5);
-        KernelTimer kt(x, d, 2, cs);
+        KernelTimer kt(x, d, 2, ci, cs);
         CK(a.bf16_tc ? launch_cnn_u2_tc(a, cs) : launch_cnn_u2(a, cs));
         kt.done(cs);
         ++d.launches;
@@ -389,7 +394,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.k5_tc = c.k5tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k5tc_off);
         a.n_pad = cnn_n5_pad(t.n5);
         a.k6_host = g.ds[t.prm[8]].src;
-        KernelTimer kt(x, d, 3, cs);
+        KernelTimer kt(x, d, 3, ci, cs);
         CK(a.bf16_tc ? launch_cnn_u3_tc(a, cs) : launch_cnn_u3(a, cs));
         kt.done(cs);
         ++d.launches;
@@ -453,7 +458,7 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
         const int s = (int)(d.seq % D);
         if (!c.device_io) {
             if (d.seq >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
-            ProfRec pr{10, nullptr, nullptr};
+            ProfRec pr{10, nullptr, nullptr, d.c0 + k};
             if (x->profiling) {
                 pr.a = pool_event(d);
                 pr.b = pool_event(d);
@@ -474,7 +479,7 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
         CK(cudaEventRecord(d.ev_comp[s], S1));
         if (!c.device_io) {
             CK(cudaStreamWaitEvent(S2, d.ev_comp[s], 0));
-            ProfRec pr{11, nullptr, nullptr};
+            ProfRec pr{11, nullptr, nullptr, d.c0 + k};
             if (x->profiling) {
                 pr.a = pool_event(d);
                 pr.b = pool_event(d);
@@ -557,6 +562,7 @@ tg_status exec_set_profiling(tg_plan* p, bool on) {
     p->exec->profiling = on;
     if (on) {
         p->exec->timing = tg_timing{};
+        p->exec->trace.clear();
     }
     return TG_OK;
 }
@@ -571,8 +577,10 @@ tg_status exec_timing(tg_plan* p, tg_timing* out) {
         CK(cudaSetDevice(d.dev));
         for (auto& r : d.prof) {
             CK(cudaEventSynchronize(r.b));
-            float ms = 0.f;
+            float ms = 0.f, t0 = 0.f;
             CK(cudaEventElapsedTime(&ms, r.a, r.b));
+            CK(cudaEventElapsedTime(&t0, d.prof.front().a, r.a));
+            x->trace.push_back({d.dev, r.kind, r.chunk, (double)t0, (double)t0 + ms});
             if (r.kind < 4) {
                 x->timing.kernel_ms[r.kind] += ms;
                 x->timing.unit_launches[r.kind] += 1;
@@ -621,6 +629,18 @@ void exec_destroy(tg_plan* p) {
     cudaGetLastError();
     delete x;
     p->exec = nullptr;
+}
+
+tg_status exec_trace(tg_plan* p, tg_trace_rec* out, size_t cap, size_t* n) {
+    tg_timing t{};
+    tg_status st = exec_timing(p, &t);  // collects pending records into the trace
+    if (st != TG_OK) return st;
+    *n = 0;
+    if (!p->exec) return TG_OK;
+    const std::vector<tg_trace_rec>& tr = p->exec->trace;
+    *n = tr.size();
+    for (size_t i = 0; i < tr.size() && i < cap; ++i) out[i] = tr[i];
+    return TG_OK;
 }
 
 uint64_t exec_registered_bytes(const tg_plan* p) { return p->exec ? p->exec->registered_bytes : 0; }

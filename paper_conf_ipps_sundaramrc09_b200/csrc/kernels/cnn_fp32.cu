@@ -16,10 +16,12 @@
 // well inside the normwise 1e-5 parity bound.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstring>
 
 #include "kernels.h"
+#include "tma_util.cuh"
 
 namespace tg {
 namespace {
@@ -28,6 +30,13 @@ __device__ __forceinline__ float tanh_f(float x) {
     x = fminf(fmaxf(x, -15.f), 15.f);
     const float e = __expf(2.f * x);
     return 1.f - __fdividef(2.f, 1.f + e);
+}
+// MUFU.TANH (one SFU op, relative error ~2^-11): only where the result is rounded to bf16
+// anyway (U1 feeding the tensor-core path), never on the fp32 path.
+__device__ __forceinline__ float tanh_mufu(float x) {
+    float y;
+    asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
 }
 
 // ============================================================================ U1
@@ -42,6 +51,7 @@ struct U1W {
 constexpr int U1_TR = 8, U1_TC = 16;                // T2 tile (rows x cols) = 128 threads
 constexpr int U1_IR = 2 * U1_TR + 4, U1_IC = 2 * U1_TC + 4;  // 20 x 36 input window
 
+template <bool kBf16>
 __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const __grid_constant__ U1W w) {
     __shared__ __align__(16) float xs[U1_IR * U1_IC];
     const int tid = threadIdx.x, ty = tid / U1_TC, tx = tid % U1_TC;
@@ -59,6 +69,26 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
     __syncthreads();
     const int64_t R2 = r2_0 + ty, C2 = c2_0 + tx;
     if (R2 >= a.t2_row0 + a.t2_rows || C2 >= a.w2) return;
+
+    // bias of the 2x2 C1 pixels under this T2 pixel, loaded before the FMA sweep so the
+    // loads are in flight while it runs (one 8-byte load per channel and row when aligned)
+    float2 bb[8][2];
+    if (a.b1_plane) {
+        const bool v2 = (a.w1 & 1) == 0 && (reinterpret_cast<uintptr_t>(a.b1) & 7) == 0;
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch)
+#pragma unroll
+            for (int ra = 0; ra < 2; ++ra) {
+                const float* bp = a.b1 + ((int64_t)ch * a.b1_rows + (2 * R2 + ra - a.b1_row0)) * a.w1 + 2 * C2;
+                bb[ch][ra] = v2 ? __ldg(reinterpret_cast<const float2*>(bp)) : make_float2(__ldg(bp), __ldg(bp + 1));
+            }
+    } else {
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch) {
+            const float b = __ldg(a.b1 + ch);
+            bb[ch][0] = bb[ch][1] = make_float2(b, b);
+        }
+    }
 
     // FFMA2 over channel pairs (2c, 2c+1): each lane rounds exactly like fmaf
     float2 acc2[4][4];
@@ -99,16 +129,14 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
         float s = 0.f;
 #pragma unroll
         for (int p = 0; p < 4; ++p) {
-            const int64_t r1 = 2 * R2 + (p >> 1), c1 = 2 * C2 + (p & 1);
-            const float b = a.b1_plane ? __ldg(a.b1 + ((int64_t)ch * a.b1_rows + (r1 - a.b1_row0)) * a.w1 + c1)
-                                       : __ldg(a.b1 + ch);
+            const float b = (p & 1) ? bb[ch][p >> 1].y : bb[ch][p >> 1].x;
             const float av = (ch & 1) ? acc2[ch >> 1][p].y : acc2[ch >> 1][p].x;
-            const float t = tanh_f(av + b);
+            const float t = kBf16 ? tanh_mufu(av + b) : tanh_f(av + b);
             s = fmaf(w.p2[ch][p], t, s);
         }
-        tv[ch] = tanh_f(s);
+        tv[ch] = kBf16 ? tanh_mufu(s) : tanh_f(s);
     }
-    if (a.bf16_out) {  // one 16-byte pixel of 8 bf16 channels (the tensor-core U2's operand rows)
+    if (kBf16) {  // one 16-byte pixel of 8 bf16 channels (the tensor-core U2's operand rows)
         uint4* d = reinterpret_cast<uint4*>(a.t2) + (img * a.t2_rows + (R2 - a.t2_row0)) * a.w2 + C2;
         uint32_t p[4];
 #pragma unroll
@@ -119,6 +147,153 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
     } else {
 #pragma unroll
         for (int ch = 0; ch < 8; ++ch) t2[ch * plane + (R2 - a.t2_row0) * a.w2 + C2] = tv[ch];
+    }
+}
+
+// ---------------------------------------------------------------------------- U1, TMA path
+// Persistent variant (W % 4 == 0): each CTA walks T2 tiles of 8 rows x 32 columns; thread
+// (ty, tx) owns T2 pixels (ty, 2tx) and (ty, 2tx+1), i.e. a 2 x 4 block of C1 pixels x 8
+// channels (32 FFMA2 accumulators) from a 6 x 8 input window (two LDS.128 per row). One
+// thread stages the NEXT tile with two TMA loads -- the 20 x 68 input window and the
+// 8 x 16 x 64 bias block of the plane -- into the other shared-memory stage while the CTA
+// computes the current one (OOB zero fill = the image edge). Same FFMA order per output as
+// the fallback kernel above, so the two give identical bits.
+constexpr int U1T_R = 8, U1T_C = 32;
+constexpr int U1T_IR = 2 * U1T_R + 4, U1T_IC = 2 * U1T_C + 4;  // 20 x 68 input window
+constexpr int U1T_BR = 2 * U1T_R, U1T_BC = 2 * U1T_C;          // 16 x 64 C1 bias block per channel
+constexpr int U1T_XBYTES = U1T_IR * U1T_IC * 4;                 // 5440
+constexpr int U1T_XSTRIDE = (U1T_XBYTES + 127) / 128 * 128;
+constexpr int U1T_BBYTES = 8 * U1T_BR * U1T_BC * 4;             // 32768
+constexpr int U1T_STAGE = U1T_XSTRIDE + U1T_BBYTES;
+
+template <bool kBf16, bool kPlane>
+__global__ void __launch_bounds__(128, 2)
+    cnn_u1_tma_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap bmap,
+                      const CnnU1Args a, const __grid_constant__ U1W w, const int tiles_c, const int tiles_r,
+                      const int64_t ntiles) {
+    extern __shared__ __align__(128) uint8_t smraw[];
+    uint8_t* base = smraw + ((128 - (tma_smem_u32(smraw) & 127)) & 127);
+    __shared__ __align__(8) uint64_t full[2];
+    const int tid = threadIdx.x, ty = tid >> 4, tx = tid & 15;
+    if (tid == 0) {
+        tma_prefetch_map(&xmap);
+        if (kPlane) tma_prefetch_map(&bmap);
+        tma_mbar_init(&full[0], 1);
+        tma_mbar_init(&full[1], 1);
+        tma_fence_init();
+    }
+    __syncthreads();
+    auto coords = [&](int64_t t, int64_t& img, int64_t& r2_0, int64_t& c2_0) {
+        const int64_t per = (int64_t)tiles_c * tiles_r;
+        img = t / per;
+        const int64_t rem = t - img * per;
+        const int64_t ry = rem / tiles_c;
+        r2_0 = a.t2_row0 + ry * U1T_R;
+        c2_0 = (rem - ry * tiles_c) * U1T_C;
+    };
+    auto issue = [&](int64_t t, int b) {
+        int64_t img, r2_0, c2_0;
+        coords(t, img, r2_0, c2_0);
+        uint8_t* st = base + b * U1T_STAGE;
+        tma_expect_tx(&full[b], U1T_XBYTES + (kPlane ? U1T_BBYTES : 0));
+        tma_load_3d(st, &xmap, (int)(2 * c2_0), (int)(2 * r2_0 - a.in_row0), (int)img, &full[b]);
+        if (kPlane) tma_load_3d(st + U1T_XSTRIDE, &bmap, (int)(2 * c2_0), (int)(2 * r2_0 - a.b1_row0), 0, &full[b]);
+    };
+    const int64_t plane = a.t2_rows * a.w2;
+    int64_t t = blockIdx.x;
+    if (tid == 0 && t < ntiles) issue(t, 0);
+    for (int k = 0; t < ntiles; ++k, t += gridDim.x) {
+        const int b = k & 1;
+        if (tid == 0 && t + gridDim.x < ntiles) issue(t + gridDim.x, b ^ 1);
+        tma_wait(&full[b], (uint32_t)((k >> 1) & 1));
+        const float* xs = reinterpret_cast<const float*>(base + b * U1T_STAGE);
+        const float* bs = reinterpret_cast<const float*>(base + b * U1T_STAGE + U1T_XSTRIDE);
+        int64_t img, r2_0, c2_0;
+        coords(t, img, r2_0, c2_0);
+
+        float2 acc[4][2][4];  // [channel pair][C1 row ra][C1 column cb]
+#pragma unroll
+        for (int cp = 0; cp < 4; ++cp)
+#pragma unroll
+            for (int ra = 0; ra < 2; ++ra)
+#pragma unroll
+                for (int cb = 0; cb < 4; ++cb) acc[cp][ra][cb] = make_float2(0.f, 0.f);
+#pragma unroll
+        for (int i = 0; i < 6; ++i) {
+            float x[8];
+            const float4* xr = reinterpret_cast<const float4*>(&xs[(2 * ty + i) * U1T_IC + 4 * tx]);
+            const float4 u = xr[0], v = xr[1];
+            x[0] = u.x; x[1] = u.y; x[2] = u.z; x[3] = u.w;
+            x[4] = v.x; x[5] = v.y; x[6] = v.z; x[7] = v.w;
+#pragma unroll
+            for (int ra = 0; ra < 2; ++ra) {
+                const int ki = i - ra;
+                if (ki < 0 || ki > 4) continue;
+#pragma unroll
+                for (int cp = 0; cp < 4; ++cp)
+#pragma unroll
+                    for (int kj = 0; kj < 5; ++kj) {
+                        const float2 wv = make_float2(w.k1[ki * 5 + kj][2 * cp], w.k1[ki * 5 + kj][2 * cp + 1]);
+#pragma unroll
+                        for (int cb = 0; cb < 4; ++cb)
+                            acc[cp][ra][cb] = __ffma2_rn(make_float2(x[cb + kj], x[cb + kj]), wv, acc[cp][ra][cb]);
+                    }
+            }
+        }
+        const int64_t R2 = r2_0 + ty;
+        const bool row_ok = R2 < a.t2_row0 + a.t2_rows;
+        float tv[2][8];
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch) {
+            float4 b4[2];
+            if (kPlane) {
+#pragma unroll
+                for (int ra = 0; ra < 2; ++ra)
+                    b4[ra] = *reinterpret_cast<const float4*>(&bs[(ch * U1T_BR + 2 * ty + ra) * U1T_BC + 4 * tx]);
+            } else {
+                const float bv = __ldg(a.b1 + ch);
+                b4[0] = b4[1] = make_float4(bv, bv, bv, bv);
+            }
+#pragma unroll
+            for (int q = 0; q < 2; ++q) {
+                float s = 0.f;
+#pragma unroll
+                for (int p = 0; p < 4; ++p) {
+                    const int ra = p >> 1, cb = 2 * q + (p & 1);
+                    const float4 bb = b4[ra];
+                    const float bias = cb == 0 ? bb.x : cb == 1 ? bb.y : cb == 2 ? bb.z : bb.w;
+                    const float av = (ch & 1) ? acc[ch >> 1][ra][cb].y : acc[ch >> 1][ra][cb].x;
+                    const float th = kBf16 ? tanh_mufu(av + bias) : tanh_f(av + bias);
+                    s = fmaf(w.p2[ch][p], th, s);
+                }
+                tv[q][ch] = kBf16 ? tanh_mufu(s) : tanh_f(s);
+            }
+        }
+        __syncthreads();  // stage b is free for the prefetch issued in iteration k+1
+        if (row_ok) {
+            const int64_t C2 = c2_0 + 2 * tx;
+            if (kBf16) {
+                uint4* d = reinterpret_cast<uint4*>(a.t2) + (img * a.t2_rows + (R2 - a.t2_row0)) * a.w2 + C2;
+#pragma unroll
+                for (int q = 0; q < 2; ++q) {
+                    if (C2 + q >= a.w2) continue;
+                    uint32_t pk[4];
+#pragma unroll
+                    for (int m = 0; m < 4; ++m)
+                        asm("cvt.rn.bf16x2.f32 %0, %1, %2;\n" : "=r"(pk[m]) : "f"(tv[q][2 * m + 1]), "f"(tv[q][2 * m]));
+                    d[q] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                }
+            } else {
+                float* t2 = a.t2 + img * a.t2_img_stride + (R2 - a.t2_row0) * a.w2 + C2;
+#pragma unroll
+                for (int ch = 0; ch < 8; ++ch) {
+                    if (C2 + 1 < a.w2)
+                        *reinterpret_cast<float2*>(t2 + ch * plane) = make_float2(tv[0][ch], tv[1][ch]);
+                    else if (C2 < a.w2)
+                        t2[ch * plane] = tv[0][ch];
+                }
+            }
+        }
     }
 }
 
@@ -321,8 +496,47 @@ cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s) {
     for (int ch = 0; ch < 8; ++ch)
         for (int t = 0; t < 25; ++t) w.k1[t][ch] = a.k1_host[ch * 25 + t];
     std::memcpy(w.p2, a.p2_host, sizeof w.p2);
+    // TMA path: 16-byte aligned rows (W % 4 == 0 makes w1, w2 even and w1 % 4 == 0),
+    // images at a uniform stride of whole rows
+    const int64_t in_rows = a.W > 0 ? a.in_img_stride / a.W : 0;
+    const bool tma_ok = (a.W & 3) == 0 && (reinterpret_cast<uintptr_t>(a.in) & 15) == 0 &&
+                        in_rows * a.W == a.in_img_stride && (!a.b1_plane || (reinterpret_cast<uintptr_t>(a.b1) & 15) == 0) &&
+                        (a.bf16_out || (reinterpret_cast<uintptr_t>(a.t2) & 7) == 0) && in_rows < (1ll << 31) &&
+                        a.nimg < (1ll << 31);
+    if (tma_ok) {
+        CUtensorMap xm, bm;
+        bool ok = tma_make_3d(&xm, a.in, (uint64_t)a.W, (uint64_t)in_rows, (uint64_t)a.nimg, (uint64_t)a.W * 4,
+                              (uint64_t)a.in_img_stride * 4, U1T_IC, U1T_IR, 1);
+        if (ok && a.b1_plane)
+            ok = tma_make_3d(&bm, a.b1, (uint64_t)a.w1, (uint64_t)a.b1_rows, 8, (uint64_t)a.w1 * 4,
+                             (uint64_t)a.b1_rows * a.w1 * 4, U1T_BC, U1T_BR, 8);
+        else
+            bm = xm;  // unused
+        if (ok) {
+            const int tiles_c = (int)((a.w2 + U1T_C - 1) / U1T_C);
+            const int tiles_r = (int)((a.t2_rows + U1T_R - 1) / U1T_R);
+            const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
+            int dev = 0, sms = 148;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            const int64_t grid = std::min<int64_t>(ntiles, 2 * (int64_t)sms);
+            const size_t smem = 2 * (size_t)U1T_STAGE + 128;
+            auto go = [&](auto kern) -> cudaError_t {
+                cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                if (e != cudaSuccess) return e;
+                kern<<<(unsigned)grid, 128, smem, s>>>(xm, bm, a, w, tiles_c, tiles_r, ntiles);
+                return cudaGetLastError();
+            };
+            if (a.bf16_out)
+                return a.b1_plane ? go(cnn_u1_tma_kernel<true, true>) : go(cnn_u1_tma_kernel<true, false>);
+            return a.b1_plane ? go(cnn_u1_tma_kernel<false, true>) : go(cnn_u1_tma_kernel<false, false>);
+        }
+    }
     dim3 grid((unsigned)((a.w2 + U1_TC - 1) / U1_TC), (unsigned)((a.t2_rows + U1_TR - 1) / U1_TR), (unsigned)a.nimg);
-    cnn_u1_kernel<<<grid, 128, 0, s>>>(a, w);
+    if (a.bf16_out)
+        cnn_u1_kernel<true><<<grid, 128, 0, s>>>(a, w);
+    else
+        cnn_u1_kernel<false><<<grid, 128, 0, s>>>(a, w);
     return cudaGetLastError();
 }
 

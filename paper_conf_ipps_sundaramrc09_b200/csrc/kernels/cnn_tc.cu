@@ -13,9 +13,10 @@
 // the next pixel's channels, i.e. tap (i, j+1) -- so C3 needs 15 K-steps (not 25 x 16-wide)
 // and C5 40 (not 50 with a 12-channel zero pad).
 //
-// Epilogues run on all 4 warps from TMEM (tcgen05.ld 32x32b): bias plane + tanh, then
+// Both kernels are persistent and warp-specialised: one thread issues the bulk copies (TMA
+// engine) and the MMAs, epilogue warps drain TMEM (tcgen05.ld 32x32b): bias plane + tanh, then
 //   U2: the 2x2 subsample pairs row 2R (tile 0) with row 2R+1 (tile 1) in the same thread and
-//       columns c, c+1 across neighbouring lanes (shfl), + tanh -> T4 (fp32);
+//       columns c, c+1 across neighbouring lanes (shfl), + tanh -> T4 (bf16 channel blocks);
 //   U3: the 1x1 C6 layer as a dot product over n5 in registers, + bias -> output (fp32).
 // Precision: bf16 operands, fp32 accumulation; parity bound 2e-2 normwise (R16).
 #include <cuda_runtime.h>
@@ -28,6 +29,9 @@
 #include "kernels.h"
 #include "tc_sm100.cuh"
 
+#ifndef U2_EXP
+#define U2_EXP 0
+#endif
 namespace tg {
 namespace {
 
@@ -39,121 +43,203 @@ __device__ __forceinline__ float tanh_approx(float x) {
     return y;
 }
 
-constexpr int kThreads = 128;
 constexpr int kTileM = 128;
 
 // ============================================================================ U2 (C3)
-// Band = C3 rows (2R, 2R+1) x 128 columns [c0, c0+128): tile 0 = row 2R, tile 1 = row 2R+1.
-// Window: T2 rows [2R, 2R+6) x cols [c0, c0 + 134), 8 channels per pixel (one plane).
+// Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns [c0, c0+128): tile 0 = C3 row 2R,
+// tile 1 = row 2R+1 (M = 128 each, N = 32: 20 maps padded). Window: T2 rows [2R, 2R+6) x
+// cols [c0, c0+134), 8 channels per pixel (one 16-byte row each).
+// Warp-specialised and persistent (one CTA per SM, 9 warps):
+//   warp 8, one thread   producer + MMA issuer: the C3 B operand (15 K-steps) once per CTA by a
+//                        bulk copy; per segment six 1-D bulk copies (TMA engine) of the window's
+//                        T2 rows into one of U2_NA buffers (prefetched U2_NA-1 segments ahead);
+//                        2 tiles x 15 tcgen05.mma into one of 4 TMEM slots; tcgen05.commit frees
+//                        the window buffer and hands the slot to the epilogue
+//   warps 0-3 / 4-7      epilogue groups for even / odd segments: bias plane (prefetched one
+//                        segment ahead), tanh, the 2x2 subsample (rows in the same thread,
+//                        columns across neighbouring lanes), tanh -> T4 bf16 channel blocks
 constexpr int U2_WR = 6, U2_WP = kTileM + 6;  // +4 taps, +1 for the (4,5) tap pair, +1 spare
 constexpr int U2_N = 32;                      // 20 maps padded to 32
 constexpr int U2_KS = 15;                     // 5 rows x pairs (0,1) (2,3) (4,5)
+constexpr int U2_NA = 4;                      // window buffers
+constexpr int U2_NT = 4;                      // TMEM slots (2 per epilogue group)
+constexpr int kThreadsU2 = 9 * 32;
 
-struct U2TcShared {
-    uint4 a[U2_WR * U2_WP];            // [row][col] -> 8 bf16 channels
-    uint4 b[U2_KS * 2 * U2_N];         // [ks][half][n] -> 8 bf16
-    float p4[20][4];
-    uint64_t mbar;
+struct U2P {
+    float p4[20][4];  // S4 weights (constant bank)
+};
+
+struct U2Smem {
+    uint4 a[U2_NA][U2_WR * U2_WP];  // [row][col] -> 8 bf16 channels
+    uint4 b[U2_KS * 2 * U2_N];      // [ks][half][n] -> 8 bf16
+    uint64_t b_full, a_full[U2_NA], a_empty[U2_NA], t_full[U2_NT], t_empty[U2_NT];
     uint32_t tmem;
 };
 
-__global__ void __launch_bounds__(kThreads) cnn_u2_tc_kernel(const CnnU2Args a) {
+__global__ void __launch_bounds__(kThreadsU2, 1)
+    cnn_u2_tc_kernel(const CnnU2Args a, const __grid_constant__ U2P pw, const int64_t nseg) {
     extern __shared__ __align__(128) uint8_t smraw[];
-    U2TcShared& S = *reinterpret_cast<U2TcShared*>(smraw);
+    U2Smem& S = *reinterpret_cast<U2Smem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int bands_per_row = (int)((a.w3 + kTileM - 1) / kTileM);
-    const int64_t img = blockIdx.z;
-    const int64_t R = a.t4_row0 + blockIdx.y;      // T4 row (global)
-    const int64_t c0 = (int64_t)blockIdx.x * kTileM;  // C3 column of position 0
-    (void)bands_per_row;
+    const int64_t segs_per_row = (a.w3 + kTileM - 1) / kTileM;
+    const int64_t per_img = a.t4_rows * segs_per_row;
+    auto seg_coords = [&](int64_t sg, int64_t& img, int64_t& R, int64_t& c0) {
+        img = sg / per_img;
+        const int64_t rem = sg - img * per_img;
+        const int64_t rr = rem / segs_per_row;
+        R = a.t4_row0 + rr;
+        c0 = (rem - rr * segs_per_row) * kTileM;
+    };
 
-    if (warp == 0) tc::tmem_alloc<64>(&S.tmem);
+    if (warp == 0) tc::tmem_alloc<256>(&S.tmem);
     if (tid == 0) {
-        tc::mbar_init(&S.mbar, 1);
+        tc::mbar_init(&S.b_full, 1);
+        for (int i = 0; i < U2_NA; ++i) {
+            tc::mbar_init(&S.a_full[i], 1);
+            tc::mbar_init(&S.a_empty[i], 1);
+        }
+        for (int i = 0; i < U2_NT; ++i) {
+            tc::mbar_init(&S.t_full[i], 1);
+            tc::mbar_init(&S.t_empty[i], 4);
+        }
         tc::mbar_fence_init();
     }
-    // stage the T2 window: U1 wrote T2 as bf16 pixels [row][col][8 ch] = one 16-byte load each
-    const uint4* t2b = reinterpret_cast<const uint4*>(a.t2) + img * a.t2_rows * a.w2;
-    for (int idx = tid; idx < U2_WR * U2_WP; idx += kThreads) {
-        const int r = idx / U2_WP, c = idx - r * U2_WP;
-        const int64_t br = 2 * R + r - a.t2_row0, gc = c0 + c;
-        const bool ok = br >= 0 && br < a.t2_rows && gc < a.w2;
-        S.a[idx] = ok ? __ldg(t2b + br * a.w2 + gc) : make_uint4(0u, 0u, 0u, 0u);
-    }
-    const uint4* kb = reinterpret_cast<const uint4*>(a.k3_tc);
-    for (int idx = tid; idx < U2_KS * 2 * U2_N; idx += kThreads) S.b[idx] = __ldg(kb + idx);
-    for (int idx = tid; idx < 80; idx += kThreads) S.p4[idx / 4][idx % 4] = __ldg(a.p4_dev + idx);
+    // windows start zeroed: pixels a copy does not cover (beyond the image) then only ever
+    // hold finite T2 values
+    for (int idx = tid; idx < U2_NA * U2_WR * U2_WP; idx += kThreadsU2) (&S.a[0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
     tc::fence_proxy_async();
     tc::fence_before_sync();
     __syncthreads();
     tc::fence_after_sync();
     const uint32_t tmem = S.tmem;
+    const int64_t my = nseg > blockIdx.x ? (nseg - 1 - blockIdx.x) / gridDim.x + 1 : 0;
 
-    if (tid == 0) {
-        const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
-        const uint32_t a0 = tc::smem_u32(S.a), b0 = tc::smem_u32(S.b);
-        for (int t = 0; t < 2; ++t) {       // tile t = C3 row 2R + t
-            for (int ks = 0; ks < U2_KS; ++ks) {
-                const int i = ks / 3, j = 2 * (ks % 3);
-                const uint32_t a_addr = a0 + (uint32_t)(((t + i) * U2_WP + j) * 16);
-                const uint64_t ad = tc::make_desc(a_addr, 16, 128);  // 2nd K-half = next pixel (tap j+1)
-                const uint64_t bd = tc::make_desc(b0 + (uint32_t)(ks * 2 * U2_N * 16), U2_N * 16, 128);
-                tc::mma_bf16(tmem + (uint32_t)(t * U2_N), ad, bd, idesc, ks > 0 ? 1u : 0u);
+    if (warp == 8) {
+        if (lane == 0) {
+            // ---------------------------------------------------------------- producer + MMA
+            const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
+            auto load_a = [&](int64_t k) {
+                int64_t img, R, c0;
+                seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
+                const int buf = (int)(k % U2_NA);
+                const int64_t r0 = 2 * R - a.t2_row0;
+                const int64_t rows = min((int64_t)U2_WR, a.t2_rows - r0);
+                const int64_t cols = min((int64_t)U2_WP, a.w2 - c0);
+                tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(rows * cols * 16));
+                const uint4* src = t2all + (img * a.t2_rows + r0) * a.w2 + c0;
+                for (int r = 0; r < rows; ++r)
+                    tc::bulk_g2s(&S.a[buf][r * U2_WP], src + r * a.w2, (uint32_t)(cols * 16), &S.a_full[buf]);
+            };
+            const uint32_t bbytes = (uint32_t)(U2_KS * 2 * U2_N * 16);
+            tc::mbar_expect_tx(&S.b_full, bbytes);
+            tc::bulk_g2s(S.b, a.k3_tc, bbytes, &S.b_full);
+            for (int64_t k = 0; k < U2_NA - 1 && k < my; ++k) load_a(k);
+            tc::mbar_wait(&S.b_full, 0);
+            const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
+            const uint32_t b0 = tc::smem_u32(S.b);
+            for (int64_t k = 0; k < my; ++k) {
+                const int buf = (int)(k % U2_NA), ts = (int)(k % U2_NT);
+                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
+                if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
+                tc::fence_after_sync();
+                const uint32_t a0 = tc::smem_u32(S.a[buf]);
+                const uint32_t d0 = tmem + (uint32_t)(ts * 2 * U2_N);
+#if U2_EXP == 2
+                if (0)
+#endif
+                for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
+                    for (int ks = 0; ks < U2_KS; ++ks) {
+                        const int i = ks / 3, j = 2 * (ks % 3);
+                        const uint32_t a_addr = a0 + (uint32_t)(((t + i) * U2_WP + j) * 16);
+                        const uint64_t ad = tc::make_desc(a_addr, 16, 128);  // 2nd K-half = next pixel (tap j+1)
+                        const uint64_t bd = tc::make_desc(b0 + (uint32_t)(ks * 2 * U2_N * 16), U2_N * 16, 128);
+                        tc::mma_bf16(d0 + (uint32_t)(t * U2_N), ad, bd, idesc, ks > 0 ? 1u : 0u);
+                    }
+                }
+                tc::commit(&S.a_empty[buf]);
+                tc::commit(&S.t_full[ts]);
+                // keep U2_NA-1 windows in flight: refill the buffer segment k-1 used (its MMAs
+                // are done or about to be: segment k's MMAs are queued behind them)
+                if (k + U2_NA - 1 < my) {
+                    if (k >= 1) tc::mbar_wait(&S.a_empty[(k - 1) % U2_NA], (uint32_t)(((k - 1) / U2_NA) & 1));
+                    load_a(k + U2_NA - 1);
+                }
             }
         }
-        tc::commit(&S.mbar);
-    }
-    tc::mbar_wait(&S.mbar, 0);
-    tc::fence_after_sync();
-
-    // epilogue: thread = C3 column c0 + 32*warp + lane, rows 2R (tile 0) and 2R+1 (tile 1)
-    float v0[32], v1[32];
-    const uint32_t lane_base = (uint32_t)(32 * warp) << 16;
-    tc::tmem_ld32(tmem + lane_base + 0, v0);
-    tc::tmem_ld32(tmem + lane_base + U2_N, v1);
-    const int64_t c = c0 + 32 * warp + lane;  // C3 column
-    const int64_t C = c >> 1;                 // T4 column
-    const bool row_ok = R < a.t4_row0 + a.t4_rows;
-    const bool col_ok = c < a.w3;
-    float tv[20];
-#pragma unroll
-    for (int co = 0; co < 20; ++co) {
-        float t0 = 0.f, t1 = 0.f;
-        if (row_ok && col_ok) {
-            float b0, b1;
-            if (a.b3_plane) {
-                b0 = __ldg(a.b3 + ((int64_t)co * a.b3_rows + (2 * R - a.b3_row0)) * a.w3 + c);
-                b1 = __ldg(a.b3 + ((int64_t)co * a.b3_rows + (2 * R + 1 - a.b3_row0)) * a.w3 + c);
-            } else {
-                b0 = b1 = __ldg(a.b3 + co);
-            }
-            t0 = tanh_approx(v0[co] + b0);
-            t1 = tanh_approx(v1[co] + b1);
-        }
-        // odd lanes hold column c+1 of the even lane's 2x2 window
-        const float t01 = __shfl_down_sync(0xffffffffu, t0, 1);
-        const float t11 = __shfl_down_sync(0xffffffffu, t1, 1);
-        if (row_ok && !(lane & 1) && C < a.w4) {
-            float s = S.p4[co][0] * t0;
-            s = fmaf(S.p4[co][1], t01, s);
-            s = fmaf(S.p4[co][2], t1, s);
-            s = fmaf(S.p4[co][3], t11, s);
-            tv[co] = tanh_approx(s);
-        }
-    }
-    if (row_ok && !(lane & 1) && C < a.w4) {
-        // T4 as bf16 channel blocks [3][rows][w4][8] (U3's tensor-core operand rows)
+    } else {
+        // -------------------------------------------------------------------- epilogue groups
+        const int grp = warp >> 2, wq = warp & 3;
+        const uint32_t lane_base = (uint32_t)(32 * wq) << 16;
         const int64_t bplane = a.t4_rows * a.w4;
-        uint4* t4 = reinterpret_cast<uint4*>(a.t4) + img * 3 * bplane + (R - a.t4_row0) * a.w4 + C;
-        t4[0] = make_uint4(tc::pack_bf16(tv[0], tv[1]), tc::pack_bf16(tv[2], tv[3]), tc::pack_bf16(tv[4], tv[5]),
-                           tc::pack_bf16(tv[6], tv[7]));
-        t4[bplane] = make_uint4(tc::pack_bf16(tv[8], tv[9]), tc::pack_bf16(tv[10], tv[11]),
-                                tc::pack_bf16(tv[12], tv[13]), tc::pack_bf16(tv[14], tv[15]));
-        t4[2 * bplane] = make_uint4(tc::pack_bf16(tv[16], tv[17]), tc::pack_bf16(tv[18], tv[19]), 0u, 0u);
+        // Bias of both C3 rows of a segment, software-pipelined across segments: the loads for
+        // this group's NEXT segment are issued as soon as the current values are consumed, so
+        // they are in flight during the stores and the wait for the next accumulator.
+        float b0v[20], b1v[20];
+        auto load_bias = [&](int64_t kk) {
+            int64_t img_, R_, c0_;
+            seg_coords(blockIdx.x + kk * gridDim.x, img_, R_, c0_);
+            const int64_t cc = min(c0_ + 32 * wq + lane, a.w3 - 1);
+#pragma unroll
+            for (int co = 0; co < 20; ++co) {
+                if (a.b3_plane) {
+                    b0v[co] = __ldg(a.b3 + ((int64_t)co * a.b3_rows + (2 * R_ - a.b3_row0)) * a.w3 + cc);
+                    b1v[co] = __ldg(a.b3 + ((int64_t)co * a.b3_rows + (2 * R_ + 1 - a.b3_row0)) * a.w3 + cc);
+                } else {
+                    b0v[co] = b1v[co] = __ldg(a.b3 + co);
+                }
+            }
+        };
+        if (grp < my) load_bias(grp);
+        for (int64_t k = grp; k < my; k += 2) {
+            const int ts = (int)(k % U2_NT);
+            int64_t img, R, c0;
+            seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
+            const int64_t c = c0 + 32 * wq + lane;  // C3 column
+            const int64_t C = c >> 1;               // T4 column
+            tc::mbar_wait(&S.t_full[ts], (uint32_t)((k / U2_NT) & 1));
+            tc::fence_after_sync();
+#if U2_EXP >= 1
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&S.t_empty[ts]);
+            continue;
+#endif
+            float v0[32], v1[32];
+            tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 2 * U2_N), v0);
+            tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 2 * U2_N + U2_N), v1);
+            tc::tmem_wait_ld();
+            tc::fence_before_sync();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&S.t_empty[ts]);
+            const bool out_ok = !(lane & 1) && C < a.w4;
+            float tv[20];
+#pragma unroll
+            for (int co = 0; co < 20; ++co) {
+                const float t0 = tanh_approx(v0[co] + b0v[co]);
+                const float t1 = tanh_approx(v1[co] + b1v[co]);
+                // odd lanes hold column c+1 of the even lane's 2x2 window
+                const float t01 = __shfl_down_sync(0xffffffffu, t0, 1);
+                const float t11 = __shfl_down_sync(0xffffffffu, t1, 1);
+                float s4 = pw.p4[co][0] * t0;
+                s4 = fmaf(pw.p4[co][1], t01, s4);
+                s4 = fmaf(pw.p4[co][2], t1, s4);
+                s4 = fmaf(pw.p4[co][3], t11, s4);
+                tv[co] = tanh_approx(s4);
+            }
+            if (k + 2 < my) load_bias(k + 2);
+            if (out_ok) {
+                // T4 as bf16 channel blocks [3][rows][w4][8] (U3's tensor-core operand rows)
+                uint4* t4 = reinterpret_cast<uint4*>(a.t4) + img * 3 * bplane + (R - a.t4_row0) * a.w4 + C;
+                t4[0] = make_uint4(tc::pack_bf16(tv[0], tv[1]), tc::pack_bf16(tv[2], tv[3]),
+                                   tc::pack_bf16(tv[4], tv[5]), tc::pack_bf16(tv[6], tv[7]));
+                t4[bplane] = make_uint4(tc::pack_bf16(tv[8], tv[9]), tc::pack_bf16(tv[10], tv[11]),
+                                        tc::pack_bf16(tv[12], tv[13]), tc::pack_bf16(tv[14], tv[15]));
+                t4[2 * bplane] = make_uint4(tc::pack_bf16(tv[16], tv[17]), tc::pack_bf16(tv[18], tv[19]), 0u, 0u);
+            }
+        }
     }
     tc::fence_before_sync();
     __syncthreads();
-    if (warp == 0) tc::tmem_dealloc<64>(tmem);
+    if (warp == 0) tc::tmem_dealloc<256>(tmem);
 }
 
 // ============================================================================ U3 (C5 + C6)
@@ -483,10 +569,16 @@ void cnn_prepare_k5_tc(const float* k5, int n5, uint16_t* dst) {
 cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s) {
     if (a.t4_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     static std::atomic<uint32_t> flags{0};
-    const size_t smem = sizeof(U2TcShared);
+    const size_t smem = sizeof(U2Smem) + 128;
     if (!set_smem_attr((const void*)cnn_u2_tc_kernel, smem, flags)) return cudaErrorInvalidValue;
-    dim3 grid((unsigned)((a.w3 + kTileM - 1) / kTileM), (unsigned)a.t4_rows, (unsigned)a.nimg);
-    cnn_u2_tc_kernel<<<grid, kThreads, smem, s>>>(a);
+    U2P pw;
+    std::memcpy(pw.p4, a.p4_host, sizeof pw.p4);
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t nseg = a.t4_rows * ((a.w3 + kTileM - 1) / kTileM) * a.nimg;
+    const unsigned grid = (unsigned)std::min<int64_t>(nseg, sms);
+    cnn_u2_tc_kernel<<<grid, kThreadsU2, smem, s>>>(a, pw, nseg);
     return cudaGetLastError();
 }
 

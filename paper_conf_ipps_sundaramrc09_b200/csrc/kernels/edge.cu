@@ -39,6 +39,7 @@
 #include <mutex>
 
 #include "kernels.h"
+#include "tma_util.cuh"
 
 namespace tg {
 namespace {
@@ -260,7 +261,9 @@ __global__ void __launch_bounds__(kThreads, 2)
     }
 }
 
-PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+}  // namespace
+
+PFN_cuTensorMapEncodeTiled_v12000 tma_encode_fn() {
     static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
     static std::once_flag once;
     std::call_once(once, [] {
@@ -272,8 +275,6 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     });
     return fn;
 }
-
-}  // namespace
 
 template <int kComb, int kPairs, int kF>
 cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s);
@@ -316,7 +317,7 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
             }
     const int tiles_c = (int)((a.W + kTileC - 1) / kTileC);
     const int tiles_r = (int)((a.out_rows + kTileR - 1) / kTileR);
-    PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
+    PFN_cuTensorMapEncodeTiled_v12000 enc = tma_encode_fn();
     const bool tma_ok = enc && (a.W & 3) == 0 && (reinterpret_cast<uintptr_t>(a.in) & 15) == 0 &&
                         a.in_img_stride == a.in_rows * a.W && a.in_rows < (1ll << 31) && a.W < (1ll << 31);
     if (tma_ok) {

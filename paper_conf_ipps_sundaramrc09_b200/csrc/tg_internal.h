@@ -177,6 +177,7 @@ namespace tg {
 tg_status exec_run(tg_plan* p, bool blocking);
 tg_status exec_set_profiling(tg_plan* p, bool on);
 tg_status exec_timing(tg_plan* p, tg_timing* out);
+tg_status exec_trace(tg_plan* p, tg_trace_rec* out, size_t cap, size_t* n);
 void exec_destroy(tg_plan* p);
 uint64_t exec_registered_bytes(const tg_plan* p);
 void exec_invalidate_params(tg_plan* p);

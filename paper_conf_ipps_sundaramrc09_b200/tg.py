@@ -73,6 +73,11 @@ class tg_timing(ctypes.Structure):
                 ("unit_launches", c_i64 * 4), ("h2d_ms", ctypes.c_double), ("d2h_ms", ctypes.c_double)]
 
 
+class tg_trace_rec(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int32), ("kind", ctypes.c_int32), ("chunk", ctypes.c_int64),
+                ("t0_ms", ctypes.c_double), ("t1_ms", ctypes.c_double)]
+
+
 _PROTOS = {
     "tg_graph_create": (c_i32, [ctypes.POINTER(vp)]),
     "tg_graph_destroy": (None, [vp]),
@@ -102,6 +107,7 @@ _PROTOS = {
     "tg_execute_async": (c_i32, [vp]),
     "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
     "tg_plan_timing_get": (c_i32, [vp, ctypes.POINTER(tg_timing)]),
+    "tg_plan_trace_get": (c_i32, [vp, ctypes.POINTER(tg_trace_rec), c_sz, ctypes.POINTER(c_sz)]),
     "tg_plan_launch_count": (c_i64, [vp]),
     "tg_plan_invalidate_params": (c_i32, [vp]),
     "tg_plan_destroy": (None, [vp]),
@@ -290,6 +296,18 @@ def tg_plan_timing_get(p) -> dict:
     _ck(_lib.tg_plan_timing_get(p, ctypes.byref(t)))
     return {"launches": t.launches, "executions": t.executions, "kernel_ms": list(t.kernel_ms),
             "unit_launches": list(t.unit_launches), "h2d_ms": t.h2d_ms, "d2h_ms": t.d2h_ms}
+
+
+TRACE_KINDS = {0: "edge", 1: "U1", 2: "U2", 3: "U3", 10: "h2d", 11: "d2h"}
+
+
+def tg_plan_trace_get(p) -> list[dict]:
+    n = c_sz(0)
+    _ck(_lib.tg_plan_trace_get(p, None, 0, ctypes.byref(n)))
+    buf = (tg_trace_rec * max(1, n.value))()
+    _ck(_lib.tg_plan_trace_get(p, buf, n.value, ctypes.byref(n)))
+    return [{"device": r.device, "kind": TRACE_KINDS.get(r.kind, str(r.kind)), "chunk": r.chunk,
+             "t0_ms": r.t0_ms, "t1_ms": r.t1_ms} for r in buf[:n.value]]
 
 
 def tg_plan_launch_count(p) -> int:
@@ -487,6 +505,10 @@ class Plan:
 
     def launches(self) -> int:
         return tg_plan_launch_count(self.h)
+
+    def trace(self) -> list[dict]:
+        """Timeline of the profiled copies and kernel launches (tg_plan_trace_get)."""
+        return tg_plan_trace_get(self.h)
 
     def invalidate_params(self) -> None:
         tg_plan_invalidate_params(self.h)

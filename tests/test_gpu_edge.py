@@ -257,3 +257,39 @@ def test_pipelined_async_executions(tg):
             p.execute(blocking=False)
         torch.cuda.synchronize()
         assert torch.equal(out_t, ref)
+
+
+def test_trace_respects_stream_dependencies(tg):
+    """tg_plan_trace_get: one record per chunk copy and launch; per chunk H2D ends before its
+    kernel starts and the kernel ends before its D2H starts; a slot (depth 2) is not
+    overwritten before the chunk that used it two steps earlier finished computing; copies
+    of one direction never overlap each other (one stream each)."""
+    n, H, W = 2, 300, 256
+    img_t = pinned((n, 1, H, W))
+    img_t.copy_(torch.from_numpy(synth.images_np(13, n, H, W)))
+    out_t = pinned((n, 1, H, W))
+    K1, _ = synth.edge_filter_np()
+    g, _ = tg.edge_graph(img_t, K1, out=out_t)
+    g.set(budget=400_000, depth=2, torch_runtime=True)
+    p = g.plan()
+    p.execute()                        # parameters resident; not profiled
+    p.profiling(True)
+    p.execute(blocking=False)
+    p.execute(blocking=False)
+    tr = p.trace()
+    nc = p.stats()["n_chunks"]
+    assert len(tr) == 2 * 3 * nc
+    eps = 1e-3
+    for e in range(2):
+        recs = tr[e * 3 * nc:(e + 1) * 3 * nc]
+        by = {(r["kind"], r["chunk"]): r for r in recs}
+        assert len(by) == 3 * nc
+        for c in range(nc):
+            h, k, d = by[("h2d", c)], by[("edge", c)], by[("d2h", c)]
+            assert h["t0_ms"] <= h["t1_ms"] <= k["t0_ms"] + eps
+            assert k["t1_ms"] <= d["t0_ms"] + eps
+            if c >= 2:
+                assert by[("edge", c - 2)]["t1_ms"] <= h["t0_ms"] + eps
+    for kind in ("h2d", "d2h", "edge"):
+        iv = sorted((r["t0_ms"], r["t1_ms"]) for r in tr if r["kind"] == kind)
+        assert all(a[1] <= b[0] + eps for a, b in zip(iv, iv[1:])), kind
