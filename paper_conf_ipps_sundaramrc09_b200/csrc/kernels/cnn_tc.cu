@@ -32,6 +32,9 @@
 #ifndef U2_EXP
 #define U2_EXP 0
 #endif
+#ifndef U3_EXP
+#define U3_EXP 0
+#endif
 namespace tg {
 namespace {
 
@@ -61,7 +64,7 @@ constexpr int kTileM = 128;
 constexpr int U2_WR = 6, U2_WP = kTileM + 6;  // +4 taps, +1 for the (4,5) tap pair, +1 spare
 constexpr int U2_N = 32;                      // 20 maps padded to 32
 constexpr int U2_KS = 15;                     // 5 rows x pairs (0,1) (2,3) (4,5)
-constexpr int U2_NA = 4;                      // window buffers
+constexpr int U2_NA = 8;                      // window buffers
 constexpr int U2_NT = 4;                      // TMEM slots (2 per epilogue group)
 constexpr int kThreadsU2 = 9 * 32;
 
@@ -115,55 +118,69 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
     const int64_t my = nseg > blockIdx.x ? (nseg - 1 - blockIdx.x) / gridDim.x + 1 : 0;
 
     if (warp == 8) {
-        if (lane == 0) {
-            // ---------------------------------------------------------------- producer + MMA
-            const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
-            auto load_a = [&](int64_t k) {
-                int64_t img, R, c0;
-                seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
-                const int buf = (int)(k % U2_NA);
-                const int64_t r0 = 2 * R - a.t2_row0;
-                const int64_t rows = min((int64_t)U2_WR, a.t2_rows - r0);
-                const int64_t cols = min((int64_t)U2_WP, a.w2 - c0);
+        // -------------------------------------------------------------------- producer + MMA
+        // (the whole warp runs the loop, so descriptors stay in uniform registers; one elected
+        // lane issues the copies, MMAs and commits)
+        const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
+        auto load_a = [&](int64_t k) {
+            int64_t img, R, c0;
+            seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
+            const int buf = (int)(k % U2_NA);
+            const int64_t r0 = 2 * R - a.t2_row0;
+            const int64_t rows = min((int64_t)U2_WR, a.t2_rows - r0);
+            const int64_t cols = min((int64_t)U2_WP, a.w2 - c0);
+            if (tc::elect_one()) {
                 tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(rows * cols * 16));
                 const uint4* src = t2all + (img * a.t2_rows + r0) * a.w2 + c0;
                 for (int r = 0; r < rows; ++r)
                     tc::bulk_g2s(&S.a[buf][r * U2_WP], src + r * a.w2, (uint32_t)(cols * 16), &S.a_full[buf]);
-            };
-            const uint32_t bbytes = (uint32_t)(U2_KS * 2 * U2_N * 16);
+            }
+            __syncwarp();
+        };
+        const uint32_t bbytes = (uint32_t)(U2_KS * 2 * U2_N * 16);
+        if (tc::elect_one()) {
             tc::mbar_expect_tx(&S.b_full, bbytes);
             tc::bulk_g2s(S.b, a.k3_tc, bbytes, &S.b_full);
-            for (int64_t k = 0; k < U2_NA - 1 && k < my; ++k) load_a(k);
-            tc::mbar_wait(&S.b_full, 0);
-            const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
-            const uint32_t b0 = tc::smem_u32(S.b);
-            for (int64_t k = 0; k < my; ++k) {
-                const int buf = (int)(k % U2_NA), ts = (int)(k % U2_NT);
-                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
-                if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
-                tc::fence_after_sync();
-                const uint32_t a0 = tc::smem_u32(S.a[buf]);
-                const uint32_t d0 = tmem + (uint32_t)(ts * 2 * U2_N);
+        }
+        __syncwarp();
+        for (int64_t k = 0; k < U2_NA - 1 && k < my; ++k) load_a(k);
+        tc::mbar_wait(&S.b_full, 0);
+        const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
+        // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding
+        const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), U2_N * 16, 128);
+        const uint64_t adesc0 = tc::make_desc(tc::smem_u32(S.a[0]), 16, 128);  // 2nd K-half = next pixel
+        for (int64_t k = 0; k < my; ++k) {
+            const int buf = (int)(k % U2_NA), ts = (int)(k % U2_NT);
+            tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
+            if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
+            tc::fence_after_sync();
+            const uint64_t abuf = adesc0 + (uint64_t)(buf * (U2_WR * U2_WP));
+            const uint32_t d0 = tmem + (uint32_t)(ts * 2 * U2_N);
 #if U2_EXP == 2
-                if (0)
+            if (0)
 #endif
+            if (tc::elect_one()) {
+#pragma unroll
                 for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
+#pragma unroll
                     for (int ks = 0; ks < U2_KS; ++ks) {
                         const int i = ks / 3, j = 2 * (ks % 3);
-                        const uint32_t a_addr = a0 + (uint32_t)(((t + i) * U2_WP + j) * 16);
-                        const uint64_t ad = tc::make_desc(a_addr, 16, 128);  // 2nd K-half = next pixel (tap j+1)
-                        const uint64_t bd = tc::make_desc(b0 + (uint32_t)(ks * 2 * U2_N * 16), U2_N * 16, 128);
-                        tc::mma_bf16(d0 + (uint32_t)(t * U2_N), ad, bd, idesc, ks > 0 ? 1u : 0u);
+                        tc::mma_bf16(d0 + (uint32_t)(t * U2_N), abuf + (uint64_t)((t + i) * U2_WP + j),
+                                     bdesc0 + (uint64_t)(ks * 2 * U2_N), idesc, ks > 0 ? 1u : 0u);
                     }
                 }
+            }
+            __syncwarp();
+            if (tc::elect_one()) {
                 tc::commit(&S.a_empty[buf]);
                 tc::commit(&S.t_full[ts]);
-                // keep U2_NA-1 windows in flight: refill the buffer segment k-1 used (its MMAs
-                // are done or about to be: segment k's MMAs are queued behind them)
-                if (k + U2_NA - 1 < my) {
-                    if (k >= 1) tc::mbar_wait(&S.a_empty[(k - 1) % U2_NA], (uint32_t)(((k - 1) / U2_NA) & 1));
-                    load_a(k + U2_NA - 1);
-                }
+            }
+            __syncwarp();
+            // keep U2_NA-1 windows in flight: refill the buffer segment k-1 used (its MMAs
+            // are done or about to be: segment k's MMAs are queued behind them)
+            if (k + U2_NA - 1 < my) {
+                if (k >= 1) tc::mbar_wait(&S.a_empty[(k - 1) % U2_NA], (uint32_t)(((k - 1) / U2_NA) & 1));
+                load_a(k + U2_NA - 1);
             }
         }
     } else {
@@ -405,6 +422,9 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                             lbo = 16;
                         }
                         const uint64_t bd = tc::make_desc(b_base + (uint32_t)(u * 2 * NP * 16), (uint32_t)(NP * 16), 128);
+#if U3_EXP == 2
+                        if (0)
+#endif
                         for (int t = 0; t < 2; ++t) {
                             const uint64_t ad = tc::make_desc(a_addr + (uint32_t)(t * kTileM * 16), lbo, 128);
                             tc::mma_bf16(d_base + (uint32_t)(t * NP), ad, bd, idesc, ks > 0 ? 1u : 0u);
@@ -436,6 +456,11 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             const U3Band g = u3_band(a, band, per_img, flat);
             tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
             tc::fence_after_sync();
+#if U3_EXP >= 1
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);
+            continue;
+#endif
             const int m = t * kTileM + 32 * (warp & 3) + lane;
             int64_t orow, ocol;
             if (flat) {
@@ -473,14 +498,15 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                     tc::tmem_wait_ld();
                     if (c + 1 < nch) issue(c + 1, (c + 1) & 1);
                     if (ok) {
+                        // branch-free over the chunk (C6 weights of the padding channels
+                        // n5..NP-1 are zero and their accumulators finite), so the tanh of
+                        // several channels are in flight at once
 #pragma unroll
                         for (int u = 0; u < 32; ++u) {
                             const int ch = 32 * c + u;
-                            if (ch < a.n5) {
-                                const float th = tanh_approx(v[c & 1][u] + bv[c & 1][u]);
+                            const float th = tanh_approx(v[c & 1][u] + bv[c & 1][u]);
 #pragma unroll
-                                for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], th, c6[o]);
-                            }
+                            for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], th, c6[o]);
                         }
                     }
                 }
