@@ -292,7 +292,7 @@ def run(args, rank, world, local):
     traffic = None
     tf_file = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf_file):
-        tr = json.load(open(tf_file)).get(f"{args.template}:{KERNEL_NAMES[k]}")
+        tr = json.load(open(tf_file)).get(f"{args.template}:{args.precision}:{KERNEL_NAMES[k]}")
         if tr:
             traffic = tr["dram_bytes_per_out_px"] * opx[k] * args.steps / nl
     roofline = {"bound": "tensor" if tensor else "alu", "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
