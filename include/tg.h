@@ -139,7 +139,7 @@ tg_status tg_set_devices(tg_graph* g, const int32_t* ordinals, int32_t n);
  * uncapped. The plan's arena never exceeds it. */
 tg_status tg_set_device_budget(tg_graph* g, uint64_t bytes_per_device);
 tg_status tg_set_precision(tg_graph* g, int32_t prec);
-/* Input pixels per chunk when memory does not bind (default 1<<24) and pipeline depth
+/* Input pixels per chunk when memory does not bind (default 1<<25) and pipeline depth
  * (in-flight chunk slots, default 3, 1..8). */
 tg_status tg_set_chunking(tg_graph* g, int64_t max_chunk_px, int32_t depth);
 /* Multi-process sharding: this process executes chunk range [floor(C*rank/world),

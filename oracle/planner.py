@@ -438,7 +438,7 @@ def fig3_graph() -> tuple[Graph, dict[str, int]]:
 
 # ============================================================================ chunk rule
 DEPTH = 3                 # pipeline slots (H2D / compute / D2H in flight)
-MAX_CHUNK_PX = 1 << 24    # input pixels per chunk when memory does not bind
+MAX_CHUNK_PX = 1 << 25    # input pixels per chunk when memory does not bind
 F32 = 4
 
 

@@ -52,7 +52,7 @@ struct Graph {
     std::vector<int32_t> devices;
     uint64_t budget = 0;
     int32_t precision = TG_FP32;
-    int64_t max_chunk_px = int64_t(1) << 24;
+    int64_t max_chunk_px = int64_t(1) << 25;
     int32_t depth = 3;
     int32_t rank = 0, world = 1;
     tg_runtime rt{};

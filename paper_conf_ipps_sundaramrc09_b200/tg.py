@@ -466,7 +466,7 @@ class Graph:
         if devices is not None:
             tg_set_devices(self.h, list(devices))
         if max_chunk_px is not None or depth is not None:
-            tg_set_chunking(self.h, max_chunk_px or (1 << 24), depth or 3)
+            tg_set_chunking(self.h, max_chunk_px or (1 << 25), depth or 3)
         if shard is not None:
             tg_set_shard(self.h, *shard)
         if torch_runtime:

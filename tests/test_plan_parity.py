@@ -80,7 +80,8 @@ def library_plan(tmpl, n, H, W, kw):
         out = np.zeros(1, np.float32)
         g._keep.append(out)
         tg.tg_output(g.h, y, out.ctypes.data)
-    g.set(budget=kw.get("budget", 0), max_chunk_px=kw.get("max_chunk_px", 1 << 24), depth=kw.get("depth", 3),
+    # chunking left unset unless the case sets it: the library's default meets the oracle's
+    g.set(budget=kw.get("budget", 0), max_chunk_px=kw.get("max_chunk_px"), depth=kw.get("depth"),
           shard=(kw.get("rank", 0), kw.get("world", 1)),
           precision=tg.TG_BF16_TC if kw.get("precision") == "bf16_tc" else tg.TG_FP32)
     return g.plan().json()
