@@ -254,14 +254,31 @@ def run(args, rank, world, local):
     p.profiling(True)
     l0 = p.launches()
     barrier(world)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    # inputs smaller than 2x the 126 MB L2: flush L2 between timed steps (a 512 MB write on the
+    # compute stream, outside the per-step events); larger inputs stream through L2 anyway
+    flush = torch.empty(128 << 20, dtype=torch.float32, device=dev) if px * 4 < (252 << 20) else None
     with ClockSampler(local) as clk:
-        e0.record(cs)
-        for _ in range(args.steps):
-            p.execute(blocking=False)
-        e1.record(cs)
-        torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / args.steps
+        if flush is None:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(cs)
+            for _ in range(args.steps):
+                p.execute(blocking=False)
+            e1.record(cs)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / args.steps
+        else:
+            evs = []
+            for _ in range(args.steps):
+                with torch.cuda.stream(cs):
+                    flush.zero_()
+                ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                ea.record(cs)
+                p.execute(blocking=False)
+                eb.record(cs)
+                evs.append((ea, eb))
+            torch.cuda.synchronize()
+            ms = sum(a.elapsed_time(b) for a, b in evs) / args.steps
+    del flush
     launches = p.launches() - l0
     tim = p.timing()
     ms_max = max_over_ranks(ms, world)
@@ -349,6 +366,10 @@ def run(args, rank, world, local):
            "split": js["split"], "bias": js["bias"], "gpu_launches": launches2,
            "kernel_ms_per_step": sum(tim2["kernel_ms"]) / args.steps,
            "h2d_ms_per_step": tim2["h2d_ms"] / args.steps, "d2h_ms_per_step": tim2["d2h_ms"] / args.steps}
+    # overlap = (sum copy + sum kernel - wall) / min(sum copy, sum kernel)
+    s_copy = (tim2["h2d_ms"] + tim2["d2h_ms"]) / args.steps
+    s_kern = sum(tim2["kernel_ms"]) / args.steps
+    e2e["overlap"] = (s_copy + s_kern - ms2) / max(min(s_copy, s_kern), 1e-9)
     if rank == 0:
         link = host_link_peak(local)
         # link roofline: each direction at its solo peak, both together at the measured
@@ -365,17 +386,26 @@ def run(args, rank, world, local):
             f"{'uncapped' if not wl['budget'] else str(wl['budget'] >> 20) + ' MiB device budget'}, streamed")
     config = {"workload": desc, "template": wl["template"], "images_per_gpu": n, "H": H, "W": W,
               "n5": wl.get("n5"), "budget_bytes_e2e": wl["budget"], "precision": args.precision,
-              "l2": f"inputs {px * 4 / 1e9:.2f} GB per step" + (" >> 126 MB L2 (no flush needed)" if px * 4 > 1e9
-                                                               else " (L2 not flushed)")}
+              "l2": f"inputs {px * 4 / 1e9:.2f} GB per step" + (" >> 126 MB L2 (no flush needed)" if px * 4 >= (252 << 20)
+                                                               else ": L2 flushed (512 MB write) before every timed step")}
     return {"value": value, "ms_per_step": ms_max, "clocks": clocks, "gpu_launches": launches,
-            "roofline": roofline, "e2e": e2e, "config": config}
+            "roofline": roofline, "e2e": e2e, "config": config, "y_host": y_host}
 
 
 # ------------------------------------------------------------------------------ CPU leg
-def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0) -> dict:
+def _normwise(g, r) -> float:
+    """max over output planes of max|g - r| / max|r| (R16)."""
+    import numpy as np
+    g = np.asarray(g, np.float64).reshape(-1, r.shape[-2] * r.shape[-1])
+    r = np.asarray(r, np.float64).reshape(-1, r.shape[-2] * r.shape[-1])
+    return float(max(np.abs(g[i] - r[i]).max() / max(np.abs(r[i]).max(), 1e-30) for i in range(r.shape[0])))
+
+
+def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0, gpu_out=None, tol: float = 1e-5) -> dict:
     """The CPU oracle (as it stands) on a bounded sample of the workload: for the edge
-    template whole 10000x10000 images of configs[1] (plus a band of rows if one image is
-    too fast); for the CNN a band of rows of the workload's image. Reports input Mpx/s."""
+    template whole 10000x10000 images of configs[1]; for the CNN one image of the workload.
+    Reports input Mpx/s. With gpu_out (the GPU run's host output, [n][c][h][w]) the sampled
+    images' oracle outputs are also compared with it: outputs verified in the same run."""
     import oracle
     import synth
     oracle.build()
@@ -383,12 +413,14 @@ def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0) -> dict:
         W = 10000
         seed = synth.seed_for_config(2)
         K1, K2 = synth.edge_filter_np()
-        done_px, t_tot, imgs = 0, 0.0, 0
+        done_px, t_tot, imgs, err = 0, 0.0, 0, 0.0
         while t_tot < target_s and imgs < 15:
             img = synth.image_np(seed, synth.DS_IMAGE, imgs, (10000, W))
             t0 = time.perf_counter()
-            oracle.edge(img, K1, K2)
+            E = oracle.edge(img, K1, K2)
             t_tot += time.perf_counter() - t0
+            if gpu_out is not None:
+                err = max(err, _normwise(gpu_out[imgs, 0], E))
             done_px += img.size
             imgs += 1
         sample = f"oracle.edge on {imgs} whole 10000x10000 images of configs[1] ({t_tot:.1f} s)"
@@ -398,12 +430,18 @@ def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0) -> dict:
         prm = synth.cnn_params_np(wl["seed"], n5, H, W)
         img = synth.image_np(wl["seed"], synth.DS_IMAGE, 0, (H, W))
         t0 = time.perf_counter()
-        oracle.cnn(img, n5, prm)
+        ref = oracle.cnn(img, n5, prm)
         t_tot = time.perf_counter() - t0
+        err = _normwise(gpu_out[0:1], ref) if gpu_out is not None else 0.0
+        imgs = 1
         done_px = H * W
         sample = f"oracle.cnn on one {H}x{W} image of the workload ({t_tot:.1f} s)"
-    return {"value": done_px / t_tot / 1e6, "unit": "Mpixels/s", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": sample}
+    out = {"value": done_px / t_tot / 1e6, "unit": "Mpixels/s", "cores": oracle.num_threads(), "kind": "oracle",
+           "sample": sample}
+    if gpu_out is not None:
+        out["verified"] = {"images": imgs, "max_normwise_err": err, "tol": tol, "ok": err <= tol,
+                           "what": "the sampled images' oracle outputs vs this run's streamed GPU outputs"}
+    return out
 
 
 def run_reference(args):
@@ -458,7 +496,8 @@ def main():
             line["paper_context"] = {"mpx_s": 24.3, "what": "edge 10000x10000, Tesla C870, host-to-host, no overlap "
                                                             "(PAPER.md:753); 25.5 on 8800 GTX"}
         if world == 1 and not args.no_cpu:
-            line["cpu_baseline"] = cpu_oracle_sample(args.template)
+            line["cpu_baseline"] = cpu_oracle_sample(args.template, gpu_out=res["y_host"].numpy(),
+                                                     tol=1e-5 if args.precision == "fp32" else 2e-2)
         print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist
