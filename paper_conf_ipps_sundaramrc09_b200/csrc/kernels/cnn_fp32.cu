@@ -301,6 +301,9 @@ __global__ void __launch_bounds__(128, 2)
 // One thread per T4 pixel and all 20 channels (the 2x2 C3 pixels under it: 80
 // accumulators). Loop over the 8 input planes; per plane a fully unrolled 6-row sweep of
 // the 6x6 window (2000 FFMA). The 20x8x25 weights are a kernel parameter (constant bank).
+// The T2 window and, in bias-plane mode, the C3 bias block under the tile reach shared
+// memory as one batch of asynchronous copies (LDGSTS, zero fill outside the chunk), so a
+// CTA waits one memory latency before computing, and the other resident CTA covers it.
 struct U2W {
     float k3[8][25][20];  // [ci][tap][co]: the 20 output channels of one tap are contiguous
     float p4[20][4];
@@ -308,23 +311,51 @@ struct U2W {
 
 constexpr int U2_TR = 8, U2_TC = 16;
 constexpr int U2_IR = 2 * U2_TR + 4, U2_IC = 2 * U2_TC + 4;  // 20 x 36 per plane
+constexpr int U2_BR = 2 * U2_TR, U2_BC = 2 * U2_TC;           // C3 bias block 16 x 32 per channel
+
+__device__ __forceinline__ void cp_async4(uint32_t dst, const float* src, bool valid) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(dst), "l"(src), "r"(valid ? 4 : 0)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
 __global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const __grid_constant__ U2W w) {
-    __shared__ __align__(16) float xs[8][U2_IR * U2_IC];
+    extern __shared__ __align__(16) float u2sm[];
+    float* xs = u2sm;                      // [8][U2_IR * U2_IC]
+    float* bs = xs + 8 * U2_IR * U2_IC;    // [20][U2_BR][U2_BC] (bias-plane mode)
     const int tid = threadIdx.x, ty = tid / U2_TC, tx = tid % U2_TC;
     const int64_t img = blockIdx.z;
     const int64_t r4_0 = a.t4_row0 + (int64_t)blockIdx.y * U2_TR;
     const int64_t c4_0 = (int64_t)blockIdx.x * U2_TC;
-    const int64_t ir0 = 2 * r4_0, ic0 = 2 * c4_0;  // global T2 row/col of the window
+    const int64_t ir0 = 2 * r4_0, ic0 = 2 * c4_0;  // global T2 row/col of the window (= C3 row/col of the bias block)
     const float* t2b = a.t2 + img * a.t2_img_stride;
     const int64_t plane = a.t2_rows * a.w2;
-    for (int idx = tid; idx < 8 * U2_IR * U2_IC; idx += 128) {
-        const int ci = idx / (U2_IR * U2_IC);
-        const int rem = idx - ci * (U2_IR * U2_IC);
+    for (int rem = tid; rem < U2_IR * U2_IC; rem += 128) {
         const int r = rem / U2_IC, c = rem - r * U2_IC;
         const int64_t br = ir0 + r - a.t2_row0, gc = ic0 + c;
-        xs[ci][rem] = (br >= 0 && br < a.t2_rows && gc < a.w2) ? t2b[ci * plane + br * a.w2 + gc] : 0.f;
+        const bool ok = br >= 0 && br < a.t2_rows && gc < a.w2;
+        const float* src = ok ? t2b + br * a.w2 + gc : a.t2;
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(xs + rem);
+#pragma unroll
+        for (int ci = 0; ci < 8; ++ci)
+            cp_async4(dst + 4u * ci * (U2_IR * U2_IC), ok ? src + ci * plane : src, ok);
     }
+    if (a.b3_plane) {
+        const int64_t b3_plane = a.b3_rows * a.w3;
+        for (int rem = tid; rem < U2_BR * U2_BC; rem += 128) {
+            const int r = rem / U2_BC, c = rem - r * U2_BC;
+            const int64_t br = ir0 + r - a.b3_row0, gc = ic0 + c;
+            const bool ok = br >= 0 && br < a.b3_rows && gc < a.w3;
+            const float* src = ok ? a.b3 + br * a.w3 + gc : a.b3;
+            const uint32_t dst = (uint32_t)__cvta_generic_to_shared(bs + rem);
+#pragma unroll 4
+            for (int co = 0; co < 20; ++co)
+                cp_async4(dst + 4u * co * (U2_BR * U2_BC), ok ? src + co * b3_plane : src, ok);
+        }
+    }
+    cp_async_commit();
+    cp_async_wait_all();
     __syncthreads();
     const int64_t R4 = r4_0 + ty, C4 = c4_0 + tx;
     if (R4 >= a.t4_row0 + a.t4_rows || C4 >= a.w4) return;
@@ -339,7 +370,7 @@ __global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const
 #pragma unroll
         for (int i = 0; i < 6; ++i) {
             float x[6];
-            const float2* xr = reinterpret_cast<const float2*>(&xs[ci][(2 * ty + i) * U2_IC + 2 * tx]);
+            const float2* xr = reinterpret_cast<const float2*>(&xs[ci * (U2_IR * U2_IC) + (2 * ty + i) * U2_IC + 2 * tx]);
 #pragma unroll
             for (int v = 0; v < 3; ++v) {
                 const float2 t = xr[v];
@@ -365,55 +396,128 @@ __global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const
     const int64_t oplane = a.t4_rows * a.w4;
 #pragma unroll
     for (int co = 0; co < 20; ++co) {
+        float bq[4];
+        if (a.b3_plane) {
+#pragma unroll
+            for (int ra = 0; ra < 2; ++ra) {
+                const float2 bb = *reinterpret_cast<const float2*>(&bs[(co * U2_BR + 2 * ty + ra) * U2_BC + 2 * tx]);
+                bq[2 * ra] = bb.x;
+                bq[2 * ra + 1] = bb.y;
+            }
+        } else {
+            const float b = __ldg(a.b3 + co);
+            bq[0] = bq[1] = bq[2] = bq[3] = b;
+        }
         float s = 0.f;
 #pragma unroll
         for (int p = 0; p < 4; ++p) {
-            const int64_t r3 = 2 * R4 + (p >> 1), c3 = 2 * C4 + (p & 1);
-            const float b = a.b3_plane ? __ldg(a.b3 + ((int64_t)co * a.b3_rows + (r3 - a.b3_row0)) * a.w3 + c3)
-                                       : __ldg(a.b3 + co);
             const float av = (co & 1) ? acc2[co >> 1][p].y : acc2[co >> 1][p].x;
-            s = fmaf(w.p4[co][p], tanh_f(av + b), s);
+            s = fmaf(w.p4[co][p], tanh_f(av + bq[p]), s);
         }
         t4[co * oplane + (R4 - a.t4_row0) * a.w4 + C4] = tanh_f(s);
     }
 }
 
 // ============================================================================ U3
-// One thread per 4 consecutive output pixels of a row. C5 channels in groups of 8: per
-// group, 4 px x 8 ch accumulators over 20 planes x 25 taps (weights staged in shared
-// memory, broadcast LDS.128), then bias + tanh and the group's contribution to the 9 C6
-// accumulators per pixel (C6 is a 1x1 conv: a dot product over n5 channels).
-constexpr int U3_TR = 8, U3_TCG = 16, U3_P = 4, U3_G = 8;
-constexpr int U3_TC = U3_TCG * U3_P;              // 64 output cols per tile
-constexpr int U3_IR = U3_TR + 4, U3_IC = U3_TC + 4;  // 12 x 68 per plane
-constexpr int U3_ICP = 68;                         // pitch (floats), 16-byte aligned rows
+// C5 + bias + tanh + C6 + bias. One CTA (256 threads, one per SM: ~150 KB of shared memory)
+// per work item of 1024 output positions; a thread owns 4 consecutive positions of a row and
+// loops over the C5 channels in groups of 8 (4 px x 8 ch accumulators over 20 planes x 25
+// taps, channel-paired FFMA2 with broadcast LDS.128 weights), then bias + tanh and the
+// group's contribution to the 9 C6 dot products (C6 is 1x1: a dot product over n5), so T5
+// never exists in memory. All loads into shared memory are asynchronous (LDGSTS with zero
+// fill for halo and out-of-range positions): the band of T4 once per item, the weights of
+// group g+1 while group g computes (double buffer), and the bias-plane values of a group are
+// fetched into registers before its tap loop so their latency hides behind it.
+// Two item geometries (chosen per launch by the fraction of wasted positions):
+//  - narrow images (padded T4 pitch P = round4(w4) <= 256): positions are flattened over
+//    (row, col) with pitch P, an item is 1024 consecutive flattened positions, and the
+//    shared band holds the flattened range [p0, p0 + 1024 + 4P + 8) of every T4 plane; the
+//    P - w5 columns past the row end are computed and dropped (2-5 % at VGA width, instead
+//    of the 20 % a 64-column tile loses on 153 columns);
+//  - wide images: 16 x 64 output tiles, T4 window 20 x 68 per plane.
+// Every output is the same FFMA sequence (ci, i, j order) wherever its item starts, so split
+// runs stay bit-identical to unsplit runs.
+constexpr int U3_THREADS = 256, U3_POS = 4 * U3_THREADS, U3_P = 4, U3_G = 8;
+constexpr int U3W_TR = 16, U3W_TC = 64, U3W_PITCH = U3W_TC + 4;  // wide tile (pitch 68)
+constexpr int U3_NARROW_MAX_PITCH = 256;
 
-__global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
+
+struct U3Geom {
+    int narrow;             // 1: flattened items, 0: 16 x 64 tiles
+    int pitch;              // shared-memory row pitch (floats)
+    int cs;                 // shared-memory plane stride (floats)
+    int stage;              // floats staged per plane
+    int tiles_c;            // wide: column tiles
+    int64_t items_per_img;
+};
+
+__global__ void __launch_bounds__(U3_THREADS, 1) cnn_u3_kernel(const CnnU3Args a, const U3Geom gm) {
     extern __shared__ __align__(16) float sm[];
-    float* xs = sm;                                  // [20][U3_IR][U3_ICP]
-    float* ws = xs + 20 * U3_IR * U3_ICP;            // [20][25][8] group weights
-    float* k6s = ws + 20 * 25 * U3_G;                // [9][n5p]
     const int n5 = a.n5, n5p = (n5 + U3_G - 1) / U3_G * U3_G;
-    const int tid = threadIdx.x, ty = tid / U3_TCG, tg = tid % U3_TCG;
-    const int64_t img = blockIdx.z;
-    const int64_t r5_0 = a.out_row0 + (int64_t)blockIdx.y * U3_TR;
-    const int64_t c5_0 = (int64_t)blockIdx.x * U3_TC;
+    float* xs = sm;                             // [20][cs]
+    float* ws = xs + 20 * gm.cs;                // [2][20*25][8] group weights (double buffer)
+    float* k6s = ws + 2 * 20 * 25 * U3_G;       // [n5p][12]: the 9 C6 weights of a channel
+    const int tid = threadIdx.x;
+    const int64_t img = blockIdx.x / gm.items_per_img;
+    const int64_t item = blockIdx.x - img * gm.items_per_img;
     const float* t4b = a.t4 + img * a.t4_img_stride;
     const int64_t plane = a.t4_rows * a.w4;
-    for (int idx = tid; idx < 20 * U3_IR * U3_IC; idx += 128) {
-        const int ci = idx / (U3_IR * U3_IC);
-        const int rem = idx - ci * (U3_IR * U3_IC);
-        const int r = rem / U3_IC, c = rem - r * U3_IC;
-        const int64_t br = r5_0 + r - a.t4_row0, gc = c5_0 + c;
-        xs[(ci * U3_IR + r) * U3_ICP + c] =
-            (br >= 0 && br < a.t4_rows && gc < a.w4) ? t4b[ci * plane + br * a.w4 + gc] : 0.f;
+
+    // geometry of the staged band and of this thread's 4 positions
+    int64_t R5, C5;  // global C5 row, column of the first position
+    int sb;          // shared offset of the first position (tap (0,0)) within a plane
+    int64_t p0 = 0, r0 = 0, c0 = 0;
+    if (gm.narrow) {
+        p0 = item * U3_POS;
+        const int64_t p = p0 + 4 * tid;
+        R5 = a.out_row0 + p / gm.pitch;
+        C5 = p % gm.pitch;
+        sb = 4 * tid;
+    } else {
+        const int64_t tr = item / gm.tiles_c, tc = item - tr * gm.tiles_c;
+        r0 = a.out_row0 + tr * U3W_TR;
+        c0 = tc * U3W_TC;
+        const int ty = tid / (U3W_TC / U3_P), tg = tid % (U3W_TC / U3_P);
+        R5 = r0 + ty;
+        C5 = c0 + tg * U3_P;
+        sb = ty * U3W_PITCH + tg * U3_P;
     }
-    for (int idx = tid; idx < 9 * n5p; idx += 128) {
-        const int o = idx / n5p, ch = idx - o * n5p;
-        k6s[idx] = ch < n5 ? __ldg(a.k6 + o * n5 + ch) : 0.f;
-    }
-    const int64_t R5 = r5_0 + ty, C5 = c5_0 + tg * U3_P;
     const bool row_ok = R5 < a.out_row0 + a.out_rows;
+
+    auto stage_weights = [&](int g0, int buf) {
+        float* wd = ws + buf * (20 * 25 * U3_G);
+        for (int idx = tid; idx < 20 * 25 * U3_G; idx += U3_THREADS) {
+            const int ch = idx / 500, k = idx - ch * 500;  // coalesced over k within a channel
+            const bool ok = g0 + ch < n5;
+            cp_async4((uint32_t)__cvta_generic_to_shared(wd + k * U3_G + ch),
+                      ok ? a.k5 + (int64_t)(g0 + ch) * 500 + k : a.k5, ok);
+        }
+    };
+    stage_weights(0, 0);
+    // the band of every T4 plane (rows are global T4 rows; zero outside the chunk's rows)
+    for (int s = tid; s < gm.stage; s += U3_THREADS) {
+        int64_t gr, gc;
+        if (gm.narrow) {
+            const int64_t q = p0 + s;
+            gr = a.out_row0 + q / gm.pitch;
+            gc = q % gm.pitch;
+        } else {
+            const int rr = s / U3W_PITCH;
+            gr = r0 + rr;
+            gc = c0 + (s - rr * U3W_PITCH);
+        }
+        const int64_t br = gr - a.t4_row0;
+        const bool ok = br >= 0 && br < a.t4_rows && gc < a.w4;
+        const float* src = ok ? t4b + br * a.w4 + gc : a.t4;
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(xs + s);
+#pragma unroll 4
+        for (int ci = 0; ci < 20; ++ci) cp_async4(dst + 4u * ci * gm.cs, ok ? src + ci * plane : src, ok);
+    }
+    cp_async_commit();
+    for (int idx = tid; idx < n5p * 12; idx += U3_THREADS) {
+        const int ch = idx / 12, o = idx - ch * 12;
+        k6s[idx] = (ch < n5 && o < 9) ? __ldg(a.k6 + o * n5 + ch) : 0.f;
+    }
 
     float c6[9][U3_P];
 #pragma unroll
@@ -421,13 +525,29 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
 #pragma unroll
         for (int p = 0; p < U3_P; ++p) c6[o][p] = 0.f;
 
-    for (int g0 = 0; g0 < n5p; g0 += U3_G) {
-        __syncthreads();  // previous group's weights fully consumed (and tile staged)
-        for (int idx = tid; idx < 20 * 25 * U3_G; idx += 128) {
-            const int k = idx / U3_G, ch = idx - k * U3_G;  // k = ci*25 + tap
-            ws[idx] = (g0 + ch < n5) ? __ldg(a.k5 + (int64_t)(g0 + ch) * 500 + k) : 0.f;
+    const int ngroups = n5p / U3_G;
+    for (int gi = 0; gi < ngroups; ++gi) {
+        const int g0 = gi * U3_G;
+        cp_async_wait_all();
+        __syncthreads();  // weights of group gi (and the band) visible; group gi-1 fully consumed
+        if (gi + 1 < ngroups) stage_weights(g0 + U3_G, (gi + 1) & 1);
+        cp_async_commit();
+        // this group's bias values (their latency hides behind the tap loop)
+        float bv[U3_G][U3_P];
+#pragma unroll
+        for (int c = 0; c < U3_G; ++c) {
+            const int ch = min(g0 + c, n5 - 1);
+#pragma unroll
+            for (int p = 0; p < U3_P; ++p) {
+                if (a.b5_plane)
+                    bv[c][p] = (row_ok && C5 + p < a.w5)
+                                   ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (R5 - a.b5_row0)) * a.w5 + C5 + p)
+                                   : 0.f;
+                else
+                    bv[c][p] = __ldg(a.b5 + ch);
+            }
         }
-        __syncthreads();
+        const float* wg = ws + (gi & 1) * (20 * 25 * U3_G);
         float2 acc2[U3_G / 2][U3_P];  // channel pairs, FFMA2
 #pragma unroll
         for (int c = 0; c < U3_G / 2; ++c)
@@ -438,13 +558,13 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
 #pragma unroll
             for (int i = 0; i < 5; ++i) {
                 float x[8];
-                const float4* xr = reinterpret_cast<const float4*>(&xs[(ci * U3_IR + ty + i) * U3_ICP + tg * U3_P]);
+                const float4* xr = reinterpret_cast<const float4*>(&xs[ci * gm.cs + sb + i * gm.pitch]);
                 const float4 x0 = xr[0], x1 = xr[1];
                 x[0] = x0.x; x[1] = x0.y; x[2] = x0.z; x[3] = x0.w;
                 x[4] = x1.x; x[5] = x1.y; x[6] = x1.z; x[7] = x1.w;
 #pragma unroll
                 for (int kj = 0; kj < 5; ++kj) {
-                    const float4* wr = reinterpret_cast<const float4*>(&ws[((ci * 25) + i * 5 + kj) * U3_G]);
+                    const float4* wr = reinterpret_cast<const float4*>(&wg[((ci * 25) + i * 5 + kj) * U3_G]);
                     const float4 wa = wr[0], wb = wr[1];
                     const float2 wv[4] = {make_float2(wa.x, wa.y), make_float2(wa.z, wa.w), make_float2(wb.x, wb.y),
                                           make_float2(wb.z, wb.w)};
@@ -456,21 +576,19 @@ __global__ void __launch_bounds__(128, 2) cnn_u3_kernel(const CnnU3Args a) {
                 }
             }
         }
-        // bias + tanh, then this group's share of the 1x1 C6 dot products
+        // bias + tanh, then this group's share of the 1x1 C6 dot products (padded channels
+        // have zero C6 weights, so they add exact zeros)
 #pragma unroll
         for (int c = 0; c < U3_G; ++c) {
-            const int ch = g0 + c;
-            if (ch >= n5) break;
+            const float4* k6r = reinterpret_cast<const float4*>(&k6s[(g0 + c) * 12]);
+            const float4 ka = k6r[0], kb = k6r[1], kc = k6r[2];
+            const float kw[9] = {ka.x, ka.y, ka.z, ka.w, kb.x, kb.y, kb.z, kb.w, kc.x};
 #pragma unroll
             for (int p = 0; p < U3_P; ++p) {
-                float b = 0.f;
-                if (row_ok && C5 + p < a.w5)
-                    b = a.b5_plane ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (R5 - a.b5_row0)) * a.w5 + C5 + p)
-                                   : __ldg(a.b5 + ch);
                 const float av = (c & 1) ? acc2[c >> 1][p].y : acc2[c >> 1][p].x;
-                const float t = tanh_f(av + b);
+                const float t = tanh_f(av + bv[c][p]);
 #pragma unroll
-                for (int o = 0; o < 9; ++o) c6[o][p] = fmaf(k6s[o * n5p + ch], t, c6[o][p]);
+                for (int o = 0; o < 9; ++o) c6[o][p] = fmaf(kw[o], t, c6[o][p]);
             }
         }
     }
@@ -547,25 +665,57 @@ cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s) {
         for (int ci = 0; ci < 8; ++ci)
             for (int t = 0; t < 25; ++t) w.k3[ci][t][co] = a.k3_host[(co * 8 + ci) * 25 + t];
     std::memcpy(w.p4, a.p4_host, sizeof w.p4);
+    const size_t smem = sizeof(float) * (8 * U2_IR * U2_IC + (a.b3_plane ? 20 * U2_BR * U2_BC : 0));
+    static std::atomic<uint32_t> configured{0};  // one bit per device
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(configured.load() & (1u << (dev & 31)))) {
+        cudaError_t e = cudaFuncSetAttribute(cnn_u2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)(sizeof(float) * (8 * U2_IR * U2_IC + 20 * U2_BR * U2_BC)));
+        if (e != cudaSuccess) return e;
+        configured.fetch_or(1u << (dev & 31));
+    }
     dim3 grid((unsigned)((a.w4 + U2_TC - 1) / U2_TC), (unsigned)((a.t4_rows + U2_TR - 1) / U2_TR), (unsigned)a.nimg);
-    cnn_u2_kernel<<<grid, 128, 0, s>>>(a, w);
+    cnn_u2_kernel<<<grid, 128, smem, s>>>(a, w);
     return cudaGetLastError();
 }
 
 cudaError_t launch_cnn_u3(const CnnU3Args& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     const int n5p = (a.n5 + U3_G - 1) / U3_G * U3_G;
-    const size_t smem = sizeof(float) * (20 * U3_IR * U3_ICP + 20 * 25 * U3_G + 9 * n5p);
+    // geometry: flattened items when the padded row fits and wastes less than 64-column tiles
+    U3Geom gm{};
+    const int64_t pitch = (a.w4 + 3) / 4 * 4;
+    const int64_t narrow_items = (a.out_rows * pitch + U3_POS - 1) / U3_POS;
+    const int64_t tiles_c = (a.w5 + U3W_TC - 1) / U3W_TC;
+    const int64_t wide_items = (a.out_rows + U3W_TR - 1) / U3W_TR * tiles_c;
+    if (pitch <= U3_NARROW_MAX_PITCH && narrow_items <= wide_items) {
+        gm.narrow = 1;
+        gm.pitch = (int)pitch;
+        gm.stage = (int)(U3_POS + 4 * pitch + 8);
+        gm.cs = gm.stage;
+        gm.items_per_img = narrow_items;
+    } else {
+        gm.narrow = 0;
+        gm.pitch = U3W_PITCH;
+        gm.stage = (U3W_TR + 4) * U3W_PITCH;
+        gm.cs = gm.stage;
+        gm.tiles_c = (int)tiles_c;
+        gm.items_per_img = wide_items;
+    }
+    const size_t smem = sizeof(float) * ((size_t)20 * gm.cs + 2 * 20 * 25 * U3_G + (size_t)n5p * 12);
     static std::atomic<uint32_t> configured{0};  // one bit per device
     int dev = 0;
     cudaGetDevice(&dev);
     if (!(configured.load() & (1u << (dev & 31)))) {
-        cudaError_t e = cudaFuncSetAttribute(cnn_u3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
+        cudaError_t e = cudaFuncSetAttribute(cnn_u3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
         if (e != cudaSuccess) return e;
         configured.fetch_or(1u << (dev & 31));
     }
-    dim3 grid((unsigned)((a.w5 + U3_TC - 1) / U3_TC), (unsigned)((a.out_rows + U3_TR - 1) / U3_TR), (unsigned)a.nimg);
-    cnn_u3_kernel<<<grid, 128, smem, s>>>(a);
+    if (smem > 227 * 1024) return cudaErrorInvalidValue;
+    const int64_t grid = gm.items_per_img * a.nimg;
+    if (grid >= (1ll << 31)) return cudaErrorInvalidValue;
+    cnn_u3_kernel<<<(unsigned)grid, U3_THREADS, smem, s>>>(a, gm);
     return cudaGetLastError();
 }
 

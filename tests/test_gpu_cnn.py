@@ -42,7 +42,9 @@ def run_cnn(tg, img, n5, prm, bias="plane", budget=0, device=False, max_chunk_px
 
 @pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
                                           (3, 67, 61, 20, "scalar"), (1, 97, 131, 120, "scalar"),
-                                          (1, 483 // 3, 643 // 3, 60, "plane"), (2, 32, 32, 7, "plane")])
+                                          (1, 483 // 3, 643 // 3, 60, "plane"), (2, 32, 32, 7, "plane"),
+                                          # wide rows (T4 pitch > 256): the U3 16 x 64 tile geometry
+                                          (1, 70, 1210, 20, "plane"), (1, 45, 1333, 120, "scalar")])
 def test_cnn_parity(tg, orc, n, H, W, n5, bias):
     seed = synth.seed_for_config(3)
     img = synth.images_np(seed, n, H, W)
