@@ -260,25 +260,28 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
 }
 
 // ============================================================================ U3 (C5 + C6)
+// Band = 256 consecutive output positions in the FLATTENED (row, col) index of the chunk with
+// pitch w4 (two M=128 tiles; the w4 - w5 = 4 positions past each row's end are computed and
+// dropped). For any width, filter row i of a band reads one contiguous run of T4: flat pixels
+// [q0 + i*w4, q0 + i*w4 + 262) -- the band's "slice" i (+4 taps, +1 for the (4,5) tap pair,
+// +1 spare).
 // Warp-specialised and persistent (one CTA per SM, 9 warps):
-//   warp 8, one thread   producer + MMA issuer: per band, 1-D bulk copies (TMA engine) of the
-//                        input window into one of two A buffers; the 40 K-steps of the C5 B
-//                        operand stream through a 4-slot ring of bulk copies (the weights are the
-//                        same for every band); tcgen05.mma into one of two TMEM accumulators
-//                        (2 tiles x NP columns each); tcgen05.commit releases the ring slot, the
-//                        A buffer and hands the accumulator to the epilogue
+//   warp 8 (warp-uniform, one elected lane issues)  producer + MMA issuer: the whole C5 B
+//                        operand (40 K-steps x NP maps, up to 160 KB) is loaded ONCE per CTA and
+//                        stays resident; the slices flow through a ring of U3_NA buffers (three
+//                        1-D bulk copies each, one per channel block, prefetched U3_NA-1 slices
+//                        ahead); per slice 8 K-steps x 2 tiles of tcgen05.mma into one of two TMEM
+//                        accumulators (2 tiles x NP columns); tcgen05.commit frees the slice
+//                        buffer, and after the 5th slice hands the accumulator to the epilogue
 //   warps 0-7            epilogue: TMEM -> registers, bias plane + tanh, the 1x1 C6 layer as a
 //                        dot product over n5 (weights in the constant bank), + bias -> output
-// so the epilogue of band k overlaps the MMAs of band k+1 and the copies of band k+2.
-// Bands are 256 output positions (two M=128 tiles): narrow images (w4 <= kFlatMax) use the
-// flattened (row, col) index with the window pitch = w4 (columns >= w5 discarded; a window is
-// a run of whole T4 rows = one contiguous copy per channel block); wide images use 256-column
-// segments of one output row (window pitch 262, 5 row copies per block).
-constexpr int kFlatMax = 180;
-constexpr int U3_KS = 40, U3_KS_STAGE = 4, U3_STAGES = U3_KS / U3_KS_STAGE, U3_BRING = 6;
+// so the epilogue of band k overlaps the MMAs of band k+1. (An earlier version re-streamed B
+// through a 6-slot ring for every band -- 160 KB of L2 reads per 256 positions -- and its MMAs
+// waited on those copies.)
+constexpr int U3_KS = 40;
 constexpr int U3_NMAX = 128;
-constexpr int U3_WP_COL = 2 * kTileM + 6;
-constexpr int U3_APX = 1320;  // window pixels per block: flat <= 7*180+8, column 5*262+8
+constexpr int U3_SPX = 2 * kTileM + 8;  // pixels per slice buffer (262 used)
+constexpr int U3_NA = 4;                // slice buffers
 constexpr int kEpiWarps = 8;
 constexpr int kThreadsU3 = (kEpiWarps + 1) * 32;
 
@@ -287,70 +290,39 @@ struct U3K6 {
 };
 
 struct U3Smem {
-    uint4 a[2][3][U3_APX];                         // double-buffered window, 3 channel blocks
-    uint4 b[U3_BRING][U3_KS_STAGE * 2 * U3_NMAX];  // B ring (4 K-steps per slot)
-    uint64_t a_full[2], a_empty[2], b_full[U3_BRING], b_empty[U3_BRING], t_full[2], t_empty[2];
+    uint4 b[U3_KS * 2 * U3_NMAX];  // resident C5 B operand: [ks][half][n] -> 8 bf16
+    uint4 a[U3_NA][3][U3_SPX];     // slice ring: [channel block][pixel] -> 8 bf16
+    uint64_t b_full, a_full[U3_NA], a_empty[U3_NA], t_full[2], t_empty[2];
     uint32_t tmem;
 };
 
-struct U3Band {
-    int64_t img, q0, wr0, wc0;
-    int WP, WR, base;
-};
-
-__device__ __forceinline__ U3Band u3_band(const CnnU3Args& a, int64_t band, int64_t per_img, bool flat) {
-    U3Band g;
-    g.img = band / per_img;
-    const int64_t bi = band - g.img * per_img;
-    if (flat) {
-        g.q0 = bi * 2 * kTileM;
-        const int64_t r_first = g.q0 / a.w4;
-        g.wr0 = a.out_row0 + r_first;
-        g.wc0 = 0;
-        g.WP = (int)a.w4;
-        g.base = (int)(g.q0 - r_first * a.w4);
-        g.WR = (g.base + 2 * kTileM - 1) / g.WP + 1 + 4;
-    } else {
-        const int64_t bpr = (a.w5 + 2 * kTileM - 1) / (2 * kTileM);
-        const int64_t row = bi / bpr;
-        g.q0 = (bi - row * bpr) * 2 * kTileM;
-        g.wr0 = a.out_row0 + row;
-        g.wc0 = g.q0;
-        g.WP = U3_WP_COL;
-        g.WR = 5;
-        g.base = 0;
-    }
-    return g;
-}
-
+template <int NCH>  // TMEM chunks of 32 columns: NP = n5 padded to 16, NCH = ceil(NP / 32)
 __global__ void __launch_bounds__(kThreadsU3, 1)
     cnn_u3_tc_kernel(const CnnU3Args a, const __grid_constant__ U3K6 k6w, const int64_t nbands) {
     extern __shared__ __align__(128) uint8_t smraw[];
     U3Smem& S = *reinterpret_cast<U3Smem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int NP = a.n_pad;
-    const bool flat = a.w4 <= kFlatMax;
-    const int64_t per_img = flat ? (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM)
-                                 : a.out_rows * ((a.w5 + 2 * kTileM - 1) / (2 * kTileM));
-    const int64_t bplane = a.t4_rows * a.w4;
+    const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
+    const int64_t bplane = a.t4_rows * a.w4;                 // pixels per channel block of one image
+    const int64_t flat0 = (a.out_row0 - a.t4_row0) * a.w4;  // flat index of output row 0 in the T4 buffer
 
     if (warp == 0) tc::tmem_alloc<512>(&S.tmem);
     if (tid == 0) {
-        for (int i = 0; i < 2; ++i) {
+        tc::mbar_init(&S.b_full, 1);
+        for (int i = 0; i < U3_NA; ++i) {
             tc::mbar_init(&S.a_full[i], 1);
             tc::mbar_init(&S.a_empty[i], 1);
+        }
+        for (int i = 0; i < 2; ++i) {
             tc::mbar_init(&S.t_full[i], 1);
             tc::mbar_init(&S.t_empty[i], kEpiWarps);
         }
-        for (int i = 0; i < U3_BRING; ++i) {
-            tc::mbar_init(&S.b_full[i], 1);
-            tc::mbar_init(&S.b_empty[i], 1);
-        }
         tc::mbar_fence_init();
     }
-    // windows start zeroed: pixels a copy does not cover (beyond the image, the spare pixels of
-    // tap pair (4,5)) then only ever hold finite T4 values
-    for (int idx = tid; idx < 2 * 3 * U3_APX; idx += kThreadsU3) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
+    // slice buffers start zeroed: pixels a copy does not cover (past the chunk's last T4 row)
+    // then only ever hold finite T4 values; they feed positions that are not stored
+    for (int idx = tid; idx < U3_NA * 3 * U3_SPX; idx += kThreadsU3) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
     tc::fence_proxy_async();
     tc::fence_before_sync();
     __syncthreads();
@@ -358,172 +330,182 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
     const uint32_t tmem = S.tmem;
 
     if (warp == kEpiWarps) {
-        if (lane == 0) {
-            // ------------------------------------------------------------ producer + MMA
-            const uint4* t4b_all = reinterpret_cast<const uint4*>(a.t4);
-            const uint4* kb = reinterpret_cast<const uint4*>(a.k5_tc);
-            const uint32_t stage_bytes = (uint32_t)(U3_KS_STAGE * 2 * NP * 16);
-            const int64_t my_bands = nbands > blockIdx.x ? (nbands - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-            const int64_t total_stages = my_bands * U3_STAGES;
-            auto load_b = [&](int64_t gs) {
-                const int slot = (int)(gs % U3_BRING);
-                tc::mbar_expect_tx(&S.b_full[slot], stage_bytes);
-                tc::bulk_g2s(S.b[slot], kb + (size_t)(gs % U3_STAGES) * (stage_bytes / 16), stage_bytes, &S.b_full[slot]);
-            };
-            auto load_a = [&](int64_t band, int buf) {
-                const U3Band g = u3_band(a, band, per_img, flat);
-                const uint4* t4b = t4b_all + g.img * 3 * bplane;
-                const int64_t r0 = g.wr0 - a.t4_row0;
-                uint32_t bytes = 0;
-                if (flat) {
-                    const int64_t rows = min((int64_t)g.WR, a.t4_rows - r0);
-                    bytes = (uint32_t)(3 * rows * a.w4 * 16);
-                    tc::mbar_expect_tx(&S.a_full[buf], bytes);
+        // ---------------------------------------------------------------- producer + MMA
+        // (the whole warp runs the loop so descriptors live in uniform registers; one elected
+        // lane issues the copies, MMAs and commits)
+        const uint4* t4all = reinterpret_cast<const uint4*>(a.t4);
+        const int64_t my_bands = nbands > blockIdx.x ? (nbands - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+        const int64_t total = my_bands * 5;  // slices
+        auto load_slice = [&](int64_t s) {
+            const int64_t band = blockIdx.x + (s / 5) * gridDim.x;
+            const int i = (int)(s % 5);
+            const int64_t img = band / per_img;
+            const int64_t q0 = (band - img * per_img) * 2 * kTileM;
+            const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
+            const int64_t n = max((int64_t)0, min((int64_t)U3_SPX, bplane - e));
+            const int slot = (int)(s % U3_NA);
+            if (tc::elect_one()) {
+                tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
+                if (n > 0) {
+                    const uint4* src = t4all + img * 3 * bplane + e;
                     for (int blk = 0; blk < 3; ++blk)
-                        tc::bulk_g2s(S.a[buf][blk], t4b + blk * bplane + r0 * a.w4, (uint32_t)(rows * a.w4 * 16),
-                                     &S.a_full[buf]);
-                } else {
-                    const int64_t cols = min((int64_t)U3_WP_COL, a.w4 - g.wc0);
-                    bytes = (uint32_t)(3 * 5 * cols * 16);
-                    tc::mbar_expect_tx(&S.a_full[buf], bytes);
-                    for (int blk = 0; blk < 3; ++blk)
-                        for (int r = 0; r < 5; ++r)
-                            tc::bulk_g2s(&S.a[buf][blk][r * U3_WP_COL], t4b + blk * bplane + (r0 + r) * a.w4 + g.wc0,
-                                         (uint32_t)(cols * 16), &S.a_full[buf]);
+                        tc::bulk_g2s(S.a[slot][blk], src + blk * bplane, (uint32_t)(n * 16), &S.a_full[slot]);
                 }
-            };
-            const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);
-            for (int64_t gs = 0; gs < (int64_t)(U3_BRING - 1) && gs < total_stages; ++gs) load_b(gs);
-            if (my_bands > 0) load_a(blockIdx.x, 0);
-            int64_t gs = 0;
-            for (int64_t k = 0; k < my_bands; ++k) {
-                const int buf = (int)(k & 1);
-                const U3Band g = u3_band(a, blockIdx.x + k * gridDim.x, per_img, flat);
-                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k >> 1) & 1));
-                if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+            }
+            __syncwarp();
+        };
+        if (my_bands > 0) {
+            const uint32_t bbytes = (uint32_t)(U3_KS * 2 * NP * 16);
+            if (tc::elect_one()) {
+                tc::mbar_expect_tx(&S.b_full, bbytes);
+                const uint8_t* kb = reinterpret_cast<const uint8_t*>(a.k5_tc);
+                for (uint32_t off = 0; off < bbytes; off += 16384u)
+                    tc::bulk_g2s(reinterpret_cast<uint8_t*>(S.b) + off, kb + off, min(16384u, bbytes - off), &S.b_full);
+            }
+            __syncwarp();
+        }
+        for (int64_t s = 0; s < U3_NA - 1 && s < total; ++s) load_slice(s);
+        if (my_bands > 0) tc::mbar_wait(&S.b_full, 0);
+        const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);
+        const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), (uint32_t)(NP * 16), 128);
+        const uint32_t plane_bytes = (uint32_t)(U3_SPX * 16);
+        for (int64_t k = 0; k < my_bands; ++k) {
+            const int buf = (int)(k & 1);
+            if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+            const uint32_t d_base = tmem + (uint32_t)(buf * 256);
+            for (int i = 0; i < 5; ++i) {
+                const int64_t s = k * 5 + i;
+                const int slot = (int)(s % U3_NA);
+                tc::mbar_wait(&S.a_full[slot], (uint32_t)((s / U3_NA) & 1));
                 tc::fence_after_sync();
-                const uint32_t a_base = tc::smem_u32(S.a[buf][0]);
-                const uint32_t plane_bytes = (uint32_t)(U3_APX * 16);
-                const uint32_t d_base = tmem + (uint32_t)(buf * 256);
-                for (int st = 0; st < U3_STAGES; ++st, ++gs) {
-                    const int slot = (int)(gs % U3_BRING);
-                    tc::mbar_wait(&S.b_full[slot], (uint32_t)((gs / U3_BRING) & 1));
-                    tc::fence_after_sync();
-                    const uint32_t b_base = tc::smem_u32(S.b[slot]);
-                    for (int u = 0; u < U3_KS_STAGE; ++u) {
-                        const int ks = st * U3_KS_STAGE + u;
-                        const int i = ks / 8, r8 = ks % 8;
-                        uint32_t a_addr, lbo;
-                        if (r8 < 5) {  // channels 0-15 of tap (i, r8): blocks 0 and 1
-                            a_addr = a_base + (uint32_t)((g.base + i * g.WP + r8) * 16);
-                            lbo = plane_bytes;
-                        } else {       // channels 16-19 of taps (i, j), (i, j+1): block 2, next pixel
-                            a_addr = a_base + 2 * plane_bytes + (uint32_t)((g.base + i * g.WP + 2 * (r8 - 5)) * 16);
-                            lbo = 16;
-                        }
-                        const uint64_t bd = tc::make_desc(b_base + (uint32_t)(u * 2 * NP * 16), (uint32_t)(NP * 16), 128);
-#if U3_EXP == 2
-                        if (0)
-#endif
+                const uint32_t a_base = tc::smem_u32(S.a[slot][0]);
+                if (tc::elect_one()) {
+#pragma unroll
+                    for (int r8 = 0; r8 < 8; ++r8) {
+                        const int ks = i * 8 + r8;
+                        // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0 and 1); r8 >= 5: channels
+                        // 16-19 of taps (i, j) and (i, j+1), j = 2(r8-5) (block 2, next pixel)
+                        const uint32_t a_addr = r8 < 5 ? a_base + (uint32_t)(r8 * 16)
+                                                       : a_base + 2 * plane_bytes + (uint32_t)(2 * (r8 - 5) * 16);
+                        const uint32_t lbo = r8 < 5 ? plane_bytes : 16u;
+                        const uint64_t bd = bdesc0 + (uint64_t)(ks * 2 * NP);  // start address in 16-B units
+#pragma unroll
                         for (int t = 0; t < 2; ++t) {
                             const uint64_t ad = tc::make_desc(a_addr + (uint32_t)(t * kTileM * 16), lbo, 128);
                             tc::mma_bf16(d_base + (uint32_t)(t * NP), ad, bd, idesc, ks > 0 ? 1u : 0u);
                         }
                     }
-                    tc::commit(&S.b_empty[slot]);
-                    // refill the slot of stage gs-1 with stage gs+BRING-1 (it has BRING-1 stages to land)
-                    if (gs + U3_BRING - 1 < total_stages) {
-                        if (gs >= 1) tc::mbar_wait(&S.b_empty[(gs - 1) % U3_BRING], (uint32_t)(((gs - 1) / U3_BRING) & 1));
-                        load_b(gs + U3_BRING - 1);
-                    }
+                    tc::commit(&S.a_empty[slot]);
+                    if (i == 4) tc::commit(&S.t_full[buf]);
                 }
-                tc::commit(&S.a_empty[buf]);
-                tc::commit(&S.t_full[buf]);
-                // prefetch the next band's window into the other buffer (freed by band k-1's MMAs)
-                if (k + 1 < my_bands) {
-                    if (k >= 1) tc::mbar_wait(&S.a_empty[buf ^ 1], (uint32_t)(((k - 1) >> 1) & 1));
-                    load_a(blockIdx.x + (k + 1) * gridDim.x, buf ^ 1);
+                __syncwarp();
+                // keep U3_NA-1 slices in flight: refill the buffer slice s-1 used (its MMAs are
+                // done or about to be: slice s's MMAs are queued behind them)
+                if (s + U3_NA - 1 < total) {
+                    if (s >= 1) tc::mbar_wait(&S.a_empty[(s - 1) % U3_NA], (uint32_t)(((s - 1) / U3_NA) & 1));
+                    load_slice(s + U3_NA - 1);
                 }
             }
         }
     } else {
         // ---------------------------------------------------------------- epilogue warps
+        // Thread = one output position of the band (tile t = warp / 4, TMEM lane group warp % 4),
+        // all NP channels in chunks of 32 TMEM columns. Bias-plane values are loaded RING chunks
+        // ahead (across band boundaries), so their L2 latency hides behind the chunk compute.
         const int t = warp >> 2;  // tile
         const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
+        const int m = t * kTileM + 32 * (warp & 3) + lane;
+        struct Pos {
+            int64_t img, orow, ocol;
+            bool ok;
+            const float* pb;
+        };
+        const uint32_t bcs = a.b5_plane ? (uint32_t)(a.b5_rows * a.w5) : 1u;  // channel stride of the bias
+        auto pos_of = [&](int64_t band) {
+            Pos q;
+            q.img = band / per_img;
+            const int64_t qq = (band - q.img * per_img) * 2 * kTileM + m;
+            q.orow = a.out_row0 + qq / a.w4;
+            q.ocol = qq - (qq / a.w4) * a.w4;
+            q.ok = q.orow < a.out_row0 + a.out_rows && q.ocol < a.w5;
+            // positions past the chunk's last row / the row's last column compute on clamped
+            // (in-bounds) bias addresses and are not stored: the drain stays branch-free
+            const int64_t orow_c = min(q.orow, a.out_row0 + a.out_rows - 1), ocol_c = min(q.ocol, a.w5 - 1);
+            q.pb = a.b5_plane ? a.b5 + (orow_c - a.b5_row0) * a.w5 + ocol_c : a.b5;
+            return q;
+        };
+        // bias ring: 2 chunk buffers loaded 2 chunks ahead when NCH is even (chunk parity is then
+        // the same in every band), else 1 buffer loaded 1 chunk ahead
+        constexpr int RING = (NCH % 2 == 0) ? 2 : 1;
+        float bv[RING][32];
+        auto load_bias = [&](const float* pb, int c, int r) {
+            const float* p = pb + (size_t)(32 * c) * bcs;
+            // chunks 0..NCH-2 are always full (NP = n5 rounded up to 16 > 32 (NCH-1)); c is a
+            // compile-time constant at every call, so only the last chunk carries predicates
+            if (c < NCH - 1) {
+#pragma unroll
+                for (int u = 0; u < 32; ++u) bv[r][u] = __ldg(p + u * bcs);
+            } else {                    // padding channels: accumulator 0, C6 weight 0
+#pragma unroll
+                for (int u = 0; u < 32; ++u) bv[r][u] = (32 * c + u < a.n5) ? __ldg(p + u * bcs) : 0.f;
+            }
+        };
+        Pos cur = pos_of(blockIdx.x);
+        if (blockIdx.x < nbands) {
+#pragma unroll
+            for (int r = 0; r < RING; ++r) load_bias(cur.pb, r, r);
+        }
         int64_t k = 0;
         for (int64_t band = blockIdx.x; band < nbands; band += gridDim.x, ++k) {
             const int buf = (int)(k & 1);
-            const U3Band g = u3_band(a, band, per_img, flat);
+            const bool has_next = band + gridDim.x < nbands;
+            const Pos nxt = pos_of(has_next ? band + gridDim.x : band);
             tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
             tc::fence_after_sync();
 #if U3_EXP >= 1
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);
+            cur = nxt;
             continue;
 #endif
-            const int m = t * kTileM + 32 * (warp & 3) + lane;
-            int64_t orow, ocol;
-            if (flat) {
-                const int64_t q = g.q0 + m;
-                orow = a.out_row0 + q / a.w4;
-                ocol = q - (q / a.w4) * a.w4;
-            } else {
-                orow = g.wr0;
-                ocol = g.q0 + m;
-            }
-            const bool ok = orow < a.out_row0 + a.out_rows && ocol < a.w5;
             float c6[9];
 #pragma unroll
             for (int o = 0; o < 9; ++o) c6[o] = 0.f;
-            // software-pipelined drain: TMEM columns and bias values of chunk c+1 are in flight
-            // while chunk c is computed (up to 4 chunks of 32 columns; NP <= 128)
-            const int nch = (NP + 31) / 32;
-            float v[2][32], bv[2][32];
-            auto issue = [&](int c, int s) {
-                tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(buf * 256 + t * NP + 32 * c), v[s]);
-                if (ok) {
 #pragma unroll
-                    for (int u = 0; u < 32; ++u) {
-                        const int ch = min(32 * c + u, a.n5 - 1);
-                        bv[s][u] = a.b5_plane
-                                       ? __ldg(a.b5 + ((int64_t)ch * a.b5_rows + (orow - a.b5_row0)) * a.w5 + ocol)
-                                       : __ldg(a.b5 + ch);
-                    }
-                }
-            };
-            issue(0, 0);
+            for (int c = 0; c < NCH; ++c) {
+                float v[32];
+                tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(buf * 256 + t * NP + 32 * c), v);
+                tc::tmem_wait_ld();
+                // all 32 MUFU tanh first (back to back in the SFU pipe), then the C6 FMAs;
+                // C6 weights of the padding channels n5..NP-1 are zero (branch-free chunk)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                if (c < nch) {
-                    tc::tmem_wait_ld();
-                    if (c + 1 < nch) issue(c + 1, (c + 1) & 1);
-                    if (ok) {
-                        // branch-free over the chunk (C6 weights of the padding channels
-                        // n5..NP-1 are zero and their accumulators finite), so the tanh of
-                        // several channels are in flight at once
+                for (int u = 0; u < 32; ++u) v[u] = tanh_approx(v[u] + bv[c % RING][u]);
+                // refill the consumed buffer with the chunk RING steps ahead
+                if (c + RING < NCH)
+                    load_bias(cur.pb, c + RING, c % RING);
+                else if (has_next)
+                    load_bias(nxt.pb, c + RING - NCH, c % RING);
 #pragma unroll
-                        for (int u = 0; u < 32; ++u) {
-                            const int ch = 32 * c + u;
-                            const float th = tanh_approx(v[c & 1][u] + bv[c & 1][u]);
+                for (int u = 0; u < 32; ++u) {
+                    const int ch = 32 * c + u;
 #pragma unroll
-                            for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], th, c6[o]);
-                        }
-                    }
+                    for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], v[u], c6[o]);
                 }
             }
             tc::fence_before_sync();
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);  // the accumulator can be reused
-            if (ok) {
-                float* ob = a.out + g.img * a.out_img_stride + (orow - a.out_row0) * a.w5 + ocol;
+            if (cur.ok) {
+                float* ob = a.out + cur.img * a.out_img_stride + (cur.orow - a.out_row0) * a.w5 + cur.ocol;
 #pragma unroll
                 for (int o = 0; o < 9; ++o) {
                     const float b = a.b6_plane
-                                        ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (orow - a.b6_row0)) * a.w5 + ocol)
+                                        ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (cur.orow - a.b6_row0)) * a.w5 + cur.ocol)
                                         : __ldg(a.b6 + o);
                     ob[o * a.out_plane_stride] = c6[o] + b;
                 }
             }
+            cur = nxt;
         }
     }
     tc::fence_before_sync();
@@ -611,12 +593,15 @@ cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s) {
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     if (a.n_pad > U3_NMAX || a.n_pad % 16 || a.n5 > U3_NMAX) return cudaErrorInvalidValue;
-    static std::atomic<uint32_t> flags{0};
     const size_t smem = sizeof(U3Smem) + 128;
-    if (!set_smem_attr((const void*)cnn_u3_tc_kernel, smem, flags)) return cudaErrorInvalidValue;
-    const bool flat = a.w4 <= kFlatMax;
-    const int64_t per_img = flat ? (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM)
-                                 : a.out_rows * ((a.w5 + 2 * kTileM - 1) / (2 * kTileM));
+    const int nch = (a.n_pad + 31) / 32;
+    const void* fns[4] = {(const void*)cnn_u3_tc_kernel<1>, (const void*)cnn_u3_tc_kernel<2>,
+                          (const void*)cnn_u3_tc_kernel<3>, (const void*)cnn_u3_tc_kernel<4>};
+    static std::atomic<uint32_t> flag_n[4];
+    if (!set_smem_attr(fns[nch - 1], smem, flag_n[nch - 1])) return cudaErrorInvalidValue;
+    const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
+    // the epilogue addresses bias channels with 32-bit offsets
+    if (a.b5_plane && (int64_t)a.n5 * a.b5_rows * a.w5 >= (1ll << 32)) return cudaErrorInvalidValue;
     U3K6 k6w{};
     for (int ch = 0; ch < a.n5; ++ch)
         for (int o = 0; o < 9; ++o) k6w.k6[ch][o] = a.k6_host[o * a.n5 + ch];
@@ -625,7 +610,12 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t nbands = per_img * a.nimg;
     const unsigned grid = (unsigned)std::min<int64_t>(nbands, sms);
-    cnn_u3_tc_kernel<<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands);
+    switch (nch) {
+        case 1: cnn_u3_tc_kernel<1><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
+        case 2: cnn_u3_tc_kernel<2><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
+        case 3: cnn_u3_tc_kernel<3><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
+        default: cnn_u3_tc_kernel<4><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
+    }
     return cudaGetLastError();
 }
 
