@@ -52,12 +52,14 @@ constexpr int kTileM = 128;
 // Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns [c0, c0+128): tile 0 = C3 row 2R,
 // tile 1 = row 2R+1 (M = 128 each, N = 32: 20 maps padded). Window: T2 rows [2R, 2R+6) x
 // cols [c0, c0+134), 8 channels per pixel (one 16-byte row each).
-// Warp-specialised and persistent (one CTA per SM, 9 warps):
-//   warp 8, one thread   producer + MMA issuer: the C3 B operand (15 K-steps) once per CTA by a
-//                        bulk copy; per segment six 1-D bulk copies (TMA engine) of the window's
-//                        T2 rows into one of U2_NA buffers (prefetched U2_NA-1 segments ahead);
-//                        2 tiles x 15 tcgen05.mma into one of 4 TMEM slots; tcgen05.commit frees
-//                        the window buffer and hands the slot to the epilogue
+// Warp-specialised and persistent (one CTA per SM, 10 warps; single-lane issue under elect.sync):
+//   warp 9               copy producer: the C3 B operand (15 K-steps) once per CTA by a bulk
+//                        copy; per segment six 1-D bulk copies (TMA engine) of the window's T2
+//                        rows into one of U2_NA buffers, as soon as the buffer is free
+//   warp 8               MMA issuer: 2 tiles x 15 tcgen05.mma into one of 4 TMEM slots;
+//                        tcgen05.commit frees the window buffer and hands the slot to the
+//                        epilogue (copy issue -- ~150 cycles per bulk copy -- no longer
+//                        serialises with MMA issue)
 //   warps 0-3 / 4-7      epilogue groups for even / odd segments: bias plane (prefetched one
 //                        segment ahead), tanh, the 2x2 subsample (rows in the same thread,
 //                        columns across neighbouring lanes), tanh -> T4 bf16 channel blocks
@@ -66,7 +68,7 @@ constexpr int U2_N = 32;                      // 20 maps padded to 32
 constexpr int U2_KS = 15;                     // 5 rows x pairs (0,1) (2,3) (4,5)
 constexpr int U2_NA = 8;                      // window buffers
 constexpr int U2_NT = 4;                      // TMEM slots (2 per epilogue group)
-constexpr int kThreadsU2 = 9 * 32;
+constexpr int kThreadsU2 = 10 * 32;
 
 struct U2P {
     float p4[20][4];  // S4 weights (constant bank)
@@ -117,15 +119,21 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
     const uint32_t tmem = S.tmem;
     const int64_t my = nseg > blockIdx.x ? (nseg - 1 - blockIdx.x) / gridDim.x + 1 : 0;
 
-    if (warp == 8) {
-        // -------------------------------------------------------------------- producer + MMA
-        // (the whole warp runs the loop, so descriptors stay in uniform registers; one elected
-        // lane issues the copies, MMAs and commits)
+    if (warp == 9) {
+        // -------------------------------------------------------------------- copy producer
+        // (the whole warp runs the loop; one elected lane issues the bulk copies)
         const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
-        auto load_a = [&](int64_t k) {
+        const uint32_t bbytes = (uint32_t)(U2_KS * 2 * U2_N * 16);
+        if (tc::elect_one()) {
+            tc::mbar_expect_tx(&S.b_full, bbytes);
+            tc::bulk_g2s(S.b, a.k3_tc, bbytes, &S.b_full);
+        }
+        __syncwarp();
+        for (int64_t k = 0; k < my; ++k) {
+            const int buf = (int)(k % U2_NA);
+            if (k >= U2_NA) tc::mbar_wait(&S.a_empty[buf], (uint32_t)(((k - U2_NA) / U2_NA) & 1));
             int64_t img, R, c0;
             seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
-            const int buf = (int)(k % U2_NA);
             const int64_t r0 = 2 * R - a.t2_row0;
             const int64_t rows = min((int64_t)U2_WR, a.t2_rows - r0);
             const int64_t cols = min((int64_t)U2_WP, a.w2 - c0);
@@ -136,14 +144,11 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
                     tc::bulk_g2s(&S.a[buf][r * U2_WP], src + r * a.w2, (uint32_t)(cols * 16), &S.a_full[buf]);
             }
             __syncwarp();
-        };
-        const uint32_t bbytes = (uint32_t)(U2_KS * 2 * U2_N * 16);
-        if (tc::elect_one()) {
-            tc::mbar_expect_tx(&S.b_full, bbytes);
-            tc::bulk_g2s(S.b, a.k3_tc, bbytes, &S.b_full);
         }
-        __syncwarp();
-        for (int64_t k = 0; k < U2_NA - 1 && k < my; ++k) load_a(k);
+    } else if (warp == 8) {
+        // -------------------------------------------------------------------- MMA issuer
+        // (the whole warp runs the loop, so descriptors stay in uniform registers; one elected
+        // lane issues the MMAs and commits)
         tc::mbar_wait(&S.b_full, 0);
         const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
         // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding
@@ -176,12 +181,6 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
                 tc::commit(&S.t_full[ts]);
             }
             __syncwarp();
-            // keep U2_NA-1 windows in flight: refill the buffer segment k-1 used (its MMAs
-            // are done or about to be: segment k's MMAs are queued behind them)
-            if (k + U2_NA - 1 < my) {
-                if (k >= 1) tc::mbar_wait(&S.a_empty[(k - 1) % U2_NA], (uint32_t)(((k - 1) / U2_NA) & 1));
-                load_a(k + U2_NA - 1);
-            }
         }
     } else {
         // -------------------------------------------------------------------- epilogue groups
@@ -192,18 +191,17 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
         // this group's NEXT segment are issued as soon as the current values are consumed, so
         // they are in flight during the stores and the wait for the next accumulator.
         float b0v[20], b1v[20];
+        const uint32_t bcs = a.b3_plane ? (uint32_t)(a.b3_rows * a.w3) : 1u;  // channel stride of the bias
+        const uint32_t brs = a.b3_plane ? (uint32_t)a.w3 : 0u;                 // row stride
         auto load_bias = [&](int64_t kk) {
             int64_t img_, R_, c0_;
             seg_coords(blockIdx.x + kk * gridDim.x, img_, R_, c0_);
             const int64_t cc = min(c0_ + 32 * wq + lane, a.w3 - 1);
+            const float* p0 = a.b3_plane ? a.b3 + (2 * R_ - a.b3_row0) * a.w3 + cc : a.b3;
 #pragma unroll
             for (int co = 0; co < 20; ++co) {
-                if (a.b3_plane) {
-                    b0v[co] = __ldg(a.b3 + ((int64_t)co * a.b3_rows + (2 * R_ - a.b3_row0)) * a.w3 + cc);
-                    b1v[co] = __ldg(a.b3 + ((int64_t)co * a.b3_rows + (2 * R_ + 1 - a.b3_row0)) * a.w3 + cc);
-                } else {
-                    b0v[co] = b1v[co] = __ldg(a.b3 + co);
-                }
+                b0v[co] = __ldg(p0 + co * bcs);
+                b1v[co] = __ldg(p0 + co * bcs + brs);
             }
         };
         if (grp < my) load_bias(grp);
@@ -578,6 +576,8 @@ cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s) {
     if (a.t4_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     static std::atomic<uint32_t> flags{0};
     const size_t smem = sizeof(U2Smem) + 128;
+    // the epilogue addresses bias channels with 32-bit offsets
+    if (a.b3_plane && 20 * a.b3_rows * a.w3 >= (1ll << 32)) return cudaErrorInvalidValue;
     if (!set_smem_attr((const void*)cnn_u2_tc_kernel, smem, flags)) return cudaErrorInvalidValue;
     U2P pw;
     std::memcpy(pw.p4, a.p4_host, sizeof pw.p4);
