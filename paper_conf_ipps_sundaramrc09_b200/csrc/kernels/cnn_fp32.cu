@@ -167,7 +167,7 @@ constexpr int U1T_BBYTES = 8 * U1T_BR * U1T_BC * 4;             // 32768
 constexpr int U1T_STAGE = U1T_XSTRIDE + U1T_BBYTES;
 
 template <bool kBf16, bool kPlane>
-__global__ void __launch_bounds__(128, 2)
+__global__ void __launch_bounds__(128, 3)
     cnn_u1_tma_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap bmap,
                       const CnnU1Args a, const __grid_constant__ U1W w, const int tiles_c, const int tiles_r,
                       const int64_t ntiles) {
@@ -637,7 +637,7 @@ cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s) {
             int dev = 0, sms = 148;
             cudaGetDevice(&dev);
             cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            const int64_t grid = std::min<int64_t>(ntiles, 2 * (int64_t)sms);
+            const int64_t grid = std::min<int64_t>(ntiles, 3 * (int64_t)sms);
             const size_t smem = 2 * (size_t)U1T_STAGE + 128;
             auto go = [&](auto kern) -> cudaError_t {
                 cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

@@ -263,40 +263,49 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
 // dropped). For any width, filter row i of a band reads one contiguous run of T4: flat pixels
 // [q0 + i*w4, q0 + i*w4 + 262) -- the band's "slice" i (+4 taps, +1 for the (4,5) tap pair,
 // +1 spare).
-// Warp-specialised and persistent (one CTA per SM, 9 warps):
-//   warp 8 (warp-uniform, one elected lane issues)  producer + MMA issuer: the whole C5 B
-//                        operand (40 K-steps x NP maps, up to 160 KB) is loaded ONCE per CTA and
-//                        stays resident; the slices flow through a ring of U3_NA buffers (three
-//                        1-D bulk copies each, one per channel block, prefetched U3_NA-1 slices
-//                        ahead); per slice 8 K-steps x 2 tiles of tcgen05.mma into one of two TMEM
-//                        accumulators (2 tiles x NP columns); tcgen05.commit frees the slice
-//                        buffer, and after the 5th slice hands the accumulator to the epilogue
-//   warps 0-7            epilogue: TMEM -> registers, bias plane + tanh, the 1x1 C6 layer as a
-//                        dot product over n5 (weights in the constant bank), + bias -> output
-// so the epilogue of band k overlaps the MMAs of band k+1. (An earlier version re-streamed B
-// through a 6-slot ring for every band -- 160 KB of L2 reads per 256 positions -- and its MMAs
-// waited on those copies.)
+// Both layers run on the tensor cores:
+//   C5  D5[px][n] = sum_k A5[px][k] B5[k][n]  (A5: the slices in smem, B5: resident in smem)
+//   C6  D6[px][o] = sum_n T5[px][n] B6[n][o]  with T5 = tanh(D5 + bias plane) written back by
+//       the epilogue into the drained TMEM columns as bf16 pairs, and the MMA reading its A
+//       operand straight from TMEM (M = 128 lanes, K = NP channels, N = 16: 9 maps padded)
+// TMEM (512 columns): accumulator buffer b in {0,1}, tile t: 128-column region at 256b + 128t
+// holding D5 in [0, NP), then T5 in [0, NP/2) and D6 in [64, 80).
+// Warp-specialised and persistent (one CTA per SM, 10 warps; single-lane issue under elect.sync):
+//   warp 9               copy producer: the whole C5 B operand (40 K-steps x NP maps, up to
+//                        160 KB) ONCE per CTA (it stays resident), then the slices through a ring
+//                        of U3_NA buffers (three 1-D bulk copies each, one per channel block)
+//   warp 8               MMA issuer: per slice 8 K-steps x 2 tiles of tcgen05.mma; after the 5th
+//                        slice the accumulator goes to the epilogue. The C6 MMAs of the previous
+//                        band are slotted in between slices as soon as its T5 is in TMEM.
+//   warps 0-7            epilogue: TMEM -> registers, + bias plane, tanh -> bf16 T5 -> TMEM;
+//                        then D6 -> registers, + C6 bias -> output (fp32)
+// so the epilogue of band k overlaps the C5 MMAs of band k+1. (Earlier versions re-streamed
+// B5 for every band, and computed C6 as 9 x n5 FFMA per position on the CUDA cores.)
 constexpr int U3_KS = 40;
 constexpr int U3_NMAX = 128;
 constexpr int U3_SPX = 2 * kTileM + 8;  // pixels per slice buffer (262 used)
 constexpr int U3_NA = 4;                // slice buffers
+constexpr int U3_C6K = U3_NMAX / 16;    // C6 K-steps (max)
+constexpr int U3_C6N = 16;              // C6 N: 9 maps padded
+constexpr int U3_C6COL = 64;            // D6 column within a tile region
 constexpr int kEpiWarps = 8;
-constexpr int kThreadsU3 = (kEpiWarps + 1) * 32;
+constexpr int kThreadsU3 = (kEpiWarps + 2) * 32;
 
-struct U3K6 {
-    float k6[U3_NMAX][12];  // [ch][o] (9 used): C6 weights, broadcast from the constant bank
+struct U3P {
+    uint4 b6[U3_C6K * 2 * U3_C6N];  // C6 B operand, bf16 [ks][half][o][8 ch] (4 KB)
 };
 
 struct U3Smem {
-    uint4 b[U3_KS * 2 * U3_NMAX];  // resident C5 B operand: [ks][half][n] -> 8 bf16
-    uint4 a[U3_NA][3][U3_SPX];     // slice ring: [channel block][pixel] -> 8 bf16
-    uint64_t b_full, a_full[U3_NA], a_empty[U3_NA], t_full[2], t_empty[2];
+    uint4 b[U3_KS * 2 * U3_NMAX];     // resident C5 B operand: [ks][half][n] -> 8 bf16
+    uint4 b6[U3_C6K * 2 * U3_C6N];    // C6 B operand
+    uint4 a[U3_NA][3][U3_SPX];        // slice ring: [channel block][pixel] -> 8 bf16
+    uint64_t b_full, a_full[U3_NA], a_empty[U3_NA], t_full[2], t_empty[2], t5_full[2], c6_full[2];
     uint32_t tmem;
 };
 
 template <int NCH>  // TMEM chunks of 32 columns: NP = n5 padded to 16, NCH = ceil(NP / 32)
 __global__ void __launch_bounds__(kThreadsU3, 1)
-    cnn_u3_tc_kernel(const CnnU3Args a, const __grid_constant__ U3K6 k6w, const int64_t nbands) {
+    cnn_u3_tc_kernel(const CnnU3Args a, const __grid_constant__ U3P pw, const int64_t nbands) {
     extern __shared__ __align__(128) uint8_t smraw[];
     U3Smem& S = *reinterpret_cast<U3Smem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -315,43 +324,28 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         for (int i = 0; i < 2; ++i) {
             tc::mbar_init(&S.t_full[i], 1);
             tc::mbar_init(&S.t_empty[i], kEpiWarps);
+            tc::mbar_init(&S.t5_full[i], kEpiWarps);
+            tc::mbar_init(&S.c6_full[i], 1);
         }
         tc::mbar_fence_init();
     }
     // slice buffers start zeroed: pixels a copy does not cover (past the chunk's last T4 row)
     // then only ever hold finite T4 values; they feed positions that are not stored
     for (int idx = tid; idx < U3_NA * 3 * U3_SPX; idx += kThreadsU3) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
+    for (int idx = tid; idx < U3_C6K * 2 * U3_C6N; idx += kThreadsU3) S.b6[idx] = pw.b6[idx];
     tc::fence_proxy_async();
     tc::fence_before_sync();
     __syncthreads();
     tc::fence_after_sync();
     const uint32_t tmem = S.tmem;
 
-    if (warp == kEpiWarps) {
-        // ---------------------------------------------------------------- producer + MMA
-        // (the whole warp runs the loop so descriptors live in uniform registers; one elected
-        // lane issues the copies, MMAs and commits)
+    const int64_t my_bands = nbands > blockIdx.x ? (nbands - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const int64_t total = my_bands * 5;  // slices
+    if (warp == kEpiWarps + 1) {
+        // ---------------------------------------------------------------- copy producer
+        // (warp-uniform loop, one elected lane issues): B5 once, then every slice as soon as
+        // its ring buffer is free
         const uint4* t4all = reinterpret_cast<const uint4*>(a.t4);
-        const int64_t my_bands = nbands > blockIdx.x ? (nbands - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-        const int64_t total = my_bands * 5;  // slices
-        auto load_slice = [&](int64_t s) {
-            const int64_t band = blockIdx.x + (s / 5) * gridDim.x;
-            const int i = (int)(s % 5);
-            const int64_t img = band / per_img;
-            const int64_t q0 = (band - img * per_img) * 2 * kTileM;
-            const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
-            const int64_t n = max((int64_t)0, min((int64_t)U3_SPX, bplane - e));
-            const int slot = (int)(s % U3_NA);
-            if (tc::elect_one()) {
-                tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
-                if (n > 0) {
-                    const uint4* src = t4all + img * 3 * bplane + e;
-                    for (int blk = 0; blk < 3; ++blk)
-                        tc::bulk_g2s(S.a[slot][blk], src + blk * bplane, (uint32_t)(n * 16), &S.a_full[slot]);
-                }
-            }
-            __syncwarp();
-        };
         if (my_bands > 0) {
             const uint32_t bbytes = (uint32_t)(U3_KS * 2 * NP * 16);
             if (tc::elect_one()) {
@@ -362,14 +356,60 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             }
             __syncwarp();
         }
-        for (int64_t s = 0; s < U3_NA - 1 && s < total; ++s) load_slice(s);
+        for (int64_t s = 0; s < total; ++s) {
+            const int slot = (int)(s % U3_NA);
+            if (s >= U3_NA) tc::mbar_wait(&S.a_empty[slot], (uint32_t)(((s - U3_NA) / U3_NA) & 1));
+            const int64_t band = blockIdx.x + (s / 5) * gridDim.x;
+            const int i = (int)(s % 5);
+            const int64_t img = band / per_img;
+            const int64_t q0 = (band - img * per_img) * 2 * kTileM;
+            const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
+            const int64_t n = max((int64_t)0, min((int64_t)U3_SPX, bplane - e));
+            if (tc::elect_one()) {
+                tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
+                if (n > 0) {
+                    const uint4* src = t4all + img * 3 * bplane + e;
+                    for (int blk = 0; blk < 3; ++blk)
+                        tc::bulk_g2s(S.a[slot][blk], src + blk * bplane, (uint32_t)(n * 16), &S.a_full[slot]);
+                }
+            }
+            __syncwarp();
+        }
+    } else if (warp == kEpiWarps) {
+        // ---------------------------------------------------------------- MMA issuer
+        // (warp-uniform loop so descriptors live in uniform registers; one elected lane issues)
         if (my_bands > 0) tc::mbar_wait(&S.b_full, 0);
         const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);
+        const uint32_t idesc6 = tc::make_idesc_bf16(kTileM, U3_C6N);
         const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), (uint32_t)(NP * 16), 128);
+        const uint64_t b6desc0 = tc::make_desc(tc::smem_u32(S.b6), (uint32_t)(U3_C6N * 16), 128);
         const uint32_t plane_bytes = (uint32_t)(U3_SPX * 16);
+        // C6 of local band kb (its T5 is in TMEM): 2 tiles x NP/16 K-steps, A from TMEM
+        int64_t c6_next = 0;
+        auto issue_c6 = [&](int64_t kb) {
+            const uint32_t base = tmem + (uint32_t)((kb & 1) * 256);
+            if (tc::elect_one()) {
+                for (int t = 0; t < 2; ++t)
+                    for (int kk = 0; kk < NP / 16; ++kk)
+                        tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL), base + (uint32_t)(t * 128 + kk * 8),
+                                        b6desc0 + (uint64_t)(kk * 2 * U3_C6N), idesc6, kk > 0 ? 1u : 0u);
+                tc::commit(&S.c6_full[kb & 1]);
+            }
+            __syncwarp();
+        };
         for (int64_t k = 0; k < my_bands; ++k) {
             const int buf = (int)(k & 1);
-            if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+            if (k >= 2) {
+                // band k-2 shares this accumulator: its C6 must be issued before its epilogue
+                // can release the buffer
+                while (c6_next <= k - 2) {
+                    tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                    tc::fence_after_sync();
+                    issue_c6(c6_next++);
+                }
+                tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+                tc::fence_after_sync();
+            }
             const uint32_t d_base = tmem + (uint32_t)(buf * 256);
             for (int i = 0; i < 5; ++i) {
                 const int64_t s = k * 5 + i;
@@ -390,20 +430,24 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
 #pragma unroll
                         for (int t = 0; t < 2; ++t) {
                             const uint64_t ad = tc::make_desc(a_addr + (uint32_t)(t * kTileM * 16), lbo, 128);
-                            tc::mma_bf16(d_base + (uint32_t)(t * NP), ad, bd, idesc, ks > 0 ? 1u : 0u);
+                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad, bd, idesc, ks > 0 ? 1u : 0u);
                         }
                     }
                     tc::commit(&S.a_empty[slot]);
                     if (i == 4) tc::commit(&S.t_full[buf]);
                 }
                 __syncwarp();
-                // keep U3_NA-1 slices in flight: refill the buffer slice s-1 used (its MMAs are
-                // done or about to be: slice s's MMAs are queued behind them)
-                if (s + U3_NA - 1 < total) {
-                    if (s >= 1) tc::mbar_wait(&S.a_empty[(s - 1) % U3_NA], (uint32_t)(((s - 1) / U3_NA) & 1));
-                    load_slice(s + U3_NA - 1);
+                // the previous band's C6 as soon as its T5 is ready (between slices)
+                if (c6_next < k && tc::mbar_test(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1))) {
+                    tc::fence_after_sync();
+                    issue_c6(c6_next++);
                 }
             }
+        }
+        while (c6_next < my_bands) {
+            tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+            tc::fence_after_sync();
+            issue_c6(c6_next++);
         }
     } else {
         // ---------------------------------------------------------------- epilogue warps
@@ -414,22 +458,25 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
         const int m = t * kTileM + 32 * (warp & 3) + lane;
         struct Pos {
-            int64_t img, orow, ocol;
+            int img, orow, ocol;  // image, global output row, column (32-bit: per-chunk extents)
             bool ok;
-            const float* pb;
+            const float* pb;      // bias-plane address of channel 0 at this position
         };
         const uint32_t bcs = a.b5_plane ? (uint32_t)(a.b5_rows * a.w5) : 1u;  // channel stride of the bias
+        const int w4 = (int)a.w4, w5 = (int)a.w5, orow_end = (int)(a.out_row0 + a.out_rows);
         auto pos_of = [&](int64_t band) {
             Pos q;
-            q.img = band / per_img;
-            const int64_t qq = (band - q.img * per_img) * 2 * kTileM + m;
-            q.orow = a.out_row0 + qq / a.w4;
-            q.ocol = qq - (qq / a.w4) * a.w4;
-            q.ok = q.orow < a.out_row0 + a.out_rows && q.ocol < a.w5;
+            const int64_t img = band / per_img;
+            const int qq = (int)(band - img * per_img) * 2 * kTileM + m;
+            q.img = (int)img;
+            const int r = qq / w4;
+            q.orow = (int)a.out_row0 + r;
+            q.ocol = qq - r * w4;
+            q.ok = q.orow < orow_end && q.ocol < w5;
             // positions past the chunk's last row / the row's last column compute on clamped
             // (in-bounds) bias addresses and are not stored: the drain stays branch-free
-            const int64_t orow_c = min(q.orow, a.out_row0 + a.out_rows - 1), ocol_c = min(q.ocol, a.w5 - 1);
-            q.pb = a.b5_plane ? a.b5 + (orow_c - a.b5_row0) * a.w5 + ocol_c : a.b5;
+            const int orow_c = min(q.orow, orow_end - 1), ocol_c = min(q.ocol, w5 - 1);
+            q.pb = a.b5_plane ? a.b5 + ((int64_t)(orow_c - a.b5_row0) * w5 + ocol_c) : a.b5;
             return q;
         };
         // bias ring: 2 chunk buffers loaded 2 chunks ahead when NCH is even (chunk parity is then
@@ -442,10 +489,10 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             // compile-time constant at every call, so only the last chunk carries predicates
             if (c < NCH - 1) {
 #pragma unroll
-                for (int u = 0; u < 32; ++u) bv[r][u] = __ldg(p + u * bcs);
-            } else {                    // padding channels: accumulator 0, C6 weight 0
+                for (int u = 0; u < 32; ++u, p += bcs) bv[r][u] = __ldg(p);
+            } else {  // padding channels: accumulator 0, C6 weight 0
 #pragma unroll
-                for (int u = 0; u < 32; ++u) bv[r][u] = (32 * c + u < a.n5) ? __ldg(p + u * bcs) : 0.f;
+                for (int u = 0; u < 32; ++u, p += bcs) bv[r][u] = (32 * c + u < a.n5) ? __ldg(p) : 0.f;
             }
         };
         Pos cur = pos_of(blockIdx.x);
@@ -456,54 +503,52 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         int64_t k = 0;
         for (int64_t band = blockIdx.x; band < nbands; band += gridDim.x, ++k) {
             const int buf = (int)(k & 1);
+            const uint32_t region = tmem + lane_base + (uint32_t)(buf * 256 + t * 128);
             const bool has_next = band + gridDim.x < nbands;
-            const Pos nxt = pos_of(has_next ? band + gridDim.x : band);
+            const float* nxt_pb = pos_of(has_next ? band + gridDim.x : band).pb;
             tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
             tc::fence_after_sync();
-#if U3_EXP >= 1
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);
-            cur = nxt;
-            continue;
-#endif
-            float c6[9];
-#pragma unroll
-            for (int o = 0; o < 9; ++o) c6[o] = 0.f;
 #pragma unroll
             for (int c = 0; c < NCH; ++c) {
                 float v[32];
-                tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(buf * 256 + t * NP + 32 * c), v);
+                tc::tmem_ld32_async(region + (uint32_t)(32 * c), v);
                 tc::tmem_wait_ld();
-                // all 32 MUFU tanh first (back to back in the SFU pipe), then the C6 FMAs;
-                // C6 weights of the padding channels n5..NP-1 are zero (branch-free chunk)
 #pragma unroll
                 for (int u = 0; u < 32; ++u) v[u] = tanh_approx(v[u] + bv[c % RING][u]);
                 // refill the consumed buffer with the chunk RING steps ahead
                 if (c + RING < NCH)
                     load_bias(cur.pb, c + RING, c % RING);
                 else if (has_next)
-                    load_bias(nxt.pb, c + RING - NCH, c % RING);
+                    load_bias(nxt_pb, c + RING - NCH, c % RING);
+                // T5 chunk c -> TMEM columns [16c, 16c+16) (already drained), bf16 pairs
+                uint32_t r[16];
 #pragma unroll
-                for (int u = 0; u < 32; ++u) {
-                    const int ch = 32 * c + u;
-#pragma unroll
-                    for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], v[u], c6[o]);
-                }
+                for (int u = 0; u < 16; ++u) r[u] = tc::pack_bf16(v[2 * u], v[2 * u + 1]);
+                tc::tmem_st16(region + (uint32_t)(16 * c), r);
             }
+            tc::tmem_wait_st();
+            tc::fence_before_sync();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&S.t5_full[buf]);  // T5 ready for the C6 MMA
+            float d6[16];
+            tc::mbar_wait(&S.c6_full[buf], (uint32_t)((k >> 1) & 1));
+            tc::fence_after_sync();
+            tc::tmem_ld16_async(region + (uint32_t)U3_C6COL, d6);
+            tc::tmem_wait_ld();
             tc::fence_before_sync();
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);  // the accumulator can be reused
             if (cur.ok) {
-                float* ob = a.out + cur.img * a.out_img_stride + (cur.orow - a.out_row0) * a.w5 + cur.ocol;
+                float* ob = a.out + cur.img * a.out_img_stride + (int64_t)(cur.orow - a.out_row0) * w5 + cur.ocol;
 #pragma unroll
                 for (int o = 0; o < 9; ++o) {
                     const float b = a.b6_plane
-                                        ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (cur.orow - a.b6_row0)) * a.w5 + cur.ocol)
+                                        ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (cur.orow - a.b6_row0)) * w5 + cur.ocol)
                                         : __ldg(a.b6 + o);
-                    ob[o * a.out_plane_stride] = c6[o] + b;
+                    ob[o * a.out_plane_stride] = d6[o] + b;
                 }
             }
-            cur = nxt;
+            if (has_next) cur = pos_of(band + gridDim.x);
         }
     }
     tc::fence_before_sync();
@@ -602,19 +647,26 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
     // the epilogue addresses bias channels with 32-bit offsets
     if (a.b5_plane && (int64_t)a.n5 * a.b5_rows * a.w5 >= (1ll << 32)) return cudaErrorInvalidValue;
-    U3K6 k6w{};
-    for (int ch = 0; ch < a.n5; ++ch)
-        for (int o = 0; o < 9; ++o) k6w.k6[ch][o] = a.k6_host[o * a.n5 + ch];
+    // C6 B operand: bf16 [ks][half][o][8 ch], value K6[o][16 ks + 8 half + e] (zero padding)
+    U3P pw{};
+    uint16_t* b6 = reinterpret_cast<uint16_t*>(pw.b6);
+    for (int ks = 0; ks < U3_C6K; ++ks)
+        for (int h = 0; h < 2; ++h)
+            for (int o = 0; o < U3_C6N; ++o)
+                for (int e = 0; e < 8; ++e) {
+                    const int ch = 16 * ks + 8 * h + e;
+                    b6[((ks * 2 + h) * U3_C6N + o) * 8 + e] = to_bf16(o < 9 && ch < a.n5 ? a.k6_host[o * a.n5 + ch] : 0.f);
+                }
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t nbands = per_img * a.nimg;
     const unsigned grid = (unsigned)std::min<int64_t>(nbands, sms);
     switch (nch) {
-        case 1: cnn_u3_tc_kernel<1><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
-        case 2: cnn_u3_tc_kernel<2><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
-        case 3: cnn_u3_tc_kernel<3><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
-        default: cnn_u3_tc_kernel<4><<<grid, kThreadsU3, smem, s>>>(a, k6w, nbands); break;
+        case 1: cnn_u3_tc_kernel<1><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
+        case 2: cnn_u3_tc_kernel<2><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
+        case 3: cnn_u3_tc_kernel<3><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
+        default: cnn_u3_tc_kernel<4><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
     }
     return cudaGetLastError();
 }
