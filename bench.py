@@ -300,7 +300,8 @@ def run(args, rank, world, local):
         peak_basis = ("bf16 dense, measured cuBLAS burst (MEASURED_PEAKS.json)" if "bf16_tflops" in peaks
                       else "bf16 dense fallback 1.59 PFLOP/s (B200_PROFILING.md)")
         fl = dict(fl)
-        fl[2], fl[3] = 4 * 20 * 200 * 2, wl["n5"] * 500 * 2   # the tensor-core part of each unit
+        # the tensor-core part of each unit: C3 (U2); C5 and the 1x1 C6 (U3)
+        fl[2], fl[3] = 4 * 20 * 200 * 2, wl["n5"] * 500 * 2 + 9 * wl["n5"] * 2
         flops_per_launch = fl[k] * opx[k] * args.steps / nl
         achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
     else:
