@@ -211,6 +211,23 @@ def unit_flops_per_px(wl) -> dict:
     return {1: 4 * 8 * 25 * 2, 2: 4 * 20 * 200 * 2, 3: n5 * 500 * 2 + 9 * n5 * 2}
 
 
+def unit_bytes(wl, precision: str) -> dict:
+    """Algorithmic HBM bytes of each unit for the whole batch: inputs read
+    once, bias planes once (shared by every image of the batch), outputs written once; T2/T4 in
+    the layout the precision path keeps between units (fp32 planes, or bf16 channel blocks)."""
+    n = wl["n"]
+    if wl["template"] == "edge":
+        return {0: n * wl["H"] * wl["W"] * 8}
+    import synth
+    (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = synth.cnn_dims(wl["H"], wl["W"])
+    bf = precision == "bf16_tc"
+    t2 = n * h2 * w2 * (16 if bf else 32)
+    t4 = n * h4 * w4 * (48 if bf else 80)
+    return {1: n * wl["H"] * wl["W"] * 4 + 8 * h1 * w1 * 4 + t2,
+            2: t2 + 20 * h3 * w3 * 4 + t4,
+            3: t4 + (wl["n5"] + 9) * h5 * w5 * 4 + n * 9 * h5 * w5 * 4}
+
+
 def unit_out_px(wl) -> dict:
     import synth
     if wl["template"] == "edge":
@@ -307,18 +324,52 @@ def run(args, rank, world, local):
     else:
         peak_tf = fp32_peak_tflops(1965.0)
         peak_basis = "FP32 FFMA: 148 SM x 128 lanes x 2 flop x 1965 MHz (clocks.max.sm)"
+    # the same kernel against the HBM roofline (measured copy bandwidth): bias planes make the
+    # single-image CNN units (cnn4) as byte-heavy as they are flop-heavy
+    peaks = json.load(open(PEAKS_FILE)) if os.path.exists(PEAKS_FILE) else {}
+    hbm_peak = float(peaks.get("hbm_gbs", 6549.0))
+    bytes_per_launch = unit_bytes(wl, args.precision)[k] * args.steps / nl
+    hbm_gbs = bytes_per_launch / (kern_ms / 1e3) / 1e9
     traffic = None
     tf_file = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf_file):
         tr = json.load(open(tf_file)).get(f"{args.template}:{args.precision}:{KERNEL_NAMES[k]}")
         if tr:
             traffic = tr["dram_bytes_per_out_px"] * opx[k] * args.steps / nl
-    roofline = {"bound": "tensor" if tensor else "alu", "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
-                "frac": achieved_tf / peak_tf, "traffic": traffic, "kernel": KERNEL_NAMES[k],
-                "kernel_ms_per_launch": kern_ms, "algorithmic_flop_per_launch": flops_per_launch,
-                "peak_basis": peak_basis,
-                "kernel_share_of_step": tim["kernel_ms"][k] / args.steps / ms,
-                "units_ms_per_step": {KERNEL_NAMES[u]: tim["kernel_ms"][u] / args.steps for u in fl}}
+    if bytes_per_launch / (hbm_peak * 1e9) > flops_per_launch / (peak_tf * 1e12):
+        # HBM is the binding roofline of this kernel at this workload
+        roofline = {"bound": "hbm", "achieved": hbm_gbs, "peak": hbm_peak, "unit": "GB/s", "frac": hbm_gbs / hbm_peak,
+                    "peak_basis": "HBM copy bandwidth, measured (MEASURED_PEAKS.json)" if "hbm_gbs" in peaks
+                    else "HBM fallback 6549 GB/s", "compute": {"achieved": achieved_tf, "peak": peak_tf,
+                                                              "unit": "TFLOP/s", "frac": achieved_tf / peak_tf,
+                                                              "basis": peak_basis}}
+    else:
+        roofline = {"bound": "tensor" if tensor else "alu", "achieved": achieved_tf, "peak": peak_tf,
+                    "unit": "TFLOP/s", "frac": achieved_tf / peak_tf, "peak_basis": peak_basis,
+                    "hbm": {"achieved": hbm_gbs, "peak": hbm_peak, "unit": "GB/s", "frac": hbm_gbs / hbm_peak}}
+    roofline.update({"traffic": traffic, "kernel": KERNEL_NAMES[k], "kernel_ms_per_launch": kern_ms,
+                     "algorithmic_flop_per_launch": flops_per_launch,
+                     "algorithmic_bytes_per_launch": bytes_per_launch,
+                     "kernel_share_of_step": tim["kernel_ms"][k] / args.steps / ms,
+                     "units_ms_per_step": {KERNEL_NAMES[u]: tim["kernel_ms"][u] / args.steps for u in fl}})
+    # every unit of the step against both rooflines (algorithmic flops and bytes per step)
+    ub, uf = unit_bytes(wl, args.precision), unit_flops_per_px(wl)
+    units = {}
+    for u in uf:
+        ms_u = tim["kernel_ms"][u] / args.steps
+        if ms_u <= 0:
+            continue
+        tens_u = args.precision == "bf16_tc" and u in (2, 3)
+        if tens_u:  # the tensor-core part: C3 (U2); C5 and C6 (U3)
+            fpx = 4 * 20 * 200 * 2 if u == 2 else wl["n5"] * 500 * 2 + 9 * wl["n5"] * 2
+        else:
+            fpx = uf[u]
+        f_u = fpx * opx[u] / (ms_u / 1e3) / 1e12
+        pk_u = float(peaks.get("bf16_tflops", 1590.0)) if tens_u else fp32_peak_tflops(1965.0)
+        units[KERNEL_NAMES[u]] = {"ms": ms_u, "tflops": f_u, "flop_frac": f_u / pk_u,
+                                  "flop_bound": "tensor" if tens_u else "alu",
+                                  "gbs": ub[u] / (ms_u / 1e3) / 1e9, "hbm_frac": ub[u] / (ms_u / 1e3) / 1e9 / hbm_peak}
+    roofline["units"] = units
     y_ref = [y_dev[0].clone(), y_dev[-1].clone()]
     del p, g, y_dev
 
