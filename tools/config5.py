@@ -102,6 +102,8 @@ def run_template(name, total_gb, share, precision, steps, dev):
            "split_equals_unsplit_first_last_image": ok}
     del p, g, x, y
     torch.cuda.empty_cache()
+    if hasattr(torch._C, "_host_emptyCache"):
+        torch._C._host_emptyCache()  # release the cached pinned host blocks for the next template
     return res
 
 
