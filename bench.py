@@ -530,6 +530,9 @@ def main():
     ap.add_argument("--template", default="edge", choices=["edge", "cnn4", "cnn3", "cnn3s"])
     ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16_tc"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--per-template", default=None,
+                    help="extra template:precision runs reported under per_template (default with --template "
+                         "edge: cnn4:fp32,cnn4:bf16_tc,cnn3:fp32,cnn3:bf16_tc; 'none' skips them)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -553,6 +556,32 @@ def main():
         if world == 1 and not args.no_cpu:
             line["cpu_baseline"] = cpu_oracle_sample(args.template, gpu_out=res["y_host"].numpy(),
                                                      tol=1e-5 if args.precision == "fp32" else 2e-2)
+    del res
+    # the metric is per template: the CNN template's configs (configs[3] cnn4, configs[2] cnn3) in
+    # both precisions, measured in the same run (value / e2e / roofline of each; full lines come
+    # from `--template cnn4 --precision ...`)
+    extra = args.per_template
+    if extra is None:
+        extra = "cnn4:fp32,cnn4:bf16_tc,cnn3:fp32,cnn3:bf16_tc" if args.template == "edge" else "none"
+    per = []
+    for item in ([] if extra == "none" else extra.split(",")):
+        t, pr = item.split(":")
+        a2 = argparse.Namespace(**vars(args))
+        a2.template, a2.precision = t, pr
+        a2.precision_code = tg.TG_FP32 if pr == "fp32" else tg.TG_BF16_TC
+        r2 = run(a2, rank, world, local)
+        per.append({"template": t, "precision": pr, "workload": r2["config"]["workload"], "value": r2["value"],
+                    "unit": "Mpixels/s", "ms_per_step": r2["ms_per_step"],
+                    "e2e": {k: r2["e2e"].get(k) for k in ("value", "ms_per_step", "h2d_bytes_per_step",
+                                                         "d2h_bytes_per_step", "bytes_vs_lower_bound", "overlap")}
+                           | {"link_roofline_frac": r2["e2e"].get("host_link", {}).get("roofline_frac")},
+                    "roofline": {k: r2["roofline"].get(k) for k in ("bound", "achieved", "peak", "unit", "frac",
+                                                                     "kernel")},
+                    "gpu_launches": r2["gpu_launches"], "clocks": r2["clocks"]})
+        del r2
+    if rank == 0:
+        if per:
+            line["per_template"] = per
         print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist
