@@ -254,6 +254,17 @@ tg_status tg_sched_dfs_order(const tg_sched* s, int32_t* order);
  * TG_E_INFEASIBLE if an operator's inputs and outputs do not fit together. */
 tg_status tg_sched_transfers(const tg_sched* s, const int32_t* order, uint64_t capacity, uint64_t* moved,
                              int32_t* trace, int64_t trace_cap, int64_t* trace_len);
+/* Exact counterpart of the heuristic for small graphs: the minimum of the
+ * transfer volume of tg_sched_transfers over EVERY operator order that respects the data
+ * dependences (PB constraints (1)-(3) of Fig. 5; the paper solved the full
+ * PB model with MiniSAT+, PAPER.md:477 -- here the eviction policy stays next-use, DESIGN.md
+ * R10, and the search is over operator orders). order[0..n_ops) receives the lexicographically
+ * smallest optimal order, *moved its volume, *n_orders (may be NULL) the number of orders
+ * enumerated and *n_optimal (may be NULL) how many reach the minimum.
+ * TG_E_UNSUPPORTED if the graph has more than max_orders orders (the enumeration is
+ * factorial: meant for graphs of ~12 operators or fewer); TG_E_INFEASIBLE if no order fits. */
+tg_status tg_sched_optimal(const tg_sched* s, uint64_t capacity, uint64_t max_orders, int32_t* order,
+                           uint64_t* moved, uint64_t* n_orders, uint64_t* n_optimal);
 
 const char* tg_last_error(void);
 /* Library version string, e.g. "tg 0.1 sm_100a". */

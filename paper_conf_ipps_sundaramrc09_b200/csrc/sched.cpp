@@ -157,6 +157,82 @@ uint64_t sched_transfers(const tg_sched& s, const std::vector<int32_t>& order, u
     return moved;
 }
 
+// Exhaustive minimum of the next-use transfer volume over every operator order that respects
+// the data dependences (PB constraints (1)-(3) of Fig. 5): the exact
+// counterpart of the DFS heuristic for small graphs (the paper solved the PB model
+// with MiniSAT+, which is out of scope). Orders are enumerated depth-first with
+// operators tried in id order, so the order returned is the lexicographically smallest optimal
+// one. Returns false if more than max_orders orders exist.
+bool sched_optimal(const tg_sched& s, uint64_t capacity, uint64_t max_orders, std::vector<int32_t>& best_order,
+                   uint64_t& best, uint64_t& n_orders, uint64_t& n_best) {
+    const int n = (int)s.ops.size();
+    std::map<int32_t, int32_t> producer;
+    for (int i = 0; i < n; ++i)
+        for (int32_t j : s.ops[i].outs) producer[j] = i;
+    std::vector<std::vector<int32_t>> preds(n);
+    for (int c = 0; c < n; ++c)
+        for (int32_t j : s.ops[c].ins) {
+            auto it = producer.find(j);
+            if (it != producer.end()) preds[c].push_back(it->second);
+        }
+    best = UINT64_MAX;
+    n_orders = n_best = 0;
+    std::vector<int32_t> prefix;
+    std::vector<char> placed(n, 0);
+    bool ok = true;
+    // explicit-stack DFS over the choices at each depth
+    std::vector<int> next(n + 1, 0);
+    int depth = 0;
+    while (depth >= 0 && ok) {
+        if (depth == n) {
+            if (++n_orders > max_orders) {
+                ok = false;
+                break;
+            }
+            const uint64_t v = sched_transfers(s, prefix, capacity, nullptr, false);
+            if (v < best) {
+                best = v;
+                n_best = 1;
+                best_order = prefix;
+            } else if (v == best && v != UINT64_MAX) {
+                ++n_best;
+            }
+            --depth;
+            if (depth >= 0) {
+                placed[prefix.back()] = 0;
+                prefix.pop_back();
+            }
+            continue;
+        }
+        int i = next[depth];
+        for (; i < n; ++i) {
+            if (placed[i]) continue;
+            bool ready = true;
+            for (int p : preds[i])
+                if (!placed[p]) {
+                    ready = false;
+                    break;
+                }
+            if (ready) break;
+        }
+        if (i >= n) {  // no more choices at this depth: backtrack
+            next[depth] = 0;
+            --depth;
+            if (depth >= 0) {
+                placed[prefix.back()] = 0;
+                prefix.pop_back();
+            }
+            continue;
+        }
+        next[depth] = i + 1;
+        placed[i] = 1;
+        prefix.push_back(i);
+        ++depth;
+        next[depth] = 0;
+    }
+    return ok;
+}
+
 }  // namespace tg
 
 using namespace tg;
@@ -231,6 +307,23 @@ tg_status tg_sched_transfers(const tg_sched* s, const int32_t* order, uint64_t c
             trace[2 * i + 1] = tr[i].second;
         }
     }
+    return TG_OK;
+}
+
+tg_status tg_sched_optimal(const tg_sched* s, uint64_t capacity, uint64_t max_orders, int32_t* order,
+                           uint64_t* moved, uint64_t* n_orders, uint64_t* n_optimal) {
+    if (!s || !moved || (!order && !s->ops.empty())) return fail(TG_E_ARG, "tg_sched_optimal: NULL argument");
+    std::vector<int32_t> best_order;
+    uint64_t best = 0, no = 0, nb = 0;
+    if (!sched_optimal(*s, capacity, max_orders, best_order, best, no, nb))
+        return fail(TG_E_UNSUPPORTED, "tg_sched_optimal: more operator orders than max_orders");
+    if (no == 0 && !s->ops.empty()) return fail(TG_E_ARG, "tg_sched_optimal: the graph has a cycle");
+    if (best == UINT64_MAX)
+        return fail(TG_E_INFEASIBLE, "tg_sched_optimal: no order fits the capacity");
+    std::copy(best_order.begin(), best_order.end(), order);
+    *moved = best;
+    if (n_orders) *n_orders = no;
+    if (n_optimal) *n_optimal = nb;
     return TG_OK;
 }
 

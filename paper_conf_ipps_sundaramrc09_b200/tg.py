@@ -117,6 +117,8 @@ _PROTOS = {
     "tg_sched_add_op": (c_i32, [vp, P_id, c_i32, P_id, c_i32, P_id]),
     "tg_sched_dfs_order": (c_i32, [vp, P_id]),
     "tg_sched_transfers": (c_i32, [vp, P_id, c_u64, ctypes.POINTER(c_u64), P_id, c_i64, ctypes.POINTER(c_i64)]),
+    "tg_sched_optimal": (c_i32, [vp, c_u64, c_u64, P_id, ctypes.POINTER(c_u64), ctypes.POINTER(c_u64),
+                                 ctypes.POINTER(c_u64)]),
     "tg_last_error": (ctypes.c_char_p, []),
     "tg_version": (ctypes.c_char_p, []),
 }
@@ -363,6 +365,15 @@ class Sched:
         buf = (c_i32 * (2 * max(1, n.value)))()
         _ck(_lib.tg_sched_transfers(self.h, o, int(capacity), ctypes.byref(moved), buf, n.value, ctypes.byref(n)))
         return moved.value, [(buf[2 * i], buf[2 * i + 1]) for i in range(n.value)]
+
+    def optimal(self, capacity: int, max_orders: int = 10 ** 7):
+        """Exhaustive optimum over all dependence-respecting operator orders (tg_sched_optimal):
+        (moved, lexicographically smallest optimal order, orders enumerated, optimal orders)."""
+        o = (c_i32 * max(1, self.n_ops))()
+        moved, n, nb = c_u64(), c_u64(), c_u64()
+        _ck(_lib.tg_sched_optimal(self.h, int(capacity), int(max_orders), o, ctypes.byref(moved), ctypes.byref(n),
+                                  ctypes.byref(nb)))
+        return moved.value, list(o)[: self.n_ops], n.value, nb.value
 
 
 def tg_version() -> str:

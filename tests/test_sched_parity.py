@@ -87,3 +87,49 @@ def test_infeasible_and_errors():
     assert e.value.code == tg.TG_E_INFEASIBLE
     with pytest.raises(tg.TGError):
         s.transfers([0, 0, 1, 2, 3, 4, 5, 6], 5)
+
+
+def test_exact_scheduler_fig6():
+    """tg_sched_optimal on the Fig. 3 / Fig. 6 instance: the optimum is Fig. 6's 8 units
+    (PAPER.md:477), the same as the brute-force oracle (264 orders), and the order it returns
+    achieves it under the heuristic transfer rule."""
+    gold = json.load(open(os.path.join(GOLDEN, "schedules.json")))
+    g, ops = P.fig3_graph()
+    s = to_sched(g)
+    cap = gold["fig3"]["capacity"]
+    moved, order, n_orders, n_best = s.optimal(cap)
+    assert moved == gold["fig6"]["optimal_units"]
+    best, n_o, n_b = P.brute_force_min_transfers(g, cap)
+    assert (moved, n_orders, n_best) == (best, n_o, n_b)
+    assert s.transfers(order, cap) == moved
+    # the paper's DFS heuristic does not reach it on this instance (SURVEY F3: 12)
+    assert s.transfers(s.dfs_order(), cap) > moved
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_exact_scheduler_random_dags(seed):
+    """Optimum, number of orders and of optimal orders equal the oracle's brute force; the
+    returned order is the lexicographically smallest optimal one."""
+    rng = random.Random(1000 + seed)
+    g = random_dag(rng, rng.randint(3, 8))
+    s = to_sched(g)
+    need = max(P.Graph.req(g, op) for op in g.ops)
+    for cap in (need, need + 3):
+        moved, order, n_orders, n_best = s.optimal(cap)
+        best, n_o, n_b = P.brute_force_min_transfers(g, cap)
+        assert (moved, n_orders, n_best) == (best, n_o, n_b)
+        first = next(o for o in P.topological_orders(g) if P.simulate_transfers(g, o, cap) == best)
+        assert order == first
+        assert moved <= s.transfers(s.dfs_order(), cap)
+
+
+def test_exact_scheduler_limits():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    g, ops = P.fig3_graph()
+    s = to_sched(g)
+    with pytest.raises(tg.TGError) as e:
+        s.optimal(5, max_orders=100)        # 264 orders
+    assert e.value.code == tg.TG_E_UNSUPPORTED
+    with pytest.raises(tg.TGError) as e:
+        s.optimal(3)                        # max needs 5 units at once
+    assert e.value.code == tg.TG_E_INFEASIBLE
