@@ -288,7 +288,8 @@ constexpr int U3_NA = 4;                // slice buffers
 constexpr int U3_C6K = U3_NMAX / 16;    // C6 K-steps (max)
 constexpr int U3_C6N = 16;              // C6 N: 9 maps padded
 constexpr int U3_C6COL = 64;            // D6 column within a tile region
-constexpr int kEpiWarps = 8;
+constexpr int kEpiGroups = 2;                 // epilogue groups, alternating bands
+constexpr int kEpiWarps = 8 * kEpiGroups;
 constexpr int kThreadsU3 = (kEpiWarps + 2) * 32;
 
 struct U3P {
@@ -323,8 +324,8 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         }
         for (int i = 0; i < 2; ++i) {
             tc::mbar_init(&S.t_full[i], 1);
-            tc::mbar_init(&S.t_empty[i], kEpiWarps);
-            tc::mbar_init(&S.t5_full[i], kEpiWarps);
+            tc::mbar_init(&S.t_empty[i], 8);   // the 8 warps of the group that owns buffer i
+            tc::mbar_init(&S.t5_full[i], 8);
             tc::mbar_init(&S.c6_full[i], 1);
         }
         tc::mbar_fence_init();
@@ -450,13 +451,18 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             issue_c6(c6_next++);
         }
     } else {
-        // ---------------------------------------------------------------- epilogue warps
-        // Thread = one output position of the band (tile t = warp / 4, TMEM lane group warp % 4),
-        // all NP channels in chunks of 32 TMEM columns. Bias-plane values are loaded RING chunks
-        // ahead (across band boundaries), so their L2 latency hides behind the chunk compute.
-        const int t = warp >> 2;  // tile
+        // ---------------------------------------------------------------- epilogue groups
+        // Two groups of 8 warps take alternate bands (group g: bands k = g, g+2, ..., always TMEM
+        // buffer g), so one group's wait for its C6 result overlaps the other group's drain.
+        // Thread = one output position of the band (tile t, TMEM lane group warp % 4), all NP
+        // channels in chunks of 16 TMEM columns. Bias-plane values are loaded RING chunks ahead
+        // (across band boundaries), so their L2 latency hides behind the chunk compute.
+        const int grp = warp >> 3;
+        const int t = (warp >> 2) & 1;  // tile
         const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
         const int m = t * kTileM + 32 * (warp & 3) + lane;
+        constexpr int NC = 2 * NCH;     // 16-column chunks (NP = 16 NC or 16 NC - 16)
+        const int nc = NP / 16;
         struct Pos {
             int img, orow, ocol;  // image, global output row, column (32-bit: per-chunk extents)
             bool ok;
@@ -479,52 +485,64 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             q.pb = a.b5_plane ? a.b5 + ((int64_t)(orow_c - a.b5_row0) * w5 + ocol_c) : a.b5;
             return q;
         };
-        // bias ring: 2 chunk buffers loaded 2 chunks ahead when NCH is even (chunk parity is then
-        // the same in every band), else 1 buffer loaded 1 chunk ahead
-        constexpr int RING = (NCH % 2 == 0) ? 2 : 1;
-        float bv[RING][32];
+        // bias ring of 2 chunk buffers loaded 2 chunks ahead (nc is even or 1 ... the ring index
+        // of chunk c is c % 2 in every band when nc is even; for odd nc the ring degenerates to
+        // one buffer loaded one chunk ahead)
+        float bv[2][16];
         auto load_bias = [&](const float* pb, int c, int r) {
-            const float* p = pb + (size_t)(32 * c) * bcs;
-            // chunks 0..NCH-2 are always full (NP = n5 rounded up to 16 > 32 (NCH-1)); c is a
-            // compile-time constant at every call, so only the last chunk carries predicates
-            if (c < NCH - 1) {
+            const float* p = pb + (size_t)(16 * c) * bcs;
+            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)
 #pragma unroll
-                for (int u = 0; u < 32; ++u, p += bcs) bv[r][u] = __ldg(p);
-            } else {  // padding channels: accumulator 0, C6 weight 0
+                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = __ldg(p);
+            } else {                    // padding channels: accumulator 0, C6 weight 0
 #pragma unroll
-                for (int u = 0; u < 32; ++u, p += bcs) bv[r][u] = (32 * c + u < a.n5) ? __ldg(p) : 0.f;
+                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = (16 * c + u < a.n5) ? __ldg(p) : 0.f;
             }
         };
-        Pos cur = pos_of(blockIdx.x);
-        if (blockIdx.x < nbands) {
-#pragma unroll
-            for (int r = 0; r < RING; ++r) load_bias(cur.pb, r, r);
+        const int ring = (nc % 2 == 0) ? 2 : 1;
+        const int64_t first = blockIdx.x + (int64_t)grp * gridDim.x;
+        Pos cur = pos_of(first);
+        if (first < nbands) {
+            load_bias(cur.pb, 0, 0);
+            if (ring == 2) load_bias(cur.pb, 1, 1);
         }
-        int64_t k = 0;
-        for (int64_t band = blockIdx.x; band < nbands; band += gridDim.x, ++k) {
+        int64_t k = grp;
+        for (int64_t band = first; band < nbands; band += kEpiGroups * gridDim.x, k += kEpiGroups) {
             const int buf = (int)(k & 1);
             const uint32_t region = tmem + lane_base + (uint32_t)(buf * 256 + t * 128);
-            const bool has_next = band + gridDim.x < nbands;
-            const float* nxt_pb = pos_of(has_next ? band + gridDim.x : band).pb;
+            const bool has_next = band + kEpiGroups * gridDim.x < nbands;
+            const float* nxt_pb = pos_of(has_next ? band + kEpiGroups * gridDim.x : band).pb;
             tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
             tc::fence_after_sync();
 #pragma unroll
-            for (int c = 0; c < NCH; ++c) {
-                float v[32];
-                tc::tmem_ld32_async(region + (uint32_t)(32 * c), v);
-                tc::tmem_wait_ld();
+            for (int c = 0; c < NC; ++c) {
+                if (c < nc) {
+                    float v[16];
+                    tc::tmem_ld16_async(region + (uint32_t)(16 * c), v);
+                    tc::tmem_wait_ld();
+                    const int rb = ring == 2 ? (c & 1) : 0;
+                    if (rb == 0) {
 #pragma unroll
-                for (int u = 0; u < 32; ++u) v[u] = tanh_approx(v[u] + bv[c % RING][u]);
-                // refill the consumed buffer with the chunk RING steps ahead
-                if (c + RING < NCH)
-                    load_bias(cur.pb, c + RING, c % RING);
-                else if (has_next)
-                    load_bias(nxt_pb, c + RING - NCH, c % RING);
-                // T5 chunk c -> TMEM columns [16c, 16c+16) (already drained), bf16 pairs
-                uint32_t r[16];
+                        for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[0][u]);
+                    } else {
 #pragma unroll
-                for (int u = 0; u < 16; ++u) r[u] = tc::pack_bf16(v[2 * u], v[2 * u + 1]);
-                tc::tmem_st16(region + (uint32_t)(16 * c), r);
+                        for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[1][u]);
+                    }
+                    // refill the consumed buffer with the chunk `ring` steps ahead
+                    const int cn = c + ring;
+                    if (rb == 0) {
+                        if (cn < nc) load_bias(cur.pb, cn, 0);
+                        else if (has_next) load_bias(nxt_pb, cn - nc, 0);
+                    } else {
+                        if (cn < nc) load_bias(cur.pb, cn, 1);
+                        else if (has_next) load_bias(nxt_pb, cn - nc, 1);
+                    }
+                    // T5 chunk c -> TMEM columns [8c, 8c+8) (already drained), bf16 pairs
+                    uint32_t r[8];
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) r[u] = tc::pack_bf16(v[2 * u], v[2 * u + 1]);
+                    tc::tmem_st8(region + (uint32_t)(8 * c), r);
+                }
             }
             tc::tmem_wait_st();
             tc::fence_before_sync();
@@ -548,7 +566,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                     ob[o * a.out_plane_stride] = d6[o] + b;
                 }
             }
-            if (has_next) cur = pos_of(band + gridDim.x);
+            if (has_next) cur = pos_of(band + kEpiGroups * gridDim.x);
         }
     }
     tc::fence_before_sync();
