@@ -95,3 +95,25 @@ def test_plan_stats_match_table1_counts():
         s = g.plan().stats()
         assert (s["total_temp_bytes"], s["io_lower_bound_bytes"]) == (total * 4, io * 4)
         assert (s["n_ops_fig7"], s["n_ds_fig7"]) == (ops, ds)
+
+
+def test_degenerate_shapes_rejected():
+    """Empty inputs are a shape error at graph construction (no plan, no launch); a CNN image
+    smaller than the receptive field (32 x 32 input -> 1 x 1 output) cannot be
+    built: its C5/C6 planes would be empty."""
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    import synth
+    for shape in [(0, 1, 8, 8), (1, 1, 0, 8), (1, 1, 8, 0)]:
+        g = tg.Graph()
+        with pytest.raises(tg.TGError) as e:
+            g.input(np.zeros(shape, np.float32))
+        assert e.value.code == tg.TG_E_SHAPE
+    prm = synth.cnn_params_np(1, 20, 32, 32)
+    g, y = tg.cnn_graph(np.zeros((1, 1, 32, 32), np.float32), 20, prm)
+    assert g.shape(y) == (1, 9, 1, 1)
+    g = tg.Graph()
+    x = g.input(np.zeros((1, 1, 4, 4), np.float32))
+    k = g.param(np.zeros((8, 1, 5, 5), np.float32))
+    with pytest.raises(tg.TGError) as e:   # VALID 5x5 on a 4x4 image: empty output
+        g.conv2d(x, k, -1, tg.TG_VALID)
+    assert e.value.code == tg.TG_E_SHAPE
