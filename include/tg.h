@@ -72,6 +72,9 @@ typedef int32_t tg_id;
 #define TG_FP32 0         /* all arithmetic in fp32 (FFMA); parity 1e-5 normwise          */
 #define TG_BF16_TC 1      /* CNN C3/C5/C6 on tcgen05 tensor cores, bf16 operands, fp32
                              accumulation; parity 2e-2 normwise                           */
+#define TG_FP32_TC 2      /* fp32-accurate CNN with C5 on tcgen05: every operand split into
+                             two TF32 numbers, three TF32 MMAs per product (3xTF32), fp32
+                             accumulation; parity 1e-5 normwise like TG_FP32               */
 #define TG_FUSED 0        /* offload units = fused templates (edge: 1 unit; CNN: 3)       */
 #define TG_PER_OP 1       /* paper mode: one operator per offload unit, DFS
                              order + latest-time-of-use transfers, one

@@ -380,7 +380,8 @@ tg_status tg_set_device_budget(tg_graph* g, uint64_t bytes) {
 }
 
 tg_status tg_set_precision(tg_graph* g, int32_t prec) {
-    if (!g || (prec != TG_FP32 && prec != TG_BF16_TC)) return fail(TG_E_ARG, "tg_set_precision: bad precision");
+    if (!g || (prec != TG_FP32 && prec != TG_BF16_TC && prec != TG_FP32_TC))
+        return fail(TG_E_ARG, "tg_set_precision: bad precision");
     g->g.precision = prec;
     return TG_OK;
 }

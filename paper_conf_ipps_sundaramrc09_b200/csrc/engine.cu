@@ -62,6 +62,7 @@ struct tg_exec {
     std::vector<tg_trace_rec> trace;  // timeline collected from the profiling events
     int64_t param_uploads = 0;
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
+    std::vector<float> k5t32;          // host copy of the 3xTF32 B operand (TG_FP32_TC)
 };
 
 namespace {
@@ -341,7 +342,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         }
         a.p4_host = g.ds[t.prm[5]].src;
         a.t4 = t4;
-        a.t4_img_stride = 20 * ch.t4.n() * w4;
+        a.t4_img_stride = 20 * ch.t4.n() * w4 * (c.precision == TG_FP32_TC ? 2 : 1);
         a.t4_row0 = ch.t4.a;
         a.t4_rows = ch.t4.n();
         a.w3 = w3;
@@ -350,6 +351,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.bf16_tc = c.precision == TG_BF16_TC;
         a.k3_tc = c.k3tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k3tc_off);
         a.p4_dev = param(5);
+        a.t4_tf32 = c.precision == TG_FP32_TC;
         KernelTimer kt(x, d, 2, ci, cs);
         CK(a.bf16_tc ? launch_cnn_u2_tc(a, cs) : launch_cnn_u2(a, cs));
         kt.done(cs);
@@ -358,7 +360,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
     {
         CnnU3Args a{};
         a.t4 = t4;
-        a.t4_img_stride = 20 * ch.t4.n() * w4;
+        a.t4_img_stride = 20 * ch.t4.n() * w4 * (c.precision == TG_FP32_TC ? 2 : 1);
         a.t4_row0 = ch.t4.a;
         a.t4_rows = ch.t4.n();
         a.w4 = w4;
@@ -395,7 +397,8 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.n_pad = cnn_n5_pad(t.n5);
         a.k6_host = g.ds[t.prm[8]].src;
         KernelTimer kt(x, d, 3, ci, cs);
-        CK(a.bf16_tc ? launch_cnn_u3_tc(a, cs) : launch_cnn_u3(a, cs));
+        CK(a.bf16_tc ? launch_cnn_u3_tc(a, cs)
+                     : c.precision == TG_FP32_TC ? launch_cnn_u3_t32(a, cs) : launch_cnn_u3(a, cs));
         kt.done(cs);
         ++d.launches;
     }
@@ -431,6 +434,14 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
             if (c.param_off[i] == UINT64_MAX) continue;
             const Ds& P = g.ds[c.param_ds[i]];
             CK(cudaMemcpyAsync(d.arena + c.param_off[i], P.src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
+        }
+        if (c.k5tc_off != UINT64_MAX && c.precision == TG_FP32_TC) {
+            // TF32-split B operand of the 3xTF32 C5 (prepared on the host once per plan)
+            if (x->k5t32.empty()) {
+                x->k5t32.resize(cnn_k5_t32_bytes(c.t.n5) / 4);
+                cnn_prepare_k5_t32(g.ds[c.t.prm[6]].src, c.t.n5, x->k5t32.data());
+            }
+            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5t32.data(), x->k5t32.size() * 4, cudaMemcpyHostToDevice, S0));
         }
         if (c.k3tc_off != UINT64_MAX) {
             // bf16 B operands of the tensor-core C3/C5 (prepared on the host once per plan)
@@ -650,6 +661,7 @@ void exec_invalidate_params(tg_plan* p) {
     for (auto& d : p->exec->devs) d.params_resident = false;
     p->exec->k3tc.clear();  // the bf16 tensor-core operands are re-derived from the new values
     p->exec->k5tc.clear();
+    p->exec->k5t32.clear();
 }
 
 }  // namespace tg

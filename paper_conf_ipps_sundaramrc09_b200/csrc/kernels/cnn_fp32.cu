@@ -31,6 +31,12 @@ __device__ __forceinline__ float tanh_f(float x) {
     const float e = __expf(2.f * x);
     return 1.f - __fdividef(2.f, 1.f + e);
 }
+// round to TF32 (10-bit mantissa; nearest, ties away): the "big" part of a 3xTF32 split
+__device__ __forceinline__ float tf32_rn(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
 // MUFU.TANH (one SFU op, relative error ~2^-11): only where the result is rounded to bf16
 // anyway (U1 feeding the tensor-core path), never on the fp32 path.
 __device__ __forceinline__ float tanh_mufu(float x) {
@@ -394,6 +400,7 @@ __global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const
     }
     float* t4 = a.t4 + img * a.t4_img_stride;
     const int64_t oplane = a.t4_rows * a.w4;
+    float tv[20];
 #pragma unroll
     for (int co = 0; co < 20; ++co) {
         float bq[4];
@@ -414,7 +421,26 @@ __global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const
             const float av = (co & 1) ? acc2[co >> 1][p].y : acc2[co >> 1][p].x;
             s = fmaf(w.p4[co][p], tanh_f(av + bq[p]), s);
         }
-        t4[co * oplane + (R4 - a.t4_row0) * a.w4 + C4] = tanh_f(s);
+        tv[co] = tanh_f(s);
+    }
+    const int64_t px = (R4 - a.t4_row0) * a.w4 + C4;
+    if (!a.t4_tf32) {
+#pragma unroll
+        for (int co = 0; co < 20; ++co) t4[co * oplane + px] = tv[co];
+    } else {
+        // TF32-split pixel blocks for the 3xTF32 U3 (cnn_t32.cu): [part][block][rows][w4][4]
+#pragma unroll
+        for (int blk = 0; blk < 5; ++blk) {
+            float big[4], small[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                big[e] = tf32_rn(tv[4 * blk + e]);
+                small[e] = tf32_rn(tv[4 * blk + e] - big[e]);
+            }
+            reinterpret_cast<float4*>(t4)[(0 * 5 + blk) * oplane + px] = make_float4(big[0], big[1], big[2], big[3]);
+            reinterpret_cast<float4*>(t4)[(1 * 5 + blk) * oplane + px] =
+                make_float4(small[0], small[1], small[2], small[3]);
+        }
     }
 }
 

@@ -50,6 +50,7 @@ struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
                             //    as bf16 [3][rows][w4][8] (channel blocks 0-7, 8-15, 16-19+pad)
     const uint16_t* k3_tc;  // bf16 B operand prepared by cnn_prepare_k3_tc (device)
     const float* p4_dev;    // [20][4] (device)
+    int t4_tf32;            // 1 (TG_FP32_TC): T4 written TF32-split [2][5][rows][w4][4] for cnn_t32.cu
 };
 struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + bias -> out
     const float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w4;
@@ -94,6 +95,10 @@ cudaError_t launch_gen_sub(const GenSubArgs& a, cudaStream_t s);
 // tcgen05 (bf16 operands, fp32 accumulation in TMEM) variants of U2 and U3 (cnn_tc.cu)
 cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s);
+// 3xTF32 U3 (fp32-accurate on tcgen05, TG_FP32_TC): B operand prepared on the host
+size_t cnn_k5_t32_bytes(int n5);
+void cnn_prepare_k5_t32(const float* k5, int n5, float* dst);
+cudaError_t launch_cnn_u3_t32(const CnnU3Args& a, cudaStream_t s);
 size_t cnn_k3_tc_bytes();
 void cnn_prepare_k3_tc(const float* k3, uint16_t* dst);
 int cnn_n5_pad(int n5);

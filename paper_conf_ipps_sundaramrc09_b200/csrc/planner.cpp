@@ -248,6 +248,7 @@ struct Sizer {
     const Template& t;
     bool device_io;
     int64_t n5;
+    uint64_t t4_mult;  // 2 for TG_FP32_TC: T4 is kept TF32-split (big and small parts)
     // slot layout for B images x R output rows with the given row ranges
     SlotLayout slot(int64_t B, int64_t R, const Chunk& rg, bool streamed) const {
         SlotLayout s;
@@ -260,7 +261,7 @@ struct Sizer {
         if (!device_io) put(s.in, (uint64_t)B * rg.in.n() * t.W * f);
         if (t.kind == Tmpl::Cnn) {
             put(s.t2, (uint64_t)B * 8 * rg.t2.n() * t.w[2] * f);
-            put(s.t4, (uint64_t)B * 20 * rg.t4.n() * t.w[4] * f);
+            put(s.t4, (uint64_t)B * 20 * rg.t4.n() * t.w[4] * f * t4_mult);
             if (!device_io) put(s.out, (uint64_t)B * 9 * R * t.w[5] * f);
             if (streamed) {
                 put(s.b1, (uint64_t)8 * rg.c1.n() * t.w[1] * f);
@@ -329,9 +330,15 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         all_pb += tc_bytes;
         nonbias_pb += tc_bytes;
     }
+    // 3xTF32 path: the TF32-split B operand of C5, kept with the parameters
+    if (t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC) {
+        tc_bytes = a256(cnn_k5_t32_bytes(t.n5));
+        all_pb += tc_bytes;
+        nonbias_pb += tc_bytes;
+    }
     int32_t depth = p.device_io ? 1 : g.depth;
     p.depth = depth;
-    Sizer sz{t, p.device_io, t.n5};
+    Sizer sz{t, p.device_io, t.n5, (uint64_t)(t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC ? 2 : 1)};
     auto fits = [&](uint64_t pb, uint64_t sb) { return g.budget == 0 || pb + (uint64_t)depth * sb <= g.budget; };
 
     auto chunk_list = [&](bool batch, int64_t B, int64_t R) {
@@ -451,11 +458,14 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         off += a256((uint64_t)g.ds[prm[i]].numel() * f);
     }
     p.k3tc_off = p.k5tc_off = UINT64_MAX;
-    if (tc_bytes) {
+    if (tc_bytes && g.precision == TG_BF16_TC) {
         p.k3tc_off = off;
         off += a256(cnn_k3_tc_bytes());
         p.k5tc_off = off;
         off += a256(cnn_k5_tc_bytes(t.n5));
+    } else if (tc_bytes) {  // TG_FP32_TC
+        p.k5tc_off = off;
+        off += a256(cnn_k5_t32_bytes(t.n5));
     }
     p.chunks = chunk_list(batch, B, R);
     const int64_t C = (int64_t)p.chunks.size();
@@ -523,8 +533,8 @@ std::string plan_json(const PlanCore& p) {
     o << "\"nf\": " << (t.kind == Tmpl::Edge ? t.nf : 0) << ", \"combine\": \"" << (t.kind == Tmpl::Edge ? kComb[t.combine] : "none") << "\", ";
     o << "\"budget\": " << p.budget << ", \"depth\": " << p.depth << ", \"max_chunk_px\": " << p.max_chunk_px << ", ";
     o << "\"device_io\": " << (p.device_io ? "true" : "false") << ", ";
-    o << "\"precision\": \"" << (t.kind == Tmpl::Cnn && p.precision == TG_BF16_TC ? "bf16_tc" : "fp32") << "\", ";
-    o << "\"precision\": \"" << (p.precision == TG_BF16_TC ? "bf16_tc" : "fp32") << "\", ";
+    o << "\"precision\": \"" << (t.kind != Tmpl::Cnn ? "fp32" : p.precision == TG_BF16_TC ? "bf16_tc" : p.precision == TG_FP32_TC ? "fp32_tc" : "fp32") << "\", ";
+    o << "\"precision\": \"" << (p.precision == TG_BF16_TC ? "bf16_tc" : p.precision == TG_FP32_TC ? "fp32_tc" : "fp32") << "\", ";
     o << "\"bias\": \"" << p.bias << "\", \"split\": \"" << p.split << "\", ";
     o << "\"B\": " << p.B << ", \"R\": " << p.R << ", ";
     o << "\"param_bytes\": " << p.param_bytes << ", \"slot_bytes\": " << p.slot_bytes

@@ -33,7 +33,7 @@ TG_VALID, TG_SAME = 0, 1
 TG_ADD, TG_NEG, TG_AFFINE, TG_ABS = 0, 1, 2, 3
 TG_MAX, TG_SUM, TG_MAXABS = 0, 1, 2
 TG_BIAS_PLANE, TG_BIAS_SCALAR = 0, 1
-TG_FP32, TG_BF16_TC = 0, 1
+TG_FP32, TG_BF16_TC, TG_FP32_TC = 0, 1, 2
 TG_FUSED, TG_PER_OP, TG_BASELINE = 0, 1, 2
 
 _STATUS = {v: k for k, v in dict(TG_E_ARG=-1, TG_E_SHAPE=-2, TG_E_INFEASIBLE=-3, TG_E_CUDA=-4,

