@@ -48,6 +48,7 @@ def lib():
         L.orc_tanh.argtypes = [f32p, f32p, i64]
         L.orc_max_fold.argtypes = [ctypes.POINTER(f32p), ctypes.c_int, f32p, i64]
         L.orc_subsample.argtypes = [f32p, i64, i64, f32p, ctypes.c_int, f32p]
+        L.orc_matmul.argtypes = [f32p, f32p, i64, i64, i64, f32p]
         L.orc_edge.argtypes = [f32p, i64, i64, f32p, f32p, ctypes.c_int, f32p, f32p, f32p]
         L.orc_edge.restype = ctypes.c_int
         L.orc_cnn.argtypes = [f32p, i64, i64, i64, ctypes.c_int, ctypes.POINTER(f32p),
@@ -130,6 +131,17 @@ def subsample(x, P) -> np.ndarray:
     y = np.empty(((H - s) // s + 1, (W - s) // s + 1), dtype=np.float32)
     lib().orc_subsample(_p(x), H, W, _p(P), s, _p(y))
     return y
+
+
+def matmul(A, B) -> np.ndarray:
+    """C = A B with fp64 accumulation (oracle.c orc_matmul)."""
+    A, B = _c(A), _c(B)
+    M, K = A.shape
+    K2, N = B.shape
+    assert K == K2
+    C = np.empty((M, N), dtype=np.float32)
+    lib().orc_matmul(_p(A), _p(B), M, K, N, _p(C))
+    return C
 
 
 def edge(img, K1, K2, return_parts: bool = False):

@@ -149,6 +149,22 @@ void orc_subsample(const float* x, int64_t H, int64_t W, const float* P, int s, 
     }
 }
 
+/* matrix-matrix multiply C = A B ("a large matrix-matrix multiply that does not
+ * fit in the GPU memory can be split by breaking up one of the input matrices and the output
+ * matrix"; the operator itself is the textbook product):
+ *   C[i][j] = sum_{l<K} A[i][l] * B[l][j],  A is M x K, B is K x N, C is M x N,
+ * accumulated in fp64 over l = 0..K-1 and rounded once to fp32. */
+void orc_matmul(const float* A, const float* B, int64_t M, int64_t K, int64_t N, float* C) {
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < M; ++i) {
+        for (int64_t j = 0; j < N; ++j) {
+            double acc = 0.0;
+            for (int64_t l = 0; l < K; ++l) acc += (double)A[i * K + l] * (double)B[l * N + j];
+            C[i * N + j] = (float)acc;
+        }
+    }
+}
+
 /* Edge-detection template, 4 orientations ("16x16 sized edge filter at four
  * different orientations (2 convolutions and 2 remaps) and combined the results using a
  * Max operation"; graph of Fig. 3 / SURVEY F1):

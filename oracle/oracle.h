@@ -16,6 +16,7 @@ void orc_neg(const float* a, float* y, int64_t n);
 void orc_tanh(const float* a, float* y, int64_t n);
 void orc_max_fold(const float* const* xs, int nx, float* y, int64_t n);
 void orc_subsample(const float* x, int64_t H, int64_t W, const float* P, int s, float* y);
+void orc_matmul(const float* A, const float* B, int64_t M, int64_t K, int64_t N, float* C);
 int orc_edge(const float* img, int64_t H, int64_t W, const float* K1, const float* K2, int ks,
              float* E, float* E1_out, float* E2_out);
 int orc_cnn(const float* img, int64_t n, int64_t H, int64_t W, int n5, const float* const* prm,

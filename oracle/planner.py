@@ -436,6 +436,200 @@ def fig3_graph() -> tuple[Graph, dict[str, int]]:
     return g, ops
 
 
+# ============================================================================ operator splitting
+# The paper's splitting algorithm (steps 1-3) on an operator graph with
+# static shapes, in the reading DESIGN.md R18:
+#   * the split axis is the output rows (R12); an operator's inputs are "row-linked" when an
+#     output row band needs only a row band of them (convolution image, bias plane,
+#     subsample input, elementwise inputs, the first matrix of a matmul -- PAPER.md:369
+#     "breaking up one of the input matrices and the output matrix") and "whole" otherwise
+#     (convolution kernels, "should not be split"; subsample weights; the
+#     second matrix of a matmul; scalar biases);
+#   * "When an operator is split, other operators that produce/receive data from the split
+#     operator also need to be modified": the operators joined by row-linked
+#     data form a component that is split into the same number k of pieces;
+#   * the pieces of every data structure are found "by traversing the split graph from the
+#     leaves to the root and inferring the sizes and offsets from the kernel and output
+#     sizes": the component's sinks are cut into k equal row bands
+#     [i*h//k, (i+1)*h//k), and each input band is the band its consumers' piece i needs
+#     (the hull over consumers), halos included -- so input pieces overlap (the paper's
+#     "two 100x52 input matrices (not 100x50)");
+#   * k starts at max ceil(req(op) / M) over the component's operators (step 2) and grows by
+#     one until every piece operator fits (step 3); a component whose operators all fit
+#     stays whole (k = 1, every data structure one piece).
+
+
+@dataclass
+class SNode:
+    """A graph operator with its row semantics (for splitting only)."""
+    kind: str                  # "conv_valid" | "conv_same" | "sub" | "elem" | "matmul"
+    ins: list[int]             # graph DS ids in the library's order (conv: x, k[, bias])
+    out: int
+    kh: int = 1                # convolution kernel rows
+    s: int = 1                 # subsample window = stride
+    bias_plane: bool = False   # conv: the third input is a bias plane (row-linked)
+
+
+def in_rows(node: SNode, slot: int, a: int, b: int, h_in: int):
+    """Rows of input `slot` that output rows [a, b) of `node` need, or None if the input is
+    read whole. (the 5x5 VALID conv's output rows [0, 48) need input rows
+    [0, 52).)"""
+    if node.kind == "conv_valid":
+        if slot == 0:
+            return (a, b + node.kh - 1)
+        return (a, b) if slot == 2 and node.bias_plane else None
+    if node.kind == "conv_same":
+        if slot == 0:
+            return (max(0, a - (node.kh - 1) // 2), min(h_in, b + node.kh // 2))
+        return (a, b) if slot == 2 and node.bias_plane else None
+    if node.kind == "sub":
+        return (node.s * a, node.s * b) if slot == 0 else None
+    if node.kind == "matmul":
+        return (a, b) if slot == 0 else None
+    return (a, b)              # elementwise / tanh / max: row for row
+
+
+def split_plan(shapes, kinds, nodes: list[SNode], output: int, capacity: int, force_k: int | None = None):
+    """Split the operators feeding `output` (reading R18) and schedule the
+    pieces with the DFS order and the next-use transfer policy.
+    shapes[d] = (n, c, h, w), kinds[d] in {"input", "param", "temp", "output"}; sizes are
+    bytes of fp32. Returns a dict with the pieces, piece operators, k per node, order and
+    trace; raises ValueError when some operator cannot be made to fit. force_k (tests only):
+    cut every component that needs splitting into exactly force_k pieces, fitting or not."""
+    def nbytes(d, rows):
+        return 4 * shapes[d][0] * shapes[d][1] * rows * shapes[d][3]
+
+    # step 0: the operators the output depends on (graph order is topological)
+    need_ds = {output}
+    live = []
+    for i in reversed(range(len(nodes))):
+        if nodes[i].out in need_ds:
+            live.append(i)
+            need_ds.update(nodes[i].ins)
+    live.reverse()
+
+    def linked(nd, slot):
+        return in_rows(nd, slot, 0, 1, shapes[nd.ins[slot]][2]) is not None
+
+    # components of row-linked data (union-find over DS ids, smallest id is the root)
+    parent = list(range(len(shapes)))
+
+    def find(x):
+        while parent[x] != x:
+            x = parent[x]
+        return x
+
+    for i in live:
+        nd = nodes[i]
+        for slot, d in enumerate(nd.ins):
+            if linked(nd, slot):
+                ra, rb = find(d), find(nd.out)
+                if ra != rb:
+                    parent[max(ra, rb)] = min(ra, rb)
+    comps = []                     # in order of their first operator
+    comp_nodes = {}
+    for i in live:
+        c = find(nodes[i].out)
+        if c not in comp_nodes:
+            comps.append(c)
+            comp_nodes[c] = []
+        comp_nodes[c].append(i)
+
+    def sinks(c):
+        consumed = {d for i in comp_nodes[c] for slot, d in enumerate(nodes[i].ins) if linked(nodes[i], slot)}
+        outs = [nodes[i].out for i in comp_nodes[c]]
+        return [d for d in dict.fromkeys(outs) if d not in consumed or d == output]
+
+    def bands_for(c, k):
+        """Piece i of every DS of component c: sinks cut into k equal row bands, every other
+        DS the hull of what its consumers' piece i needs (leaves to root)."""
+        band = {d: [(i * shapes[d][2] // k, (i + 1) * shapes[d][2] // k) for i in range(k)] for d in sinks(c)}
+        for i in reversed(comp_nodes[c]):
+            nd = nodes[i]
+            for slot, d in enumerate(nd.ins):
+                if not linked(nd, slot):
+                    continue
+                h = shapes[d][2]
+                want = []
+                for a, b in band[nd.out]:
+                    ra, rb = in_rows(nd, slot, a, b, h)
+                    want.append((max(0, ra), min(h, rb)))
+                if d in band:
+                    band[d] = [(min(p[0], q[0]), max(p[1], q[1])) for p, q in zip(band[d], want)]
+                else:
+                    band[d] = want
+        return band
+
+    k_of = {}
+    band_of = {}
+
+    def bands(d, cur=None, cur_k=1, cur_band=None):
+        c = find(d)
+        if c == cur and cur_k > 1:
+            return cur_band[d]
+        if k_of.get(c, 1) > 1:
+            return band_of[c][d]
+        return [(0, shapes[d][2])]
+
+    def op_pieces(nd, p, k, c, band):
+        """DS pieces (d, r0, r1) that piece p of operator nd reads and writes."""
+        keys = []
+        for slot, d in enumerate(nd.ins):
+            if linked(nd, slot) and k > 1:
+                keys.append((d, *band[d][p]))
+            else:
+                keys.extend((d, *r) for r in bands(d, c, k, band))
+        keys.append((nd.out, *(band[nd.out][p] if k > 1 else (0, shapes[nd.out][2]))))
+        return keys
+
+    def req(keys):
+        return sum(nbytes(d, b - a) for d, a, b in dict.fromkeys(keys))
+
+    for c in comps:
+        cn = comp_nodes[c]
+        k0 = max(-(-req(op_pieces(nodes[i], 0, 1, c, None)) // capacity) for i in cn)   # step 1-2
+        if k0 <= 1:
+            k_of[c] = 1
+            continue
+        kmax = min(shapes[d][2] for d in sinks(c))
+        k = k0 if force_k is None else force_k
+        while force_k is None:                                                             # step 3
+            if k > kmax:
+                raise ValueError("infeasible: an operator does not fit even split into single rows")
+            band = bands_for(c, k)
+            if all(req(op_pieces(nodes[i], p, k, c, band)) <= capacity for i in cn for p in range(k)):
+                break
+            k += 1
+        k_of[c] = k
+        band_of[c] = bands_for(c, k)
+    # the split graph for the scheduler: DS pieces by first appearance, piece operators in
+    # (node, piece) order
+    g = Graph()
+    pieces = []
+    pid = {}
+    op_piece = []
+    for i in live:
+        nd = nodes[i]
+        c = find(nd.out)
+        k = k_of[c]
+        for p in range(k):
+            ids = []
+            for d, a, b in op_pieces(nd, p, k, c, band_of.get(c)):
+                if (d, a, b) not in pid:
+                    pid[(d, a, b)] = g.add_ds(f"d{d}[{a}:{b}]", nbytes(d, b - a), kinds[d])
+                    pieces.append([d, a, b])
+                ids.append(pid[(d, a, b)])
+            g.add_op(f"n{i}.{p}", ids[:-1], ids[-1:])
+            op_piece.append([i, p])
+    if force_k is not None:
+        return {"graph": g, "pieces": pieces, "op_piece": op_piece}
+    order = dfs_order(g)
+    tr = []
+    moved = simulate_transfers(g, order, capacity, tr)
+    return {"graph": g, "pieces": pieces, "op_piece": op_piece, "order": order, "trace": tr,
+            "moved": moved, "k": {i: k_of[find(nodes[i].out)] for i in live}}
+
+
 # ============================================================================ chunk rule
 DEPTH = 3                 # pipeline slots (H2D / compute / D2H in flight)
 MAX_CHUNK_PX = 1 << 25    # input pixels per chunk when memory does not bind (DESIGN.md §4)
