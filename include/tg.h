@@ -76,9 +76,10 @@ typedef int32_t tg_id;
                              two TF32 numbers, three TF32 MMAs per product (3xTF32), fp32
                              accumulation; parity 1e-5 normwise like TG_FP32               */
 #define TG_FUSED 0        /* offload units = fused templates (edge: 1 unit; CNN: 3)       */
-#define TG_PER_OP 1       /* paper mode: one operator per offload unit, DFS
-                             order + latest-time-of-use transfers, one
-                             stream, generic per-operator kernels, no splitting           */
+#define TG_PER_OP 1       /* paper mode: operators that exceed the budget are split into row
+                             pieces (R19), one operator piece
+                             per offload unit, DFS order + latest-time-of-use
+                             transfers, one stream, generic kernels    */
 #define TG_BASELINE 2     /* paper baseline: per operator copy inputs in,
                              run, copy outputs out, keep nothing                          */
 
@@ -134,6 +135,14 @@ tg_status tg_find_edges(tg_graph* g, tg_id img, tg_id kernel, int32_t num_orient
 tg_status tg_cnn(tg_graph* g, tg_id img, int32_t n5, const tg_id params[10], int32_t bias_mode,
                  tg_id* out);
 
+/* Matrix-matrix multiply C = A B: a [1][1][m][k], b [1][1][k][n] (any DS
+ * kinds), result [1][1][m][n]. When it does not fit, TG_PER_OP splits it by rows of A and C,
+ * B read whole ("breaking up one of the input matrices and the output matrix", DESIGN.md
+ * R20). fp32 with fp32 accumulation in order l = 0..k-1. TG_E_SHAPE if the inner dimensions
+ * differ or an operand is not a matrix. Executed by TG_PER_OP / TG_BASELINE plans (TG_FUSED
+ * plans only the edge and CNN templates: TG_E_UNSUPPORTED). */
+tg_status tg_matmul(tg_graph* g, tg_id a, tg_id b, tg_id* y);
+
 /* ------------------------------------------------------------------ target parameters */
 /* Devices the plan runs on (one host thread per device; chunks are split contiguously).
  * Default: the current CUDA device. */
@@ -163,9 +172,12 @@ tg_status tg_set_runtime(tg_graph* g, const tg_runtime* rt);
 /* ------------------------------------------------------------------ plan / execute */
 /* Build the execution plan: recognise the template's offload units, split into chunks
  * (PAPER.md:359-371), order them and size every transfer. Pure host
- * code: works without a GPU. mode = TG_FUSED (edge/CNN templates, split into chunks),
- * TG_PER_OP or TG_BASELINE (any graph, host I/O, one device, operators run whole:
- * TG_E_INFEASIBLE if one does not fit). The graph must outlive the plan. */
+ * code: works without a GPU. mode = TG_FUSED (edge/CNN templates, split into chunks);
+ * TG_PER_OP (any graph, host I/O, one device: operators that do not fit within 7/8 of the
+ * budget are split into row pieces, PAPER.md:359-367 / DESIGN.md R19 -- TG_E_INFEASIBLE if
+ * even single-row pieces do not fit, TG_E_UNSUPPORTED if a whole-read operand would span
+ * more than 8 pieces); TG_BASELINE (any graph, operators run whole: TG_E_INFEASIBLE if one
+ * does not fit). The graph must outlive the plan. */
 tg_status tg_plan_create(const tg_graph* g, int32_t mode, tg_plan** plan);
 
 typedef struct {

@@ -302,7 +302,7 @@ def dfs_order(g: Graph) -> list[int]:
     return done
 
 
-def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None) -> int:
+def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None, frees: bool = False) -> int:
     """Transfer volume of an operator order under the 'latest time of use' policy
     (read as next use -- DESIGN.md R10):
       * the inputs and outputs of the running operator must be resident; a missing input is
@@ -313,7 +313,8 @@ def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None) ->
       * data is deleted eagerly once no later operator uses it (template outputs are
         instead copied to the CPU when evicted or at the end);
       * initially everything is on the CPU, nothing on the GPU (PB constraints (11),(12)).
-    Returns the number of floats moved (H2D + D2H)."""
+    Returns the number of floats moved (H2D + D2H). With frees=True the trace also records
+    ("free", name) whenever a DS leaves the GPU (evicted, or deleted eagerly in id order)."""
     uses = {j: [] for j in range(len(g.ds))}
     for t, i in enumerate(order):
         for j in set(g.ops[i].ins) | set(g.ops[i].outs):
@@ -352,6 +353,8 @@ def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None) ->
                     if trace is not None:
                         trace.append(("d2h", g.ds[v].name))
                 del on_gpu[v]
+                if trace is not None and frees:
+                    trace.append(("free", g.ds[v].name))
             if j in op.ins:
                 assert j in host_valid, g.ds[j].name
                 moved += sz
@@ -364,9 +367,11 @@ def simulate_transfers(g: Graph, order: list[int], capacity: int, trace=None) ->
         if trace is not None:
             trace.append(("run", op.name))
         # eager deletion of data no later operator needs (outputs stay until copied back)
-        for j in list(on_gpu):
+        for j in sorted(on_gpu):
             if next_use(j, t) == math.inf and j not in outputs:
                 del on_gpu[j]
+                if trace is not None and frees:
+                    trace.append(("free", g.ds[j].name))
     for j in sorted(on_gpu):          # outputs still on the GPU go to the host, in id order
         if j in outputs and on_gpu[j]:
             moved += g.ds[j].size
@@ -438,7 +443,7 @@ def fig3_graph() -> tuple[Graph, dict[str, int]]:
 
 # ============================================================================ operator splitting
 # The paper's splitting algorithm (steps 1-3) on an operator graph with
-# static shapes, in the reading DESIGN.md R18:
+# static shapes, in the reading DESIGN.md R19:
 #   * the split axis is the output rows (R12); an operator's inputs are "row-linked" when an
 #     output row band needs only a row band of them (convolution image, bias plane,
 #     subsample input, elementwise inputs, the first matrix of a matmul -- PAPER.md:369
@@ -490,7 +495,7 @@ def in_rows(node: SNode, slot: int, a: int, b: int, h_in: int):
 
 
 def split_plan(shapes, kinds, nodes: list[SNode], output: int, capacity: int, force_k: int | None = None):
-    """Split the operators feeding `output` (reading R18) and schedule the
+    """Split the operators feeding `output` (reading R19) and schedule the
     pieces with the DFS order and the next-use transfer policy.
     shapes[d] = (n, c, h, w), kinds[d] in {"input", "param", "temp", "output"}; sizes are
     bytes of fp32. Returns a dict with the pieces, piece operators, k per node, order and
@@ -628,6 +633,82 @@ def split_plan(shapes, kinds, nodes: list[SNode], output: int, capacity: int, fo
     moved = simulate_transfers(g, order, capacity, tr)
     return {"graph": g, "pieces": pieces, "op_piece": op_piece, "order": order, "trace": tr,
             "moved": moved, "k": {i: k_of[find(nodes[i].out)] for i in live}}
+
+
+def arena_layout(g: Graph, trace, arena: int):
+    """Static arena layout of a transfer trace (with frees). Every residency interval of a DS
+    piece -- from its copy-in or production to its free (or the end) -- is a buffer of its
+    size rounded up to 256 B. Buffers are placed largest first (ties: earlier start, then lower
+    DS id), each at the lowest offset where it overlaps no already placed buffer that is live
+    at the same time. Returns the offset each trace step touches, or None when a buffer would
+    end beyond the arena (fragmentation)."""
+    a256 = lambda v: (max(v, 1) + 255) // 256 * 256
+    names = {d.name: i for i, d in enumerate(g.ds)}
+    ops = {o.name: o for o in g.ops}
+    opened = {}
+    iv = []                       # (start step, end step, DS)
+    for t, (kind, nm) in enumerate(trace):
+        if kind in ("h2d", "run"):
+            j = names[nm] if kind == "h2d" else ops[nm].outs[0]
+            if j not in opened:
+                opened[j] = t
+        elif kind == "free":
+            j = names[nm]
+            if j in opened:
+                iv.append((opened.pop(j), t, j))
+    for j, t0 in opened.items():
+        iv.append((t0, len(trace), j))
+    off = {}
+    placed = []
+    for t0, t1, j in sorted(iv, key=lambda v: (-a256(g.ds[v[2]].size), v[0], v[2])):
+        sz = a256(g.ds[j].size)
+        cur = 0
+        for lo, hi in sorted((o, o + s) for a, b, o, s in placed if a < t1 and t0 < b):
+            if lo - cur >= sz:
+                break
+            cur = max(cur, hi)
+        if cur + sz > arena:
+            return None
+        placed.append((t0, t1, cur, sz))
+        off[(j, t0)] = cur
+    offs = []
+    start = {}
+    for t, (kind, nm) in enumerate(trace):
+        j = ops[nm].outs[0] if kind == "run" else names[nm]
+        if kind in ("h2d", "run") and j not in start:
+            start[j] = t
+        offs.append(off[(j, start[j])])
+        if kind == "free":
+            del start[j]
+    return offs
+
+
+def per_op_plan(shapes, kinds, nodes: list[SNode], output: int, budget: int):
+    """TG_PER_OP end to end: split (R19) and schedule within the scheduling capacity M, then
+    lay the arena out (arena_layout). M starts at the budget less 1/8 ("set to a value less than
+    the actual amount of GPU memory present in the system to account for fragmentation",
+    PAPER.md:409) and, while the layout does not fit the arena, drops by another 1/16 of the
+    budget. Uncapped (budget 0): M = every DS once, no layout constraint."""
+    total = 4 * sum(math.prod(sh) for d, sh in enumerate(shapes)
+                    if d == output or any(d in nd.ins or d == nd.out for nd in nodes))
+    if budget == 0:
+        r = split_plan(shapes, kinds, nodes, output, max(total, 1))
+        r["capacity"] = max(total, 1)
+        return r
+    cap = budget - budget // 8
+    arena = budget // 256 * 256
+    while cap > 0:
+        r = split_plan(shapes, kinds, nodes, output, cap)
+        tr = []
+        simulate_transfers(r["graph"], r["order"], cap, tr, frees=True)
+        offs = arena_layout(r["graph"], tr, arena)
+        if offs is not None:
+            r["capacity"] = cap
+            r["trace_full"] = tr
+            r["trace_off"] = offs
+            return r
+        cap -= budget // 16
+    raise ValueError("infeasible: no capacity gives a layout that fits the arena")
 
 
 # ============================================================================ chunk rule

@@ -210,6 +210,25 @@ tg_status tg_subsample(tg_graph* g, tg_id x, tg_id p, int32_t s, tg_id* y) {
     TG_GUARD_END
 }
 
+tg_status tg_matmul(tg_graph* g, tg_id a, tg_id b, tg_id* y) {
+    if (!g || !y) return fail(TG_E_ARG, "tg_matmul: NULL argument");
+    Graph& G = g->g;
+    if (!valid_id(G, a) || !valid_id(G, b)) return fail(TG_E_ARG, "tg_matmul: unknown DS id");
+    const Ds& A = G.ds[a];
+    const Ds& B = G.ds[b];
+    if (A.d[0] * A.d[1] != 1 || B.d[0] * B.d[1] != 1)
+        return fail(TG_E_SHAPE, "tg_matmul: operands must be matrices [1][1][m][k] and [1][1][k][n]");
+    if (A.d[3] != B.d[2]) return fail(TG_E_SHAPE, "tg_matmul: inner dimensions differ");
+    TG_GUARD_BEGIN
+    Node nd;
+    nd.op = OpKind::Matmul;
+    nd.ins = {a, b};
+    int64_t d[4] = {1, 1, A.d[2], B.d[3]};
+    *y = add_node(G, nd, d);
+    return TG_OK;
+    TG_GUARD_END
+}
+
 static tg_status output_common(tg_graph* g, tg_id y, float* dst, Loc loc) {
     if (!g || !dst) return fail(TG_E_ARG, "tg_output: NULL argument");
     Graph& G = g->g;

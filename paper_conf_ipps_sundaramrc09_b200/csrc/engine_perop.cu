@@ -1,11 +1,11 @@
 // engine_perop.cu -- executor of the paper-faithful plans (TG_PER_OP, TG_BASELINE).
 //
 // Replays the plan's schedule (planner_perop.cpp) literally on one stream, the way the paper
-// ran its plans (no copy/compute overlap): H2D copies of whole data
-// structures, one generic kernel per operator (the "operator library", Fig. 4), D2H copies
-// of evicted or final data, and eager frees. Device memory is one arena of plan.arena_bytes
-// carved with a first-fit allocator; data structures evicted to the host live in staging
-// buffers owned by the plan.
+// ran its plans (no copy/compute overlap): H2D copies of data-structure pieces
+// (row bands of the host arrays), one generic kernel per operator piece (the
+// "operator library", Fig. 4), D2H copies of evicted or final pieces, and eager frees. Device
+// memory is one arena of plan.arena_bytes laid out statically by the planner (first fit over
+// the trace); pieces evicted to the host live in staging buffers owned by the plan.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -24,7 +24,6 @@ struct tg_perop_exec {
     char* arena = nullptr;
     bool own_arena = false;
     std::vector<std::vector<float>> staging;  // per sched DS: host copy of evicted temporaries
-    std::map<uint64_t, uint64_t> free_list;   // offset -> size
     std::vector<int64_t> off;                 // per sched DS: arena offset or -1
     bool profiling = false;
     bool ready = false;
@@ -46,58 +45,54 @@ namespace {
         }                                                                                          \
     } while (0)
 
-uint64_t a256(uint64_t x) { return (x + 255) / 256 * 256; }
-
-bool arena_alloc(tg_perop_exec& x, uint64_t bytes, uint64_t& out) {
-    bytes = a256(std::max<uint64_t>(bytes, 1));
-    for (auto it = x.free_list.begin(); it != x.free_list.end(); ++it)
-        if (it->second >= bytes) {
-            out = it->first;
-            const uint64_t rest = it->second - bytes;
-            const uint64_t noff = it->first + bytes;
-            x.free_list.erase(it);
-            if (rest) x.free_list[noff] = rest;
-            return true;
-        }
-    return false;
-}
-
-void arena_free(tg_perop_exec& x, uint64_t off, uint64_t bytes) {
-    bytes = a256(std::max<uint64_t>(bytes, 1));
-    auto it = x.free_list.emplace(off, bytes).first;
-    auto nx = std::next(it);  // coalesce with the next and previous blocks
-    if (nx != x.free_list.end() && it->first + it->second == nx->first) {
-        it->second += nx->second;
-        x.free_list.erase(nx);
+// view of the resident pieces `ids` (sched DS ids, all of one graph DS) for a kernel
+bool make_view(const PlanCore& c, const tg_perop_exec& x, const std::vector<int32_t>& ids, GenView& v) {
+    v = GenView{};
+    for (int32_t id : ids) {
+        if (x.off[id] < 0 || v.nseg >= kGenMaxSeg) return false;
+        v.seg[v.nseg++] = GenSeg{(const float*)(x.arena + x.off[id]), c.po_r0[id], c.po_r1[id]};
     }
-    if (it != x.free_list.begin()) {
-        auto pv = std::prev(it);
-        if (pv->first + pv->second == it->first) {
-            pv->second += it->second;
-            x.free_list.erase(it);
-        }
-    }
+    return true;
 }
 
 tg_status launch_node(const Graph& g, const PlanCore& c, tg_perop_exec& x, int op) {
     const Node& nd = g.nodes[c.po_ops[op]];
-    auto dptr = [&](int gid) -> float* {
-        for (size_t k = 0; k < c.po_ds.size(); ++k)
-            if (c.po_ds[k] == gid) return x.off[k] < 0 ? nullptr : (float*)(x.arena + x.off[k]);
-        return nullptr;
-    };
+    // the operator's input slots in order (conv x, k[, bias]); each slot's pieces are the
+    // consecutive entries of po_ins that belong to its DS
+    std::vector<int> slots = nd.ins;
+    if (nd.op == OpKind::Conv && nd.bias >= 0) slots.push_back(nd.bias);
+    std::vector<std::vector<int32_t>> pieces(slots.size());
+    {
+        const std::vector<int32_t>& ins = c.po_ins[op];
+        size_t i = 0;
+        for (size_t s = 0; s < slots.size(); ++s) {
+            while (i < ins.size() && c.po_ds[ins[i]] == slots[s]) pieces[s].push_back(ins[i++]);
+            if (pieces[s].empty()) {  // repeated operand (e.g. add(x, x)): same pieces again
+                for (size_t t = 0; t < s; ++t)
+                    if (slots[t] == slots[s]) pieces[s] = pieces[t];
+            }
+        }
+    }
+    GenView v[kGenMaxInputs];
+    for (size_t s = 0; s < slots.size() && s < (size_t)kGenMaxInputs; ++s)
+        if (!make_view(c, x, pieces[s], v[s])) return fail(TG_E_STATE, "per-op executor: input not resident");
+    const int32_t yo = c.po_outs[op][0];
+    if (x.off[yo] < 0) return fail(TG_E_STATE, "per-op executor: output not resident");
+    float* y = (float*)(x.arena + x.off[yo]);
+    const int64_t r0 = c.po_r0[yo], r1 = c.po_r1[yo];
     const Ds& Y = g.ds[nd.out];
-    float* y = dptr(nd.out);
-    if (!y) return fail(TG_E_STATE, "per-op executor: output not resident");
     cudaError_t e = cudaSuccess;
     switch (nd.op) {
         case OpKind::Conv: {
             const Ds& X = g.ds[nd.ins[0]];
             const Ds& K = g.ds[nd.ins[1]];
             GenConvArgs a{};
-            a.x = dptr(nd.ins[0]);
-            a.k = dptr(nd.ins[1]);
+            a.x = v[0];
+            if (v[1].nseg != 1 || v[1].seg[0].r0 != 0) return fail(TG_E_STATE, "per-op executor: split kernel");
+            a.k = v[1].seg[0].p;
             a.y = y;
+            a.r0 = r0;
+            a.r1 = r1;
             a.n = X.d[0];
             a.ci = X.d[1];
             a.h = X.d[2];
@@ -105,45 +100,56 @@ tg_status launch_node(const Graph& g, const PlanCore& c, tg_perop_exec& x, int o
             a.co = K.d[0];
             a.kh = K.d[2];
             a.kw = K.d[3];
-            a.ho = Y.d[2];
             a.wo = Y.d[3];
             a.pt = nd.pad == TG_SAME ? (int)(K.d[2] - 1) / 2 : 0;
             a.pl = nd.pad == TG_SAME ? (int)(K.d[3] - 1) / 2 : 0;
             a.bias_kind = 0;
             if (nd.bias >= 0) {
-                a.bias = dptr(nd.bias);
+                a.bias = v[2];
                 a.bias_kind = g.ds[nd.bias].numel() == K.d[0] ? 1 : 2;
             }
-            if (!a.x || !a.k || (nd.bias >= 0 && !a.bias)) return fail(TG_E_STATE, "per-op executor: input not resident");
             e = launch_gen_conv(a, x.stream);
             break;
         }
         case OpKind::Sub: {
             const Ds& X = g.ds[nd.ins[0]];
             GenSubArgs a{};
-            a.x = dptr(nd.ins[0]);
-            a.p = dptr(nd.ins[1]);
+            a.x = v[0];
+            if (v[1].nseg != 1) return fail(TG_E_STATE, "per-op executor: split subsample kernel");
+            a.p = v[1].seg[0].p;
             a.y = y;
+            a.r0 = r0;
+            a.r1 = r1;
             a.n = X.d[0];
             a.c = X.d[1];
             a.h = X.d[2];
             a.w = X.d[3];
-            a.ho = Y.d[2];
             a.wo = Y.d[3];
             a.s = nd.s;
-            if (!a.x || !a.p) return fail(TG_E_STATE, "per-op executor: input not resident");
             e = launch_gen_sub(a, x.stream);
+            break;
+        }
+        case OpKind::Matmul: {
+            GenMatmulArgs a{};
+            a.a = v[0];
+            a.b = v[1];
+            a.c = y;
+            a.r0 = r0;
+            a.r1 = r1;
+            a.k = g.ds[nd.ins[0]].d[3];
+            a.n = Y.d[3];
+            e = launch_gen_matmul(a, x.stream);
             break;
         }
         default: {
             GenElemArgs a{};
             a.nx = (int)nd.ins.size();
-            for (int i = 0; i < a.nx; ++i) {
-                a.xs[i] = dptr(nd.ins[i]);
-                if (!a.xs[i]) return fail(TG_E_STATE, "per-op executor: input not resident");
-            }
+            for (int i = 0; i < a.nx; ++i) a.xs[i] = v[i];
             a.y = y;
-            a.numel = Y.numel();
+            a.r0 = r0;
+            a.r1 = r1;
+            a.planes = Y.d[0] * Y.d[1];
+            a.w = Y.d[3];
             a.op = nd.op == OpKind::Tanh ? 4 : nd.op == OpKind::Max ? 5 : nd.elem;
             a.a = nd.a;
             a.b = nd.b;
@@ -152,6 +158,17 @@ tg_status launch_node(const Graph& g, const PlanCore& c, tg_perop_exec& x, int o
     }
     if (e != cudaSuccess) return fail(TG_E_CUDA, std::string("generic kernel launch failed: ") + cudaGetErrorString(e));
     return TG_OK;
+}
+
+// copy rows [r0, r1) of every [n][c] plane between a whole host DS and a piece buffer
+cudaError_t copy_rows(void* dst, const void* src, const Ds& d, int64_t r0, int64_t r1, bool h2d, cudaStream_t s) {
+    const size_t row = (size_t)d.d[3] * 4, planes = (size_t)(d.d[0] * d.d[1]);
+    const size_t piece = (size_t)(r1 - r0) * row, whole = (size_t)d.d[2] * row;
+    if (r0 == 0 && r1 == d.d[2])
+        return cudaMemcpyAsync(dst, src, planes * whole, h2d ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToHost, s);
+    if (h2d)
+        return cudaMemcpy2DAsync(dst, piece, (const char*)src + r0 * row, whole, piece, planes, cudaMemcpyHostToDevice, s);
+    return cudaMemcpy2DAsync((char*)dst + r0 * row, whole, src, piece, piece, planes, cudaMemcpyDeviceToHost, s);
 }
 
 }  // namespace
@@ -188,35 +205,26 @@ tg_status exec_run_per_op(tg_plan* p, bool blocking) {
     }
     tg_perop_exec& x = *p->perop;
     CK(cudaSetDevice(x.dev));
-    x.free_list.clear();
-    x.free_list[0] = std::max<uint64_t>(c.arena_bytes, 256) / 256 * 256;
     x.off.assign(c.po_ds.size(), -1);
-    auto host_src = [&](int sd) -> const float* {
-        const Ds& d = g.ds[c.po_ds[sd]];
-        if (d.kind != DsKind::Temp) return d.src;
-        return x.staging[sd].empty() ? nullptr : x.staging[sd].data();
-    };
-    for (auto& e : c.po_trace) {
+    for (size_t t = 0; t < c.po_trace.size(); ++t) {
+        const auto& e = c.po_trace[t];
         const int id = e.second;
+        const uint64_t off = c.po_trace_off[t];  // static first-fit layout (planner_perop.cpp)
         switch (e.first) {
-            case 0: {  // H2D
-                if (x.off[id] < 0) {
-                    uint64_t o;
-                    if (!arena_alloc(x, c.po_size[id], o)) return fail(TG_E_OOM, "per-op arena fragmented (H2D)");
-                    x.off[id] = (int64_t)o;
+            case 0: {  // H2D of a piece: rows [r0, r1) of its DS
+                x.off[id] = (int64_t)off;
+                const Ds& d = g.ds[c.po_ds[id]];
+                if (d.kind != DsKind::Temp) {
+                    CK(copy_rows(x.arena + off, d.src, d, c.po_r0[id], c.po_r1[id], true, x.stream));
+                } else {
+                    if (x.staging[id].empty()) return fail(TG_E_STATE, "per-op executor: no host copy to load");
+                    CK(cudaMemcpyAsync(x.arena + off, x.staging[id].data(), c.po_size[id], cudaMemcpyHostToDevice,
+                                       x.stream));
                 }
-                const float* src = host_src(id);
-                if (!src) return fail(TG_E_STATE, "per-op executor: no host copy to load");
-                CK(cudaMemcpyAsync(x.arena + x.off[id], src, c.po_size[id], cudaMemcpyHostToDevice, x.stream));
                 break;
             }
             case 1: {  // run
-                for (int32_t j : c.po_outs[id])
-                    if (x.off[j] < 0) {
-                        uint64_t o;
-                        if (!arena_alloc(x, c.po_size[j], o)) return fail(TG_E_OOM, "per-op arena fragmented (output)");
-                        x.off[j] = (int64_t)o;
-                    }
+                x.off[c.po_outs[id][0]] = (int64_t)off;
                 cudaEvent_t a = nullptr, b = nullptr;
                 if (x.profiling) {
                     cudaEventCreate(&a);
@@ -232,24 +240,20 @@ tg_status exec_run_per_op(tg_plan* p, bool blocking) {
                 ++p->launches;
                 break;
             }
-            case 2: {  // D2H
+            case 2: {  // D2H: outputs into their rows of the host buffer, temporaries to staging
                 const Ds& d = g.ds[c.po_ds[id]];
-                float* dst;
                 if (c.po_kind[id] == TG_DS_OUTPUT) {
-                    dst = d.dst;
+                    CK(copy_rows(d.dst, x.arena + x.off[id], d, c.po_r0[id], c.po_r1[id], false, x.stream));
                 } else {
                     x.staging[id].resize(c.po_size[id] / 4);
-                    dst = x.staging[id].data();
+                    CK(cudaMemcpyAsync(x.staging[id].data(), x.arena + x.off[id], c.po_size[id],
+                                       cudaMemcpyDeviceToHost, x.stream));
+                    CK(cudaStreamSynchronize(x.stream));  // staging is pageable
                 }
-                CK(cudaMemcpyAsync(dst, x.arena + x.off[id], c.po_size[id], cudaMemcpyDeviceToHost, x.stream));
-                if (c.po_kind[id] != TG_DS_OUTPUT) CK(cudaStreamSynchronize(x.stream));  // staging is pageable
                 break;
             }
             default:  // free
-                if (x.off[id] >= 0) {
-                    arena_free(x, (uint64_t)x.off[id], c.po_size[id]);
-                    x.off[id] = -1;
-                }
+                x.off[id] = -1;
         }
     }
     if (blocking) CK(cudaStreamSynchronize(x.stream));

@@ -70,27 +70,53 @@ cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3(const CnnU3Args& a, cudaStream_t s);
 
-// Generic per-operator kernels (generic.cu) for the TG_PER_OP / TG_BASELINE modes.
+// Generic per-operator kernels (generic.cu) for the TG_PER_OP / TG_BASELINE modes. Every
+// kernel computes output rows [r0, r1) of its operator (a piece of a split operator,
+// PAPER.md:359-367, or the whole operator) into a piece buffer laid out [n][c][r1-r0][w].
+// Inputs are views: the pieces of a data structure that the operator reads, each a row band
+// [r0, r1) stored [n][c][r1-r0][w]; a row is looked up in the first piece that holds it
+// (overlapping pieces hold identical rows).
+constexpr int kGenMaxSeg = 8;
+struct GenSeg {
+    const float* p;
+    int64_t r0, r1;
+};
+struct GenView {
+    GenSeg seg[kGenMaxSeg];
+    int32_t nseg;
+};
 struct GenConvArgs {
-    const float* x; const float* k; const float* bias; float* y;
-    int64_t n, ci, h, w, co, kh, kw, ho, wo;
+    GenView x, bias;        // image [n][ci][h][w]; bias plane [1][co][ho][wo] or scalar [co]
+    const float* k;         // kernel [co][ci][kh][kw] (whole parameter)
+    float* y;               // output rows [r0, r1): [n][co][r1-r0][wo]
+    int64_t r0, r1;
+    int64_t n, ci, h, w, co, kh, kw, wo;
     int pt, pl;             // top/left padding (0 for VALID)
     int bias_kind;          // 0 none, 1 scalar [co], 2 plane [co][ho][wo]
 };
 constexpr int kGenMaxInputs = 16;
 struct GenElemArgs {
-    const float* xs[kGenMaxInputs]; int nx;
-    float* y; int64_t numel;
+    GenView xs[kGenMaxInputs]; int nx;
+    float* y;               // rows [r0, r1) of [n][c][h][w]: [n][c][r1-r0][w]
+    int64_t r0, r1, planes, w;
     int op;                 // 0 add, 1 neg, 2 affine, 3 abs, 4 tanh, 5 max
     float a, b;
 };
 struct GenSubArgs {
-    const float* x; const float* p; float* y;
-    int64_t n, c, h, w, ho, wo; int s;
+    GenView x; const float* p; float* y;
+    int64_t r0, r1;
+    int64_t n, c, h, w, wo; int s;
+};
+// C = A B over rows [r0, r1) of A and C; A [m][k] (view), B [k][n] (view,
+// read whole), C rows [r0, r1) of [m][n]
+struct GenMatmulArgs {
+    GenView a, b; float* c;
+    int64_t r0, r1, k, n;
 };
 cudaError_t launch_gen_conv(const GenConvArgs& a, cudaStream_t s);
 cudaError_t launch_gen_elem(const GenElemArgs& a, cudaStream_t s);
 cudaError_t launch_gen_sub(const GenSubArgs& a, cudaStream_t s);
+cudaError_t launch_gen_matmul(const GenMatmulArgs& a, cudaStream_t s);
 
 // tcgen05 (bf16 operands, fp32 accumulation in TMEM) variants of U2 and U3 (cnn_tc.cu)
 cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s);

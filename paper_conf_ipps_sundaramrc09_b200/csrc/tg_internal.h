@@ -32,11 +32,11 @@ struct Ds {
     int64_t numel() const { return d[0] * d[1] * d[2] * d[3]; }
 };
 
-enum class OpKind { Conv, Elem, Tanh, Max, Sub };
+enum class OpKind { Conv, Elem, Tanh, Max, Sub, Matmul };
 
 struct Node {
     OpKind op;
-    std::vector<int> ins;  // DS ids (conv: x, k[, bias]; sub: x, p)
+    std::vector<int> ins;  // DS ids (conv: x, k; sub: x, p; matmul: a, b)
     int out = -1;
     int32_t pad = TG_VALID;  // conv
     int32_t bias = -1;       // conv bias DS id or -1
@@ -127,6 +127,13 @@ struct PlanCore {
     std::vector<int32_t> po_order;
     std::vector<std::pair<int32_t, int32_t>> po_trace;  // (0 h2d | 1 run | 2 d2h | 3 free, id)
     uint64_t po_capacity = 0;
+    // operator splitting (TG_PER_OP, R19): sched DS k is rows
+    // [po_r0[k], po_r1[k]) of graph DS po_ds[k]; sched op j is piece po_piece[j] of node po_ops[j]
+    std::vector<int64_t> po_r0, po_r1;
+    std::vector<int32_t> po_piece;
+    std::vector<int32_t> po_k;    // split factor per graph node (0: not needed)
+    std::vector<uint64_t> po_trace_off;  // arena offset of the DS each trace step touches (static
+                                         // first-fit layout, PAPER.md:409 fragmentation margin)
 };
 
 tg_status recognise(const Graph& g, Template& t);

@@ -89,6 +89,7 @@ _PROTOS = {
     "tg_tanh": (c_i32, [vp, c_i32, P_id]),
     "tg_max_combine": (c_i32, [vp, P_id, c_i32, P_id]),
     "tg_subsample": (c_i32, [vp, c_i32, c_i32, c_i32, P_id]),
+    "tg_matmul": (c_i32, [vp, c_i32, c_i32, P_id]),
     "tg_output": (c_i32, [vp, c_i32, vp]),
     "tg_output_device": (c_i32, [vp, c_i32, vp]),
     "tg_shape": (c_i32, [vp, c_i32, ctypes.POINTER(c_i64)]),
@@ -209,6 +210,10 @@ def tg_max_combine(g, xs: Sequence[int]) -> int:
 
 def tg_subsample(g, x, p, s=2) -> int:
     return _id_call(_lib.tg_subsample, g, x, p, s)
+
+
+def tg_matmul(g, a, b) -> int:
+    return _id_call(_lib.tg_matmul, g, a, b)
 
 
 def tg_output(g, y, host_ptr) -> None:
@@ -463,6 +468,18 @@ class Graph:
 
     def neg(self, x):
         return tg_elementwise(self.h, TG_NEG, [x])
+
+    def elementwise(self, op, xs, a=1.0, b=0.0):
+        return tg_elementwise(self.h, op, list(xs), a, b)
+
+    def tanh(self, x):
+        return tg_tanh(self.h, x)
+
+    def subsample(self, x, p, s=2):
+        return tg_subsample(self.h, x, p, s)
+
+    def matmul(self, a, b):
+        return tg_matmul(self.h, a, b)
 
     def max_combine(self, xs):
         return tg_max_combine(self.h, xs)

@@ -233,3 +233,39 @@ def run_split(spec, plan):
         if d == spec.output:
             out[:, :, a:b] = store[opid]
     return out
+
+
+# ------------------------------------------------------------------------------ library graph
+def lib_graph(spec, out, budget=0, torch_runtime=False):
+    """The same graph through the C ABI (DS ids in the same creation order as the spec)."""
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    g = tg.Graph()
+    made = {}
+    node_of = {nd.out: i for i, nd in enumerate(spec.nodes)}
+    codes = {"add": tg.TG_ADD, "neg": tg.TG_NEG, "affine": tg.TG_AFFINE, "abs": tg.TG_ABS}
+    for d in range(len(spec.shapes)):
+        if d in spec.data:
+            a = spec.data[d]
+            made[d] = g.input(a) if spec.kinds[d] == "input" else g.param(a)
+            continue
+        i = node_of[d]
+        nd, op = spec.nodes[i], spec.ops[i]
+        xs = [made[x] for x in nd.ins]
+        if op["op"] == "conv":
+            y = g.conv2d(xs[0], xs[1], xs[2] if len(xs) > 2 else -1, tg.TG_SAME if op["pad"] == "same" else tg.TG_VALID)
+        elif op["op"] == "sub":
+            y = g.subsample(xs[0], xs[1], op["s"])
+        elif op["op"] == "matmul":
+            y = g.matmul(xs[0], xs[1])
+        elif op["op"] == "tanh":
+            y = g.tanh(xs[0])
+        elif op["op"] == "max":
+            y = g.max_combine(xs)
+        else:
+            y = g.elementwise(codes[op["op"]], xs, op["a"], op["b"])
+        assert y == d, (y, d)
+        assert tuple(g.shape(y)) == tuple(spec.shapes[d])
+        made[d] = y
+    g.output(made[spec.output], out)
+    g.set(budget=budget, torch_runtime=torch_runtime)
+    return g

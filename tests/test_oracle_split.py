@@ -1,4 +1,4 @@
-"""Pins of the splitting oracle (oracle/planner.py::split_plan, reading R18)
+"""Pins of the splitting oracle (oracle/planner.py::split_plan, reading R19)
 and of the matmul oracle (oracle.c orc_matmul), against what the paper and the
 mathematics fix:
   * the paper's own example: a 100x100 image and a 5x5 kernel split in two give

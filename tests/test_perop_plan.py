@@ -68,11 +68,15 @@ def test_edge_per_op_schedule_matches_oracle(budget):
     check_against_oracle(edge_plan(tg.TG_BASELINE, budget=budget).json())
 
 
-def test_per_op_infeasible_without_splitting():
+def test_baseline_infeasible_per_op_splits():
+    """The max operator needs 5 x 4 MB: the baseline (operators whole) cannot
+    run it in 16 MB, the paper's method splits it (tests/test_split_plan.py)."""
     from paper_conf_ipps_sundaramrc09_b200 import tg
     with pytest.raises(tg.TGError) as e:
-        edge_plan(tg.TG_PER_OP, budget=16 << 20)   # max needs 5 x 4 MB
+        edge_plan(tg.TG_BASELINE, budget=16 << 20)
     assert e.value.code == tg.TG_E_INFEASIBLE
+    j = edge_plan(tg.TG_PER_OP, budget=16 << 20).json()
+    assert max(j["k"].values()) > 1 and len(j["ops"]) > 5
 
 
 @pytest.mark.parametrize("budget", [0, 12 << 20, 6 << 20])

@@ -1,0 +1,114 @@
+"""The library's operator splitting (TG_PER_OP, reading R19) built through
+the C ABI on a CPU-only box, bit-exact against the splitting oracle (oracle/planner.py::
+split_plan): the same pieces (DS, row band), the same piece operators, the same DFS order
+(PAPER.md:381), the same next-use transfer trace and byte counts, for the
+edge template, the CNN and a conv/tanh/subsample/matmul/affine chain at several budgets."""
+import numpy as np
+import pytest
+
+import synth
+from split_graphs import cnn_spec, edge_spec, lib_graph, mixed_spec
+
+KIND = {"input": 0, "param": 1, "temp": 2, "output": 3}
+
+
+def compare(spec, budget):
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    out = np.zeros(spec.shapes[spec.output], np.float32)
+    g = lib_graph(spec, out, budget=budget)
+    j = g.plan(tg.TG_PER_OP).json()
+    from oracle import planner as P
+    r = P.per_op_plan(spec.shapes, spec.kinds, spec.nodes, spec.output, budget)
+    assert j["capacity"] == r["capacity"]
+    og = r["graph"]
+    assert j["pieces"] == r["pieces"]
+    assert j["ds"] == [[d.size, KIND[d.kind]] for d in og.ds]
+    assert j["ops"] == [[o.ins, o.outs] for o in og.ops]
+    assert j["op_piece"] == r["op_piece"]
+    assert {int(k): v for k, v in j["k"].items()} == r["k"]
+    assert j["order"] == r["order"]
+    kind = {"h2d": 0, "run": 1, "d2h": 2}
+    names_ds = {d.name: i for i, d in enumerate(og.ds)}
+    names_op = {o.name: i for i, o in enumerate(og.ops)}
+    assert j["trace"] == [[kind[k], names_op[n] if k == "run" else names_ds[n]] for k, n in r["trace"]]
+    assert j["h2d_bytes"] + j["d2h_bytes"] == r["moved"]
+    if budget:   # the static arena layout (first fit over the trace with frees)
+        kf = {"h2d": 0, "run": 1, "d2h": 2, "free": 3}
+        assert j["trace_full"] == [[kf[k], names_op[n] if k == "run" else names_ds[n]] for k, n in r["trace_full"]]
+        assert j["trace_off"] == r["trace_off"]
+    return j, r
+
+
+@pytest.mark.parametrize("frac", [0, 0.5, 0.2, 0.08])
+def test_edge_split_plan_matches_oracle(frac):
+    K1, K2 = synth.random_edge_filters_np(7)
+    spec = edge_spec(301, 64, K1, K2, n=2, rng=3)
+    budget = int(spec.total_bytes() * frac) // 256 * 256
+    j, r = compare(spec, budget)
+    if frac and frac < 0.5:
+        assert max(r["k"].values()) > 1
+
+
+@pytest.mark.parametrize("frac", [0, 0.3, 0.25, 0.2])
+def test_cnn_split_plan_matches_oracle(frac):
+    H, W, n5 = 77, 41, 4
+    spec = cnn_spec(1, H, W, n5, synth.cnn_params_np(11, n5, H, W))
+    compare(spec, int(spec.total_bytes() * frac) // 256 * 256)
+
+
+@pytest.mark.parametrize("frac", [0, 0.4, 0.15])
+def test_mixed_split_plan_matches_oracle(frac):
+    spec = mixed_spec(83, 30, 7)
+    compare(spec, int(spec.total_bytes() * frac) // 256 * 256)
+
+
+def test_paper_example_367_through_the_library():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    x = np.zeros((1, 1, 100, 100), np.float32)
+    g = tg.Graph()
+    xi = g.input(x)
+    k = g.param(np.zeros((1, 1, 5, 5), np.float32))
+    y = g.conv2d(xi, k)
+    g.output(y, np.zeros((1, 1, 96, 96), np.float32))
+    g.set(budget=45568)                   # capacity 39,872 B: two pieces
+    j = g.plan(tg.TG_PER_OP).json()
+    assert [p[1:] for p in j["pieces"] if p[0] == xi] == [[0, 52], [48, 100]]
+    assert [p[1:] for p in j["pieces"] if p[0] == y] == [[0, 48], [48, 96]]
+    with pytest.raises(tg.TGError) as e:   # the baseline never splits
+        g.plan(tg.TG_BASELINE)
+    assert e.value.code == tg.TG_E_INFEASIBLE
+
+
+def test_infeasible_when_nothing_fits():
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    g = tg.Graph()
+    xi = g.input(np.zeros((1, 1, 64, 64), np.float32))
+    k = g.param(np.zeros((1, 1, 32, 32), np.float32))
+    g.output(g.conv2d(xi, k), np.zeros((1, 1, 33, 33), np.float32))
+    g.set(budget=4608)
+    with pytest.raises(tg.TGError) as e:
+        g.plan(tg.TG_PER_OP)
+    assert e.value.code == tg.TG_E_INFEASIBLE
+
+
+def test_static_arena_layout_is_consistent():
+    """Every allocation of the static layout lies inside the arena and no two resident
+    pieces overlap at any step of the trace."""
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    K1, K2 = synth.random_edge_filters_np(7)
+    spec = edge_spec(301, 64, K1, K2, n=2, rng=3)
+    budget = int(spec.total_bytes() * 0.2) // 256 * 256
+    g = lib_graph(spec, np.zeros(spec.shapes[spec.output], np.float32), budget=budget)
+    j = g.plan(tg.TG_PER_OP).json()
+    a256 = lambda v: (max(v, 1) + 255) // 256 * 256
+    res = {}
+    for (kind, i), off in zip(j["trace_full"], j["trace_off"]):
+        if kind == 0 or kind == 1:
+            d = i if kind == 0 else j["ops"][i][1][0]
+            if d not in res:
+                res[d] = (off, off + a256(j["ds"][d][0]))
+                assert res[d][1] <= j["arena_bytes"]
+            iv = sorted(res.values())
+            assert all(iv[t][1] <= iv[t + 1][0] for t in range(len(iv) - 1))
+        elif kind == 3:
+            res.pop(i, None)
