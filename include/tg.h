@@ -244,6 +244,61 @@ int64_t tg_plan_launch_count(const tg_plan* plan);
 
 void tg_plan_destroy(tg_plan* plan);
 
+/* ------------------------------------------------------------------ operator library */
+/* The operator library of Fig. 4: one call runs output rows [r0, r1) of one
+ * operator -- a piece of a split operator or the whole operator -- on the
+ * device. TG_PER_OP / TG_BASELINE plans execute through it, and the code generator below emits
+ * calls to it. All pointers are DEVICE pointers owned by the caller. A data structure piece
+ * holding rows [r0, r1) of a DS [n][c][h][w] is stored [n][c][r1-r0][w]; an input is a view
+ * of up to TG_OPLIB_MAX_SEG such pieces (a row is read from the first piece that holds it;
+ * overlapping pieces must hold identical rows). Returns TG_E_ARG for malformed descriptors
+ * (unknown kind, too many inputs/pieces, a kernel or subsample weight not in one piece at row
+ * 0), TG_E_CUDA if the launch fails; the call is asynchronous on `stream` (a cudaStream_t,
+ * NULL = legacy default stream). */
+#define TG_OPLIB_MAX_SEG 8
+#define TG_OPLIB_MAX_IN 16
+#define TG_OPLIB_CONV 0     /* in: x, kernel[, bias] ; pad, dims as tg_conv2d              */
+#define TG_OPLIB_ELEM 1     /* in: xs ; elem = TG_ADD..TG_ABS, 4 = tanh, 5 = max; a, b       */
+#define TG_OPLIB_SUB 2      /* in: x, p ; s                                                 */
+#define TG_OPLIB_MATMUL 3   /* in: a, b (b read whole)                                      */
+typedef struct {
+    const float* p;         /* piece buffer [n][c][r1-r0][w]                                */
+    int64_t r0, r1;         /* rows of the DS it holds                                      */
+} tg_oplib_seg;
+typedef struct {
+    tg_oplib_seg seg[TG_OPLIB_MAX_SEG];
+    int32_t nseg;
+} tg_oplib_view;
+typedef struct {
+    int32_t kind;                       /* TG_OPLIB_*                                        */
+    int32_t nin;                        /* inputs used in in[] / in_dims[]                   */
+    tg_oplib_view in[TG_OPLIB_MAX_IN];
+    int64_t in_dims[TG_OPLIB_MAX_IN][4];  /* [n][c][h][w] of each input DS                   */
+    float* y;                           /* output piece: rows [r0, r1) of y_dims, [n][c][r1-r0][w] */
+    int64_t y_dims[4];
+    int64_t r0, r1;
+    int32_t pad;                        /* conv: TG_VALID | TG_SAME                          */
+    int32_t elem;                       /* elementwise op (see TG_OPLIB_ELEM)                */
+    int32_t s;                          /* subsample window = stride                         */
+    float a, b;                         /* TG_AFFINE coefficients                            */
+} tg_oplib_op;
+tg_status tg_oplib_run(const tg_oplib_op* op, void* stream);
+
+/* Code generator ("A code generator takes the execution plan generated by the
+ * previous steps, and generates a hybrid CPU/GPU program ... compiled together with a larger
+ * application"): C source replaying a TG_PER_OP / TG_BASELINE plan -- every H2D copy of a
+ * piece (2-D copies of its rows), every tg_oplib_run call, every D2H copy, with the plan's
+ * static arena offsets baked in. The source defines
+ *   int tg_generated_execute(float* const* host, char* arena, void* stream);
+ *   TG_GEN_ARENA_BYTES, TG_GEN_NUM_DS
+ * where host[d] is the host buffer of graph DS d (inputs, parameters and the output; others
+ * may be NULL), arena a device buffer of TG_GEN_ARENA_BYTES bytes, stream a cudaStream_t; it
+ * returns 0 when the output is complete on the host, a tg_status otherwise. Compile with the
+ * CUDA runtime headers and link against this library and cudart. Writes at most cap bytes
+ * incl. NUL; *needed = required size incl. NUL; TG_E_ARG if buf is too small,
+ * TG_E_UNSUPPORTED for TG_FUSED plans. */
+tg_status tg_plan_codegen(const tg_plan* plan, char* buf, size_t cap, size_t* needed);
+
 /* ------------------------------------------------------------------ transfer scheduling */
 /* The paper's heuristic offload/transfer scheduler (Section 3.3.1) over an
  * abstract operator graph whose data structures have sizes in any unit (floats, bytes, or

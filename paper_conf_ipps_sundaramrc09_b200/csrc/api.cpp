@@ -481,6 +481,20 @@ tg_status tg_plan_dump_json(const tg_plan* p, char* buf, size_t cap, size_t* nee
     TG_GUARD_END
 }
 
+tg_status tg_plan_codegen(const tg_plan* p, char* buf, size_t cap, size_t* needed) {
+    if (!p) return fail(TG_E_ARG, "tg_plan_codegen: NULL plan");
+    if (p->core.mode == TG_FUSED)
+        return fail(TG_E_UNSUPPORTED, "tg_plan_codegen: generates TG_PER_OP / TG_BASELINE plans");
+    TG_GUARD_BEGIN
+    std::string s = plan_codegen(p);
+    if (s.empty()) return fail(TG_E_STATE, "tg_plan_codegen: inconsistent plan");
+    if (needed) *needed = s.size() + 1;
+    if (!buf || cap < s.size() + 1) return fail(TG_E_ARG, "tg_plan_codegen: buffer too small");
+    std::memcpy(buf, s.c_str(), s.size() + 1);
+    return TG_OK;
+    TG_GUARD_END
+}
+
 tg_status tg_execute(tg_plan* p) {
     if (!p) return fail(TG_E_ARG, "tg_execute: NULL plan");
     TG_GUARD_BEGIN

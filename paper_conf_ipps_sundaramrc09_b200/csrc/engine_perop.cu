@@ -45,119 +45,64 @@ namespace {
         }                                                                                          \
     } while (0)
 
-// view of the resident pieces `ids` (sched DS ids, all of one graph DS) for a kernel
-bool make_view(const PlanCore& c, const tg_perop_exec& x, const std::vector<int32_t>& ids, GenView& v) {
-    v = GenView{};
-    for (int32_t id : ids) {
-        if (x.off[id] < 0 || v.nseg >= kGenMaxSeg) return false;
-        v.seg[v.nseg++] = GenSeg{(const float*)(x.arena + x.off[id]), c.po_r0[id], c.po_r1[id]};
-    }
-    return true;
-}
+// The tg_oplib_op descriptor of sched op `op` (graph node piece) with the arena offsets
+// `off` of its resident pieces (-1: not resident). Shared with the code generator.
+}  // namespace
 
-tg_status launch_node(const Graph& g, const PlanCore& c, tg_perop_exec& x, int op) {
+bool oplib_desc(const Graph& g, const PlanCore& c, int op, const std::vector<int64_t>& off, const char* arena,
+                tg_oplib_op& d) {
     const Node& nd = g.nodes[c.po_ops[op]];
+    d = tg_oplib_op{};
     // the operator's input slots in order (conv x, k[, bias]); each slot's pieces are the
     // consecutive entries of po_ins that belong to its DS
     std::vector<int> slots = nd.ins;
     if (nd.op == OpKind::Conv && nd.bias >= 0) slots.push_back(nd.bias);
+    if (slots.size() > (size_t)TG_OPLIB_MAX_IN) return false;
     std::vector<std::vector<int32_t>> pieces(slots.size());
-    {
-        const std::vector<int32_t>& ins = c.po_ins[op];
-        size_t i = 0;
-        for (size_t s = 0; s < slots.size(); ++s) {
-            while (i < ins.size() && c.po_ds[ins[i]] == slots[s]) pieces[s].push_back(ins[i++]);
-            if (pieces[s].empty()) {  // repeated operand (e.g. add(x, x)): same pieces again
-                for (size_t t = 0; t < s; ++t)
-                    if (slots[t] == slots[s]) pieces[s] = pieces[t];
-            }
-        }
+    const std::vector<int32_t>& ins = c.po_ins[op];
+    size_t i = 0;
+    for (size_t s = 0; s < slots.size(); ++s) {
+        while (i < ins.size() && c.po_ds[ins[i]] == slots[s]) pieces[s].push_back(ins[i++]);
+        if (pieces[s].empty())  // repeated operand (e.g. add(x, x)): same pieces again
+            for (size_t t = 0; t < s; ++t)
+                if (slots[t] == slots[s]) pieces[s] = pieces[t];
     }
-    GenView v[kGenMaxInputs];
-    for (size_t s = 0; s < slots.size() && s < (size_t)kGenMaxInputs; ++s)
-        if (!make_view(c, x, pieces[s], v[s])) return fail(TG_E_STATE, "per-op executor: input not resident");
+    d.nin = (int32_t)slots.size();
+    for (size_t s = 0; s < slots.size(); ++s) {
+        if (pieces[s].empty() || pieces[s].size() > (size_t)TG_OPLIB_MAX_SEG) return false;
+        for (int32_t id : pieces[s]) {
+            if (off[id] < 0) return false;
+            d.in[s].seg[d.in[s].nseg++] = tg_oplib_seg{(const float*)((uintptr_t)arena + (uint64_t)off[id]), c.po_r0[id], c.po_r1[id]};
+        }
+        for (int q = 0; q < 4; ++q) d.in_dims[s][q] = g.ds[slots[s]].d[q];
+    }
     const int32_t yo = c.po_outs[op][0];
-    if (x.off[yo] < 0) return fail(TG_E_STATE, "per-op executor: output not resident");
-    float* y = (float*)(x.arena + x.off[yo]);
-    const int64_t r0 = c.po_r0[yo], r1 = c.po_r1[yo];
-    const Ds& Y = g.ds[nd.out];
-    cudaError_t e = cudaSuccess;
+    if (off[yo] < 0) return false;
+    d.y = (float*)((uintptr_t)arena + (uint64_t)off[yo]);
+    for (int q = 0; q < 4; ++q) d.y_dims[q] = g.ds[nd.out].d[q];
+    d.r0 = c.po_r0[yo];
+    d.r1 = c.po_r1[yo];
+    d.pad = nd.pad;
+    d.s = nd.s;
+    d.a = nd.a;
+    d.b = nd.b;
     switch (nd.op) {
-        case OpKind::Conv: {
-            const Ds& X = g.ds[nd.ins[0]];
-            const Ds& K = g.ds[nd.ins[1]];
-            GenConvArgs a{};
-            a.x = v[0];
-            if (v[1].nseg != 1 || v[1].seg[0].r0 != 0) return fail(TG_E_STATE, "per-op executor: split kernel");
-            a.k = v[1].seg[0].p;
-            a.y = y;
-            a.r0 = r0;
-            a.r1 = r1;
-            a.n = X.d[0];
-            a.ci = X.d[1];
-            a.h = X.d[2];
-            a.w = X.d[3];
-            a.co = K.d[0];
-            a.kh = K.d[2];
-            a.kw = K.d[3];
-            a.wo = Y.d[3];
-            a.pt = nd.pad == TG_SAME ? (int)(K.d[2] - 1) / 2 : 0;
-            a.pl = nd.pad == TG_SAME ? (int)(K.d[3] - 1) / 2 : 0;
-            a.bias_kind = 0;
-            if (nd.bias >= 0) {
-                a.bias = v[2];
-                a.bias_kind = g.ds[nd.bias].numel() == K.d[0] ? 1 : 2;
-            }
-            e = launch_gen_conv(a, x.stream);
-            break;
-        }
-        case OpKind::Sub: {
-            const Ds& X = g.ds[nd.ins[0]];
-            GenSubArgs a{};
-            a.x = v[0];
-            if (v[1].nseg != 1) return fail(TG_E_STATE, "per-op executor: split subsample kernel");
-            a.p = v[1].seg[0].p;
-            a.y = y;
-            a.r0 = r0;
-            a.r1 = r1;
-            a.n = X.d[0];
-            a.c = X.d[1];
-            a.h = X.d[2];
-            a.w = X.d[3];
-            a.wo = Y.d[3];
-            a.s = nd.s;
-            e = launch_gen_sub(a, x.stream);
-            break;
-        }
-        case OpKind::Matmul: {
-            GenMatmulArgs a{};
-            a.a = v[0];
-            a.b = v[1];
-            a.c = y;
-            a.r0 = r0;
-            a.r1 = r1;
-            a.k = g.ds[nd.ins[0]].d[3];
-            a.n = Y.d[3];
-            e = launch_gen_matmul(a, x.stream);
-            break;
-        }
-        default: {
-            GenElemArgs a{};
-            a.nx = (int)nd.ins.size();
-            for (int i = 0; i < a.nx; ++i) a.xs[i] = v[i];
-            a.y = y;
-            a.r0 = r0;
-            a.r1 = r1;
-            a.planes = Y.d[0] * Y.d[1];
-            a.w = Y.d[3];
-            a.op = nd.op == OpKind::Tanh ? 4 : nd.op == OpKind::Max ? 5 : nd.elem;
-            a.a = nd.a;
-            a.b = nd.b;
-            e = launch_gen_elem(a, x.stream);
-        }
+        case OpKind::Conv: d.kind = TG_OPLIB_CONV; break;
+        case OpKind::Sub: d.kind = TG_OPLIB_SUB; break;
+        case OpKind::Matmul: d.kind = TG_OPLIB_MATMUL; break;
+        default:
+            d.kind = TG_OPLIB_ELEM;
+            d.elem = nd.op == OpKind::Tanh ? 4 : nd.op == OpKind::Max ? 5 : nd.elem;
     }
-    if (e != cudaSuccess) return fail(TG_E_CUDA, std::string("generic kernel launch failed: ") + cudaGetErrorString(e));
-    return TG_OK;
+    return true;
+}
+
+namespace {
+
+tg_status launch_node(const Graph& g, const PlanCore& c, tg_perop_exec& x, int op) {
+    tg_oplib_op d;
+    if (!oplib_desc(g, c, op, x.off, x.arena, d)) return fail(TG_E_STATE, "per-op executor: operand not resident");
+    return oplib_run(d, x.stream);
 }
 
 // copy rows [r0, r1) of every [n][c] plane between a whole host DS and a piece buffer

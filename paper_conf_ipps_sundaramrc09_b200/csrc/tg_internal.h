@@ -192,4 +192,11 @@ tg_status exec_run_per_op(tg_plan* p, bool blocking);
 tg_status exec_timing_per_op(tg_plan* p, tg_timing* out);
 void exec_set_profiling_per_op(tg_plan* p, bool on);
 void exec_destroy_per_op(tg_plan* p);
+// descriptor of sched op `op` of a per-op plan given the arena offsets of its pieces
+bool oplib_desc(const Graph& g, const PlanCore& c, int op, const std::vector<int64_t>& off, const char* arena,
+                tg_oplib_op& d);
+// operator library (oplib.cu): one operator piece on `stream` (a cudaStream_t)
+tg_status oplib_run(const tg_oplib_op& op, void* stream);
+// code generator (codegen.cpp)
+std::string plan_codegen(const tg_plan* p);
 }  // namespace tg

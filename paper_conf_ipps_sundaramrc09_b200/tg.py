@@ -104,6 +104,8 @@ _PROTOS = {
     "tg_plan_create": (c_i32, [vp, c_i32, ctypes.POINTER(vp)]),
     "tg_plan_stats_get": (c_i32, [vp, ctypes.POINTER(tg_plan_stats)]),
     "tg_plan_dump_json": (c_i32, [vp, ctypes.c_char_p, c_sz, ctypes.POINTER(c_sz)]),
+    "tg_plan_codegen": (c_i32, [vp, ctypes.c_char_p, c_sz, ctypes.POINTER(c_sz)]),
+    "tg_oplib_run": (c_i32, [vp, vp]),
     "tg_execute": (c_i32, [vp]),
     "tg_execute_async": (c_i32, [vp]),
     "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
@@ -284,6 +286,17 @@ def tg_plan_dump_json(p) -> dict:
     buf = ctypes.create_string_buffer(need.value)
     _ck(_lib.tg_plan_dump_json(p, buf, need.value, ctypes.byref(need)))
     return json.loads(buf.value.decode())
+
+
+def tg_plan_codegen(p) -> str:
+    """C source replaying the plan (tg_plan_codegen)."""
+    need = c_sz(0)
+    _lib.tg_plan_codegen(p, None, 0, ctypes.byref(need))
+    if need.value == 0:
+        raise TGError(TG_E_UNSUPPORTED, last_error())
+    buf = ctypes.create_string_buffer(need.value)
+    _ck(_lib.tg_plan_codegen(p, buf, need.value, ctypes.byref(need)))
+    return buf.value.decode()
 
 
 def tg_execute(p) -> None:
@@ -521,6 +534,9 @@ class Plan:
 
     def json(self) -> dict:
         return tg_plan_dump_json(self.h)
+
+    def codegen(self) -> str:
+        return tg_plan_codegen(self.h)
 
     def execute(self, blocking: bool = True) -> None:
         (tg_execute if blocking else tg_execute_async)(self.h)
