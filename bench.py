@@ -221,7 +221,7 @@ def unit_bytes(wl, precision: str) -> dict:
     import synth
     (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = synth.cnn_dims(wl["H"], wl["W"])
     bf = precision == "bf16_tc"
-    t2 = n * h2 * w2 * (16 if bf else 32)
+    t2 = n * h2 * w2 * (16 if bf else 64 if precision == "fp32_tc" else 32)
     t4 = n * h4 * w4 * (48 if bf else 160 if precision == "fp32_tc" else 80)
     return {1: n * wl["H"] * wl["W"] * 4 + 8 * h1 * w1 * 4 + t2,
             2: t2 + 20 * h3 * w3 * 4 + t4,
@@ -308,7 +308,7 @@ def run(args, rank, world, local):
     kern_ms = tim["kernel_ms"][k] / nl
     flops_per_launch = fl[k] * opx[k] * args.steps / nl
     achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
-    tensor = (args.precision == "bf16_tc" and k in (2, 3)) or (args.precision == "fp32_tc" and k == 3)
+    tensor = args.precision in ("bf16_tc", "fp32_tc") and k in (2, 3)
     if tensor and args.precision == "fp32_tc":
         # 3xTF32 C5 on tcgen05 against the TF32 dense peak (the measured bf16 peak x the nominal
         # TF32/BF16 ratio 1/2); three MMAs per product, so the algorithmic ceiling is 1/3 of it
@@ -317,7 +317,7 @@ def run(args, rank, world, local):
         peak_basis = ("tf32 dense = 0.5 x measured bf16 burst (MEASURED_PEAKS.json); 3xTF32 issues 3 MMAs "
                       "per product: algorithmic ceiling = peak / 3")
         fl = dict(fl)
-        fl[3] = wl["n5"] * 500 * 2  # C5 (C6 runs on the CUDA cores on this path)
+        fl[3] = wl["n5"] * 500 * 2  # C5 (C6 runs on the CUDA cores on this path); C3 in U2
         flops_per_launch = fl[k] * opx[k] * args.steps / nl
         achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
     elif tensor:
@@ -370,9 +370,9 @@ def run(args, rank, world, local):
         ms_u = tim["kernel_ms"][u] / args.steps
         if ms_u <= 0:
             continue
-        tens_u = (args.precision == "bf16_tc" and u in (2, 3)) or (args.precision == "fp32_tc" and u == 3)
-        if tens_u and args.precision == "fp32_tc":  # C5 (3xTF32)
-            fpx = wl["n5"] * 500 * 2
+        tens_u = args.precision in ("bf16_tc", "fp32_tc") and u in (2, 3)
+        if tens_u and args.precision == "fp32_tc":  # C3 / C5 (3xTF32; C6 on the CUDA cores)
+            fpx = 4 * 20 * 200 * 2 if u == 2 else wl["n5"] * 500 * 2
         elif tens_u:  # the tensor-core part: C3 (U2); C5 and C6 (U3)
             fpx = 4 * 20 * 200 * 2 if u == 2 else wl["n5"] * 500 * 2 + 9 * wl["n5"] * 2
         else:
@@ -393,7 +393,8 @@ def run(args, rank, world, local):
     del x_dev
     y_host = torch.empty(out_shape, dtype=torch.float32).pin_memory()
     g2 = build_graph(tg, wl, x_host, y_host, False, params)
-    g2.set(budget=wl["budget"], torch_runtime=True, precision=args.precision_code)
+    g2.set(budget=wl["budget"], torch_runtime=True, precision=args.precision_code,
+           max_chunk_px=args.max_chunk_px)
     p2 = g2.plan()
     st = p2.stats()
     js = p2.json()
@@ -544,9 +545,11 @@ def main():
     ap.add_argument("--template", default="edge", choices=["edge", "cnn4", "cnn3", "cnn3s"])
     ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16_tc", "fp32_tc"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--max-chunk-px", type=int, default=None,
+                    help="chunk cap of the e2e plan (tg_set_chunking; default: the library's 2^25)")
     ap.add_argument("--per-template", default=None,
                     help="extra template:precision runs reported under per_template (default with --template "
-                         "edge: cnn4:fp32,cnn4:bf16_tc,cnn3:fp32,cnn3:bf16_tc; 'none' skips them)")
+                         "edge: cnn4 and cnn3 in fp32, fp32_tc and bf16_tc; 'none' skips them)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -577,7 +580,8 @@ def main():
     # from `--template cnn4 --precision ...`)
     extra = args.per_template
     if extra is None:
-        extra = "cnn4:fp32,cnn4:bf16_tc,cnn3:fp32,cnn3:bf16_tc" if args.template == "edge" else "none"
+        extra = ("cnn4:fp32,cnn4:fp32_tc,cnn4:bf16_tc,cnn3:fp32,cnn3:fp32_tc,cnn3:bf16_tc"
+                 if args.template == "edge" else "none")
     per = []
     for item in ([] if extra == "none" else extra.split(",")):
         t, pr = item.split(":")

@@ -150,6 +150,19 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
             asm("cvt.rn.bf16x2.f32 %0, %1, %2;\n" : "=r"(p[k]) : "f"(tv[2 * k + 1]), "f"(tv[2 * k]));
         }
         *d = make_uint4(p[0], p[1], p[2], p[3]);
+    } else if (a.t2_tf32) {  // TF32-split pixel blocks for the 3xTF32 U2: [part][block][rows][w2][4]
+        float4* d = reinterpret_cast<float4*>(a.t2) + img * 4 * plane + (R2 - a.t2_row0) * a.w2 + C2;
+#pragma unroll
+        for (int blk = 0; blk < 2; ++blk) {
+            float big[4], small[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                big[e] = tf32_rn(tv[4 * blk + e]);
+                small[e] = tf32_rn(tv[4 * blk + e] - big[e]);
+            }
+            d[blk * plane] = make_float4(big[0], big[1], big[2], big[3]);
+            d[(2 + blk) * plane] = make_float4(small[0], small[1], small[2], small[3]);
+        }
     } else {
 #pragma unroll
         for (int ch = 0; ch < 8; ++ch) t2[ch * plane + (R2 - a.t2_row0) * a.w2 + C2] = tv[ch];
@@ -288,6 +301,23 @@ __global__ void __launch_bounds__(128, 3)
                     for (int m = 0; m < 4; ++m)
                         asm("cvt.rn.bf16x2.f32 %0, %1, %2;\n" : "=r"(pk[m]) : "f"(tv[q][2 * m + 1]), "f"(tv[q][2 * m]));
                     d[q] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                }
+            } else if (a.t2_tf32) {  // TF32-split pixel blocks [part][block][rows][w2][4]
+                float4* d = reinterpret_cast<float4*>(a.t2) + img * 4 * plane + (R2 - a.t2_row0) * a.w2 + C2;
+#pragma unroll
+                for (int q = 0; q < 2; ++q) {
+                    if (C2 + q >= a.w2) continue;
+#pragma unroll
+                    for (int blk = 0; blk < 2; ++blk) {
+                        float big[4], small[4];
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            big[e] = tf32_rn(tv[q][4 * blk + e]);
+                            small[e] = tf32_rn(tv[q][4 * blk + e] - big[e]);
+                        }
+                        d[blk * plane + q] = make_float4(big[0], big[1], big[2], big[3]);
+                        d[(2 + blk) * plane + q] = make_float4(small[0], small[1], small[2], small[3]);
+                    }
                 }
             } else {
                 float* t2 = a.t2 + img * a.t2_img_stride + (R2 - a.t2_row0) * a.w2 + C2;

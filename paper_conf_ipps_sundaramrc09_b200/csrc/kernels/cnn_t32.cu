@@ -45,6 +45,14 @@ __device__ __forceinline__ float tanh_acc(float x) {
     return 1.f - __fdividef(2.f, 1.f + e);
 }
 
+// round to TF32 (10-bit mantissa; nearest, ties away): the "big" part of a 3xTF32 split (the
+// same rounding as U1 and the FFMA U2 in cnn_fp32.cu)
+__device__ __forceinline__ float tf32_rn_dev(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
+
 constexpr int kTileM = 128;
 constexpr int T3_KS = 65;                        // K-steps (K = 8) per tile
 constexpr int T3_KST = 4;                        // K-steps per B stage
@@ -301,6 +309,225 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (warp == 0) tc::tmem_dealloc<512>(tmem);
 }
 
+// ============================================================================ U2 (C3, 3xTF32)
+// C3 (8 x 25 -> 20) with fp32 accuracy: the bf16 U2's implicit GEMM (cnn_tc.cu) with TF32-split
+// operands. Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns: tile t = C3 row 2R + t
+// (M = 128), one K = 8 step per tap (the pixel's 8 channels: block 0 = channels 0-3, block 1 =
+// 4-7, LBO = one block plane of the window). With N = 20 maps (padded to 32) an MMA is bound by
+// reading its A operand from shared memory (4 KB per 128 x 8 tf32 slice), so the big part of
+// A is read ONCE for both of its products: per tap and tile
+//   MMA 1  A_big   x [B_big | B_small]  (N = 64)  -> columns [0, 32) big.big, [32, 64) big.small
+//   MMA 2  A_small x  B_big             (N = 32)  -> accumulates onto columns [32, 64)
+// and the epilogue adds the two halves (2 A reads per tap instead of 3). Window: T2 rows
+// [2R, 2R+6) x cols [c0, c0+134) of both parts and both blocks, [part][block][row][col] -> 4 tf32.
+// Warp-specialised and persistent (one CTA per SM, 10 warps), as the bf16 U2:
+//   warp 9   copy producer: the B operand once per CTA, per segment 24 row copies
+//   warp 8   MMA issuer: 2 tiles x 25 K-steps x 2 MMAs into one of 4 TMEM slots (128 columns)
+//   0-3/4-7  epilogue groups (even / odd segments): bias plane, tanh (fp32 formula), the 2x2
+//            subsample (rows in the thread, columns across lanes), tanh -> T4 TF32-split
+//            [part][block][rows][w4][4] for the 3xTF32 U3 above
+constexpr int U2T_WR = 6, U2T_WP = kTileM + 6;
+constexpr int U2T_N = 32;                      // 20 maps padded; B rows per K half = 2 x U2T_N
+constexpr int U2T_KS = 25;
+constexpr int U2T_NA = 3;
+constexpr int U2T_NT = 4;
+constexpr int U2T_PLANE = U2T_WR * U2T_WP;     // pixels per block plane of one window
+
+struct U2TP {
+    float p4[20][4];  // S4 weights (constant bank)
+};
+
+struct U2TSmem {
+    uint4 a[U2T_NA][2][2][U2T_PLANE];          // [buf][part][block][row*WP + col] -> 4 tf32
+    uint4 b[U2T_KS * 2 * 2 * U2T_N];           // [ks][half][row < 64: big maps, then small] -> 4 tf32
+    uint64_t b_full, a_full[U2T_NA], a_empty[U2T_NA], t_full[U2T_NT], t_empty[U2T_NT];
+    uint32_t tmem;
+};
+
+__global__ void __launch_bounds__(kThreads, 1)
+    cnn_u2_t32_kernel(const CnnU2Args a, const __grid_constant__ U2TP pw, const int64_t nseg) {
+    extern __shared__ __align__(128) uint8_t smraw[];
+    U2TSmem& S = *reinterpret_cast<U2TSmem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int64_t segs_per_row = (a.w3 + kTileM - 1) / kTileM;
+    const int64_t per_img = a.t4_rows * segs_per_row;
+    auto seg_coords = [&](int64_t sg, int64_t& img, int64_t& R, int64_t& c0) {
+        img = sg / per_img;
+        const int64_t rem = sg - img * per_img;
+        const int64_t rr = rem / segs_per_row;
+        R = a.t4_row0 + rr;
+        c0 = (rem - rr * segs_per_row) * kTileM;
+    };
+
+    if (warp == 0) tc::tmem_alloc<512>(&S.tmem);
+    if (tid == 0) {
+        tc::mbar_init(&S.b_full, 1);
+        for (int i = 0; i < U2T_NA; ++i) {
+            tc::mbar_init(&S.a_full[i], 1);
+            tc::mbar_init(&S.a_empty[i], 1);
+        }
+        for (int i = 0; i < U2T_NT; ++i) {
+            tc::mbar_init(&S.t_full[i], 1);
+            tc::mbar_init(&S.t_empty[i], 4);
+        }
+        tc::mbar_fence_init();
+    }
+    // windows start zeroed: pixels a copy does not cover (beyond the image) only ever hold
+    // finite T2 values; they feed C3 columns that are not stored
+    for (int idx = tid; idx < U2T_NA * 4 * U2T_PLANE; idx += kThreads) (&S.a[0][0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
+    tc::fence_proxy_async();
+    tc::fence_before_sync();
+    __syncthreads();
+    tc::fence_after_sync();
+    const uint32_t tmem = S.tmem;
+    const int64_t my = nseg > blockIdx.x ? (nseg - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+
+    if (warp == kEpiWarps + 1) {
+        // ---------------------------------------------------------------- copy producer
+        const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
+        const int64_t tplane = a.t2_rows * a.w2;  // pixels per block plane of one image's T2
+        const uint32_t bbytes = (uint32_t)(U2T_KS * 2 * 2 * U2T_N * 16);
+        if (tc::elect_one()) {
+            tc::mbar_expect_tx(&S.b_full, bbytes);
+            tc::bulk_g2s(S.b, a.k3_t32, bbytes, &S.b_full);
+        }
+        __syncwarp();
+        for (int64_t k = 0; k < my; ++k) {
+            const int buf = (int)(k % U2T_NA);
+            if (k >= U2T_NA) tc::mbar_wait(&S.a_empty[buf], (uint32_t)(((k - U2T_NA) / U2T_NA) & 1));
+            int64_t img, R, c0;
+            seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
+            const int64_t r0 = 2 * R - a.t2_row0;
+            const int64_t rows = min((int64_t)U2T_WR, a.t2_rows - r0);
+            const int64_t cols = min((int64_t)U2T_WP, a.w2 - c0);
+            // the 4 planes x `rows` window rows are issued by as many lanes in ONE warp
+            // instruction (a single thread would serialise ~150 cycles per bulk copy)
+            if (lane == 0) tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(4 * rows * cols * 16));
+            __syncwarp();
+            if (lane < 4 * rows) {
+                const int pb = lane / (int)rows, r = lane - pb * (int)rows;  // plane = part * 2 + block
+                const uint4* src = t2all + (img * 4 + pb) * tplane + (r0 + r) * a.w2 + c0;
+                tc::bulk_g2s(&S.a[buf][pb >> 1][pb & 1][r * U2T_WP], src, (uint32_t)(cols * 16), &S.a_full[buf]);
+            }
+            __syncwarp();
+        }
+    } else if (warp == kEpiWarps) {
+        // ---------------------------------------------------------------- MMA issuer
+        tc::mbar_wait(&S.b_full, 0);
+        const uint32_t idesc64 = idesc_tf32(kTileM, 2 * U2T_N), idesc32 = idesc_tf32(kTileM, U2T_N);
+        const uint32_t blk_bytes = (uint32_t)(U2T_PLANE * 16);
+        const uint64_t a_desc0 = tc::make_desc(tc::smem_u32(S.a[0][0][0]), blk_bytes, 128);  // K half 2 = block 1
+        const uint64_t b_desc0 = tc::make_desc(tc::smem_u32(S.b), 2 * U2T_N * 16, 128);
+        for (int64_t k = 0; k < my; ++k) {
+            const int buf = (int)(k % U2T_NA), ts = (int)(k % U2T_NT);
+            tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2T_NA) & 1));
+            if (k >= U2T_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2T_NT) / U2T_NT) & 1));
+            tc::fence_after_sync();
+            // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding
+            const uint64_t abuf = a_desc0 + (uint64_t)(buf * (4 * U2T_PLANE));
+            const uint32_t d0 = tmem + (uint32_t)(ts * 4 * U2T_N);
+            if (tc::elect_one()) {
+#pragma unroll
+                for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
+#pragma unroll
+                    for (int ks = 0; ks < U2T_KS; ++ks) {
+                        const int i = ks / 5, j = ks % 5;
+                        const uint64_t a_big = abuf + (uint64_t)((t + i) * U2T_WP + j);
+                        const uint64_t a_small = a_big + (uint64_t)(2 * U2T_PLANE);
+                        const uint64_t b_ks = b_desc0 + (uint64_t)(ks * 2 * 2 * U2T_N);  // rows 0..31 = B_big
+                        const uint32_t d = d0 + (uint32_t)(t * 2 * U2T_N);
+                        mma_tf32(d, a_big, b_ks, idesc64, ks > 0 ? 1u : 0u);
+                        mma_tf32(d + U2T_N, a_small, b_ks, idesc32, 1u);
+                    }
+                }
+                tc::commit(&S.a_empty[buf]);
+                tc::commit(&S.t_full[ts]);
+            }
+            __syncwarp();
+        }
+    } else {
+        // ---------------------------------------------------------------- epilogue groups
+        const int grp = warp >> 2, wq = warp & 3;
+        const uint32_t lane_base = (uint32_t)(32 * wq) << 16;
+        const int64_t bplane = a.t4_rows * a.w4;
+        float b0v[20], b1v[20];
+        const uint32_t bcs = a.b3_plane ? (uint32_t)(a.b3_rows * a.w3) : 1u;
+        const uint32_t brs = a.b3_plane ? (uint32_t)a.w3 : 0u;
+        auto load_bias = [&](int64_t kk) {
+            int64_t img_, R_, c0_;
+            seg_coords(blockIdx.x + kk * gridDim.x, img_, R_, c0_);
+            const int64_t cc = min(c0_ + 32 * wq + lane, a.w3 - 1);
+            const float* p0 = a.b3_plane ? a.b3 + (2 * R_ - a.b3_row0) * a.w3 + cc : a.b3;
+#pragma unroll
+            for (int co = 0; co < 20; ++co) {
+                b0v[co] = __ldg(p0 + co * bcs);
+                b1v[co] = __ldg(p0 + co * bcs + brs);
+            }
+        };
+        if (grp < my) load_bias(grp);
+        for (int64_t k = grp; k < my; k += 2) {
+            const int ts = (int)(k % U2T_NT);
+            int64_t img, R, c0;
+            seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
+            const int64_t c = c0 + 32 * wq + lane;  // C3 column
+            const int64_t C = c >> 1;               // T4 column
+            tc::mbar_wait(&S.t_full[ts], (uint32_t)((k / U2T_NT) & 1));
+            tc::fence_after_sync();
+            float v0[32], v1[32];
+            {
+                float x0[32], x1[32];
+                const uint32_t tb = tmem + lane_base + (uint32_t)(ts * 4 * U2T_N);
+                tc::tmem_ld32_async(tb, v0);                     // tile 0: big.big
+                tc::tmem_ld32_async(tb + U2T_N, x0);             //         big.small + small.big
+                tc::tmem_ld32_async(tb + 2 * U2T_N, v1);         // tile 1
+                tc::tmem_ld32_async(tb + 3 * U2T_N, x1);
+                tc::tmem_wait_ld();
+#pragma unroll
+                for (int co = 0; co < 20; ++co) {
+                    v0[co] += x0[co];
+                    v1[co] += x1[co];
+                }
+            }
+            tc::fence_before_sync();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(&S.t_empty[ts]);
+            const bool out_ok = !(lane & 1) && C < a.w4;
+            float tv[20];
+#pragma unroll
+            for (int co = 0; co < 20; ++co) {
+                const float t0 = tanh_acc(v0[co] + b0v[co]);
+                const float t1 = tanh_acc(v1[co] + b1v[co]);
+                const float t01 = __shfl_down_sync(0xffffffffu, t0, 1);  // column c+1
+                const float t11 = __shfl_down_sync(0xffffffffu, t1, 1);
+                float s4 = 0.f;
+                s4 = fmaf(pw.p4[co][0], t0, s4);
+                s4 = fmaf(pw.p4[co][1], t01, s4);
+                s4 = fmaf(pw.p4[co][2], t1, s4);
+                s4 = fmaf(pw.p4[co][3], t11, s4);
+                tv[co] = tanh_acc(s4);
+            }
+            if (k + 2 < my) load_bias(k + 2);
+            if (out_ok) {
+                float4* t4 = reinterpret_cast<float4*>(a.t4) + img * 10 * bplane + (R - a.t4_row0) * a.w4 + C;
+#pragma unroll
+                for (int blk = 0; blk < 5; ++blk) {
+                    float big[4], small[4];
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) {
+                        big[e] = tf32_rn_dev(tv[4 * blk + e]);
+                        small[e] = tf32_rn_dev(tv[4 * blk + e] - big[e]);
+                    }
+                    t4[blk * bplane] = make_float4(big[0], big[1], big[2], big[3]);
+                    t4[(5 + blk) * bplane] = make_float4(small[0], small[1], small[2], small[3]);
+                }
+            }
+        }
+    }
+    tc::fence_before_sync();
+    __syncthreads();
+    if (warp == 0) tc::tmem_dealloc<512>(tmem);
+}
+
 // round to TF32 (10-bit mantissa), nearest even, on the host
 float to_tf32(float f) {
     uint32_t u;
@@ -352,6 +579,41 @@ void cnn_prepare_k5_t32(const float* k5, int n5, float* dst) {
                     dst[(((size_t)(ks * 2 + 1) * 2 + h) * NP + n) * 4 + e] = small;
                 }
     }
+}
+
+// B operand of the 3xTF32 C3: [ks < 25][half][row < 64][4] fp32, K-step ks = tap (i, j) =
+// (ks / 5, ks % 5), half h = channels 4h..4h+3; row n < 32: big part tf32_rn(w) of map n,
+// row 32 + n: small part tf32_rn(w - big) of map n, w = K3[n][4h + e][i][j]; maps 20..31 zero.
+size_t cnn_k3_t32_bytes() { return (size_t)U2T_KS * 2 * 2 * U2T_N * 4 * 4; }
+void cnn_prepare_k3_t32(const float* k3, float* dst) {
+    std::memset(dst, 0, cnn_k3_t32_bytes());
+    for (int ks = 0; ks < U2T_KS; ++ks)
+        for (int h = 0; h < 2; ++h)
+            for (int n = 0; n < 20; ++n)
+                for (int e = 0; e < 4; ++e) {
+                    const float w = k3[((size_t)n * 8 + 4 * h + e) * 25 + ks];
+                    const float big = to_tf32(w), small = to_tf32(w - big);
+                    dst[(((size_t)ks * 2 + h) * 2 * U2T_N + n) * 4 + e] = big;
+                    dst[(((size_t)ks * 2 + h) * 2 * U2T_N + U2T_N + n) * 4 + e] = small;
+                }
+}
+
+cudaError_t launch_cnn_u2_t32(const CnnU2Args& a, cudaStream_t s) {
+    if (a.t4_rows <= 0 || a.nimg <= 0) return cudaSuccess;
+    if (!a.k3_t32) return cudaErrorInvalidValue;
+    if (a.b3_plane && 20 * a.b3_rows * a.w3 >= (1ll << 32)) return cudaErrorInvalidValue;
+    static std::atomic<uint32_t> flags{0};
+    const size_t smem = sizeof(U2TSmem) + 128;
+    if (!set_smem_attr_t32((const void*)cnn_u2_t32_kernel, smem, flags)) return cudaErrorInvalidValue;
+    U2TP pw;
+    std::memcpy(pw.p4, a.p4_host, sizeof pw.p4);
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t nseg = a.t4_rows * ((a.w3 + kTileM - 1) / kTileM) * a.nimg;
+    const unsigned grid = (unsigned)std::min<int64_t>(nseg, sms);
+    cnn_u2_t32_kernel<<<grid, kThreads, smem, s>>>(a, pw, nseg);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_cnn_u3_t32(const CnnU3Args& a, cudaStream_t s) {

@@ -248,7 +248,7 @@ struct Sizer {
     const Template& t;
     bool device_io;
     int64_t n5;
-    uint64_t t4_mult;  // 2 for TG_FP32_TC: T4 is kept TF32-split (big and small parts)
+    uint64_t t4_mult;  // 2 for TG_FP32_TC: T2 and T4 are kept TF32-split (big and small parts)
     // slot layout for B images x R output rows with the given row ranges
     SlotLayout slot(int64_t B, int64_t R, const Chunk& rg, bool streamed) const {
         SlotLayout s;
@@ -260,7 +260,7 @@ struct Sizer {
         const uint64_t f = 4;
         if (!device_io) put(s.in, (uint64_t)B * rg.in.n() * t.W * f);
         if (t.kind == Tmpl::Cnn) {
-            put(s.t2, (uint64_t)B * 8 * rg.t2.n() * t.w[2] * f);
+            put(s.t2, (uint64_t)B * 8 * rg.t2.n() * t.w[2] * f * t4_mult);
             put(s.t4, (uint64_t)B * 20 * rg.t4.n() * t.w[4] * f * t4_mult);
             if (!device_io) put(s.out, (uint64_t)B * 9 * R * t.w[5] * f);
             if (streamed) {
@@ -330,9 +330,9 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         all_pb += tc_bytes;
         nonbias_pb += tc_bytes;
     }
-    // 3xTF32 path: the TF32-split B operand of C5, kept with the parameters
+    // 3xTF32 path: the TF32-split B operands of C3 and C5, kept with the parameters
     if (t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC) {
-        tc_bytes = a256(cnn_k5_t32_bytes(t.n5));
+        tc_bytes = a256(cnn_k3_t32_bytes()) + a256(cnn_k5_t32_bytes(t.n5));
         all_pb += tc_bytes;
         nonbias_pb += tc_bytes;
     }
@@ -464,6 +464,8 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         p.k5tc_off = off;
         off += a256(cnn_k5_tc_bytes(t.n5));
     } else if (tc_bytes) {  // TG_FP32_TC
+        p.k3tc_off = off;
+        off += a256(cnn_k3_t32_bytes());
         p.k5tc_off = off;
         off += a256(cnn_k5_t32_bytes(t.n5));
     }
