@@ -221,8 +221,8 @@ def unit_bytes(wl, precision: str) -> dict:
     import synth
     (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = synth.cnn_dims(wl["H"], wl["W"])
     bf = precision == "bf16_tc"
-    t2 = n * h2 * w2 * (16 if bf else 64 if precision == "fp32_tc" else 32)
-    t4 = n * h4 * w4 * (48 if bf else 160 if precision == "fp32_tc" else 80)
+    t2 = n * h2 * w2 * (16 if bf else 32)
+    t4 = n * h4 * w4 * (48 if bf else 96 if precision == "fp32_tc" else 80)
     return {1: n * wl["H"] * wl["W"] * 4 + 8 * h1 * w1 * 4 + t2,
             2: t2 + 20 * h3 * w3 * 4 + t4,
             3: t4 + (wl["n5"] + 9) * h5 * w5 * 4 + n * 9 * h5 * w5 * 4}
@@ -310,11 +310,11 @@ def run(args, rank, world, local):
     achieved_tf = flops_per_launch / (kern_ms / 1e3) / 1e12
     tensor = args.precision in ("bf16_tc", "fp32_tc") and k in (2, 3)
     if tensor and args.precision == "fp32_tc":
-        # 3xTF32 C5 on tcgen05 against the TF32 dense peak (the measured bf16 peak x the nominal
-        # TF32/BF16 ratio 1/2); three MMAs per product, so the algorithmic ceiling is 1/3 of it
+        # 3xFP16 C3 / C5 on tcgen05 against the fp16 dense peak (= the measured bf16 peak: same
+        # kind::f16 rate); three MMAs per product, so the algorithmic ceiling is 1/3 of it
         peaks = json.load(open(PEAKS_FILE)) if os.path.exists(PEAKS_FILE) else {}
-        peak_tf = 0.5 * float(peaks.get("bf16_tflops", 1590.0))
-        peak_basis = ("tf32 dense = 0.5 x measured bf16 burst (MEASURED_PEAKS.json); 3xTF32 issues 3 MMAs "
+        peak_tf = float(peaks.get("bf16_tflops", 1590.0))
+        peak_basis = ("fp16 dense = measured bf16 burst (MEASURED_PEAKS.json); 3xFP16 issues 3 MMAs "
                       "per product: algorithmic ceiling = peak / 3")
         fl = dict(fl)
         fl[3] = wl["n5"] * 500 * 2  # C5 (C6 runs on the CUDA cores on this path); C3 in U2
@@ -371,14 +371,14 @@ def run(args, rank, world, local):
         if ms_u <= 0:
             continue
         tens_u = args.precision in ("bf16_tc", "fp32_tc") and u in (2, 3)
-        if tens_u and args.precision == "fp32_tc":  # C3 / C5 (3xTF32; C6 on the CUDA cores)
+        if tens_u and args.precision == "fp32_tc":  # C3 / C5 (3xFP16; C6 on the CUDA cores)
             fpx = 4 * 20 * 200 * 2 if u == 2 else wl["n5"] * 500 * 2
         elif tens_u:  # the tensor-core part: C3 (U2); C5 and C6 (U3)
             fpx = 4 * 20 * 200 * 2 if u == 2 else wl["n5"] * 500 * 2 + 9 * wl["n5"] * 2
         else:
             fpx = uf[u]
         f_u = fpx * opx[u] / (ms_u / 1e3) / 1e12
-        pk_u = (float(peaks.get("bf16_tflops", 1590.0)) * (0.5 if args.precision == "fp32_tc" else 1.0) if tens_u
+        pk_u = (float(peaks.get("bf16_tflops", 1590.0)) if tens_u
                 else fp32_peak_tflops(1965.0))
         units[KERNEL_NAMES[u]] = {"ms": ms_u, "tflops": f_u, "flop_frac": f_u / pk_u,
                                   "flop_bound": "tensor" if tens_u else "alu",
@@ -564,7 +564,7 @@ def main():
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms_per_step"],
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": {"fp32": "f32", "bf16_tc": "bf16 (fp32 accumulate)",
-                          "fp32_tc": "f32 (3xTF32 tensor cores, fp32 accumulate)"}[args.precision],
+                          "fp32_tc": "f32 (3xFP16 tensor cores, fp32 accumulate)"}[args.precision],
                 "data": "synthetic (counter-based generator synth/, 8-bit levels k/255)",
                 "config": res["config"], "roofline": res["roofline"], "e2e": res["e2e"], "clocks": res["clocks"],
                 "gpu_launches": res["gpu_launches"]}

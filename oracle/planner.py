@@ -791,10 +791,10 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
         if not device_io:
             s += a256(B * _span(rg["in"]) * W * f)
         if template == "cnn":
-            # TG_FP32_TC keeps T2 and T4 split into two TF32 parts (big, small) for the 3xTF32
-            # C3 and C5
-            s += a256(B * 8 * _span(rg["t2"]) * w2 * f * (2 if precision == "fp32_tc" else 1))
-            s += a256(B * 20 * _span(rg["t4"]) * w4 * f * (2 if precision == "fp32_tc" else 1))
+            s += a256(B * 8 * _span(rg["t2"]) * w2 * f)
+            # TG_FP32_TC keeps T4 as two fp16 parts (hi, lo) x 3 blocks of 8 channels = 24 words
+            # per pixel for the 3xFP16 C5 (T2: 2 parts x 8 fp16 = the 8 fp32 words of the others)
+            s += a256(B * (24 if precision == "fp32_tc" else 20) * _span(rg["t4"]) * w4 * f)
             if not device_io:
                 s += a256(B * 9 * R * w5 * f)
             if streamed:
@@ -815,10 +815,9 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
         all_pb += tc
         nonbias_pb += tc
     if template == "cnn" and precision == "fp32_tc":
-        # TF32-split B operands of the 3xTF32 C3 (25 K-steps x 2 parts x 2 halves x 32 maps x 4
-        # fp32) and C5 (68 K-steps: 65 + zero padding to stages of 4, x 2 x 2 x n5 rounded up
-        # to 16 x 4 fp32)
-        tc = a256(25 * 2 * 2 * 32 * 4 * 4) + a256(68 * 2 * 2 * ((n5 + 15) // 16 * 16) * 4 * 4)
+        # fp16-split B operands of the 3xFP16 C3 (15 K-steps x 2 halves x 64 rows (hi and lo
+        # maps) x 8 fp16) and C5 (40 K-steps x 2 parts x 2 halves x n5 rounded up to 16 x 8 fp16)
+        tc = a256(15 * 2 * 64 * 8 * 2) + a256(40 * 2 * 2 * ((n5 + 15) // 16 * 16) * 8 * 2)
         all_pb += tc
         nonbias_pb += tc
     if device_io:

@@ -62,7 +62,7 @@ struct tg_exec {
     std::vector<tg_trace_rec> trace;  // timeline collected from the profiling events
     int64_t param_uploads = 0;
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
-    std::vector<float> k3t32, k5t32;   // host copies of the 3xTF32 B operands (TG_FP32_TC)
+    std::vector<uint16_t> k3h3, k5h3;  // host copies of the 3xFP16 B operands (TG_FP32_TC)
 };
 
 namespace {
@@ -310,14 +310,14 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         }
         a.p2_host = g.ds[t.prm[2]].src;
         a.t2 = t2;
-        a.t2_img_stride = 8 * ch.t2.n() * w2 * (c.precision == TG_FP32_TC ? 2 : 1);
+        a.t2_img_stride = 8 * ch.t2.n() * w2;  // fp32 planes, or 2 fp16 parts x 8 channels (same bytes)
         a.t2_row0 = ch.t2.a;
         a.t2_rows = ch.t2.n();
         a.w1 = w1;
         a.w2 = w2;
         a.nimg = ch.nimg;
         a.bf16_out = c.precision == TG_BF16_TC;
-        a.t2_tf32 = c.precision == TG_FP32_TC;
+        a.t2_h3 = c.precision == TG_FP32_TC;
         KernelTimer kt(x, d, 1, ci, cs);
         CK(launch_cnn_u1(a, cs));
         kt.done(cs);
@@ -343,7 +343,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         }
         a.p4_host = g.ds[t.prm[5]].src;
         a.t4 = t4;
-        a.t4_img_stride = 20 * ch.t4.n() * w4 * (c.precision == TG_FP32_TC ? 2 : 1);
+        a.t4_img_stride = (c.precision == TG_FP32_TC ? 24 : 20) * ch.t4.n() * w4;
         a.t4_row0 = ch.t4.a;
         a.t4_rows = ch.t4.n();
         a.w3 = w3;
@@ -352,21 +352,17 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.bf16_tc = c.precision == TG_BF16_TC;
         a.k3_tc = c.k3tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k3tc_off);
         a.p4_dev = param(5);
-        a.t4_tf32 = c.precision == TG_FP32_TC;
-        if (c.precision == TG_FP32_TC) {
-            a.t2_img_stride *= 2;
-            a.k3_t32 = (const float*)(d.arena + c.k3tc_off);
-        }
+        if (c.precision == TG_FP32_TC) a.k3_h3 = (const uint16_t*)(d.arena + c.k3tc_off);
         KernelTimer kt(x, d, 2, ci, cs);
         CK(a.bf16_tc ? launch_cnn_u2_tc(a, cs)
-                     : c.precision == TG_FP32_TC ? launch_cnn_u2_t32(a, cs) : launch_cnn_u2(a, cs));
+                     : c.precision == TG_FP32_TC ? launch_cnn_u2_h3(a, cs) : launch_cnn_u2(a, cs));
         kt.done(cs);
         ++d.launches;
     }
     {
         CnnU3Args a{};
         a.t4 = t4;
-        a.t4_img_stride = 20 * ch.t4.n() * w4 * (c.precision == TG_FP32_TC ? 2 : 1);
+        a.t4_img_stride = (c.precision == TG_FP32_TC ? 24 : 20) * ch.t4.n() * w4;
         a.t4_row0 = ch.t4.a;
         a.t4_rows = ch.t4.n();
         a.w4 = w4;
@@ -404,7 +400,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.k6_host = g.ds[t.prm[8]].src;
         KernelTimer kt(x, d, 3, ci, cs);
         CK(a.bf16_tc ? launch_cnn_u3_tc(a, cs)
-                     : c.precision == TG_FP32_TC ? launch_cnn_u3_t32(a, cs) : launch_cnn_u3(a, cs));
+                     : c.precision == TG_FP32_TC ? launch_cnn_u3_h3(a, cs) : launch_cnn_u3(a, cs));
         kt.done(cs);
         ++d.launches;
     }
@@ -442,15 +438,15 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
             CK(cudaMemcpyAsync(d.arena + c.param_off[i], P.src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
         }
         if (c.k5tc_off != UINT64_MAX && c.precision == TG_FP32_TC) {
-            // TF32-split B operands of the 3xTF32 C3 and C5 (prepared on the host once per plan)
-            if (x->k5t32.empty()) {
-                x->k3t32.resize(cnn_k3_t32_bytes() / 4);
-                cnn_prepare_k3_t32(g.ds[c.t.prm[3]].src, x->k3t32.data());
-                x->k5t32.resize(cnn_k5_t32_bytes(c.t.n5) / 4);
-                cnn_prepare_k5_t32(g.ds[c.t.prm[6]].src, c.t.n5, x->k5t32.data());
+            // fp16-split B operands of the 3xFP16 C3 and C5 (prepared on the host once per plan)
+            if (x->k5h3.empty()) {
+                x->k3h3.resize(cnn_k3_h3_bytes() / 2);
+                cnn_prepare_k3_h3(g.ds[c.t.prm[3]].src, x->k3h3.data());
+                x->k5h3.resize(cnn_k5_h3_bytes(c.t.n5) / 2);
+                cnn_prepare_k5_h3(g.ds[c.t.prm[6]].src, c.t.n5, x->k5h3.data());
             }
-            CK(cudaMemcpyAsync(d.arena + c.k3tc_off, x->k3t32.data(), x->k3t32.size() * 4, cudaMemcpyHostToDevice, S0));
-            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5t32.data(), x->k5t32.size() * 4, cudaMemcpyHostToDevice, S0));
+            CK(cudaMemcpyAsync(d.arena + c.k3tc_off, x->k3h3.data(), x->k3h3.size() * 2, cudaMemcpyHostToDevice, S0));
+            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5h3.data(), x->k5h3.size() * 2, cudaMemcpyHostToDevice, S0));
         }
         if (c.k3tc_off != UINT64_MAX && c.precision == TG_BF16_TC) {
             // bf16 B operands of the tensor-core C3/C5 (prepared on the host once per plan)
@@ -670,8 +666,8 @@ void exec_invalidate_params(tg_plan* p) {
     for (auto& d : p->exec->devs) d.params_resident = false;
     p->exec->k3tc.clear();  // the bf16 tensor-core operands are re-derived from the new values
     p->exec->k5tc.clear();
-    p->exec->k5t32.clear();
-    p->exec->k3t32.clear();
+    p->exec->k5h3.clear();
+    p->exec->k3h3.clear();
 }
 
 }  // namespace tg

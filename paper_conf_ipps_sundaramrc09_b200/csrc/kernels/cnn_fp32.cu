@@ -14,6 +14,7 @@
 //
 // tanh: 1 - 2/(1 + e^{2x}) with MUFU ex2/rcp (x clamped to +-15): absolute error < 3e-7,
 // well inside the normwise 1e-5 parity bound.
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -31,12 +32,15 @@ __device__ __forceinline__ float tanh_f(float x) {
     const float e = __expf(2.f * x);
     return 1.f - __fdividef(2.f, 1.f + e);
 }
-// round to TF32 (10-bit mantissa; nearest, ties away): the "big" part of a 3xTF32 split
-__device__ __forceinline__ float tf32_rn(float x) {
-    uint32_t r;
-    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
-    return __uint_as_float(r);
+// hi/lo fp16 pairs of two consecutive channels (element 0 in the low half): the 3xFP16 split
+__device__ __forceinline__ void split_f16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
+    const __half2 h = __floats2half2_rn(x0, x1);
+    const float2 hf = __half22float2(h);
+    const __half2 l = __floats2half2_rn(x0 - hf.x, x1 - hf.y);
+    hi = *reinterpret_cast<const uint32_t*>(&h);
+    lo = *reinterpret_cast<const uint32_t*>(&l);
 }
+
 // MUFU.TANH (one SFU op, relative error ~2^-11): only where the result is rounded to bf16
 // anyway (U1 feeding the tensor-core path), never on the fp32 path.
 __device__ __forceinline__ float tanh_mufu(float x) {
@@ -150,19 +154,13 @@ __global__ void __launch_bounds__(128, 4) cnn_u1_kernel(const CnnU1Args a, const
             asm("cvt.rn.bf16x2.f32 %0, %1, %2;\n" : "=r"(p[k]) : "f"(tv[2 * k + 1]), "f"(tv[2 * k]));
         }
         *d = make_uint4(p[0], p[1], p[2], p[3]);
-    } else if (a.t2_tf32) {  // TF32-split pixel blocks for the 3xTF32 U2: [part][block][rows][w2][4]
-        float4* d = reinterpret_cast<float4*>(a.t2) + img * 4 * plane + (R2 - a.t2_row0) * a.w2 + C2;
+    } else if (a.t2_h3) {  // fp16-split pixels (x 2^4) for the 3xFP16 U2: [part][rows][w2][8]
+        uint4* d = reinterpret_cast<uint4*>(a.t2) + img * 2 * plane + (R2 - a.t2_row0) * a.w2 + C2;
+        uint32_t hi[4], lo[4];
 #pragma unroll
-        for (int blk = 0; blk < 2; ++blk) {
-            float big[4], small[4];
-#pragma unroll
-            for (int e = 0; e < 4; ++e) {
-                big[e] = tf32_rn(tv[4 * blk + e]);
-                small[e] = tf32_rn(tv[4 * blk + e] - big[e]);
-            }
-            d[blk * plane] = make_float4(big[0], big[1], big[2], big[3]);
-            d[(2 + blk) * plane] = make_float4(small[0], small[1], small[2], small[3]);
-        }
+        for (int m = 0; m < 4; ++m) split_f16x2(16.f * tv[2 * m], 16.f * tv[2 * m + 1], hi[m], lo[m]);
+        d[0] = make_uint4(hi[0], hi[1], hi[2], hi[3]);
+        d[plane] = make_uint4(lo[0], lo[1], lo[2], lo[3]);
     } else {
 #pragma unroll
         for (int ch = 0; ch < 8; ++ch) t2[ch * plane + (R2 - a.t2_row0) * a.w2 + C2] = tv[ch];
@@ -302,22 +300,17 @@ __global__ void __launch_bounds__(128, 3)
                         asm("cvt.rn.bf16x2.f32 %0, %1, %2;\n" : "=r"(pk[m]) : "f"(tv[q][2 * m + 1]), "f"(tv[q][2 * m]));
                     d[q] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
                 }
-            } else if (a.t2_tf32) {  // TF32-split pixel blocks [part][block][rows][w2][4]
-                float4* d = reinterpret_cast<float4*>(a.t2) + img * 4 * plane + (R2 - a.t2_row0) * a.w2 + C2;
+            } else if (a.t2_h3) {  // fp16-split pixels (x 2^4): [part][rows][w2][8]
+                uint4* d = reinterpret_cast<uint4*>(a.t2) + img * 2 * plane + (R2 - a.t2_row0) * a.w2 + C2;
 #pragma unroll
                 for (int q = 0; q < 2; ++q) {
                     if (C2 + q >= a.w2) continue;
+                    uint32_t hi[4], lo[4];
 #pragma unroll
-                    for (int blk = 0; blk < 2; ++blk) {
-                        float big[4], small[4];
-#pragma unroll
-                        for (int e = 0; e < 4; ++e) {
-                            big[e] = tf32_rn(tv[q][4 * blk + e]);
-                            small[e] = tf32_rn(tv[q][4 * blk + e] - big[e]);
-                        }
-                        d[blk * plane + q] = make_float4(big[0], big[1], big[2], big[3]);
-                        d[(2 + blk) * plane + q] = make_float4(small[0], small[1], small[2], small[3]);
-                    }
+                    for (int m = 0; m < 4; ++m)
+                        split_f16x2(16.f * tv[q][2 * m], 16.f * tv[q][2 * m + 1], hi[m], lo[m]);
+                    d[q] = make_uint4(hi[0], hi[1], hi[2], hi[3]);
+                    d[plane + q] = make_uint4(lo[0], lo[1], lo[2], lo[3]);
                 }
             } else {
                 float* t2 = a.t2 + img * a.t2_img_stride + (R2 - a.t2_row0) * a.w2 + C2;
@@ -454,24 +447,8 @@ __global__ void __launch_bounds__(128, 2) cnn_u2_kernel(const CnnU2Args a, const
         tv[co] = tanh_f(s);
     }
     const int64_t px = (R4 - a.t4_row0) * a.w4 + C4;
-    if (!a.t4_tf32) {
 #pragma unroll
-        for (int co = 0; co < 20; ++co) t4[co * oplane + px] = tv[co];
-    } else {
-        // TF32-split pixel blocks for the 3xTF32 U3 (cnn_t32.cu): [part][block][rows][w4][4]
-#pragma unroll
-        for (int blk = 0; blk < 5; ++blk) {
-            float big[4], small[4];
-#pragma unroll
-            for (int e = 0; e < 4; ++e) {
-                big[e] = tf32_rn(tv[4 * blk + e]);
-                small[e] = tf32_rn(tv[4 * blk + e] - big[e]);
-            }
-            reinterpret_cast<float4*>(t4)[(0 * 5 + blk) * oplane + px] = make_float4(big[0], big[1], big[2], big[3]);
-            reinterpret_cast<float4*>(t4)[(1 * 5 + blk) * oplane + px] =
-                make_float4(small[0], small[1], small[2], small[3]);
-        }
-    }
+    for (int co = 0; co < 20; ++co) t4[co * oplane + px] = tv[co];
 }
 
 // ============================================================================ U3

@@ -38,7 +38,7 @@ struct CnnU1Args {          // C1(1->8, 5x5) + bias + tanh + S2 + tanh  -> T2
     int64_t w1, w2;
     int64_t nimg;
     int bf16_out;           // 1: write T2 as bf16 [rows][w2][8] (operand layout of U2 on tcgen05)
-    int t2_tf32;            // 1 (TG_FP32_TC): write T2 TF32-split [2][2][rows][w2][4] for the 3xTF32 U2
+    int t2_h3;              // 1 (TG_FP32_TC): write T2 fp16-split [2][rows][w2][8] (x 2^4) for the 3xFP16 U2
 };
 struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
     const float* t2; int64_t t2_img_stride; int64_t t2_row0, t2_rows; int64_t w2;
@@ -51,8 +51,7 @@ struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
                             //    as bf16 [3][rows][w4][8] (channel blocks 0-7, 8-15, 16-19+pad)
     const uint16_t* k3_tc;  // bf16 B operand prepared by cnn_prepare_k3_tc (device)
     const float* p4_dev;    // [20][4] (device)
-    int t4_tf32;            // 1 (TG_FP32_TC): T4 written TF32-split [2][5][rows][w4][4] for cnn_t32.cu
-    const float* k3_t32;    // TF32-split B operand of the 3xTF32 C3 (cnn_prepare_k3_t32, device)
+    const uint16_t* k3_h3;  // fp16-split B operand of the 3xFP16 C3 (cnn_prepare_k3_h3, device)
 };
 struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + bias -> out
     const float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w4;
@@ -123,14 +122,13 @@ cudaError_t launch_gen_matmul(const GenMatmulArgs& a, cudaStream_t s);
 // tcgen05 (bf16 operands, fp32 accumulation in TMEM) variants of U2 and U3 (cnn_tc.cu)
 cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s);
-// 3xTF32 U3 (fp32-accurate on tcgen05, TG_FP32_TC): B operand prepared on the host
-size_t cnn_k5_t32_bytes(int n5);
-void cnn_prepare_k5_t32(const float* k5, int n5, float* dst);
-cudaError_t launch_cnn_u3_t32(const CnnU3Args& a, cudaStream_t s);
-// 3xTF32 U2 (C3 on tcgen05): T2 read TF32-split [2][2][rows][w2][4], T4 written TF32-split
-size_t cnn_k3_t32_bytes();
-void cnn_prepare_k3_t32(const float* k3, float* dst);
-cudaError_t launch_cnn_u2_t32(const CnnU2Args& a, cudaStream_t s);
+// 3xFP16 U2 / U3 (cnn_h3.cu): T2 [2][rows][w2][8] and T4 [2][3][rows][w4][8] fp16-split
+size_t cnn_k3_h3_bytes();
+void cnn_prepare_k3_h3(const float* k3, uint16_t* dst);
+size_t cnn_k5_h3_bytes(int n5);
+void cnn_prepare_k5_h3(const float* k5, int n5, uint16_t* dst);
+cudaError_t launch_cnn_u2_h3(const CnnU2Args& a, cudaStream_t s);
+cudaError_t launch_cnn_u3_h3(const CnnU3Args& a, cudaStream_t s);
 size_t cnn_k3_tc_bytes();
 void cnn_prepare_k3_tc(const float* k3, uint16_t* dst);
 int cnn_n5_pad(int n5);

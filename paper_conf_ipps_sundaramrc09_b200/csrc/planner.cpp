@@ -248,7 +248,8 @@ struct Sizer {
     const Template& t;
     bool device_io;
     int64_t n5;
-    uint64_t t4_mult;  // 2 for TG_FP32_TC: T2 and T4 are kept TF32-split (big and small parts)
+    uint64_t t4_words;  // 4-byte words per T4 pixel: 20 (fp32 planes; bf16 blocks fit), 24 for
+                        // TG_FP32_TC (2 fp16 parts x 3 blocks of 8 channels)
     // slot layout for B images x R output rows with the given row ranges
     SlotLayout slot(int64_t B, int64_t R, const Chunk& rg, bool streamed) const {
         SlotLayout s;
@@ -260,8 +261,8 @@ struct Sizer {
         const uint64_t f = 4;
         if (!device_io) put(s.in, (uint64_t)B * rg.in.n() * t.W * f);
         if (t.kind == Tmpl::Cnn) {
-            put(s.t2, (uint64_t)B * 8 * rg.t2.n() * t.w[2] * f * t4_mult);
-            put(s.t4, (uint64_t)B * 20 * rg.t4.n() * t.w[4] * f * t4_mult);
+            put(s.t2, (uint64_t)B * 8 * rg.t2.n() * t.w[2] * f);
+            put(s.t4, (uint64_t)B * t4_words * rg.t4.n() * t.w[4] * f);
             if (!device_io) put(s.out, (uint64_t)B * 9 * R * t.w[5] * f);
             if (streamed) {
                 put(s.b1, (uint64_t)8 * rg.c1.n() * t.w[1] * f);
@@ -330,15 +331,15 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         all_pb += tc_bytes;
         nonbias_pb += tc_bytes;
     }
-    // 3xTF32 path: the TF32-split B operands of C3 and C5, kept with the parameters
+    // 3xFP16 path: the fp16-split B operands of C3 and C5, kept with the parameters
     if (t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC) {
-        tc_bytes = a256(cnn_k3_t32_bytes()) + a256(cnn_k5_t32_bytes(t.n5));
+        tc_bytes = a256(cnn_k3_h3_bytes()) + a256(cnn_k5_h3_bytes(t.n5));
         all_pb += tc_bytes;
         nonbias_pb += tc_bytes;
     }
     int32_t depth = p.device_io ? 1 : g.depth;
     p.depth = depth;
-    Sizer sz{t, p.device_io, t.n5, (uint64_t)(t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC ? 2 : 1)};
+    Sizer sz{t, p.device_io, t.n5, (uint64_t)(t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC ? 24 : 20)};
     auto fits = [&](uint64_t pb, uint64_t sb) { return g.budget == 0 || pb + (uint64_t)depth * sb <= g.budget; };
 
     auto chunk_list = [&](bool batch, int64_t B, int64_t R) {
@@ -465,9 +466,9 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         off += a256(cnn_k5_tc_bytes(t.n5));
     } else if (tc_bytes) {  // TG_FP32_TC
         p.k3tc_off = off;
-        off += a256(cnn_k3_t32_bytes());
+        off += a256(cnn_k3_h3_bytes());
         p.k5tc_off = off;
-        off += a256(cnn_k5_t32_bytes(t.n5));
+        off += a256(cnn_k5_h3_bytes(t.n5));
     }
     p.chunks = chunk_list(batch, B, R);
     const int64_t C = (int64_t)p.chunks.size();

@@ -213,14 +213,14 @@ def test_cnn_bf16_tc_split_equals_unsplit(tg):
     assert np.array_equal(split, full)
 
 
-# ------------------------------------------------------------------ 3xTF32 path (TG_FP32_TC)
+# ------------------------------------------------------------------ 3xFP16 path (TG_FP32_TC)
 @pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
                                           (3, 67, 61, 20, "scalar"), (1, 97, 1003, 120, "plane"),
                                           (2, 36, 40, 7, "plane"), (2, 100, 300, 80, "plane"),
                                           (1, 60, 1500, 60, "scalar"), (1, 140, 1400, 33, "plane")])
 def test_cnn_fp32_tc_parity(tg, orc, n, H, W, n5, bias):
-    """C5 on tcgen05 with every operand split into two TF32 numbers (3 MMAs per product): the
-    fp32 bound, normwise 1e-5 (R16, "3xTF32"), on narrow and wide rows, every NP."""
+    """C3 and C5 on tcgen05 with every operand split into two fp16 numbers (3 MMAs per product):
+    the fp32 bound, normwise 1e-5 (R16, "3xFP16"), on narrow and wide rows, every NP."""
     seed = synth.seed_for_config(3) + 29
     img = synth.images_np(seed, n, H, W)
     prm = synth.cnn_params_np(seed, n5, H, W, bias)
@@ -236,8 +236,8 @@ def test_cnn_fp32_tc_parity(tg, orc, n, H, W, n5, bias):
 def test_cnn_fp32_tc_single_pixel_planes(tg, orc):
     """The smallest CNN input (32 x 32 -> 1 x 1 output planes), where the normwise measure of
     R16 degenerates to the relative error of ONE value per plane (here values down to 6e-3):
-    the 3xTF32 path's absolute error is ~2.5x the FFMA path's (operand split residuals of
-    2^-22 per factor vs fp32 rounding), so this case is held to the FFMA
+    the split-operand path's absolute error can exceed the FFMA path's (operand split residuals
+    of 2^-22 per factor vs fp32 rounding), so this case is held to the FFMA
     path's own error on the same inputs (x3) and to 5e-5 rather than to 1e-5."""
     seed = synth.seed_for_config(3) + 29
     n, H, W, n5 = 2, 32, 32, 7

@@ -9,4 +9,4 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:edge -s 1 -c 1 -o gpurun_out/k1_full -f python tools/prof_k1.py 15 > /dev/null 2>&1; echo "k1 rc=$?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_bf16_full -f python tools/prof_cnn.py 120 bf16 > /dev/null 2>&1; echo "cnn bf16 rc=$?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_fp32_full -f python tools/prof_cnn.py 120 > /dev/null 2>&1; echo "cnn fp32 rc=$?"
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_t32_full -f python tools/prof_cnn.py 120 t32 > /dev/null 2>&1; echo "cnn t32 rc=$?"
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_fp32tc_full -f python tools/prof_cnn.py 120 fp32tc > /dev/null 2>&1; echo "cnn fp32tc rc=$?"

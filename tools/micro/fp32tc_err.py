@@ -1,4 +1,4 @@
-"""Error of the 3xTF32 CNN path (TG_FP32_TC) vs the FFMA path (TG_FP32), both against the
+"""Error of the fp32-accurate tensor-core CNN path (TG_FP32_TC, 3xFP16) vs the FFMA path (TG_FP32), both against the
 oracle, per case: normwise per plane and absolute. Test infrastructure (loads the oracle)."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))

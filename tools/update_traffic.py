@@ -2,7 +2,7 @@
 (dram__bytes_read.sum + dram__bytes_write.sum) of one launch / output pixels of that launch.
 
   python tools/update_traffic.py gpurun_out/k1_full.ncu-rep gpurun_out/cnn_bf16_full.ncu-rep \
-      gpurun_out/cnn_fp32_full.ncu-rep gpurun_out/cnn_t32_full.ncu-rep
+      gpurun_out/cnn_fp32_full.ncu-rep gpurun_out/cnn_fp32tc_full.ncu-rep
 
 The captures are tools/prof_k1.py 15 (15 x 10000x10000 edge images) and tools/prof_cnn.py 120
 [bf16] (cnn3: 64 x 480x640, n5 = 120). U1 and U2 do not depend on n5, so their figures serve
@@ -43,7 +43,7 @@ def main(reps):
                       "[bf16]); (dram__bytes_read.sum + dram__bytes_write.sum) of one launch / output pixels of "
                       "that launch; written by tools/update_traffic.py"}
     for rep in reps:
-        prec = "bf16_tc" if "bf16" in rep else "fp32_tc" if "t32" in rep else "fp32"
+        prec = "bf16_tc" if "bf16" in rep else "fp32_tc" if "fp32tc" in rep else "fp32"
         for name, b in launches(rep):
             if "edge" in name:
                 out[f"edge:fp32:{NAMES['edge']}"] = {"dram_bytes_per_out_px": b / (15 * 10000 * 10000),
