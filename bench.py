@@ -394,7 +394,7 @@ def run(args, rank, world, local):
     y_host = torch.empty(out_shape, dtype=torch.float32).pin_memory()
     g2 = build_graph(tg, wl, x_host, y_host, False, params)
     g2.set(budget=wl["budget"], torch_runtime=True, precision=args.precision_code,
-           max_chunk_px=args.max_chunk_px)
+           max_chunk_px=args.max_chunk_px, depth=args.depth)
     p2 = g2.plan()
     st = p2.stats()
     js = p2.json()
@@ -545,6 +545,8 @@ def main():
     ap.add_argument("--template", default="edge", choices=["edge", "cnn4", "cnn3", "cnn3s"])
     ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16_tc", "fp32_tc"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--depth", type=int, default=None,
+                    help="pipeline slots of the e2e plan (tg_set_chunking; default: the library's 3)")
     ap.add_argument("--max-chunk-px", type=int, default=None,
                     help="chunk cap of the e2e plan (tg_set_chunking; default: the library's 2^25)")
     ap.add_argument("--per-template", default=None,
