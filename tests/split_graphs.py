@@ -269,3 +269,62 @@ def lib_graph(spec, out, budget=0, torch_runtime=False):
     g.output(made[spec.output], out)
     g.set(budget=budget, torch_runtime=torch_runtime)
     return g
+
+
+# ------------------------------------------------------------------------------ random graphs
+def random_spec(seed: int) -> Spec:
+    """A random operator graph for fuzzing the splitting rule: a chain of 3-8 operators over a
+    small image with side branches (elementwise ops of two same-shape data structures), VALID
+    and SAME convolutions (1/3/5-tap kernels, 1-3 maps, bias plane / scalar / none), tanh,
+    remap, abs, affine, subsample and -- on single-plane data -- matmul."""
+    rng = np.random.default_rng(seed)
+    s = Spec()
+    n, c = int(rng.integers(1, 3)), int(rng.integers(1, 3))
+    if rng.random() < 0.3:
+        n = c = 1
+    h, w = int(rng.integers(24, 90)), int(rng.integers(12, 40))
+    x = s.ds((n, c, h, w), "input", rng.random((n, c, h, w)))
+    cur = x
+    pool = [x]
+    for _ in range(int(rng.integers(3, 9))):
+        N, C, H, W = s.shapes[cur]
+        r = rng.random()
+        if r < 0.3 and H >= 6 and W >= 6:
+            kh = int(rng.choice([1, 3, 5]))
+            co = int(rng.integers(1, 4))
+            pad = "same" if rng.random() < 0.5 else "valid"
+            k = s.ds((co, C, kh, kh), "param", rng.uniform(-0.5, 0.5, (co, C, kh, kh)))
+            ho, wo = (H, W) if pad == "same" else (H - kh + 1, W - kh + 1)
+            bk = rng.random()
+            if bk < 0.4:
+                b = s.ds((1, co, ho, wo), "param", rng.uniform(-0.1, 0.1, (1, co, ho, wo)))
+            elif bk < 0.7:
+                b = s.ds((co,), "param", rng.uniform(-0.1, 0.1, (co,)))
+            else:
+                b = -1
+            cur = s.conv(cur, k, b, pad)
+        elif r < 0.45:
+            cur = s.elem("tanh", [cur])
+        elif r < 0.55:
+            cur = s.elem(str(rng.choice(["neg", "abs"])), [cur])
+        elif r < 0.62:
+            cur = s.elem("affine", [cur], a=float(rng.uniform(-2, 2)), b=float(rng.uniform(-1, 1)))
+        elif r < 0.77:
+            same = [d for d in pool if s.shapes[d] == s.shapes[cur] and d != cur]
+            if same:
+                other = int(rng.choice(same))
+                cur = s.elem(str(rng.choice(["add", "max"])), [cur, other] if rng.random() < 0.5 else [other, cur])
+            else:
+                cur = s.elem("tanh", [cur])
+        elif r < 0.9 and H >= 4 and W >= 4:
+            p = s.ds((C, 2, 2), "param", rng.uniform(-0.5, 0.5, (C, 2, 2)))
+            cur = s.sub(cur, p)
+        elif N == 1 and C == 1:
+            m = int(rng.integers(3, 30))
+            B = s.ds((1, 1, W, m), "param", rng.uniform(-1, 1, (1, 1, W, m)))
+            cur = s.matmul(cur, B)
+        else:
+            cur = s.elem("tanh", [cur])
+        pool.append(cur)
+    s.set_output(cur)
+    return s

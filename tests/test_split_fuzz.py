@@ -1,0 +1,70 @@
+"""Fuzzing the splitting rule (reading R19) on random operator graphs (conv VALID/SAME with
+plane/scalar/no bias, tanh, remap, abs, affine, add/max branches, subsample, matmul):
+  * CPU: the library's TG_PER_OP plan through the C ABI equals the oracle's per_op_plan
+    bit for bit (pieces, piece operators, k, DFS order, transfer trace, capacity, arena
+    offsets), or both find the budget infeasible; the oracle's pieces executed by the numpy
+    piece executor reproduce the unsplit graph bit for bit;
+  * GPU: the library executes the split plan to the numpy evaluation of the unsplit graph
+    within 1e-5 normwise and bit-identical to its own unsplit execution."""
+import numpy as np
+import pytest
+
+from split_graphs import lib_graph, random_spec, run_split, run_unsplit
+
+SEEDS = list(range(40))
+FRACS = [0.5, 0.3, 0.15]
+
+
+def budget_of(spec, frac):
+    return int(spec.total_bytes() * frac) // 256 * 256
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+def test_random_graph_plan_matches_oracle(seed):
+    from oracle import planner as P
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    from test_split_plan import compare
+    spec = random_spec(seed)
+    ref = run_unsplit(spec)
+    for frac in FRACS:
+        budget = budget_of(spec, frac)
+        try:
+            r = P.per_op_plan(spec.shapes, spec.kinds, spec.nodes, spec.output, budget)
+        except ValueError:
+            out = np.zeros(spec.shapes[spec.output], np.float32)
+            with pytest.raises(tg.TGError) as e:
+                lib_graph(spec, out, budget=budget).plan(tg.TG_PER_OP)
+            assert e.value.code in (tg.TG_E_INFEASIBLE, tg.TG_E_UNSUPPORTED)
+            continue
+        compare(spec, budget)
+        assert np.array_equal(run_split(spec, r), ref)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("seed", SEEDS[:16])
+def test_random_graph_split_gpu(seed):
+    from gpu_util import need_gpu, normwise, torch
+    need_gpu()
+    from oracle import planner as P
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    torch.cuda.set_device(0)
+    spec = random_spec(seed)
+    ref = run_unsplit(spec)
+    full = np.full(spec.shapes[spec.output], np.nan, np.float32)
+    g = lib_graph(spec, full, torch_runtime=True)
+    g.plan(tg.TG_PER_OP).execute()
+    assert normwise(full.reshape(-1, *full.shape[-2:]), ref.reshape(-1, *ref.shape[-2:])) <= 1e-5
+    ran = 0
+    for frac in FRACS:
+        budget = budget_of(spec, frac)
+        try:
+            P.per_op_plan(spec.shapes, spec.kinds, spec.nodes, spec.output, budget)
+        except ValueError:
+            continue
+        out = np.full_like(full, np.nan)
+        g = lib_graph(spec, out, budget=budget, torch_runtime=True)
+        p = g.plan(tg.TG_PER_OP)
+        p.execute()
+        assert np.array_equal(out, full), frac
+        ran += 1
+    assert ran >= 1
