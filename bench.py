@@ -406,7 +406,9 @@ def run(args, rank, world, local):
     assert torch.equal(y_host[0].to(dev), y_ref[0]) and torch.equal(y_host[-1].to(dev), y_ref[1]), \
         "streamed != resident"
     del y_ref
-    p2.profiling(True)
+    # the e2e number is timed with the library's per-launch profiling OFF (its events cost up to
+    # 25 % of a streamed step); a second, profiled pass of the same steps gives the breakdown
+    # (kernel / copy busy times, overlap) reported beside it
     l2 = p2.launches()
     barrier(world)
     f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -419,8 +421,17 @@ def run(args, rank, world, local):
     wall = (time.perf_counter() - t0) / args.steps
     ms2 = f0.elapsed_time(f1) / args.steps
     launches2 = p2.launches() - l2
-    tim2 = p2.timing()
     ms2_max = max_over_ranks(ms2, world)
+    p2.profiling(True)
+    g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    g0.record(cs2)
+    for _ in range(args.steps):
+        p2.execute(blocking=False)
+    g1.record(cs2)
+    torch.cuda.synchronize()
+    ms2_prof = g0.elapsed_time(g1) / args.steps
+    tim2 = p2.timing()
+    p2.profiling(False)
     e2e_value = world * px / (ms2_max / 1e3) / 1e6
     # parameters stay resident after the first execution: a timed step moves the images,
     # the streamed bias rows (if any) and the outputs
@@ -431,6 +442,7 @@ def run(args, rank, world, local):
            "bytes_vs_lower_bound": (h2d + d2h) / st["io_lower_bound_bytes"],
            "budget_bytes": wl["budget"], "arena_bytes": st["peak_device_bytes"][0], "chunks": st["n_chunks"],
            "split": js["split"], "bias": js["bias"], "gpu_launches": launches2,
+           "profiled_ms_per_step": ms2_prof,
            "kernel_ms_per_step": sum(tim2["kernel_ms"]) / args.steps,
            "h2d_ms_per_step": tim2["h2d_ms"] / args.steps, "d2h_ms_per_step": tim2["d2h_ms"] / args.steps}
     # SURVEY 8(d) overlap = (sum copy + sum kernel - wall) / min(sum copy, sum kernel), with the copy
@@ -438,8 +450,9 @@ def run(args, rank, world, local):
     # copy direction, kernels} is completely hidden behind the longer, 0 = fully serialised
     s_copy = max(tim2["h2d_ms"], tim2["d2h_ms"]) / args.steps
     s_kern = sum(tim2["kernel_ms"]) / args.steps
-    e2e["overlap"] = (s_copy + s_kern - ms2) / max(min(s_copy, s_kern), 1e-9)
-    e2e["overlap_def"] = "(max(H2D, D2H) busy + kernel busy - step) / min(max(H2D, D2H) busy, kernel busy)"
+    e2e["overlap"] = (s_copy + s_kern - ms2_prof) / max(min(s_copy, s_kern), 1e-9)
+    e2e["overlap_def"] = ("(max(H2D, D2H) busy + kernel busy - step) / min(max(H2D, D2H) busy, kernel busy), "
+                          "all from the profiled pass")
     if rank == 0:
         link = host_link_peak(local)
         # link roofline: each direction at its solo peak, both together at the measured

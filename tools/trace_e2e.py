@@ -41,7 +41,7 @@ else:
     y = torch.empty(out_shape, dtype=torch.float32).pin_memory()
 g = bench.build_graph(tg, wl, x, y, a.device, params)
 g.set(budget=0 if a.device else wl["budget"], torch_runtime=True,
-      precision=tg.TG_FP32 if a.precision == "fp32" else tg.TG_BF16_TC,
+      precision={"fp32": tg.TG_FP32, "fp32_tc": tg.TG_FP32_TC, "bf16_tc": tg.TG_BF16_TC}[a.precision],
       max_chunk_px=a.max_chunk_px, depth=a.depth)
 p = g.plan()
 for _ in range(3):
