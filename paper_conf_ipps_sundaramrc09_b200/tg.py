@@ -35,6 +35,7 @@ TG_MAX, TG_SUM, TG_MAXABS = 0, 1, 2
 TG_BIAS_PLANE, TG_BIAS_SCALAR = 0, 1
 TG_FP32, TG_BF16_TC, TG_FP32_TC = 0, 1, 2
 TG_FUSED, TG_PER_OP, TG_BASELINE = 0, 1, 2
+TG_OPLIB_CONV, TG_OPLIB_ELEM, TG_OPLIB_SUB, TG_OPLIB_MATMUL = 0, 1, 2, 3
 
 _STATUS = {v: k for k, v in dict(TG_E_ARG=-1, TG_E_SHAPE=-2, TG_E_INFEASIBLE=-3, TG_E_CUDA=-4,
                                    TG_E_OOM=-5, TG_E_STATE=-6, TG_E_UNSUPPORTED=-7).items()}
@@ -58,6 +59,22 @@ STREAM_FN = ctypes.CFUNCTYPE(vp, c_i32, c_i32, vp)
 
 class tg_runtime(ctypes.Structure):
     _fields_ = [("alloc", ALLOC_FN), ("free", FREE_FN), ("stream", STREAM_FN), ("ctx", vp)]
+
+
+class tg_oplib_seg(ctypes.Structure):
+    _fields_ = [("p", ctypes.c_void_p), ("r0", ctypes.c_int64), ("r1", ctypes.c_int64)]
+
+
+class tg_oplib_view(ctypes.Structure):
+    _fields_ = [("seg", tg_oplib_seg * 8), ("nseg", ctypes.c_int32)]
+
+
+class tg_oplib_op(ctypes.Structure):
+    """One operator piece for tg_oplib_run (include/tg.h "operator library")."""
+    _fields_ = [("kind", ctypes.c_int32), ("nin", ctypes.c_int32), ("in_", tg_oplib_view * 16),
+                ("in_dims", (ctypes.c_int64 * 4) * 16), ("y", ctypes.c_void_p), ("y_dims", ctypes.c_int64 * 4),
+                ("r0", ctypes.c_int64), ("r1", ctypes.c_int64), ("pad", ctypes.c_int32), ("elem", ctypes.c_int32),
+                ("s", ctypes.c_int32), ("a", ctypes.c_float), ("b", ctypes.c_float)]
 
 
 class tg_plan_stats(ctypes.Structure):
@@ -286,6 +303,11 @@ def tg_plan_dump_json(p) -> dict:
     buf = ctypes.create_string_buffer(need.value)
     _ck(_lib.tg_plan_dump_json(p, buf, need.value, ctypes.byref(need)))
     return json.loads(buf.value.decode())
+
+
+def tg_oplib_run(op: "tg_oplib_op", stream=None) -> None:
+    """Run one operator piece on the device (device pointers in `op`)."""
+    _ck(_lib.tg_oplib_run(ctypes.byref(op), stream))
 
 
 def tg_plan_codegen(p) -> str:

@@ -117,3 +117,44 @@ def test_degenerate_shapes_rejected():
     with pytest.raises(tg.TGError) as e:   # VALID 5x5 on a 4x4 image: empty output
         g.conv2d(x, k, -1, tg.TG_VALID)
     assert e.value.code == tg.TG_E_SHAPE
+
+
+def test_oplib_descriptor_abi_and_validation(tmp_path):
+    """tg_oplib_op has the same layout in C and in the binding (sizeof and field offsets from a
+    program compiled against include/tg.h), and malformed descriptors are refused with TG_E_ARG
+    before anything reaches the device (so this runs without a GPU)."""
+    import subprocess
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    src = tmp_path / "abi.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "tg.h"\nint main(void) {\n'
+                   '  printf("%zu %zu %zu %zu %zu %zu\\n", sizeof(tg_oplib_op), offsetof(tg_oplib_op, in_dims),\n'
+                   '         offsetof(tg_oplib_op, y), offsetof(tg_oplib_op, r0), offsetof(tg_oplib_op, a),\n'
+                   '         sizeof(tg_oplib_view));\n  return 0;\n}\n')
+    exe = tmp_path / "abi"
+    subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), "-o", str(exe), str(src)])
+    got = [int(v) for v in subprocess.check_output([str(exe)], text=True).split()]
+    T = tg.tg_oplib_op
+    assert got == [ctypes.sizeof(T), T.in_dims.offset, T.y.offset, T.r0.offset, T.a.offset,
+                   ctypes.sizeof(tg.tg_oplib_view)]
+    op = tg.tg_oplib_op()
+    with pytest.raises(tg.TGError) as e:          # no inputs
+        tg.tg_oplib_run(op)
+    assert e.value.code == tg.TG_E_ARG
+    op.nin, op.kind, op.y = 1, 7, 256            # unknown kind (the view is checked first: give one)
+    op.y_dims[:] = [1, 1, 4, 4]
+    op.r0, op.r1 = 0, 4
+    op.in_[0].nseg = 1
+    op.in_[0].seg[0].p, op.in_[0].seg[0].r0, op.in_[0].seg[0].r1 = 512, 0, 4
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_oplib_run(op)
+    assert e.value.code == tg.TG_E_ARG and "kind" in str(e.value)
+    op.kind, op.nin = tg.TG_OPLIB_CONV, 2        # kernel not in one whole piece
+    op.in_dims[1][:] = [1, 1, 3, 3]
+    op.in_[1].nseg = 2
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_oplib_run(op)
+    assert e.value.code == tg.TG_E_ARG
+    op.kind, op.nin, op.r1 = tg.TG_OPLIB_ELEM, 1, 9   # rows beyond the output
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_oplib_run(op)
+    assert e.value.code == tg.TG_E_ARG
