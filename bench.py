@@ -161,7 +161,8 @@ def workload(name: str, rank: int) -> dict:
 
 
 def host_link_peak(dev: int) -> dict:
-    """Pinned 1 GiB H2D and D2H concurrently on two streams, best of 5."""
+    """Pinned 1 GiB H2D, D2H, and both concurrently on two streams, best of 5.
+    Called by every rank at once under torchrun, so at N GPUs it measures the concurrent link."""
     import torch
     n = 1 << 28
     h1 = torch.empty(n, dtype=torch.float32).pin_memory()
@@ -453,8 +454,13 @@ def run(args, rank, world, local):
     e2e["overlap"] = (s_copy + s_kern - ms2_prof) / max(min(s_copy, s_kern), 1e-9)
     e2e["overlap_def"] = ("(max(H2D, D2H) busy + kernel busy - step) / min(max(H2D, D2H) busy, kernel busy), "
                           "all from the profiled pass")
+    # every rank measures its link at the same time (the concurrent figure is the one that
+    # bounds a multi-GPU streamed run: host DRAM and root-complex bandwidth are shared); the
+    # denominator is the slowest rank's
+    barrier(world)
+    link = host_link_peak(local)
+    link = {k: -max_over_ranks(-v, world) for k, v in link.items()}
     if rank == 0:
-        link = host_link_peak(local)
         # link roofline: each direction at its solo peak, both together at the measured
         # concurrent (bidirectional) rate
         t_link = max(h2d / (link["h2d"] * 1e9), d2h / (link["d2h"] * 1e9),
