@@ -121,7 +121,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
 
     if (warp == 9) {
         // -------------------------------------------------------------------- copy producer
-        // (the whole warp runs the loop; one elected lane issues the bulk copies)
+        // (the whole warp runs the loop; the window rows are issued by one lane each)
         const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
         const uint32_t bbytes = (uint32_t)(U2_KS * 2 * U2_N * 16);
         if (tc::elect_one()) {
@@ -137,11 +137,13 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             const int64_t r0 = 2 * R - a.t2_row0;
             const int64_t rows = min((int64_t)U2_WR, a.t2_rows - r0);
             const int64_t cols = min((int64_t)U2_WP, a.w2 - c0);
-            if (tc::elect_one()) {
-                tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(rows * cols * 16));
-                const uint4* src = t2all + (img * a.t2_rows + r0) * a.w2 + c0;
-                for (int r = 0; r < rows; ++r)
-                    tc::bulk_g2s(&S.a[buf][r * U2_WP], src + r * a.w2, (uint32_t)(cols * 16), &S.a_full[buf]);
+            // one window row per lane, all issued in ONE warp instruction (a single thread
+            // serialises ~150 cycles per bulk copy)
+            if (lane == 0) tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(rows * cols * 16));
+            __syncwarp();
+            if (lane < rows) {
+                const uint4* src = t2all + (img * a.t2_rows + r0 + lane) * a.w2 + c0;
+                tc::bulk_g2s(&S.a[buf][lane * U2_WP], src, (uint32_t)(cols * 16), &S.a_full[buf]);
             }
             __syncwarp();
         }
@@ -366,14 +368,10 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             const int64_t q0 = (band - img * per_img) * 2 * kTileM;
             const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
             const int64_t n = max((int64_t)0, min((int64_t)U3_SPX, bplane - e));
-            if (tc::elect_one()) {
-                tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
-                if (n > 0) {
-                    const uint4* src = t4all + img * 3 * bplane + e;
-                    for (int blk = 0; blk < 3; ++blk)
-                        tc::bulk_g2s(S.a[slot][blk], src + blk * bplane, (uint32_t)(n * 16), &S.a_full[slot]);
-                }
-            }
+            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
+            __syncwarp();
+            if (n > 0 && lane < 3)  // one channel block per lane, in one warp instruction
+                tc::bulk_g2s(S.a[slot][lane], t4all + (img * 3 + lane) * bplane + e, (uint32_t)(n * 16), &S.a_full[slot]);
             __syncwarp();
         }
     } else if (warp == kEpiWarps) {
