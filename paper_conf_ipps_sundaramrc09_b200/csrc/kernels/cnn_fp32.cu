@@ -200,13 +200,14 @@ __global__ void __launch_bounds__(128, 3)
         tma_fence_init();
     }
     __syncthreads();
+    // tile -> (image, first T2 row, first T2 column) in 32-bit arithmetic (the launcher checks
+    // that tile counts fit; 64-bit division is a long software sequence)
+    const uint32_t per = (uint32_t)tiles_c * (uint32_t)tiles_r;
     auto coords = [&](int64_t t, int64_t& img, int64_t& r2_0, int64_t& c2_0) {
-        const int64_t per = (int64_t)tiles_c * tiles_r;
-        img = t / per;
-        const int64_t rem = t - img * per;
-        const int64_t ry = rem / tiles_c;
-        r2_0 = a.t2_row0 + ry * U1T_R;
-        c2_0 = (rem - ry * tiles_c) * U1T_C;
+        const uint32_t tu = (uint32_t)t, im = tu / per, rem = tu - im * per, ry = rem / (uint32_t)tiles_c;
+        img = im;
+        r2_0 = a.t2_row0 + (int64_t)ry * U1T_R;
+        c2_0 = (int64_t)(rem - ry * (uint32_t)tiles_c) * U1T_C;
     };
     auto issue = [&](int64_t t, int b) {
         int64_t img, r2_0, c2_0;
@@ -667,6 +668,7 @@ cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s) {
             const int tiles_c = (int)((a.w2 + U1T_C - 1) / U1T_C);
             const int tiles_r = (int)((a.t2_rows + U1T_R - 1) / U1T_R);
             const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
+            if (ntiles >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit tile indexing in the kernel
             int dev = 0, sms = 148;
             cudaGetDevice(&dev);
             cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);

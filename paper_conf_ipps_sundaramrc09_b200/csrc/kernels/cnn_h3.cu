@@ -116,12 +116,14 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t segs_per_row = (a.w3 + kTileM - 1) / kTileM;
     const int64_t per_img = a.t4_rows * segs_per_row;
+    // segment -> (image, T4 row, first C3 column) in 32-bit arithmetic (the launcher checks that
+    // segment counts fit; 64-bit division is a ~100-instruction software sequence)
+    const uint32_t per_img_u = (uint32_t)per_img, spr_u = (uint32_t)segs_per_row;
     auto seg_coords = [&](int64_t sg, int64_t& img, int64_t& R, int64_t& c0) {
-        img = sg / per_img;
-        const int64_t rem = sg - img * per_img;
-        const int64_t rr = rem / segs_per_row;
+        const uint32_t s = (uint32_t)sg, im = s / per_img_u, rem = s - im * per_img_u, rr = rem / spr_u;
+        img = im;
         R = a.t4_row0 + rr;
-        c0 = (rem - rr * segs_per_row) * kTileM;
+        c0 = (int64_t)(rem - rr * spr_u) * kTileM;
     };
 
     if (warp == 0) tc::tmem_alloc<512>(&S.tmem);
@@ -378,7 +380,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         int64_t si = 0, gi = 0;  // slices and B stages issued so far
         for (int64_t k = 0; k < my_bands; ++k) {
             const int64_t band = blockIdx.x + k * gridDim.x;
-            const int64_t img = band / per_img;
+            const int64_t img = (uint32_t)band / (uint32_t)per_img;
             const int64_t q0 = (band - img * per_img) * 2 * kTileM;
             for (int ks = 0; ks < U3H_KS; ++ks) {
                 if (ks % 8 == 0) {  // slice i = ks / 8
@@ -475,7 +477,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         };
         auto pos_of = [&](int64_t band) {
             Pos q;
-            const int64_t img = band / per_img;
+            const int64_t img = (uint32_t)band / (uint32_t)per_img;
             const int qq = (int)(band - img * per_img) * 2 * kTileM + m;
             q.img = (int)img;
             const int r = qq / w4;
@@ -611,6 +613,7 @@ cudaError_t launch_cnn_u2_h3(const CnnU2Args& a, cudaStream_t s) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t nseg = a.t4_rows * ((a.w3 + kTileM - 1) / kTileM) * a.nimg;
+    if (nseg >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit segment indexing in the kernel
     const unsigned grid = (unsigned)std::min<int64_t>(nseg, sms);
     cnn_u2_h3_kernel<<<grid, kThreads, smem, s>>>(a, pw, nseg);
     return cudaGetLastError();
@@ -634,6 +637,7 @@ cudaError_t launch_cnn_u3_h3(const CnnU3Args& a, cudaStream_t s) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t nbands = per_img * a.nimg;
+    if (nbands >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit band indexing in the kernel
     const unsigned grid = (unsigned)std::min<int64_t>(nbands, sms);
     switch (nch) {
         case 1: cnn_u3_h3_kernel<1><<<grid, kThreads, smem, s>>>(a, k6w, nbands); break;

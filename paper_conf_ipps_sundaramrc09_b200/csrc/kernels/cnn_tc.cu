@@ -88,12 +88,14 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t segs_per_row = (a.w3 + kTileM - 1) / kTileM;
     const int64_t per_img = a.t4_rows * segs_per_row;
+    // segment -> (image, T4 row, first C3 column) in 32-bit arithmetic (the launcher checks that
+    // segment counts fit; 64-bit division is a ~100-instruction software sequence)
+    const uint32_t per_img_u = (uint32_t)per_img, spr_u = (uint32_t)segs_per_row;
     auto seg_coords = [&](int64_t sg, int64_t& img, int64_t& R, int64_t& c0) {
-        img = sg / per_img;
-        const int64_t rem = sg - img * per_img;
-        const int64_t rr = rem / segs_per_row;
+        const uint32_t s = (uint32_t)sg, im = s / per_img_u, rem = s - im * per_img_u, rr = rem / spr_u;
+        img = im;
         R = a.t4_row0 + rr;
-        c0 = (rem - rr * segs_per_row) * kTileM;
+        c0 = (int64_t)(rem - rr * spr_u) * kTileM;
     };
 
     if (warp == 0) tc::tmem_alloc<256>(&S.tmem);
@@ -364,7 +366,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             if (s >= U3_NA) tc::mbar_wait(&S.a_empty[slot], (uint32_t)(((s - U3_NA) / U3_NA) & 1));
             const int64_t band = blockIdx.x + (s / 5) * gridDim.x;
             const int i = (int)(s % 5);
-            const int64_t img = band / per_img;
+            const int64_t img = (uint32_t)band / (uint32_t)per_img;
             const int64_t q0 = (band - img * per_img) * 2 * kTileM;
             const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
             const int64_t n = max((int64_t)0, min((int64_t)U3_SPX, bplane - e));
@@ -470,7 +472,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         const int w4 = (int)a.w4, w5 = (int)a.w5, orow_end = (int)(a.out_row0 + a.out_rows);
         auto pos_of = [&](int64_t band) {
             Pos q;
-            const int64_t img = band / per_img;
+            const int64_t img = (uint32_t)band / (uint32_t)per_img;
             const int qq = (int)(band - img * per_img) * 2 * kTileM + m;
             q.img = (int)img;
             const int r = qq / w4;
@@ -646,6 +648,7 @@ cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t nseg = a.t4_rows * ((a.w3 + kTileM - 1) / kTileM) * a.nimg;
+    if (nseg >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit segment indexing in the kernel
     const unsigned grid = (unsigned)std::min<int64_t>(nseg, sms);
     cnn_u2_tc_kernel<<<grid, kThreadsU2, smem, s>>>(a, pw, nseg);
     return cudaGetLastError();
@@ -677,6 +680,7 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t nbands = per_img * a.nimg;
+    if (nbands >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit band indexing in the kernel
     const unsigned grid = (unsigned)std::min<int64_t>(nbands, sms);
     switch (nch) {
         case 1: cnn_u3_tc_kernel<1><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;

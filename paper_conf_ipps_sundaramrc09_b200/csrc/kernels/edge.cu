@@ -214,13 +214,14 @@ __global__ void __launch_bounds__(kThreads, 2)
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
     __syncthreads();
+    // tile -> (image, first row, first column) in 32-bit arithmetic (the launcher checks that the
+    // tile count fits; 64-bit division is a long software sequence)
+    const uint32_t per_img = (uint32_t)tiles_c * (uint32_t)tiles_r;
     auto coords = [&](int64_t t, int64_t& img, int64_t& tr0, int64_t& tc0) {
-        const int64_t per_img = (int64_t)tiles_c * tiles_r;
-        img = t / per_img;
-        const int64_t rem = t - img * per_img;
-        const int64_t ty = rem / tiles_c;
-        tr0 = a.out_row0 + ty * kTileR;
-        tc0 = (rem - ty * tiles_c) * kTileC;
+        const uint32_t tu = (uint32_t)t, im = tu / per_img, rem = tu - im * per_img, ty = rem / (uint32_t)tiles_c;
+        img = im;
+        tr0 = a.out_row0 + (int64_t)ty * kTileR;
+        tc0 = (int64_t)(rem - ty * (uint32_t)tiles_c) * kTileC;
     };
     auto issue = [&](int64_t t, int b) {
         int64_t img, tr0, tc0;
@@ -342,6 +343,7 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
                 configured.fetch_or(1u << (dev & 31));
             }
             const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
+            if (ntiles >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit tile indexing in the kernel
             const int64_t grid = std::min<int64_t>(ntiles, 2 * (int64_t)sms);
             edge_fused_tma_kernel<kComb, kPairs, kF><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
             return cudaGetLastError();
