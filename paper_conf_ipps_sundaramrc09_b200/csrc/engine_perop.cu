@@ -4,7 +4,7 @@
 // ran its plans (no copy/compute overlap): H2D copies of data-structure pieces
 // (row bands of the host arrays), one generic kernel per operator piece (the
 // "operator library", Fig. 4), D2H copies of evicted or final pieces, and eager frees. Device
-// memory is one arena of plan.arena_bytes laid out statically by the planner (first fit over
+// memory is one arena of plan.arena_bytes laid out statically by the planner (largest buffer first over
 // the trace); pieces evicted to the host live in staging buffers owned by the plan.
 #include <cuda_runtime.h>
 
@@ -154,7 +154,7 @@ tg_status exec_run_per_op(tg_plan* p, bool blocking) {
     for (size_t t = 0; t < c.po_trace.size(); ++t) {
         const auto& e = c.po_trace[t];
         const int id = e.second;
-        const uint64_t off = c.po_trace_off[t];  // static first-fit layout (planner_perop.cpp)
+        const uint64_t off = c.po_trace_off[t];  // static arena layout (planner_perop.cpp)
         switch (e.first) {
             case 0: {  // H2D of a piece: rows [r0, r1) of its DS
                 x.off[id] = (int64_t)off;

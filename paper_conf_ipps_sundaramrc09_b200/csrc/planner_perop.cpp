@@ -11,7 +11,7 @@
 //               GPU memory." -- operators run whole (the paper's baseline failed
 //               once an operator no longer fit): TG_E_INFEASIBLE.
 // The splitting rule is restated in oracle/planner.py::split_plan; the two agree bit-exactly
-// (tests/test_split_plan.py). Arena offsets are assigned statically by first fit over the
+// (tests/test_split_plan.py). Arena offsets are assigned statically (largest buffer first, lowest free offset) over the
 // trace, so the executor and the generated code (codegen.cpp) replay the same layout.
 #include <algorithm>
 #include <map>
@@ -305,7 +305,7 @@ tg_status make_plan_per_op(const Graph& g, int32_t mode, PlanCore& p) {
     }
     if (g.world != 1) return fail(TG_E_UNSUPPORTED, "plan: TG_PER_OP / TG_BASELINE run on one device");
     // "Total GPU Memory" below the arena to account for fragmentation: the
-    // budget less 1/8, lowered by another 1/16 of the budget while the static first-fit
+    // budget less 1/8, lowered by another 1/16 of the budget while the static
     // layout of the schedule does not fit the arena (restated in oracle per_op_plan)
     uint64_t cap = g.budget ? g.budget - g.budget / 8 : std::max<uint64_t>(whole_total, 1);
     for (;;) {

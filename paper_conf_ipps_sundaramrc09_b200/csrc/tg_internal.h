@@ -133,7 +133,7 @@ struct PlanCore {
     std::vector<int32_t> po_piece;
     std::vector<int32_t> po_k;    // split factor per graph node (0: not needed)
     std::vector<uint64_t> po_trace_off;  // arena offset of the DS each trace step touches (static
-                                         // first-fit layout, PAPER.md:409 fragmentation margin)
+                                         // layout, PAPER.md:409 fragmentation margin)
 };
 
 tg_status recognise(const Graph& g, Template& t);
