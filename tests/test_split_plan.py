@@ -112,3 +112,42 @@ def test_static_arena_layout_is_consistent():
             assert all(iv[t][1] <= iv[t + 1][0] for t in range(len(iv) - 1))
         elif kind == 3:
             res.pop(i, None)
+
+
+@pytest.mark.parametrize("S_over_M,regime", [(0.09, "all_fit"), (0.107, "max_separate"), (0.133, "max_split"),
+                                             (0.533, "conv_remap_split"), (1.07, "input_chunked")])
+def test_fig1c_regimes_on_real_plans(S_over_M, regime):
+    """Fig. 1(c) on real TG_PER_OP plans of the 8-orientation edge graph
+    (tg_find_edges, 4 convolutions + 4 remaps + one 8-input max): with the image S bytes and the
+    scheduling capacity M,
+      all_fit           (10 S <= M)       nothing split, only the I/O lower bound moves;
+      max_separate      (9 S <= M < 10 S) nothing split although the whole graph does not fit at
+                        once (the DFS order with eager deletion keeps it to the I/O bound here);
+      max_split / conv_remap_split / input_chunked (9 S > M) the graph is split, into at least
+                        ceil(9 S / M) pieces (the paper's k for max; R19 splits the connected
+                        operators together).
+    The oracle's closed-form regime (fig1c_regime) names the case at the same S / M."""
+    from oracle import planner as P
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    assert P.fig1c_regime(S_over_M * 1500.0, 1500.0) == regime
+    H = W = 384
+    S = 4 * H * W
+    M = int(S / S_over_M)
+    budget = (M * 8 + 6) // 7 + 16 * 1024          # capacity = budget - budget/8 >= M (kernels: 8 x 1 KB)
+    img = np.zeros((1, 1, H, W), np.float32)
+    g = tg.Graph()
+    x = g.input(img)
+    k = g.param(synth.edge_filter_np()[0].reshape(1, 1, 16, 16))
+    e = g.find_edges(x, k, 8, tg.TG_MAX)
+    g.output(e, np.zeros_like(img))
+    g.set(budget=budget)
+    j = g.plan(tg.TG_PER_OP).json()
+    assert len(j["ops"]) >= 9
+    kmax = max(j["k"].values())
+    moved = j["h2d_bytes"] + j["d2h_bytes"]
+    if regime == "all_fit":
+        assert kmax == 1 and moved == j["io_lower_bound_bytes"]
+    elif regime == "max_separate":
+        assert kmax == 1 and j["total_temp_bytes"] > j["capacity"] and moved >= j["io_lower_bound_bytes"]
+    else:
+        assert kmax >= -(-9 * S // j["capacity"])
