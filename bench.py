@@ -490,6 +490,16 @@ def _normwise(g, r) -> float:
     return float(max(np.abs(g[i] - r[i]).max() / max(np.abs(r[i]).max(), 1e-30) for i in range(r.shape[0])))
 
 
+def _cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0, gpu_out=None, tol: float = 1e-5) -> dict:
     """The CPU oracle (as it stands) on a bounded sample of the workload: for the edge
     template whole 10000x10000 images of configs[1]; for the CNN one image of the workload.
@@ -526,7 +536,27 @@ def cpu_oracle_sample(template: str = "edge", target_s: float = 12.0, gpu_out=No
         done_px = H * W
         sample = f"oracle.cnn on one {H}x{W} image of the workload ({t_tot:.1f} s)"
     out = {"value": done_px / t_tot / 1e6, "unit": "Mpixels/s", "cores": oracle.num_threads(), "kind": "oracle",
-           "sample": sample}
+           "sample": sample, "nproc": os.cpu_count(), "cpu_model": _cpu_model()}
+    # the same oracle on ONE core (SURVEY 8(d) "and once on 1 core"), on a small crop of the sample
+    nt = oracle.num_threads()
+    oracle.set_num_threads(1)
+    try:
+        if template == "edge":
+            crop = synth.image_np(seed, synth.DS_IMAGE, 0, (10000, W))[:1000]
+            t0 = time.perf_counter()
+            oracle.edge(crop, K1, K2)
+            t1 = time.perf_counter() - t0
+            what = "oracle.edge on the first 1000 rows of one 10000x10000 image"
+        else:
+            crop = img[:min(H, 480), :min(W, 640)].copy()
+            cprm = synth.cnn_params_np(wl["seed"], n5, crop.shape[0], crop.shape[1])
+            t0 = time.perf_counter()
+            oracle.cnn(crop[None, None], n5, cprm)
+            t1 = time.perf_counter() - t0
+            what = f"oracle.cnn on a {crop.shape[0]}x{crop.shape[1]} crop"
+        out["single_core"] = {"value": crop.size / t1 / 1e6, "unit": "Mpixels/s", "sample": f"{what} ({t1:.1f} s)"}
+    finally:
+        oracle.set_num_threads(nt)
     if gpu_out is not None:
         out["verified"] = {"images": imgs, "max_normwise_err": err, "tol": tol, "ok": err <= tol,
                            "what": "the sampled images' oracle outputs vs this run's streamed GPU outputs"}
