@@ -21,8 +21,9 @@
 //   U2: N = 20 maps is A-read bound, so A_hi is read ONCE for both of its products:
 //       A_hi x [B_hi | B_lo] (N = 64) and A_lo x B_hi (N = 32) accumulated onto the cross-term
 //       columns; the epilogue adds the two 32-column halves.
-//   U3: three MMAs per K-step into one accumulator (N = n5 padded to 16); the B operand (40
-//       K-steps x 2 parts, up to 320 KB) streams through a ring of 32 KB stages.
+//   U3: three MMAs per K-step into one accumulator (N = n5 padded to 16), or for NP <= 64 the
+//       same read-once fusion as U2; the B operand (40 K-steps x 2 parts, up to 320 KB) streams
+//       through a ring of 32 KB stages.
 // Both kernels are persistent and warp-specialised (copy producer warp, MMA issuer warp, epilogue
 // warps), like their bf16 and 3xTF32 counterparts.
 #include <cuda_fp16.h>
@@ -335,12 +336,16 @@ struct U3HSmem {
     uint32_t tmem;
 };
 
+// NCH <= 2 (NP <= 64, the small net): like U2, A_hi is read once for both of its products --
+// [B_hi | B_lo] at N = 2 NP, A_lo x B_hi onto the cross-term columns -- and a tile's accumulator is
+// 2 NP columns (2 tiles x 2 buffers fit the 512 TMEM columns); larger NP: three MMAs into NP columns.
 template <int NCH>  // TMEM chunks of 32 columns: NP = n5 padded to 16, NCH = ceil(NP / 32)
 __global__ void __launch_bounds__(kThreads, 1)
     cnn_u3_h3_kernel(const CnnU3Args a, const __grid_constant__ U3HK6 k6w, const int64_t nbands) {
     extern __shared__ __align__(128) uint8_t smraw[];
     U3HSmem& S = *reinterpret_cast<U3HSmem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    constexpr bool kFuse = NCH <= 2;
     const int NP = a.n_pad;
     const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
     const int64_t bplane = a.t4_rows * a.w4;                 // pixels per block plane of one image
@@ -412,7 +417,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
     } else if (warp == kEpiWarps) {
         // ---------------------------------------------------------------- MMA issuer
-        const uint32_t idesc = idesc_f16(kTileM, NP);
+        const uint32_t idesc = idesc_f16(kTileM, NP), idesc2 = idesc_f16(kTileM, 2 * NP);
         const uint32_t plane_bytes = (uint32_t)(U3H_SPX * 16), part_bytes = 3 * plane_bytes;
         int64_t si = 0, gi = 0;
         for (int64_t k = 0; k < my_bands; ++k) {
@@ -447,12 +452,19 @@ __global__ void __launch_bounds__(kThreads, 1)
                         const uint64_t a_hi = tc::make_desc(ab, lbo, 128);
                         const uint64_t a_lo = tc::make_desc(ab + part_bytes, lbo, 128);
                         const uint32_t bb = b_base + (uint32_t)(u * 2 * 2 * NP * 16);
-                        const uint64_t b_hi = tc::make_desc(bb, (uint32_t)(NP * 16), 128);
-                        const uint64_t b_lo = tc::make_desc(bb + (uint32_t)(2 * NP * 16), (uint32_t)(NP * 16), 128);
-                        const uint32_t d = d_base + (uint32_t)(t * NP);
-                        tc::mma_bf16(d, a_hi, b_hi, idesc, ks > 0 ? 1u : 0u);
-                        tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);
-                        tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);
+                        if (kFuse) {  // A_hi read once: [B_hi | B_lo] at N = 2 NP, then A_lo x B_hi
+                            const uint64_t b_ks = tc::make_desc(bb, (uint32_t)(2 * NP * 16), 128);
+                            const uint32_t d = d_base + (uint32_t)(t * 2 * NP);
+                            tc::mma_bf16(d, a_hi, b_ks, idesc2, ks > 0 ? 1u : 0u);
+                            tc::mma_bf16(d + (uint32_t)NP, a_lo, b_ks, idesc, 1u);
+                        } else {
+                            const uint64_t b_hi = tc::make_desc(bb, (uint32_t)(NP * 16), 128);
+                            const uint64_t b_lo = tc::make_desc(bb + (uint32_t)(2 * NP * 16), (uint32_t)(NP * 16), 128);
+                            const uint32_t d = d_base + (uint32_t)(t * NP);
+                            tc::mma_bf16(d, a_hi, b_hi, idesc, ks > 0 ? 1u : 0u);
+                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);
+                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);
+                        }
                     }
                     if (u == U3H_KST - 1) tc::commit(&S.b_empty[bslot]);
                     if (r8 == 7) tc::commit(&S.a_empty[aslot]);
@@ -514,8 +526,17 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
             for (int c = 0; c < NCH; ++c) {
                 float v[32];
-                tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(buf * 256 + t * NP + 32 * c), v);
-                tc::tmem_wait_ld();
+                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);
+                tc::tmem_ld32_async(tmem + lane_base + col, v);
+                if (kFuse) {  // + the cross terms hi.lo + lo.hi, NP columns further
+                    float x[32];
+                    tc::tmem_ld32_async(tmem + lane_base + col + (uint32_t)NP, x);
+                    tc::tmem_wait_ld();
+#pragma unroll
+                    for (int u = 0; u < 32; ++u) v[u] += x[u];
+                } else {
+                    tc::tmem_wait_ld();
+                }
 #pragma unroll
                 for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], kUnscale, bv[u]));
                 if (c + 1 < NCH)
@@ -572,9 +593,10 @@ void cnn_prepare_k3_h3(const float* k3, uint16_t* dst) {
     }
 }
 
-// B operand of the 3xFP16 C5: [ks < 40][part][half][n < NP][8] fp16 (stages of 4 K-steps are
-// contiguous); K-step ks = 8 i + r8 of filter row i as the bf16 C5 (cnn_prepare_k5_tc); part 0 =
-// hi, 1 = lo of w * 2^8.
+// B operand of the 3xFP16 C5, 40 K-steps (stages of 4 are contiguous); K-step ks = 8 i + r8 of
+// filter row i as the bf16 C5 (cnn_prepare_k5_tc); part 0 = hi, 1 = lo of w * 2^8. NP > 64:
+// [ks][part][half][n < NP][8] fp16; NP <= 64 (the fused MMAs): [ks][half][part][n < NP][8], i.e.
+// each K half is the 2 NP rows [B_hi | B_lo].
 size_t cnn_k5_h3_bytes(int n5) { return (size_t)U3H_KS * 2 * 2 * cnn_n5_pad(n5) * 8 * 2; }
 void cnn_prepare_k5_h3(const float* k5, int n5, uint16_t* dst) {
     const int NP = cnn_n5_pad(n5);
@@ -593,9 +615,14 @@ void cnn_prepare_k5_h3(const float* k5, int n5, uint16_t* dst) {
                         j = 2 * (r8 - 5) + h;
                     }
                     const float w = (ci < 20 && j < 5) ? k5[((size_t)n * 20 + ci) * 25 + i * 5 + j] * kWScale : 0.f;
-                    const uint16_t hi = to_f16(w);
-                    dst[(((size_t)(ks * 2 + 0) * 2 + h) * NP + n) * 8 + e] = hi;
-                    dst[(((size_t)(ks * 2 + 1) * 2 + h) * NP + n) * 8 + e] = to_f16(w - from_f16(hi));
+                    const uint16_t hi = to_f16(w), lo = to_f16(w - from_f16(hi));
+                    if (NP <= 64) {
+                        dst[(((size_t)(ks * 2 + h) * 2 + 0) * NP + n) * 8 + e] = hi;
+                        dst[(((size_t)(ks * 2 + h) * 2 + 1) * NP + n) * 8 + e] = lo;
+                    } else {
+                        dst[(((size_t)(ks * 2 + 0) * 2 + h) * NP + n) * 8 + e] = hi;
+                        dst[(((size_t)(ks * 2 + 1) * 2 + h) * NP + n) * 8 + e] = lo;
+                    }
                 }
     }
 }

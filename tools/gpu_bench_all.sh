@@ -10,7 +10,8 @@ timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_
 for t in ${TEMPLATES:-edge cnn4 cnn3 cnn3s}; do
   for p in fp32 fp32_tc bf16_tc; do
     [ "$t" = edge ] && [ "$p" != fp32 ] && continue
-    timeout 900 python bench.py --template $t --precision $p $BENCH_EXTRA > gpurun_out/bench_${t}_$p.json 2> gpurun_out/bench_${t}_$p.log
+    steps=5; [ "$t" != edge ] && steps=20   # CNN steps are 1-2 ms: time 20 of them
+    timeout 900 python bench.py --template $t --precision $p --steps $steps $BENCH_EXTRA > gpurun_out/bench_${t}_$p.json 2> gpurun_out/bench_${t}_$p.log
     echo "bench $t $p rc=$?"
     python -c "import json,sys; d=json.loads(open('gpurun_out/bench_${t}_$p.json').read().strip().splitlines()[-1]); print(' value', round(d['value']), 'e2e', round(d['e2e']['value']), 'frac', round(d['roofline']['frac'],3), d['roofline']['kernel'], 'units', {k: round(v,3) for k,v in d['roofline'].get('units_ms_per_step',{}).items()})"
   done
