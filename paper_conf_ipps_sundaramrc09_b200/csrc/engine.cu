@@ -63,6 +63,7 @@ struct tg_exec {
     int64_t param_uploads = 0;
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
     std::vector<uint16_t> k3h3, k5h3;  // host copies of the 3xFP16 B operands (TG_FP32_TC)
+    float k3_scale = 1.f, k5_scale = 1.f;  // their power-of-two weight scales
 };
 
 namespace {
@@ -352,7 +353,10 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.bf16_tc = c.precision == TG_BF16_TC;
         a.k3_tc = c.k3tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k3tc_off);
         a.p4_dev = param(5);
-        if (c.precision == TG_FP32_TC) a.k3_h3 = (const uint16_t*)(d.arena + c.k3tc_off);
+        if (c.precision == TG_FP32_TC) {
+            a.k3_h3 = (const uint16_t*)(d.arena + c.k3tc_off);
+            a.w_unscale = 1.f / (cnn_h3_act_scale() * x->k3_scale);
+        }
         KernelTimer kt(x, d, 2, ci, cs);
         CK(a.bf16_tc ? launch_cnn_u2_tc(a, cs)
                      : c.precision == TG_FP32_TC ? launch_cnn_u2_h3(a, cs) : launch_cnn_u2(a, cs));
@@ -396,6 +400,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.nimg = ch.nimg;
         a.bf16_tc = c.precision == TG_BF16_TC;
         a.k5_tc = c.k5tc_off == UINT64_MAX ? nullptr : (const uint16_t*)(d.arena + c.k5tc_off);
+        a.w_unscale = c.precision == TG_FP32_TC ? 1.f / (cnn_h3_act_scale() * x->k5_scale) : 1.f;
         a.n_pad = cnn_n5_pad(t.n5);
         a.k6_host = g.ds[t.prm[8]].src;
         KernelTimer kt(x, d, 3, ci, cs);
@@ -440,10 +445,14 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
         if (c.k5tc_off != UINT64_MAX && c.precision == TG_FP32_TC) {
             // fp16-split B operands of the 3xFP16 C3 and C5 (prepared on the host once per plan)
             if (x->k5h3.empty()) {
+                const Ds& K3 = g.ds[c.t.prm[3]];
+                const Ds& K5 = g.ds[c.t.prm[6]];
+                x->k3_scale = cnn_h3_weight_scale(K3.src, (size_t)K3.numel());
+                x->k5_scale = cnn_h3_weight_scale(K5.src, (size_t)K5.numel());
                 x->k3h3.resize(cnn_k3_h3_bytes() / 2);
-                cnn_prepare_k3_h3(g.ds[c.t.prm[3]].src, x->k3h3.data());
+                cnn_prepare_k3_h3(K3.src, x->k3_scale, x->k3h3.data());
                 x->k5h3.resize(cnn_k5_h3_bytes(c.t.n5) / 2);
-                cnn_prepare_k5_h3(g.ds[c.t.prm[6]].src, c.t.n5, x->k5h3.data());
+                cnn_prepare_k5_h3(K5.src, c.t.n5, x->k5_scale, x->k5h3.data());
             }
             CK(cudaMemcpyAsync(d.arena + c.k3tc_off, x->k3h3.data(), x->k3h3.size() * 2, cudaMemcpyHostToDevice, S0));
             CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5h3.data(), x->k5h3.size() * 2, cudaMemcpyHostToDevice, S0));

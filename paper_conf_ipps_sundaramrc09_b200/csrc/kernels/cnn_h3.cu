@@ -3,11 +3,12 @@
 //
 // Every operand is scaled by a power of two and split into two fp16 numbers,
 //   x' = x * 2^s,  hi = fp16_rn(x'),  lo = fp16_rn(x' - hi),   |x' - hi - lo| <= 2^-22 |x'|
-// (activations T2/T4 in [-1, 1]: s = 4; weights, |w| < 0.1: s = 8 -- both keep hi and lo in the
-// fp16 normal range for every value that matters; a lo that falls into the subnormals errs by at
-// most 2^-25 absolute). A product is accumulated from three MMAs, hi.hi + hi.lo + lo.hi, in fp32
-// in TMEM (lo.lo < 2^-22 of the product is dropped), and the result is scaled back by 2^-12
-// exactly. fp16 carries as many mantissa bits as TF32 (11) at half the bytes, and kind::f16 MMAs
+// (activations T2/T4 in [-1, 1]: s = 4; weights: s chosen per layer on the host so that max |w| x 2^s
+// lies in [2^13, 2^14) -- both keep hi and lo in the fp16 normal range for every value that
+// matters, for any weight magnitude; a lo that falls into the subnormals errs by at most 2^-25
+// of the scaled range). A product is accumulated from three MMAs, hi.hi + hi.lo + lo.hi, in fp32
+// in TMEM (lo.lo < 2^-22 of the product is dropped), and the result is scaled back by the exact
+// power of two w_unscale. fp16 carries as many mantissa bits as TF32 (11) at half the bytes, and kind::f16 MMAs
 // take K = 16 at twice the TF32 rate: the same fp32 accuracy as the 3xTF32 kernels (cnn_t32.cu)
 // for half the shared-memory operand traffic per K element and half the MMA time (this replaced a
 // 3xTF32 implementation of the same layers: U2 0.43 -> 0.32 ms, U3 0.88 -> 0.55 ms on cnn3).
@@ -31,6 +32,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <cmath>
 #include <cstring>
 #include <vector>
 
@@ -51,9 +53,7 @@ __device__ __forceinline__ float tanh_acc(float x) {
     return fmaf(-2.f, r, 1.f);
 }
 
-constexpr float kActScale = 16.f;          // 2^4: activations (T2, T4)
-constexpr float kWScale = 256.f;           // 2^8: weights (K3, K5)
-constexpr float kUnscale = 1.f / 4096.f;   // 2^-12
+constexpr float kActScale = 16.f;          // 2^4: activations (T2, T4: tanh outputs, |x| <= 1)
 
 // hi/lo fp16 pairs of two consecutive channels (element 0 in the low half, as the MMA reads K)
 __device__ __forceinline__ void split2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
@@ -252,22 +252,22 @@ __global__ void __launch_bounds__(kThreads, 1)
                 tc::tmem_ld16_async(tb + U2H_N, q);
                 tc::tmem_wait_ld();
 #pragma unroll
-                for (int co = 0; co < 16; ++co) v0[co] = (p[co] + q[co]) * kUnscale;
+                for (int co = 0; co < 16; ++co) v0[co] = (p[co] + q[co]) * a.w_unscale;
                 tc::tmem_ld16_async(tb + 16, p);
                 tc::tmem_ld16_async(tb + U2H_N + 16, q);
                 tc::tmem_wait_ld();
 #pragma unroll
-                for (int co = 16; co < 20; ++co) v0[co] = (p[co - 16] + q[co - 16]) * kUnscale;
+                for (int co = 16; co < 20; ++co) v0[co] = (p[co - 16] + q[co - 16]) * a.w_unscale;
                 tc::tmem_ld16_async(tb + 2 * U2H_N, p);
                 tc::tmem_ld16_async(tb + 3 * U2H_N, q);
                 tc::tmem_wait_ld();
 #pragma unroll
-                for (int co = 0; co < 16; ++co) v1[co] = (p[co] + q[co]) * kUnscale;
+                for (int co = 0; co < 16; ++co) v1[co] = (p[co] + q[co]) * a.w_unscale;
                 tc::tmem_ld16_async(tb + 2 * U2H_N + 16, p);
                 tc::tmem_ld16_async(tb + 3 * U2H_N + 16, q);
                 tc::tmem_wait_ld();
 #pragma unroll
-                for (int co = 16; co < 20; ++co) v1[co] = (p[co - 16] + q[co - 16]) * kUnscale;
+                for (int co = 16; co < 20; ++co) v1[co] = (p[co - 16] + q[co - 16]) * a.w_unscale;
             }
             tc::fence_before_sync();
             __syncwarp();
@@ -541,7 +541,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                     tc::tmem_wait_ld();
                 }
 #pragma unroll
-                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], kUnscale, bv[u]));
+                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], a.w_unscale, bv[u]));
                 if (c + 1 < NCH)
                     load_bias(cur.pb, c + 1);
                 else if (has_next)
@@ -580,7 +580,17 @@ __global__ void __launch_bounds__(kThreads, 1)
 // i = ks / 3, taps j0 = 2 (ks % 3) + half (tap 5 = zero); row n < 32: hi of map n, row 32 + n:
 // lo of map n, of w * 2^8 with w = K3[n][e][i][j]; maps 20..31 zero.
 size_t cnn_k3_h3_bytes() { return (size_t)U2H_KS * 2 * 2 * U2H_N * 8 * 2; }
-void cnn_prepare_k3_h3(const float* k3, uint16_t* dst) {
+float cnn_h3_act_scale() { return kActScale; }
+float cnn_h3_weight_scale(const float* w, size_t n) {
+    float m = 0.f;
+    for (size_t i = 0; i < n; ++i) m = std::max(m, std::fabs(w[i]));
+    if (!(m > 0.f) || !std::isfinite(m)) return 1.f;
+    int e = 0;
+    std::frexp(m, &e);             // m = f 2^e, f in [0.5, 1)
+    return std::ldexp(1.f, 14 - e);  // m x scale in [2^13, 2^14)
+}
+
+void cnn_prepare_k3_h3(const float* k3, float scale, uint16_t* dst) {
     std::memset(dst, 0, cnn_k3_h3_bytes());
     for (int ks = 0; ks < U2H_KS; ++ks) {
         const int i = ks / 3, j0 = 2 * (ks % 3);
@@ -588,7 +598,7 @@ void cnn_prepare_k3_h3(const float* k3, uint16_t* dst) {
             for (int n = 0; n < 20; ++n)
                 for (int e = 0; e < 8; ++e) {
                     const int j = j0 + h;
-                    const float w = j < 5 ? k3[(n * 8 + e) * 25 + i * 5 + j] * kWScale : 0.f;
+                    const float w = j < 5 ? k3[(n * 8 + e) * 25 + i * 5 + j] * scale : 0.f;
                     const uint16_t hi = to_f16(w);
                     dst[(((size_t)ks * 2 + h) * 2 * U2H_N + n) * 8 + e] = hi;
                     dst[(((size_t)ks * 2 + h) * 2 * U2H_N + U2H_N + n) * 8 + e] = to_f16(w - from_f16(hi));
@@ -601,7 +611,7 @@ void cnn_prepare_k3_h3(const float* k3, uint16_t* dst) {
 // [ks][part][half][n < NP][8] fp16; NP <= 64 (the fused MMAs): [ks][half][part][n < NP][8], i.e.
 // each K half is the 2 NP rows [B_hi | B_lo].
 size_t cnn_k5_h3_bytes(int n5) { return (size_t)U3H_KS * 2 * 2 * cnn_n5_pad(n5) * 8 * 2; }
-void cnn_prepare_k5_h3(const float* k5, int n5, uint16_t* dst) {
+void cnn_prepare_k5_h3(const float* k5, int n5, float scale, uint16_t* dst) {
     const int NP = cnn_n5_pad(n5);
     std::memset(dst, 0, cnn_k5_h3_bytes(n5));
     for (int ks = 0; ks < U3H_KS; ++ks) {
@@ -617,7 +627,7 @@ void cnn_prepare_k5_h3(const float* k5, int n5, uint16_t* dst) {
                         ci = 16 + e;
                         j = 2 * (r8 - 5) + h;
                     }
-                    const float w = (ci < 20 && j < 5) ? k5[((size_t)n * 20 + ci) * 25 + i * 5 + j] * kWScale : 0.f;
+                    const float w = (ci < 20 && j < 5) ? k5[((size_t)n * 20 + ci) * 25 + i * 5 + j] * scale : 0.f;
                     const uint16_t hi = to_f16(w), lo = to_f16(w - from_f16(hi));
                     if (NP <= 64) {
                         dst[(((size_t)(ks * 2 + h) * 2 + 0) * NP + n) * 8 + e] = hi;

@@ -52,6 +52,7 @@ struct CnnU2Args {          // C3(8->20, 5x5) + bias + tanh + S4 + tanh -> T4
     const uint16_t* k3_tc;  // bf16 B operand prepared by cnn_prepare_k3_tc (device)
     const float* p4_dev;    // [20][4] (device)
     const uint16_t* k3_h3;  // fp16-split B operand of the 3xFP16 C3 (cnn_prepare_k3_h3, device)
+    float w_unscale;        // 3xFP16: 1 / (activation scale x the weight scale of cnn_h3_weight_scale)
 };
 struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + bias -> out
     const float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w4;
@@ -66,6 +67,7 @@ struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + 
     const uint16_t* k5_tc;  // bf16 B operand prepared by cnn_prepare_k5_tc (device)
     const float* k6_host;   // [9][n5] (host; passed by value to the tensor-core kernel)
     int n_pad;              // n5 rounded up to a multiple of 16
+    float w_unscale;        // 3xFP16: 1 / (activation scale x the weight scale of cnn_h3_weight_scale)
 };
 cudaError_t launch_cnn_u1(const CnnU1Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u2(const CnnU2Args& a, cudaStream_t s);
@@ -123,10 +125,14 @@ cudaError_t launch_gen_matmul(const GenMatmulArgs& a, cudaStream_t s);
 cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s);
 // 3xFP16 U2 / U3 (cnn_h3.cu): T2 [2][rows][w2][8] and T4 [2][3][rows][w4][8] fp16-split
+// weights are scaled by a power of two (max |w| x scale in [2^13, 2^14)) before the split, so the fp16
+// parts neither overflow nor lose their low part for any weight magnitude
+float cnn_h3_weight_scale(const float* w, size_t n);
+float cnn_h3_act_scale();
 size_t cnn_k3_h3_bytes();
-void cnn_prepare_k3_h3(const float* k3, uint16_t* dst);
+void cnn_prepare_k3_h3(const float* k3, float scale, uint16_t* dst);
 size_t cnn_k5_h3_bytes(int n5);
-void cnn_prepare_k5_h3(const float* k5, int n5, uint16_t* dst);
+void cnn_prepare_k5_h3(const float* k5, int n5, float scale, uint16_t* dst);
 cudaError_t launch_cnn_u2_h3(const CnnU2Args& a, cudaStream_t s);
 cudaError_t launch_cnn_u3_h3(const CnnU3Args& a, cudaStream_t s);
 size_t cnn_k3_tc_bytes();

@@ -339,3 +339,25 @@ def test_cnn_pipelined_async_executions(tg, bias):
             p.execute(blocking=False)
         torch.cuda.synchronize()
         assert torch.equal(out_t, ref)
+
+
+@pytest.mark.parametrize("k3_mul,k5_mul", [(1e4, 1.0), (1.0, 1e4), (1e-4, 1e-3), (3.0, 1e-5)])
+def test_cnn_fp32_tc_weight_magnitudes(tg, orc, k3_mul, k5_mul):
+    """3xFP16 scales each layer's weights by a power of two chosen from its largest magnitude
+    (cnn_h3_weight_scale), so weights far outside the synthetic +-1/sqrt(fan_in) range -- large
+    enough to overflow fp16 at a fixed scale, or small enough to lose their low parts -- stay
+    finite and as accurate as the FFMA fp32 path: within 1e-5 normwise, or, where huge weights
+    make the net ill-conditioned (pre-activations ~1e3 magnify every fp32 rounding at the tanh
+    zero crossings), within 3x the FFMA path's own error on the same inputs."""
+    seed = synth.seed_for_config(3) + 41
+    n, H, W, n5 = 2, 92, 100, 60
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    prm[3] = (prm[3] * np.float32(k3_mul)).astype(np.float32)
+    prm[6] = (prm[6] * np.float32(k5_mul)).astype(np.float32)
+    out, _ = run_cnn(tg, img, n5, prm, precision=tg.TG_FP32_TC)
+    ff, _ = run_cnn(tg, img, n5, prm)
+    ref = orc.cnn(img, n5, prm)
+    assert np.isfinite(out).all()
+    e_tc, e_ff = normwise(out, ref), normwise(ff, ref)
+    assert e_tc <= max(1e-5, 3 * e_ff), (e_tc, e_ff)
