@@ -66,16 +66,20 @@ def test_codegen_refuses_fused():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("name", ["edge", "cnn", "mixed"])
-def test_generated_program_runs(tmp_path, orc, name):
+@pytest.mark.parametrize("name,mode_name", [("edge", "TG_PER_OP"), ("cnn", "TG_PER_OP"), ("mixed", "TG_PER_OP"),
+                                            ("cnn", "TG_BASELINE"), ("mixed", "TG_BASELINE")])
+def test_generated_program_runs(tmp_path, orc, name, mode_name):
     from gpu_util import need_gpu, normwise, torch
     need_gpu()
     from paper_conf_ipps_sundaramrc09_b200 import tg
     torch.cuda.set_device(0)
     spec, frac = specs()[name]
-    g, p, out = plan_of(spec, frac, torch_runtime=True)
+    if mode_name == "TG_BASELINE":
+        frac = 0                                     # the baseline runs operators whole
+    g, p, out = plan_of(spec, frac, mode_name, torch_runtime=True)
     p.execute()                                      # the library's own executor
-    assert max(p.json()["k"].values()) > 1
+    if mode_name == "TG_PER_OP":
+        assert max(p.json()["k"].values()) > 1
     src = tmp_path / "gen.c"
     src.write_text(p.codegen())
     so = tmp_path / "libgen.so"

@@ -1,12 +1,12 @@
 #!/bin/bash
-# Benches of every template workload in both CNN precisions + GPU tests (one gpurun call).
+# Benches of every template workload in the three CNN precisions + GPU tests (one gpurun call).
 # Writes gpurun_out/bench_<template>_<precision>.json (the JSON line) and .log (stderr).
 cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 if [ -z "$SKIP_TESTS" ]; then
   timeout 1200 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
 fi
-timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.log; echo "bench default rc=$?"
+t0=$(date +%s); timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.log; echo "bench default rc=$? ($(( $(date +%s) - t0 )) s)"
 for t in ${TEMPLATES:-edge cnn4 cnn3 cnn3s}; do
   for p in fp32 fp32_tc bf16_tc; do
     [ "$t" = edge ] && [ "$p" != fp32 ] && continue
