@@ -16,6 +16,7 @@
 #include <algorithm>
 #include <map>
 #include <sstream>
+#include <tuple>
 
 #include "kernels/kernels.h"
 #include "tg_internal.h"
@@ -330,11 +331,13 @@ static tg_status plan_at(const Graph& g, int32_t mode, int out, const std::vecto
     // abstract schedule graph: DS pieces in order of first appearance, piece operators in
     // (node, piece) order
     tg_sched s;
-    std::vector<Splitter::Key> keys;
+    std::map<std::tuple<int, int64_t, int64_t>, int32_t> keys;  // (DS, r0, r1) -> sched DS id
     auto piece_id = [&](const Splitter::Key& kk) {
-        for (size_t i = 0; i < keys.size(); ++i)
-            if (keys[i] == kk) return (int32_t)i;
-        keys.push_back(kk);
+        const auto key = std::make_tuple(kk.d, kk.a, kk.b);
+        auto it = keys.find(key);
+        if (it != keys.end()) return it->second;
+        const int32_t id = (int32_t)keys.size();
+        keys.emplace(key, id);
         const Ds& d = g.ds[kk.d];
         int32_t kind = d.kind == DsKind::Input ? TG_DS_INPUT : d.kind == DsKind::Param ? TG_DS_PARAM : TG_DS_TEMP;
         if (kk.d == out) kind = TG_DS_OUTPUT;
@@ -342,7 +345,7 @@ static tg_status plan_at(const Graph& g, int32_t mode, int out, const std::vecto
         p.po_ds.push_back(kk.d);
         p.po_r0.push_back(kk.a);
         p.po_r1.push_back(kk.b);
-        return (int32_t)(keys.size() - 1);
+        return id;
     };
     p.po_k.assign(g.nodes.size(), 0);
     for (int n : sp.live) {
