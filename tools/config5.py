@@ -13,7 +13,7 @@ Outputs are checked, without the oracle (tools may not use it), against a device
 unsplit run of the first and last image through the same library: split/streamed == unsplit,
 bit for bit.
 
-  python tools/config5.py [--share 8] [--total-gb 400] [--precision fp32|bf16_tc] [--steps 1]
+  python tools/config5.py [--share 8] [--total-gb 400] [--precision fp32|fp32_tc|bf16_tc] [--steps 1]
 """
 import argparse
 import json
@@ -111,12 +111,12 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--share", type=int, default=8, help="G: this process runs 1/G of the images")
     ap.add_argument("--total-gb", type=float, default=400.0)
-    ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16_tc"])
+    ap.add_argument("--precision", default="fp32", choices=["fp32", "fp32_tc", "bf16_tc"])
     ap.add_argument("--steps", type=int, default=1)
     ap.add_argument("--templates", default="edge,cnn")
     args = ap.parse_args()
     dev = torch.device("cuda:0")
-    prec = tg.TG_BF16_TC if args.precision == "bf16_tc" else tg.TG_FP32
+    prec = {"fp32": tg.TG_FP32, "fp32_tc": tg.TG_FP32_TC, "bf16_tc": tg.TG_BF16_TC}[args.precision]
     out = {"config": "configs[4]: CNN + edge over ~400 GB host-resident input, split chunks sharded over 8 B200",
            "run": f"one GPU's share (1/{args.share}) of {args.total_gb:g} GB per template, uncapped budget, "
                   f"precision {args.precision}", "gpu": torch.cuda.get_device_name(0), "results": []}
