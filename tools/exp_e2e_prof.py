@@ -32,7 +32,7 @@ for prec_name in sys.argv[2:] or ["bf16_tc", "fp32_tc"]:
     cs = p.compute_stream(0)
     for _ in range(3):
         p.execute()
-    for prof in (False, True, False):
+    for prof in (False, True, True, False):
         p.profiling(prof)
         K = 10
         f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
