@@ -132,6 +132,10 @@ def max_over_ranks(x: float, world: int) -> float:
     return float(t.item())
 
 
+def min_over_ranks(x: float, world: int) -> float:
+    return -max_over_ranks(-x, world)
+
+
 def sum_over_ranks(x: float, world: int) -> float:
     if world == 1:
         return x
@@ -459,7 +463,7 @@ def run(args, rank, world, local):
     # denominator is the slowest rank's
     barrier(world)
     link = host_link_peak(local)
-    link = {k: -max_over_ranks(-v, world) for k, v in link.items()}
+    link = {k: min_over_ranks(v, world) for k, v in link.items()}
     if rank == 0:
         # link roofline: each direction at its solo peak, both together at the measured
         # concurrent (bidirectional) rate

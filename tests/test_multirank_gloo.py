@@ -3,7 +3,7 @@ path. Each rank plans its shard through the C ABI (planning need
 the shards partition the global chunk list with no overlap, chunk boundaries do not depend
 on the world size, every rank's chunks executed on the oracle and assembled into disjoint
 output slices reproduce the unsplit template exactly (no collective on the data path), and
-bench.py's max-over-ranks timing reduction works over gloo."""
+bench.py's max-over-ranks timing and min-over-ranks host-link reductions work over gloo."""
 import os
 import socket
 import sys
@@ -64,6 +64,7 @@ def _worker(rank, world, port, q):
         res["same_chunks"] = g1.plan().json()["chunks"] == plan["chunks"]
         # ---- timing reduction used by bench.py
         res["max"] = bench.max_over_ranks(float(rank + 1), world)
+        res["min"] = bench.min_over_ranks(float(rank + 1), world)  # the host-link denominator
         res["sum"] = bench.sum_over_ranks(1.0, world)
         q.put((rank, res))
         dist.destroy_process_group()
@@ -90,4 +91,4 @@ def test_two_rank_sharding_gloo():
     assert ranges[0][0] == 0 and ranges[0][1] == ranges[1][0] and ranges[1][1] == C and C >= 4
     for r in range(world):
         assert results[r]["edge_exact"] and results[r]["edge_disjoint"] and results[r]["same_chunks"]
-        assert results[r]["max"] == 2.0 and results[r]["sum"] == 2.0
+        assert results[r]["max"] == 2.0 and results[r]["sum"] == 2.0 and results[r]["min"] == 1.0
