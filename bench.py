@@ -101,8 +101,16 @@ def dist_setup(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         import torch.distributed as dist
+        # TG_BENCH_DIST_BACKEND=gloo with more ranks than GPUs runs the multi-rank code path on
+        # one GPU (a functional check of the sharding, barriers and reductions -- its timings
+        # mean nothing); the measured runs are one rank per GPU over NCCL
+        backend = os.environ.get("TG_BENCH_DIST_BACKEND", "nccl")
+        local = local % max(1, torch.cuda.device_count())
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        else:
+            dist.init_process_group(backend)
     elif torch.cuda.is_available():
         torch.cuda.set_device(0)
     return rank, world, local
