@@ -1,0 +1,40 @@
+"""The recorded bench line (profiles/r01/bench_default.json, written by `python bench.py` on a B200)
+carries every key of the bench contract: the base keys, roofline (bound / achieved / peak / unit /
+frac / traffic), cpu_baseline (value / unit / cores / kind / sample), e2e (value / unit / bytes per
+step), clocks and gpu_launches -- and the reference arm's line shape is produced by bench.py's own
+code (checked on CPU with a tiny oracle sample)."""
+import json
+import os
+
+import pytest
+
+from conftest import ROOT
+
+LINE = os.path.join(ROOT, "profiles", "r01", "bench_default.json")
+
+
+@pytest.mark.skipif(not os.path.exists(LINE), reason="no recorded bench line")
+def test_recorded_line_has_the_contract_keys():
+    j = json.loads(open(LINE).read().strip().splitlines()[-1])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e", "clocks", "gpu_launches"):
+        assert k in j, k
+    assert j["warmup"] >= 3 and j["higher_is_better"] is True and j["scaling"] == "weak"
+    assert "workload" in j["config"]
+    r = j["roofline"]
+    for k in ("bound", "achieved", "peak", "unit", "frac", "traffic"):
+        assert k in r, k
+    assert r["bound"] in ("hbm", "tensor", "alu") and 0 < r["frac"] <= 1
+    assert abs(r["achieved"] / r["peak"] - r["frac"]) < 1e-6
+    c = j["cpu_baseline"]
+    for k in ("value", "unit", "cores", "kind", "sample"):
+        assert k in c, k
+    assert c["kind"] == "oracle" and c["verified"]["ok"]
+    e = j["e2e"]
+    for k in ("value", "unit", "h2d_bytes_per_step", "d2h_bytes_per_step"):
+        assert k in e, k
+    assert e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0
+    assert set(j["clocks"]) >= {"sm_mhz", "sm_max_mhz", "reasons"}
+    assert not {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"} & set(j["clocks"]["reasons"])
+    assert j["gpu_launches"] > 0
+    assert {t["precision"] for t in j["per_template"]} == {"fp32", "fp32_tc", "bf16_tc"}
