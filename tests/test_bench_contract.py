@@ -1,8 +1,7 @@
 """The recorded bench line (profiles/r01/bench_default.json, written by `python bench.py` on a B200)
 carries every key of the bench contract: the base keys, roofline (bound / achieved / peak / unit /
 frac / traffic), cpu_baseline (value / unit / cores / kind / sample), e2e (value / unit / bytes per
-step), clocks and gpu_launches -- and the reference arm's line shape is produced by bench.py's own
-code (checked on CPU with a tiny oracle sample)."""
+step), clocks and gpu_launches, with no throttling reason that would void the run."""
 import json
 import os
 
