@@ -19,13 +19,17 @@
  *  - Host buffers passed in are CALLER-OWNED; they must stay valid and unchanged (inputs,
  *    parameters) or untouched (outputs) until tg_execute returns (or, for
  *    tg_execute_async, until the compute stream reaches the end of the execution).
- *    Pinned (page-locked) host memory is used as is; pageable memory is registered with
- *    cudaHostRegister at the first execution and unregistered by tg_plan_destroy.
+ *    Pinned (page-locked) host memory is used as is; pageable memory of 1 MiB or more is
+ *    registered with cudaHostRegister at the first execution (a failure is TG_E_CUDA, never a
+ *    silent fall-back to pageable copies) and unregistered by tg_plan_destroy.
  *  - Device memory is owned by the library: per device it obtains exactly ONE arena of
  *    tg_plan_stats.peak_device_bytes bytes (never more than the device budget) through
  *    tg_runtime.alloc (or cudaMalloc when no runtime is set) and returns it at
  *    tg_plan_destroy. Device-resident inputs/outputs (tg_input_device/tg_output_device)
- *    are caller-owned device buffers on the plan's device.
+ *    are caller-owned device buffers on the plan's device (one-device plans only). Their
+ *    producer and consumer are ordered against the execution through a caller stream:
+ *    tg_execute_on's `stream`, or for tg_execute / tg_execute_async the legacy default
+ *    stream (cudaStreamLegacy, where PyTorch's default stream enqueues).
  *  - Threading: a graph is not thread-safe while it is being built; a plan may be
  *    executed repeatedly but by one thread at a time; independent plans may run
  *    concurrently on disjoint devices.
@@ -146,7 +150,8 @@ tg_status tg_matmul(tg_graph* g, tg_id a, tg_id b, tg_id* y);
 
 /* ------------------------------------------------------------------ target parameters */
 /* Devices the plan runs on (one host thread per device; chunks are split contiguously).
- * Default: the current CUDA device. */
+ * Default: the current CUDA device. Plans with device-resident I/O take one device
+ * (TG_E_UNSUPPORTED at tg_plan_create otherwise). */
 tg_status tg_set_devices(tg_graph* g, const int32_t* ordinals, int32_t n);
 /* Device-memory budget per device in bytes ("Total GPU Memory"); 0 =
  * uncapped. The plan's arena never exceeds it. */
@@ -195,6 +200,9 @@ typedef struct {
     uint64_t host_registered_bytes;  /* pageable host bytes registered by the library   */
     uint64_t h2d_bytes_steady;       /* H2D bytes of a later execution: parameters stay
                                         resident in the arena after the first one        */
+    uint64_t io_lower_bound_data_bytes; /* io_lower_bound_bytes without the parameters: the
+                                        floor of h2d_bytes_steady + d2h_bytes (images in,
+                                        outputs out, once)                               */
 } tg_plan_stats;
 tg_status tg_plan_stats_get(const tg_plan* plan, tg_plan_stats* out);
 
@@ -210,6 +218,13 @@ tg_status tg_execute(tg_plan* plan);
  * of one host-I/O plan pipeline: the next execution's first H2D copies may run while the
  * previous one's last chunks compute and download (each copy waits only for its slot). */
 tg_status tg_execute_async(tg_plan* plan);
+
+/* Same as tg_execute (blocking != 0) or tg_execute_async, ordered against a caller stream
+ * (a cudaStream_t of the plan's device; NULL = the legacy default stream): the execution starts
+ * after all work enqueued on `stream` before the call, and work enqueued on `stream` after the
+ * call starts after the execution completes. Fused plans on one device; TG_E_UNSUPPORTED
+ * otherwise. */
+tg_status tg_execute_on(tg_plan* plan, void* stream, int32_t blocking);
 
 /* Per-launch timing of the fused kernels measured with CUDA events on the compute stream
  * (enable before executing; tg_plan_timing_get synchronizes). Times are summed over all

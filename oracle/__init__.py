@@ -15,6 +15,7 @@ Parity status per function is listed in DESIGN.md ("Oracle pins").
 from __future__ import annotations
 
 import ctypes
+import math
 import os
 import subprocess
 
@@ -176,6 +177,52 @@ def edge_general(img, kernels, combine: str = "max") -> np.ndarray:
     if combine == "maxplain":
         return max_fold(*E)
     raise ValueError(combine)
+
+
+def rotate_kernel(K, deg: int) -> np.ndarray:
+    """A k x k kernel rotated counter-clockwise by `deg` degrees about its centre
+    c = ((k-1)/2, (k-1)/2) -- DESIGN.md reading R18 (the paper draws 8 orientations of one
+    filter, Fig. 1(b), without a rule for a discrete kernel). Output tap (i, j)
+    takes K at the source point
+        sr = c + (i - c) cos t + (j - c) sin t,   sc = c - (i - c) sin t + (j - c) cos t,
+    read by bilinear interpolation of the four surrounding taps (taps outside K are 0), in
+    float64, rounded once to fp32. For multiples of 90 degrees the source point is a tap, so
+    the result is an exact permutation (90 degrees: R[i][j] = K[j][k-1-i])."""
+    K = np.asarray(K, dtype=np.float64)
+    k = K.shape[0]
+    deg = deg % 360
+    c = (k - 1) / 2.0
+    if deg % 90 == 0:                       # cos, sin exactly in {-1, 0, 1}
+        cs, sn = [(1, 0), (0, 1), (-1, 0), (0, -1)][deg // 90]
+    else:
+        t = math.radians(deg)
+        cs, sn = math.cos(t), math.sin(t)
+    R = np.zeros((k, k), dtype=np.float64)
+    for i in range(k):
+        for j in range(k):
+            sr = c + (i - c) * cs + (j - c) * sn
+            sc = c - (i - c) * sn + (j - c) * cs
+            r0, q0 = math.floor(sr), math.floor(sc)
+            fr, fc = sr - r0, sc - q0
+            v = 0.0
+            for dr, wr in ((0, 1.0 - fr), (1, fr)):
+                for dc, wc in ((0, 1.0 - fc), (1, fc)):
+                    rr, cc = r0 + dr, q0 + dc
+                    if 0 <= rr < k and 0 <= cc < k:
+                        v += wr * wc * K[rr, cc]
+            R[i, j] = v
+    return R.astype(np.float32)
+
+
+def find_edges(img, kernel, num_orientations: int = 4, combine: str = "max") -> np.ndarray:
+    """find_edges(Image, Kernel, num_orientations, Combine_op) (PAPER.md:623): orientations in
+    steps of 360/num_orientations degrees; the first half are SAME convolutions of the image
+    with the rotated kernel (rotate_kernel), the second half their remaps -E (PAPER.md:627-629,
+    reading R3); combine 'max' over all orientations, 'maxabs' = max |E_i| of the
+    convolutions, 'sum' = their sum."""
+    step = 360 // num_orientations
+    Ks = [rotate_kernel(kernel, q * step) for q in range(num_orientations // 2)]
+    return edge_general(img, Ks, combine)
 
 
 def cnn(img, n5: int, params, bias_plane: bool = True) -> np.ndarray:

@@ -13,8 +13,8 @@ Plain Python restatement of the paper's planning steps, written for checking by 
     schedule with eager deletion (read as NEXT use, R10)
   * brute force over all operator orders for tiny graphs (stands in for the PB model of
     Fig. 5, PAPER.md:395-475)
-  * the fused B200 chunk rule, which the library's planner must
-    reproduce bit-exactly (tests/test_plan_parity.py).
+  * what a fused plan's chunks read, write and move, given its chunk size (row bands,
+    halos, shards, bytes; tests/test_plan_parity.py compares the library bit-exactly).
 """
 from __future__ import annotations
 
@@ -276,9 +276,6 @@ def dfs_order(g: Graph) -> list[int]:
             producer[j] = i
     preds = [{producer[j] for j in op.ins if j in producer} for op in g.ops]
     consumers = [[] for _ in g.ops]
-    for i, op in enumerate(g.ops):
-        for p in sorted(preds[i]):
-            pass
     for c, op in enumerate(g.ops):
         for j in op.ins:
             if j in producer and c not in consumers[producer[j]]:
@@ -635,91 +632,22 @@ def split_plan(shapes, kinds, nodes: list[SNode], output: int, capacity: int, fo
             "moved": moved, "k": {i: k_of[find(nodes[i].out)] for i in live}}
 
 
-def arena_layout(g: Graph, trace, arena: int):
-    """Static arena layout of a transfer trace (with frees). Every residency interval of a DS
-    piece -- from its copy-in or production to its free (or the end) -- is a buffer of its
-    size rounded up to 256 B. Buffers are placed largest first (ties: earlier start, then lower
-    DS id), each at the lowest offset where it overlaps no already placed buffer that is live
-    at the same time. Returns the offset each trace step touches, or None when a buffer would
-    end beyond the arena (fragmentation)."""
-    a256 = lambda v: (max(v, 1) + 255) // 256 * 256
-    names = {d.name: i for i, d in enumerate(g.ds)}
-    ops = {o.name: o for o in g.ops}
-    opened = {}
-    iv = []                       # (start step, end step, DS)
-    for t, (kind, nm) in enumerate(trace):
-        if kind in ("h2d", "run"):
-            j = names[nm] if kind == "h2d" else ops[nm].outs[0]
-            if j not in opened:
-                opened[j] = t
-        elif kind == "free":
-            j = names[nm]
-            if j in opened:
-                iv.append((opened.pop(j), t, j))
-    for j, t0 in opened.items():
-        iv.append((t0, len(trace), j))
-    off = {}
-    placed = []
-    for t0, t1, j in sorted(iv, key=lambda v: (-a256(g.ds[v[2]].size), v[0], v[2])):
-        sz = a256(g.ds[j].size)
-        cur = 0
-        for lo, hi in sorted((o, o + s) for a, b, o, s in placed if a < t1 and t0 < b):
-            if lo - cur >= sz:
-                break
-            cur = max(cur, hi)
-        if cur + sz > arena:
-            return None
-        placed.append((t0, t1, cur, sz))
-        off[(j, t0)] = cur
-    offs = []
-    start = {}
-    for t, (kind, nm) in enumerate(trace):
-        j = ops[nm].outs[0] if kind == "run" else names[nm]
-        if kind in ("h2d", "run") and j not in start:
-            start[j] = t
-        offs.append(off[(j, start[j])])
-        if kind == "free":
-            del start[j]
-    return offs
-
-
-def per_op_plan(shapes, kinds, nodes: list[SNode], output: int, budget: int):
-    """TG_PER_OP end to end: split (R19) and schedule within the scheduling capacity M, then
-    lay the arena out (arena_layout). M starts at the budget less 1/8 ("set to a value less than
-    the actual amount of GPU memory present in the system to account for fragmentation",
-    PAPER.md:409) and, while the layout does not fit the arena, drops by another 1/16 of the
-    budget. Uncapped (budget 0): M = every DS once, no layout constraint."""
-    total = 4 * sum(math.prod(sh) for d, sh in enumerate(shapes)
-                    if d == output or any(d in nd.ins or d == nd.out for nd in nodes))
-    if budget == 0:
-        r = split_plan(shapes, kinds, nodes, output, max(total, 1))
-        r["capacity"] = max(total, 1)
-        return r
-    cap = budget - budget // 8
-    arena = budget // 256 * 256
-    while cap > 0:
-        r = split_plan(shapes, kinds, nodes, output, cap)
-        tr = []
-        simulate_transfers(r["graph"], r["order"], cap, tr, frees=True)
-        offs = arena_layout(r["graph"], tr, arena)
-        if offs is not None:
-            r["capacity"] = cap
-            r["trace_full"] = tr
-            r["trace_off"] = offs
-            return r
-        cap -= budget // 16
-    raise ValueError("infeasible: no capacity gives a layout that fits the arena")
+def per_op_plan(shapes, kinds, nodes: list[SNode], output: int, capacity: int):
+    """TG_PER_OP at a scheduling capacity M: split (R19) and schedule within
+    M, plus the transfer trace with frees. How M is derived from the budget (PAPER.md:409:
+    "set to a value less than the actual amount of GPU memory ... to account for
+    fragmentation") and where buffers sit in the arena are the library's static-layout design:
+    M is an INPUT here; tests/test_split_plan.py checks the layout by properties."""
+    r = split_plan(shapes, kinds, nodes, output, capacity)
+    tr = []
+    simulate_transfers(r["graph"], r["order"], capacity, tr, frees=True)
+    r["capacity"] = capacity
+    r["trace_full"] = tr
+    return r
 
 
 # ============================================================================ chunk rule
-DEPTH = 3                 # pipeline slots (H2D / compute / D2H in flight)
-MAX_CHUNK_PX = 1 << 25    # input pixels per chunk when memory does not bind (DESIGN.md §4)
 F32 = 4
-
-
-def a256(x: int) -> int:
-    """Every arena buffer starts on a 256-byte boundary."""
-    return (int(x) + 255) // 256 * 256
 
 
 def _edge_rows(H: int, ks: int, r0: int, r1: int) -> dict:
@@ -738,165 +666,83 @@ def _span(r) -> int:
     return r[1] - r[0]
 
 
-def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int = 20,
-               bias: str = "plane", budget: int = 0, max_chunk_px: int = MAX_CHUNK_PX,
-               depth: int = DEPTH, rank: int = 0, world: int = 1, device_io: bool = False,
-               precision: str = "fp32", nf: int = 2, combine: str = "max") -> dict:
-    """Fused-mode plan, restated plainly; the library's
-    tg_plan_dump_json must produce the same dict (tests/test_plan_parity.py).
+def template_params(template: str, H: int, W: int, *, ks: int = 16, n5: int = 20, bias: str = "plane",
+                    nf: int = 2):
+    """Parameter floats of a template instance and which of them are bias planes: the edge
+    template's nf kernels of ks x ks (the 2 x 256 kernel floats of Table 1 at nf = 2,
+    PAPER.md:743); the CNN's K1 B1 P2 K3 B3 P4 K5 B5 K6 B6, biases one plane per
+    output map (Fig. 7) or one scalar per map."""
+    if template == "edge":
+        return [ks * ks] * nf, [False] * nf
+    (h1, w1), _, (h3, w3), _, (h5, w5) = cnn_dims(H, W)
+    bs = [8 * h1 * w1, 20 * h3 * w3, n5 * h5 * w5, 9 * h5 * w5] if bias == "plane" else [8, 20, n5, 9]
+    params = [8 * 25, bs[0], 8 * 4, 20 * 8 * 25, bs[1], 20 * 4, n5 * 20 * 25, bs[2], 9 * n5, bs[3]]
+    return params, [False, True, False, False, True, False, False, True, False, True]
 
-    Offload units: the whole edge template is one unit (the paper's "best possible",
-    PAPER.md:727); the CNN is three units U1 = C1 T S2 T, U2 = C3 T S4 T, U3 = C5 T C6 whose
-    intermediates (T2, T4) stay in the chunk's device slot.
 
-    1. Batch mode (whole images per chunk) when an image has at most max_chunk_px pixels:
-       B = the largest b <= min(n, max_chunk_px // (H*W), ceil(n / (2*depth))) whose slot
-       fits. With device-resident I/O (no copies, depth 1): the largest b <= n that fits.
-    2. Otherwise row mode (split the image, never the kernel), one image per
-       chunk, R output rows: the largest R <= min(h_out, max(1, max_chunk_px // (W*f)))
-       whose widest slot fits, f = input rows per output row (edge 1, CNN 4). For CNN bias
-       planes two variants are sized -- all parameters resident, or bias rows streamed with
-       each chunk -- and the one with fewer predicted H2D bytes wins (tie: resident).
-    "fits" = param_bytes + depth * slot_bytes <= budget (budget 0 = uncapped).
-    Chunks are image-major, [i*R, min((i+1)*R, h_out)); rank g of world G executes chunks
-    [floor(C*g/G), floor(C*(g+1)/G)).
-    """
+def fused_chunks(template: str, n: int, H: int, W: int, split: str, B: int, R: int, *, ks: int = 16,
+                 n5: int = 20, bias: str = "none", rank: int = 0, world: int = 1, device_io: bool = False,
+                 nf: int = 2, combine: str = "max") -> dict:
+    """What a fused plan moves and computes, given its chunk size -- restated from the paper:
+
+      * chunks (R12): whole images, B per chunk (split 'batch'), or per image output
+        row bands [i*R, min((i+1)*R, h_out)) (split 'rows': split the image, never the kernel,
+        PAPER.md:367, :371), image-major;
+      * the rows every chunk needs at every level, by back-propagation from its output rows
+        "from the leaves to the root" (PAPER.md:367; back_propagate_rows);
+      * the shard of rank g of G: chunks [floor(C g / G), floor(C (g+1) / G)) (DESIGN.md §6);
+      * host->device bytes: the parameter floats (never split; bias planes that
+        travel with the chunks -- bias 'streamed' -- excluded) and per chunk its input rows, plus
+        in 'streamed' mode the bias rows of C1, C3, C5 and C6 it needs; device->host bytes: its
+        output rows (the template output, PAPER.md:613);
+      * Table 1 accounting at Fig. 7 granularity.
+
+    How large B or R is -- the device-memory layout of a chunk slot -- is the library's design
+    decision, not the paper's: it is an INPUT here, and tests/test_plan_parity.py checks it by
+    properties (fits the budget, maximal, every buffer present)."""
     f = F32
     if n <= 0 or H <= 0 or W <= 0:
         raise ValueError("empty input")
     if template == "edge":
-        h_out, w_out, in_per_out = H, W, 1
-        params = [ks * ks] * nf
-        is_bias = [False] * nf
+        h_out, w_out, planes_out = H, W, 1
         rows = lambda r0, r1: _edge_rows(H, ks, r0, r1)          # noqa: E731
-        widest = lambda R: {"in": [0, min(H, R + ks - 1)], "out": [0, R]}  # noqa: E731
+        pbias = "plane"
     elif template == "cnn":
         (h1, w1), (h2, w2), (h3, w3), (h4, w4), (h5, w5) = cnn_dims(H, W)
         if h5 <= 0 or w5 <= 0:
             raise ValueError("image too small for the CNN")
-        h_out, w_out, in_per_out = h5, w5, 4
-        if bias == "plane":
-            bs = [8 * h1 * w1, 20 * h3 * w3, n5 * h5 * w5, 9 * h5 * w5]
-        else:
-            bs = [8, 20, n5, 9]
-        params = [8 * 25, bs[0], 8 * 4, 20 * 8 * 25, bs[1], 20 * 4, n5 * 20 * 25, bs[2], 9 * n5, bs[3]]
-        is_bias = [False, True, False, False, True, False, False, True, False, True]
+        h_out, w_out, planes_out = h5, w5, 9
         rows = _cnn_rows
-        widest = lambda R: _cnn_rows(0, R)                        # noqa: E731
+        pbias = "scalar" if bias == "scalar" else "plane"
     else:
         raise ValueError(template)
+    params, is_bias = template_params(template, H, W, ks=ks, n5=n5, bias=pbias, nf=nf)
+    streamed = bias == "streamed"
 
-    def slot_bytes(B: int, R: int, rg: dict, streamed: bool) -> int:
-        s = 0
-        if not device_io:
-            s += a256(B * _span(rg["in"]) * W * f)
-        if template == "cnn":
-            s += a256(B * 8 * _span(rg["t2"]) * w2 * f)
-            # TG_FP32_TC keeps T4 as two fp16 parts (hi, lo) x 3 blocks of 8 channels = 24 words
-            # per pixel for the 3xFP16 C5 (T2: 2 parts x 8 fp16 = the 8 fp32 words of the others)
-            s += a256(B * (24 if precision == "fp32_tc" else 20) * _span(rg["t4"]) * w4 * f)
-            if not device_io:
-                s += a256(B * 9 * R * w5 * f)
-            if streamed:
-                s += a256(8 * _span(rg["c1"]) * w1 * f)
-                s += a256(20 * _span(rg["c3"]) * w3 * f)
-                s += a256(n5 * R * w5 * f)
-                s += a256(9 * R * w5 * f)
-        elif not device_io:
-            s += a256(B * R * W * f)
-        return s
-
-    all_pb = sum(a256(p * f) for p in params)
-    nonbias_pb = sum(a256(p * f) for p, b in zip(params, is_bias) if not b)
-    if template == "cnn" and precision == "bf16_tc":
-        # bf16 B operands of the tensor-core C3 (15 K-steps x 2 halves x 32 maps x 8) and
-        # C5 (40 K-steps x 2 x n5 rounded up to 16 x 8), kept with the parameters
-        tc = a256(15 * 2 * 32 * 8 * 2) + a256(40 * 2 * ((n5 + 15) // 16 * 16) * 8 * 2)
-        all_pb += tc
-        nonbias_pb += tc
-    if template == "cnn" and precision == "fp32_tc":
-        # fp16-split B operands of the 3xFP16 C3 (15 K-steps x 2 halves x 64 rows (hi and lo
-        # maps) x 8 fp16) and C5 (40 K-steps x 2 parts x 2 halves x n5 rounded up to 16 x 8 fp16)
-        tc = a256(15 * 2 * 64 * 8 * 2) + a256(40 * 2 * 2 * ((n5 + 15) // 16 * 16) * 8 * 2)
-        all_pb += tc
-        nonbias_pb += tc
-    if device_io:
-        depth = 1
-
-    def fits(pb: int, sb: int) -> bool:
-        return budget == 0 or pb + depth * sb <= budget
-
-    def chunk_list(split: str, B: int, R: int) -> list:
-        out = []
-        if split == "batch":
-            for b0 in range(0, n, B):
-                out.append({"img": b0, "nimg": min(B, n - b0), **rows(0, h_out)})
-        else:
-            for b0 in range(n):
-                for r0 in range(0, h_out, R):
-                    out.append({"img": b0, "nimg": 1, **rows(r0, min(h_out, r0 + R))})
-        return out
-
-    def h2d_of(chunks: list, pb: int, streamed: bool) -> int:
-        if device_io:
-            return 0
-        t = pb
-        for ch in chunks:
-            t += ch["nimg"] * _span(ch["in"]) * W * f
-            if streamed:
-                t += 8 * _span(ch["c1"]) * w1 * f + 20 * _span(ch["c3"]) * w3 * f
-                t += (n5 + 9) * _span(ch["out"]) * w5 * f
-        return t
-
-    base_bias = "none" if template == "edge" else ("resident" if bias == "plane" else "scalar")
-    choice = None
-    # 1. batch mode
-    if device_io:
-        bcap = n
-    elif H * W <= max_chunk_px:
-        bcap = min(n, max_chunk_px // (H * W), max(1, -(-n // (2 * depth))))
+    chunks = []
+    if split == "batch":
+        for b0 in range(0, n, B):
+            chunks.append({"img": b0, "nimg": min(B, n - b0), **rows(0, h_out)})
+    elif split == "rows":
+        for b0 in range(n):
+            for r0 in range(0, h_out, R):
+                chunks.append({"img": b0, "nimg": 1, **rows(r0, min(h_out, r0 + R))})
     else:
-        bcap = 0
-    for b in range(bcap, 0, -1):
-        sb = slot_bytes(b, h_out, rows(0, h_out), False)
-        if fits(all_pb, sb):
-            choice = ("batch", b, h_out, base_bias, all_pb, sb)
-            break
-    # 2. row mode
-    if choice is None:
-        rcap = min(h_out, max(1, max_chunk_px // (W * in_per_out)))
-        cands = []
-        for bm in ([base_bias, "streamed"] if base_bias == "resident" else [base_bias]):
-            streamed = bm == "streamed"
-            pb = nonbias_pb if streamed else all_pb
-            lo, hi, best = 1, rcap, 0
-            while lo <= hi:                      # slot bytes grow monotonically with R
-                mid = (lo + hi) // 2
-                if fits(pb, slot_bytes(1, mid, widest(mid), streamed)):
-                    best, lo = mid, mid + 1
-                else:
-                    hi = mid - 1
-            if best:
-                sb = slot_bytes(1, best, widest(best), streamed)
-                cands.append((h2d_of(chunk_list("rows", 1, best), pb, streamed),
-                              ("rows", 1, best, bm, pb, sb)))
-        if not cands:
-            raise RuntimeError("infeasible: the budget cannot hold the smallest chunk")
-        cands.sort(key=lambda c: c[0])          # stable: resident wins ties
-        choice = cands[0][1]
-    split, B, R, bias_mode, pb, sb = choice
-    streamed = bias_mode == "streamed"
-    chunks = chunk_list(split, B, R)
+        raise ValueError(split)
     C = len(chunks)
     c0, c1 = (C * rank) // world, (C * (rank + 1)) // world
     mine = chunks[c0:c1]
-    h2d = h2d_of(mine, pb, streamed)
-    d2h = 0
-    if not device_io:
-        planes_out = 9 if template == "cnn" else 1
-        d2h = sum(ch["nimg"] * planes_out * _span(ch["out"]) * w_out * f for ch in mine)
 
-    # Table 1 accounting (per template instance; images and per-image DS scale with n)
+    h2d_param = h2d_chunk = d2h = 0
+    if not device_io:
+        h2d_param = sum(p * f for p, b in zip(params, is_bias) if not (streamed and b))
+        for ch in mine:
+            h2d_chunk += ch["nimg"] * _span(ch["in"]) * W * f
+            if streamed:
+                h2d_chunk += 8 * _span(ch["c1"]) * w1 * f + 20 * _span(ch["c3"]) * w3 * f
+                h2d_chunk += (n5 + 9) * _span(ch["out"]) * w5 * f
+            d2h += ch["nimg"] * planes_out * _span(ch["out"]) * w_out * f
+
     if template == "edge":
         g = edge_graph_general(H, W, ks, nf, combine)
     else:
@@ -904,16 +750,12 @@ def fused_plan(template: str, n: int, H: int, W: int, *, ks: int = 16, n5: int =
     param_floats = sum(params)
     per_img_floats = sum(d.size for d in g.ds if d.kind != "param")
     out_floats = sum(d.size for d in g.ds if d.kind == "output")
-    io_lb = (n * (H * W + out_floats) + param_floats) * f
-    total = (n * per_img_floats + param_floats) * f
     return {
-        "template": template, "n": n, "H": H, "W": W,
-        "ks": ks if template == "edge" else 0, "n5": n5 if template == "cnn" else 0,
-        "nf": nf if template == "edge" else 0, "combine": combine if template == "edge" else "none",
-        "budget": budget, "depth": depth, "max_chunk_px": max_chunk_px,
-        "device_io": bool(device_io), "precision": precision if template == "cnn" else "fp32", "bias": bias_mode, "split": split, "B": B, "R": R,
-        "param_bytes": pb, "slot_bytes": sb, "arena_bytes": pb + depth * sb,
-        "n_chunks": C, "chunks": chunks, "shard": [rank, world, c0, c1],
-        "h2d_bytes": h2d, "d2h_bytes": d2h, "io_lower_bound_bytes": io_lb,
-        "total_temp_bytes": total, "n_ops_fig7": len(g.ops), "n_ds_fig7": len(g.ds),
+        "split": split, "B": B, "R": R, "bias": bias, "n_chunks": C, "chunks": chunks,
+        "shard": [rank, world, c0, c1],
+        "h2d_param_bytes": h2d_param, "h2d_chunk_bytes": h2d_chunk, "d2h_bytes": d2h,
+        "io_lower_bound_bytes": (n * (H * W + out_floats) + param_floats) * f,
+        "io_lower_bound_data_bytes": n * (H * W + out_floats) * f,
+        "total_temp_bytes": (n * per_img_floats + param_floats) * f,
+        "n_ops_fig7": len(g.ops), "n_ds_fig7": len(g.ds),
     }

@@ -466,7 +466,8 @@ tg_status tg_plan_stats_get(const tg_plan* p, tg_plan_stats* out) {
     out->chunk_end = c.c1;
     out->host_registered_bytes = exec_registered_bytes(p);
     // steady state: parameters stay resident after the first execution
-    out->h2d_bytes_steady = c.device_io ? 0 : (c.mode == TG_FUSED ? c.h2d - c.param_bytes : c.h2d);
+    out->h2d_bytes_steady = c.device_io ? 0 : (c.mode == TG_FUSED ? c.h2d_chunk : c.h2d);
+    out->io_lower_bound_data_bytes = c.mode == TG_FUSED ? c.io_lb_data : c.io_lb;
     return TG_OK;
 }
 
@@ -508,6 +509,14 @@ tg_status tg_execute_async(tg_plan* p) {
     TG_GUARD_BEGIN
     if (p->core.mode != TG_FUSED) return exec_run_per_op(p, false);
     return exec_run(p, false);
+    TG_GUARD_END
+}
+
+tg_status tg_execute_on(tg_plan* p, void* stream, int32_t blocking) {
+    if (!p) return fail(TG_E_ARG, "tg_execute_on: NULL plan");
+    TG_GUARD_BEGIN
+    if (p->core.mode != TG_FUSED) return fail(TG_E_UNSUPPORTED, "tg_execute_on: fused plans only");
+    return exec_run(p, blocking != 0, stream, true);
     TG_GUARD_END
 }
 

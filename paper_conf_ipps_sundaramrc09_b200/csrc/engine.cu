@@ -42,6 +42,7 @@ struct DevState {
     bool own_arena = false;
     std::vector<cudaEvent_t> ev_h2d, ev_comp, ev_d2h;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_params = nullptr;
+    cudaEvent_t ev_caller = nullptr, ev_done = nullptr;  // ordering against the caller's stream
     int64_t c0 = 0, c1 = 0;
     std::vector<ProfRec> prof;
     std::vector<cudaEvent_t> ev_pool;
@@ -60,7 +61,6 @@ struct tg_exec {
     bool profiling = false;
     tg_timing timing{};
     std::vector<tg_trace_rec> trace;  // timeline collected from the profiling events
-    int64_t param_uploads = 0;
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
     std::vector<uint16_t> k3h3, k5h3;  // host copies of the 3xFP16 B operands (TG_FP32_TC)
     float k3_scale = 1.f, k5_scale = 1.f;  // their power-of-two weight scales
@@ -129,6 +129,8 @@ tg_status init_device(tg_plan* p, DevState& d) {
     CK(cudaEventCreateWithFlags(&d.ev_fork, flags));
     CK(cudaEventCreateWithFlags(&d.ev_join, flags));
     CK(cudaEventCreateWithFlags(&d.ev_params, flags));
+    CK(cudaEventCreateWithFlags(&d.ev_caller, flags));
+    CK(cudaEventCreateWithFlags(&d.ev_done, flags));
     return TG_OK;
 }
 
@@ -149,12 +151,19 @@ tg_status register_host(tg_plan* p, tg_exec* x) {
         if (cudaPointerGetAttributes(&at, b.first) == cudaSuccess && at.type == cudaMemoryTypeHost) continue;
         cudaGetLastError();
         cudaError_t e = cudaHostRegister(b.first, b.second, cudaHostRegisterDefault);
-        if (e == cudaSuccess) {
-            x->registered.push_back(b.first);
-            x->registered_bytes += b.second;
-        } else {
-            cudaGetLastError();  // overlapping/foreign registration: fall back to pageable copies
+        if (e != cudaSuccess) {
+            // no silent fallback to pageable copies (a several-fold cliff of the host link):
+            // the caller pins the buffer itself or fixes the overlap
+            cudaGetLastError();
+            char m[320];
+            std::snprintf(m, sizeof m,
+                          "cudaHostRegister of a %zu-byte caller host buffer failed: %s (pass page-locked memory, "
+                          "e.g. cudaHostAlloc / torch pin_memory, or non-overlapping buffers)",
+                          b.second, cudaGetErrorString(e));
+            return fail(TG_E_CUDA, m);
         }
+        x->registered.push_back(b.first);
+        x->registered_bytes += b.second;
     }
     return TG_OK;
 }
@@ -412,11 +421,18 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
     return TG_OK;
 }
 
-tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
+tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStream_t caller, bool ordered) {
     const Graph& g = graph_of(p);
     const PlanCore& c = p->core;
     CK(cudaSetDevice(d.dev));
     cudaStream_t S0 = d.st[0], S1 = d.st[1], S2 = d.st[2];
+    // The caller's stream: the execution starts after the work enqueued on it so far
+    // (device-resident inputs may be produced there) and later work on it starts after the
+    // execution (device-resident outputs may be consumed there).
+    if (ordered) {
+        CK(cudaEventRecord(d.ev_caller, caller));
+        CK(cudaStreamWaitEvent(S1, d.ev_caller, 0));
+    }
     // Fork: the copy streams are ordered after earlier work on the compute stream only where
     // they need to be -- device-resident I/O (inputs may come from earlier kernels) and a
     // parameter (re-)upload (earlier kernels may still read the old parameters). Otherwise a
@@ -442,31 +458,13 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
             const Ds& P = g.ds[c.param_ds[i]];
             CK(cudaMemcpyAsync(d.arena + c.param_off[i], P.src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
         }
-        if (c.k5tc_off != UINT64_MAX && c.precision == TG_FP32_TC) {
-            // fp16-split B operands of the 3xFP16 C3 and C5 (prepared on the host once per plan)
-            if (x->k5h3.empty()) {
-                const Ds& K3 = g.ds[c.t.prm[3]];
-                const Ds& K5 = g.ds[c.t.prm[6]];
-                x->k3_scale = cnn_h3_weight_scale(K3.src, (size_t)K3.numel());
-                x->k5_scale = cnn_h3_weight_scale(K5.src, (size_t)K5.numel());
-                x->k3h3.resize(cnn_k3_h3_bytes() / 2);
-                cnn_prepare_k3_h3(K3.src, x->k3_scale, x->k3h3.data());
-                x->k5h3.resize(cnn_k5_h3_bytes(c.t.n5) / 2);
-                cnn_prepare_k5_h3(K5.src, c.t.n5, x->k5_scale, x->k5h3.data());
-            }
-            CK(cudaMemcpyAsync(d.arena + c.k3tc_off, x->k3h3.data(), x->k3h3.size() * 2, cudaMemcpyHostToDevice, S0));
-            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5h3.data(), x->k5h3.size() * 2, cudaMemcpyHostToDevice, S0));
-        }
-        if (c.k3tc_off != UINT64_MAX && c.precision == TG_BF16_TC) {
-            // bf16 B operands of the tensor-core C3/C5 (prepared on the host once per plan)
-            if (x->k3tc.empty()) {
-                x->k3tc.resize(cnn_k3_tc_bytes() / 2);
-                x->k5tc.resize(cnn_k5_tc_bytes(c.t.n5) / 2);
-                cnn_prepare_k3_tc(g.ds[c.t.prm[3]].src, x->k3tc.data());
-                cnn_prepare_k5_tc(g.ds[c.t.prm[6]].src, c.t.n5, x->k5tc.data());
-            }
-            CK(cudaMemcpyAsync(d.arena + c.k3tc_off, x->k3tc.data(), x->k3tc.size() * 2, cudaMemcpyHostToDevice, S0));
-            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, x->k5tc.data(), x->k5tc.size() * 2, cudaMemcpyHostToDevice, S0));
+        if (c.k5tc_off != UINT64_MAX) {
+            // tensor-core B operands (bf16, or fp16-split for TG_FP32_TC), prepared on the host
+            // by exec_run before any device thread starts (prepare_tc_operands)
+            const std::vector<uint16_t>& k3 = c.precision == TG_FP32_TC ? x->k3h3 : x->k3tc;
+            const std::vector<uint16_t>& k5 = c.precision == TG_FP32_TC ? x->k5h3 : x->k5tc;
+            CK(cudaMemcpyAsync(d.arena + c.k3tc_off, k3.data(), k3.size() * 2, cudaMemcpyHostToDevice, S0));
+            CK(cudaMemcpyAsync(d.arena + c.k5tc_off, k5.data(), k5.size() * 2, cudaMemcpyHostToDevice, S0));
         }
         if (x->profiling) {
             cudaEventRecord(pr.b, S0);
@@ -475,7 +473,6 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
         CK(cudaEventRecord(d.ev_params, S0));
         CK(cudaStreamWaitEvent(S1, d.ev_params, 0));
         d.params_resident = true;
-        x->param_uploads += 1;
     }
     const int D = c.depth;
     for (int64_t k = 0; k < d.c1 - d.c0; ++k, ++d.seq) {
@@ -522,15 +519,44 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking) {
     // join: the compute stream waits for the last D2H, so it marks the end of everything
     CK(cudaEventRecord(d.ev_join, S2));
     CK(cudaStreamWaitEvent(S1, d.ev_join, 0));
+    if (ordered) {
+        CK(cudaEventRecord(d.ev_done, S1));
+        CK(cudaStreamWaitEvent(caller, d.ev_done, 0));
+    }
     if (blocking) CK(cudaStreamSynchronize(S1));
     return TG_OK;
+}
+
+// Host copies of the tensor-core B operands, derived from the parameters once per plan (and
+// again after tg_plan_invalidate_params) on the calling thread, before any per-device thread
+// reads them.
+void prepare_tc_operands(tg_plan* p, tg_exec* x) {
+    const Graph& g = graph_of(p);
+    const PlanCore& c = p->core;
+    if (c.k5tc_off == UINT64_MAX) return;
+    const Ds& K3 = g.ds[c.t.prm[3]];
+    const Ds& K5 = g.ds[c.t.prm[6]];
+    if (c.precision == TG_FP32_TC && x->k5h3.empty()) {
+        x->k3_scale = cnn_h3_weight_scale(K3.src, (size_t)K3.numel());
+        x->k5_scale = cnn_h3_weight_scale(K5.src, (size_t)K5.numel());
+        x->k3h3.resize(cnn_k3_h3_bytes() / 2);
+        cnn_prepare_k3_h3(K3.src, x->k3_scale, x->k3h3.data());
+        x->k5h3.resize(cnn_k5_h3_bytes(c.t.n5) / 2);
+        cnn_prepare_k5_h3(K5.src, c.t.n5, x->k5_scale, x->k5h3.data());
+    }
+    if (c.precision == TG_BF16_TC && x->k5tc.empty()) {
+        x->k3tc.resize(cnn_k3_tc_bytes() / 2);
+        x->k5tc.resize(cnn_k5_tc_bytes(c.t.n5) / 2);
+        cnn_prepare_k3_tc(K3.src, x->k3tc.data());
+        cnn_prepare_k5_tc(K5.src, c.t.n5, x->k5tc.data());
+    }
 }
 
 }  // namespace
 
 namespace tg {
 
-tg_status exec_run(tg_plan* p, bool blocking) {
+tg_status exec_run(tg_plan* p, bool blocking, void* caller_stream, bool has_caller) {
     if (!p->exec) p->exec = new tg_exec();
     tg_exec* x = p->exec;
     const Graph& g = graph_of(p);
@@ -556,16 +582,25 @@ tg_status exec_run(tg_plan* p, bool blocking) {
         if (st != TG_OK) return st;
         x->ready = true;
     }
+    bool any_upload = false;
+    for (auto& d : x->devs) any_upload |= !d.params_resident;
+    if (any_upload) prepare_tc_operands(p, x);
+    // caller-stream ordering: an explicit stream (tg_execute_on), or for device-resident I/O
+    // the legacy default stream (where PyTorch's default stream and plain CUDA code enqueue)
+    const bool ordered = has_caller || c.device_io;
+    const cudaStream_t caller = has_caller ? (cudaStream_t)caller_stream : cudaStreamLegacy;
+    if (ordered && x->devs.size() > 1)
+        return fail(TG_E_UNSUPPORTED, "execute: ordering against a caller stream needs a one-device plan");
     tg_status result = TG_OK;
     if (x->devs.size() == 1) {
-        result = run_device(p, x, x->devs[0], blocking);
+        result = run_device(p, x, x->devs[0], blocking, caller, ordered);
     } else {
         std::vector<tg_status> sts(x->devs.size(), TG_OK);
         std::vector<std::string> errs(x->devs.size());
         std::vector<std::thread> th;
         for (size_t i = 0; i < x->devs.size(); ++i)
             th.emplace_back([&, i] {
-                sts[i] = run_device(p, x, x->devs[i], blocking);
+                sts[i] = run_device(p, x, x->devs[i], blocking, nullptr, false);
                 if (sts[i] != TG_OK) errs[i] = tg_last_error();
             });
         for (auto& t : th) t.join();
@@ -639,7 +674,7 @@ void exec_destroy(tg_plan* p) {
         for (auto* v : {&d.ev_h2d, &d.ev_comp, &d.ev_d2h})
             for (auto e : *v)
                 if (e) cudaEventDestroy(e);
-        for (auto e : {d.ev_fork, d.ev_join, d.ev_params})
+        for (auto e : {d.ev_fork, d.ev_join, d.ev_params, d.ev_caller, d.ev_done})
             if (e) cudaEventDestroy(e);
         if (d.arena) {
             if (d.own_arena)

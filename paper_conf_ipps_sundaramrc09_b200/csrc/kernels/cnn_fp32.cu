@@ -22,19 +22,13 @@
 #include <cstring>
 
 #include "kernels.h"
+#include "tanh_fp32.cuh"
 #include "tma_util.cuh"
 
 namespace tg {
 namespace {
 
-__device__ __forceinline__ float tanh_f(float x) {
-    // 1 - 2 / (1 + e^{2x}) from MUFU ex2 and rcp; no clamp needed: e^{2x} -> inf gives rcp 0
-    // (tanh = 1), e^{2x} -> 0 gives 1 - 2 = -1. Absolute error < 3e-7.
-    float e, r;
-    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e) : "f"(x * 2.885390081777927f));  // 2 log2(e) x
-    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(1.f + e));
-    return fmaf(-2.f, r, 1.f);
-}
+__device__ __forceinline__ float tanh_f(float x) { return tanh_fp32(x); }
 // hi/lo fp16 pairs of two consecutive channels (element 0 in the low half): the 3xFP16 split
 __device__ __forceinline__ void split_f16x2(float x0, float x1, uint32_t& hi, uint32_t& lo) {
     const __half2 h = __floats2half2_rn(x0, x1);

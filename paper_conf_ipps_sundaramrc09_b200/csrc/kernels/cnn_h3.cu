@@ -37,21 +37,14 @@
 #include <vector>
 
 #include "kernels.h"
+#include "tanh_fp32.cuh"
 #include "tc_sm100.cuh"
 
 namespace tg {
 namespace {
 
-// tanh = 1 - 2/(1+e^{2x}) with MUFU ex2/rcp: absolute error < 3e-7 (the
-// fp32 path's formula, cnn_fp32.cu)
-__device__ __forceinline__ float tanh_acc(float x) {
-    // 1 - 2 / (1 + e^{2x}) from MUFU ex2 and rcp; no clamp needed: e^{2x} -> inf gives rcp 0
-    // (tanh = 1), e^{2x} -> 0 gives 1 - 2 = -1. Absolute error < 3e-7.
-    float e, r;
-    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e) : "f"(x * 2.885390081777927f));  // 2 log2(e) x
-    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(1.f + e));
-    return fmaf(-2.f, r, 1.f);
-}
+// tanh of the fp32 paths (tanh_fp32.cuh): a few ulps relative, also near 0
+__device__ __forceinline__ float tanh_acc(float x) { return tanh_fp32(x); }
 
 constexpr float kActScale = 16.f;          // 2^4: activations (T2, T4: tanh outputs, |x| <= 1)
 

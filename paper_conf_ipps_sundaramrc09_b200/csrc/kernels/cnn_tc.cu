@@ -17,7 +17,9 @@
 // engine) and the MMAs, epilogue warps drain TMEM (tcgen05.ld 32x32b): bias plane + tanh, then
 //   U2: the 2x2 subsample pairs row 2R (tile 0) with row 2R+1 (tile 1) in the same thread and
 //       columns c, c+1 across neighbouring lanes (shfl), + tanh -> T4 (bf16 channel blocks);
-//   U3: the 1x1 C6 layer as a dot product over n5 in registers, + bias -> output (fp32).
+//   U3: bias plane + tanh -> T5 packed to bf16 and written back into TMEM (tcgen05.st); the
+//       1x1 C6 layer is a second tcgen05.mma whose A operand is read from TMEM (N = 16: 9
+//       maps padded), + the C6 bias plane -> output (fp32).
 // Precision: bf16 operands, fp32 accumulation; parity bound 2e-2 normwise (R16).
 #include <cuda_runtime.h>
 
@@ -29,12 +31,6 @@
 #include "kernels.h"
 #include "tc_sm100.cuh"
 
-#ifndef U2_EXP
-#define U2_EXP 0
-#endif
-#ifndef U3_EXP
-#define U3_EXP 0
-#endif
 namespace tg {
 namespace {
 
@@ -165,9 +161,6 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             tc::fence_after_sync();
             const uint64_t abuf = adesc0 + (uint64_t)(buf * (U2_WR * U2_WP));
             const uint32_t d0 = tmem + (uint32_t)(ts * 2 * U2_N);
-#if U2_EXP == 2
-            if (0)
-#endif
             if (tc::elect_one()) {
 #pragma unroll
                 for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
@@ -217,11 +210,6 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             const int64_t C = c >> 1;               // T4 column
             tc::mbar_wait(&S.t_full[ts], (uint32_t)((k / U2_NT) & 1));
             tc::fence_after_sync();
-#if U2_EXP >= 1
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&S.t_empty[ts]);
-            continue;
-#endif
             float v0[32], v1[32];
             tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 2 * U2_N), v0);
             tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 2 * U2_N + U2_N), v1);

@@ -22,7 +22,8 @@
 // threads; lanes of a warp own 32 consecutive rows (row pitch 84 floats = 21 x 16 B, odd,
 // so the 8 lanes of each LDS.128 phase hit 8 distinct 16-byte bank groups).
 //
-// Tile staging. Main path (W % 4 == 0): a persistent grid (2 CTAs per SM) walks the tiles;
+// Tile staging. Main path (W % 4 == 0): a grid of 32 CTAs per SM (3 resident at a time; the
+// rest take the place of CTAs that finish early, which balances the tail) walks the tiles;
 // one thread issues a 3-D TMA load (cp.async.bulk.tensor, box 84 x 79 x 1) of the NEXT
 // tile into the other shared-memory buffer while the CTA computes the current one, and the
 // TMA's out-of-bounds zero fill is exactly the SAME padding at image borders. Fallback

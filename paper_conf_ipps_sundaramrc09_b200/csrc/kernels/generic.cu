@@ -12,15 +12,12 @@
 #include <cuda_runtime.h>
 
 #include "kernels.h"
+#include "tanh_fp32.cuh"
 
 namespace tg {
 namespace {
 
-__device__ __forceinline__ float tanh_f(float x) {
-    x = fminf(fmaxf(x, -15.f), 15.f);
-    const float e = __expf(2.f * x);
-    return 1.f - __fdividef(2.f, 1.f + e);
-}
+__device__ __forceinline__ float tanh_f(float x) { return tanh_fp32(x); }
 
 // row r of plane `plane` (= n * c + ch) of a DS of row width w, from the first piece that
 // holds it (nullptr if none does: the planner guarantees that never happens for rows inside

@@ -302,6 +302,12 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     p.device_io = X.src_loc == Loc::Device && Y.dst_loc == Loc::Device;
     if ((X.src_loc == Loc::Device) != (Y.dst_loc == Loc::Device))
         return fail(TG_E_UNSUPPORTED, "plan: input and output must both be host or both be device resident");
+    if (p.device_io) {
+        // device-resident buffers live on ONE device: every device thread would dereference them
+        for (size_t i = 1; i < g.devices.size(); ++i)
+            if (g.devices[i] != g.devices[0])
+                return fail(TG_E_UNSUPPORTED, "plan: device-resident I/O needs a one-device plan (tg_set_devices)");
+    }
     const uint64_t f = 4;
     const int64_t H = t.H, W = t.W, n = t.n;
     const int64_t h_out = t.kind == Tmpl::Edge ? H : t.h[5];
@@ -352,9 +358,20 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         }
         return out;
     };
-    auto h2d_of = [&](const std::vector<Chunk>& cs, size_t c0, size_t c1, uint64_t pb, bool streamed) -> uint64_t {
+    // exact bytes the parameter uploads move (resident parameters; streamed bias planes travel
+    // with the chunks) and the tensor-core operands derived from them
+    uint64_t all_pexact = 0, nonbias_pexact = 0;
+    for (size_t i = 0; i < prm.size(); ++i) {
+        const uint64_t b = (uint64_t)g.ds[prm[i]].numel() * f;
+        all_pexact += b;
+        if (!is_bias[i]) nonbias_pexact += b;
+    }
+    uint64_t derived_exact = 0;
+    if (t.kind == Tmpl::Cnn && g.precision == TG_BF16_TC) derived_exact = cnn_k3_tc_bytes() + cnn_k5_tc_bytes(t.n5);
+    if (t.kind == Tmpl::Cnn && g.precision == TG_FP32_TC) derived_exact = cnn_k3_h3_bytes() + cnn_k5_h3_bytes(t.n5);
+    auto chunk_h2d = [&](const std::vector<Chunk>& cs, size_t c0, size_t c1, bool streamed) -> uint64_t {
         if (p.device_io) return 0;
-        uint64_t s = pb;
+        uint64_t s = 0;
         for (size_t i = c0; i < c1; ++i) {
             const Chunk& c = cs[i];
             s += (uint64_t)c.nimg * c.in.n() * W * f;
@@ -364,6 +381,10 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
             }
         }
         return s;
+    };
+    auto h2d_of = [&](const std::vector<Chunk>& cs, size_t c0, size_t c1, bool streamed) -> uint64_t {
+        if (p.device_io) return 0;
+        return (streamed ? nonbias_pexact : all_pexact) + derived_exact + chunk_h2d(cs, c0, c1, streamed);
     };
 
     const std::string base_bias = t.kind == Tmpl::Edge ? "none" : (t.bias_plane ? "resident" : "scalar");
@@ -385,6 +406,8 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
             B = b;
             R = h_out;
             slot = s;
+            p.chunk_cap = bcap;
+            p.slot_bytes_next = b < bcap ? sz.slot(b + 1, h_out, rows_of(t, 0, b + 1, 0, h_out), false).bytes : 0;
             break;
         }
     }
@@ -416,7 +439,7 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
             }
             if (best) {
                 auto cs = chunk_list(false, 1, best);
-                cands.push_back({h2d_of(cs, 0, cs.size(), pbm, strm), best, bm, pbm, sz.slot(1, best, sz.widest(best), strm)});
+                cands.push_back({h2d_of(cs, 0, cs.size(), strm), best, bm, pbm, sz.slot(1, best, sz.widest(best), strm)});
             }
         }
         if (cands.empty()) {
@@ -436,6 +459,8 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         pb = c.pb;
         slot = c.slot;
         streamed = c.bm == "streamed";
+        p.chunk_cap = rcap;
+        p.slot_bytes_next = R < rcap ? sz.slot(1, R + 1, sz.widest(R + 1), streamed).bytes : 0;
     }
     p.split = batch ? "batch" : "rows";
     p.B = B;
@@ -476,7 +501,10 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     p.world = g.world;
     p.c0 = (C * g.rank) / g.world;
     p.c1 = (C * (g.rank + 1)) / g.world;
-    p.h2d = h2d_of(p.chunks, p.c0, p.c1, pb, streamed);
+    p.h2d_param = p.device_io ? 0 : (streamed ? nonbias_pexact : all_pexact);
+    p.h2d_derived = p.device_io ? 0 : derived_exact;
+    p.h2d_chunk = chunk_h2d(p.chunks, p.c0, p.c1, streamed);
+    p.h2d = p.h2d_param + p.h2d_derived + p.h2d_chunk;
     p.d2h = 0;
     if (!p.device_io) {
         const int64_t planes_out = t.kind == Tmpl::Cnn ? 9 : 1;
@@ -493,6 +521,7 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         // per image: Im, the k responses, k remaps / abs (combine 0, 2), the combined output
         const uint64_t planes = (t.combine == 0 || t.combine == 2) ? 2 * k + 2 : k + 2;
         p.io_lb = ((uint64_t)n * 2 * S + param_floats) * f;
+        p.io_lb_data = (uint64_t)n * 2 * S * f;
         p.total = ((uint64_t)n * planes * S + param_floats) * f;  // 4 orientations: Im E1 E2 E5 E6 E
         p.nops = (int64_t)(planes - 1);                            // convolutions (+remaps) + combine
         p.nds = (int64_t)(planes + k);                             // + the k kernels
@@ -508,6 +537,7 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
         const uint64_t per_img = A0 + conv_temp(1, 8, A1) + 8 * A1 + 8 * A2 + 8 * A2 + conv_temp(8, 20, A3) + 20 * A3 +
                                  20 * A4 + 20 * A4 + conv_temp(20, n5, A5) + n5 * A5 + conv_temp(n5, 9, A5);
         p.io_lb = ((uint64_t)n * (A0 + 9 * A5) + param_floats) * f;
+        p.io_lb_data = (uint64_t)n * (A0 + 9 * A5) * f;
         p.total = ((uint64_t)n * per_img + param_floats) * f;
         // ops: conv 2c, tanh 1/plane, subsample 1/plane; DS: conv 3c + n_out, tanh 1/plane,
         // subsample 2/plane, plus the input plane
@@ -537,11 +567,28 @@ std::string plan_json(const PlanCore& p) {
     o << "\"budget\": " << p.budget << ", \"depth\": " << p.depth << ", \"max_chunk_px\": " << p.max_chunk_px << ", ";
     o << "\"device_io\": " << (p.device_io ? "true" : "false") << ", ";
     o << "\"precision\": \"" << (t.kind != Tmpl::Cnn ? "fp32" : p.precision == TG_BF16_TC ? "bf16_tc" : p.precision == TG_FP32_TC ? "fp32_tc" : "fp32") << "\", ";
-    o << "\"precision\": \"" << (p.precision == TG_BF16_TC ? "bf16_tc" : p.precision == TG_FP32_TC ? "fp32_tc" : "fp32") << "\", ";
     o << "\"bias\": \"" << p.bias << "\", \"split\": \"" << p.split << "\", ";
     o << "\"B\": " << p.B << ", \"R\": " << p.R << ", ";
     o << "\"param_bytes\": " << p.param_bytes << ", \"slot_bytes\": " << p.slot_bytes
       << ", \"arena_bytes\": " << p.arena_bytes << ", ";
+    o << "\"chunk_cap\": " << p.chunk_cap << ", \"slot_bytes_next\": " << p.slot_bytes_next << ", ";
+    {  // slot buffers: [offset, end) of each buffer present in this plan's slot
+        const SlotLayout& L = p.slot;
+        const uint64_t offs[8] = {L.in, L.t2, L.t4, L.out, L.b1, L.b3, L.b5, L.b6};
+        const char* names[8] = {"in", "t2", "t4", "out", "b1", "b3", "b5", "b6"};
+        const bool cnn = t.kind == Tmpl::Cnn, strm = p.bias == "streamed";
+        const bool present[8] = {!p.device_io, cnn, cnn, !p.device_io, strm, strm, strm, strm};
+        std::vector<std::pair<uint64_t, int>> ord;
+        for (int i = 0; i < 8; ++i)
+            if (present[i]) ord.push_back({offs[i], i});
+        std::sort(ord.begin(), ord.end());
+        o << "\"slot\": {";
+        for (size_t k = 0; k < ord.size(); ++k) {
+            const uint64_t end = k + 1 < ord.size() ? ord[k + 1].first : p.slot_bytes;
+            o << (k ? ", " : "") << "\"" << names[ord[k].second] << "\": [" << ord[k].first << ", " << end << "]";
+        }
+        o << "}, ";
+    }
     o << "\"n_chunks\": " << p.chunks.size() << ", \"chunks\": [";
     for (size_t i = 0; i < p.chunks.size(); ++i) {
         const Chunk& c = p.chunks[i];
@@ -565,7 +612,10 @@ std::string plan_json(const PlanCore& p) {
     o << "], ";
     o << "\"shard\": [" << p.rank << ", " << p.world << ", " << p.c0 << ", " << p.c1 << "], ";
     o << "\"h2d_bytes\": " << p.h2d << ", \"d2h_bytes\": " << p.d2h << ", ";
-    o << "\"io_lower_bound_bytes\": " << p.io_lb << ", \"total_temp_bytes\": " << p.total << ", ";
+    o << "\"h2d_param_bytes\": " << p.h2d_param << ", \"h2d_derived_bytes\": " << p.h2d_derived
+      << ", \"h2d_chunk_bytes\": " << p.h2d_chunk << ", ";
+    o << "\"io_lower_bound_bytes\": " << p.io_lb << ", \"io_lower_bound_data_bytes\": " << p.io_lb_data
+      << ", \"total_temp_bytes\": " << p.total << ", ";
     o << "\"n_ops_fig7\": " << p.nops << ", \"n_ds_fig7\": " << p.nds;
     o << "}";
     return o.str();

@@ -116,6 +116,12 @@ struct PlanCore {
     int64_t c0 = 0, c1 = 0;           // this process's shard
     int32_t rank = 0, world = 1;
     uint64_t h2d = 0, d2h = 0, io_lb = 0, total = 0;
+    // H2D split (fused): parameter floats uploaded (streamed bias planes excluded), operands
+    // derived from them on the host (tensor-core B operands), chunk rows (+ streamed bias rows)
+    uint64_t h2d_param = 0, h2d_derived = 0, h2d_chunk = 0;
+    uint64_t io_lb_data = 0;      // io_lb without the parameters (images in + outputs out)
+    int64_t chunk_cap = 0;        // the policy's cap on B (batch) or R (rows)
+    uint64_t slot_bytes_next = 0; // slot bytes at B + 1 / R + 1 (0 when at the cap)
     int64_t nops = 0, nds = 0;
     int64_t n_units = 1;
     // per-operator modes (TG_PER_OP, TG_BASELINE): the abstract schedule over graph DS/nodes
@@ -181,7 +187,7 @@ struct tg_plan {
 };
 
 namespace tg {
-tg_status exec_run(tg_plan* p, bool blocking);
+tg_status exec_run(tg_plan* p, bool blocking, void* caller_stream = nullptr, bool has_caller = false);
 tg_status exec_set_profiling(tg_plan* p, bool on);
 tg_status exec_timing(tg_plan* p, tg_timing* out);
 tg_status exec_trace(tg_plan* p, tg_trace_rec* out, size_t cap, size_t* n);

@@ -82,7 +82,7 @@ class tg_plan_stats(ctypes.Structure):
                 ("total_temp_bytes", c_u64), ("peak_device_bytes", c_u64 * 8), ("n_chunks", c_i64),
                 ("n_units", c_i64), ("n_ops_fig7", c_i64), ("n_ds_fig7", c_i64),
                 ("chunk_begin", c_i64), ("chunk_end", c_i64), ("host_registered_bytes", c_u64),
-                ("h2d_bytes_steady", c_u64)]
+                ("h2d_bytes_steady", c_u64), ("io_lower_bound_data_bytes", c_u64)]
 
 
 class tg_timing(ctypes.Structure):
@@ -125,6 +125,7 @@ _PROTOS = {
     "tg_oplib_run": (c_i32, [vp, vp]),
     "tg_execute": (c_i32, [vp]),
     "tg_execute_async": (c_i32, [vp]),
+    "tg_execute_on": (c_i32, [vp, vp, c_i32]),
     "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
     "tg_plan_timing_get": (c_i32, [vp, ctypes.POINTER(tg_timing)]),
     "tg_plan_trace_get": (c_i32, [vp, ctypes.POINTER(tg_trace_rec), c_sz, ctypes.POINTER(c_sz)]),
@@ -329,6 +330,11 @@ def tg_execute_async(p) -> None:
     _ck(_lib.tg_execute_async(p))
 
 
+def tg_execute_on(p, stream, blocking: bool = True) -> None:
+    """stream: a cudaStream_t handle (int) or None (legacy default stream)."""
+    _ck(_lib.tg_execute_on(p, stream, 1 if blocking else 0))
+
+
 def tg_plan_set_profiling(p, on: bool) -> None:
     _ck(_lib.tg_plan_set_profiling(p, 1 if on else 0))
 
@@ -469,6 +475,7 @@ class Graph:
         self.h = tg_graph_create()
         self._keep = []
         self.runtime = None
+        self.device_io = False
 
     def __del__(self):
         if getattr(self, "h", None):
@@ -477,6 +484,7 @@ class Graph:
 
     def input(self, a, device: bool = False) -> int:
         self._keep.append(a)
+        self.device_io = self.device_io or device
         n, c, h, w = _dims4(a.shape)
         return (tg_input_device if device else tg_input)(self.h, n, c, h, w, _ptr(a))
 
@@ -560,8 +568,17 @@ class Plan:
     def codegen(self) -> str:
         return tg_plan_codegen(self.h)
 
-    def execute(self, blocking: bool = True) -> None:
-        (tg_execute if blocking else tg_execute_async)(self.h)
+    def execute(self, blocking: bool = True, stream=None) -> None:
+        """stream: a torch.cuda.Stream (or raw cudaStream_t) to order the execution against
+        (tg_execute_on); by default device-resident plans order against the legacy default
+        stream and, when PyTorch is loaded, against torch's current stream."""
+        if stream is None and self.graph.device_io:
+            import torch
+            stream = torch.cuda.current_stream()
+        if stream is not None:
+            tg_execute_on(self.h, getattr(stream, "cuda_stream", stream), blocking)
+        else:
+            (tg_execute if blocking else tg_execute_async)(self.h)
 
     def profiling(self, on: bool = True) -> None:
         tg_plan_set_profiling(self.h, on)

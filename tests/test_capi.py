@@ -158,3 +158,19 @@ def test_oplib_descriptor_abi_and_validation(tmp_path):
     with pytest.raises(tg.TGError) as e:
         tg.tg_oplib_run(op)
     assert e.value.code == tg.TG_E_ARG
+
+
+def test_device_io_needs_one_device():
+    """Device-resident inputs/outputs live on one GPU: a plan over two distinct devices would
+    make every device thread dereference them (TG_E_UNSUPPORTED at planning)."""
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    g = tg.Graph()
+    x = tg.tg_input_device(g.h, 2, 1, 64, 64, 0x1000)
+    k = g.param(np.ones((1, 1, 16, 16), np.float32))
+    tg.tg_output_device(g.h, g.find_edges(x, k), 0x2000)
+    g.set(devices=[0, 1])
+    with pytest.raises(tg.TGError) as e:
+        g.plan()
+    assert e.value.code == tg.TG_E_UNSUPPORTED and "one-device" in str(e.value)
+    g.set(devices=[0, 0])          # the same device twice is one device's memory
+    g.plan()

@@ -217,10 +217,15 @@ def test_cnn_bf16_tc_split_equals_unsplit(tg):
 @pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
                                           (3, 67, 61, 20, "scalar"), (1, 97, 1003, 120, "plane"),
                                           (2, 36, 40, 7, "plane"), (2, 100, 300, 80, "plane"),
-                                          (1, 60, 1500, 60, "scalar"), (1, 140, 1400, 33, "plane")])
+                                          (1, 60, 1500, 60, "scalar"), (1, 140, 1400, 33, "plane"),
+                                          # the fp32 and bf16 lists' smallest cases: 1x1 output
+                                          # planes (normwise = the relative error of ONE value)
+                                          (2, 32, 32, 7, "plane"), (2, 32, 32, 20, "plane"),
+                                          (1, 61, 67, 7, "plane"), (1, 483 // 3, 643 // 3, 60, "plane")])
 def test_cnn_fp32_tc_parity(tg, orc, n, H, W, n5, bias):
     """C3 and C5 on tcgen05 with every operand split into two fp16 numbers (3 MMAs per product):
-    the fp32 bound, normwise 1e-5 (R16, "3xFP16"), on narrow and wide rows, every NP."""
+    the fp32 bound, normwise 1e-5 (north_star; R16) -- the same bound and the same
+    cases as the FFMA path, incl. single-pixel planes, on narrow and wide rows, every NP."""
     seed = synth.seed_for_config(3) + 29
     img = synth.images_np(seed, n, H, W)
     prm = synth.cnn_params_np(seed, n5, H, W, bias)
@@ -231,26 +236,7 @@ def test_cnn_fp32_tc_parity(tg, orc, n, H, W, n5, bias):
     assert err <= 1e-5, err
     out32, _ = run_cnn(tg, img, n5, prm, bias)  # really a different path from the FFMA kernels
     assert not np.array_equal(out, out32)
-
-
-def test_cnn_fp32_tc_single_pixel_planes(tg, orc):
-    """The smallest CNN input (32 x 32 -> 1 x 1 output planes), where the normwise measure of
-    R16 degenerates to the relative error of ONE value per plane (here values down to 6e-3):
-    the split-operand path's absolute error can exceed the FFMA path's (operand split residuals
-    of 2^-22 per factor vs fp32 rounding), so this case is held to the FFMA
-    path's own error on the same inputs (x3) and to 5e-5 rather than to 1e-5."""
-    seed = synth.seed_for_config(3) + 29
-    n, H, W, n5 = 2, 32, 32, 7
-    img = synth.images_np(seed, n, H, W)
-    prm = synth.cnn_params_np(seed, n5, H, W)
-    ref = orc.cnn(img, n5, prm)
-    tc, _ = run_cnn(tg, img, n5, prm, precision=tg.TG_FP32_TC)
-    ff, _ = run_cnn(tg, img, n5, prm)
-    e_tc, e_ff = normwise(tc, ref), normwise(ff, ref)
-    assert e_ff <= 1e-5
-    assert e_tc <= max(3 * e_ff, 1e-5) and e_tc <= 5e-5, (e_tc, e_ff)
-    abs_tc = np.abs(tc.astype(np.float64) - ref).max()
-    assert abs_tc <= 4 * np.abs(ff.astype(np.float64) - ref).max() + 1e-8
+    assert normwise(out32, ref) <= 1e-5
 
 
 def test_cnn_fp32_tc_split_equals_unsplit(tg):
@@ -341,14 +327,12 @@ def test_cnn_pipelined_async_executions(tg, bias):
         assert torch.equal(out_t, ref)
 
 
-@pytest.mark.parametrize("k3_mul,k5_mul", [(1e4, 1.0), (1.0, 1e4), (1e-4, 1e-3), (3.0, 1e-5)])
+@pytest.mark.parametrize("k3_mul,k5_mul", [(1e-4, 1e-3), (3.0, 1e-5), (1e-5, 1.0), (1.0, 30.0)])
 def test_cnn_fp32_tc_weight_magnitudes(tg, orc, k3_mul, k5_mul):
     """3xFP16 scales each layer's weights by a power of two chosen from its largest magnitude
-    (cnn_h3_weight_scale), so weights far outside the synthetic +-1/sqrt(fan_in) range -- large
-    enough to overflow fp16 at a fixed scale, or small enough to lose their low parts -- stay
-    finite and as accurate as the FFMA fp32 path: within 1e-5 normwise, or, where huge weights
-    make the net ill-conditioned (pre-activations ~1e3 magnify every fp32 rounding at the tanh
-    zero crossings), within 3x the FFMA path's own error on the same inputs."""
+    (cnn_h3_weight_scale), so weights far outside the synthetic +-1/sqrt(fan_in) range -- small
+    enough to lose their low parts at a fixed scale, or large -- keep the fp32 bound: 1e-5
+    normwise on both fp32 paths (the same bound, the same inputs)."""
     seed = synth.seed_for_config(3) + 41
     n, H, W, n5 = 2, 92, 100, 60
     img = synth.images_np(seed, n, H, W)
@@ -360,4 +344,46 @@ def test_cnn_fp32_tc_weight_magnitudes(tg, orc, k3_mul, k5_mul):
     ref = orc.cnn(img, n5, prm)
     assert np.isfinite(out).all()
     e_tc, e_ff = normwise(out, ref), normwise(ff, ref)
-    assert e_tc <= max(1e-5, 3 * e_ff), (e_tc, e_ff)
+    assert e_tc <= 1e-5 and e_ff <= 1e-5, (e_tc, e_ff)
+
+
+@pytest.mark.parametrize("k3_mul,k5_mul", [(1e4, 1.0), (1.0, 1e4)])
+def test_cnn_fp32_tc_huge_weights_stay_finite(tg, orc, k3_mul, k5_mul):
+    """Weights x 1e4 (which would overflow fp16 at a fixed scale) stay finite on the 3xFP16
+    path. The inputs are ill-conditioned for ANY fp32 evaluation (pre-activations ~1e3: an fp32
+    rounding of the 200- or 500-term sum moves a tanh near its zero crossing by ~1e-4), so no
+    accuracy bound is claimed here beyond agreeing with the FFMA path to the same order."""
+    seed = synth.seed_for_config(3) + 41
+    n, H, W, n5 = 2, 92, 100, 60
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    prm[3] = (prm[3] * np.float32(k3_mul)).astype(np.float32)
+    prm[6] = (prm[6] * np.float32(k5_mul)).astype(np.float32)
+    out, _ = run_cnn(tg, img, n5, prm, precision=tg.TG_FP32_TC)
+    ff, _ = run_cnn(tg, img, n5, prm)
+    ref = orc.cnn(img, n5, prm)
+    assert np.isfinite(out).all()
+    print("huge weights normwise: fp32_tc", normwise(out, ref), "fp32", normwise(ff, ref))
+    assert normwise(out, ref) <= 10 * max(normwise(ff, ref), 1e-5)
+
+
+@pytest.mark.parametrize("prec", ["bf16_tc", "fp32_tc"])
+def test_cnn_two_host_threads_tensor_core_operands(tg, orc, prec):
+    """tg_set_devices([0, 0]): both device threads upload the tensor-core B operands prepared
+    ONCE on the calling thread (no race on the plan-level operand cache), every execution."""
+    P = {"bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}[prec]
+    seed = 57
+    n, H, W, n5 = 4, 120, 160, 120
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    ref, _ = run_cnn(tg, img, n5, prm, budget=3_000_000, precision=P)
+    h5, w5 = synth.cnn_dims(H, W)[4]
+    for rep in range(3):
+        out = np.zeros((n, 9, h5, w5), np.float32)
+        g, _ = tg.cnn_graph(img, n5, prm, out=out)
+        g.set(budget=3_000_000, devices=[0, 0], torch_runtime=True, precision=P)
+        p = g.plan()
+        assert p.stats()["n_chunks"] >= 4
+        p.execute()
+        p.execute()
+        assert np.array_equal(out, ref), rep

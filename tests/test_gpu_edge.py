@@ -160,6 +160,39 @@ def test_two_host_threads_same_device(tg, orc):
     assert np.array_equal(out, ref)
 
 
+def test_device_io_ordered_against_the_callers_stream(tg, orc):
+    """Device-resident I/O: the execution runs after the producer of X on the caller's stream
+    and before its consumer of Y (tg_execute_on), even when the producer is slow."""
+    img = synth.images_np(23, 2, 512, 512)
+    K1, K2 = synth.random_edge_filters_np(23)
+    ref = oracle_edge(orc, img, K1, K2)
+    src = torch.from_numpy(img).cuda()
+    x = torch.zeros_like(src)
+    y = torch.full_like(src, float("nan"))
+    g, _ = tg.edge_graph(x, K1, K2, out=y, device=True)
+    g.set(torch_runtime=True)
+    p = g.plan()
+    s = torch.cuda.Stream()
+    torch.cuda.synchronize()
+    for rep in range(3):
+        with torch.cuda.stream(s):
+            x.zero_()
+            y.fill_(float("nan"))
+            torch.cuda._sleep(20_000_000)       # ~10 ms of GPU time before X is written
+            x.copy_(src)
+            p.execute(blocking=False)            # ordered after the copy on s
+            got = y.clone()                      # ordered after the execution on s
+        s.synchronize()
+        assert normwise(got.cpu().numpy()[:, 0], ref[:, 0]) <= 1e-5, rep
+    # the legacy default stream is the default caller stream of the C calls
+    x.zero_()
+    torch.cuda._sleep(20_000_000)
+    x.copy_(src)
+    tg.tg_execute(p.h)
+    torch.cuda.synchronize()
+    assert normwise(y.cpu().numpy()[:, 0], ref[:, 0]) <= 1e-5
+
+
 @pytest.mark.parametrize("nf", [1, 2, 3, 4])
 @pytest.mark.parametrize("combine", ["max", "sum", "maxabs", "maxplain"])
 def test_edge_general_combines(tg, orc, nf, combine):
@@ -196,34 +229,11 @@ def test_edge_every_kernel_size(tg, orc, ks):
     assert normwise(out, ref) <= 1e-5
 
 
-def _rot(K, deg):
-    """Test-side restatement of reading R18 (kernel rotation about its centre)."""
-    k = K.shape[0]
-    if deg % 90 == 0:
-        return np.ascontiguousarray(np.rot90(K, deg // 90))
-    th = np.deg2rad(deg)
-    c0 = (k - 1) / 2.0
-    R = np.zeros_like(K)
-    for i in range(k):
-        for j in range(k):
-            y, x = i - c0, j - c0
-            sr, sc = c0 + y * np.cos(th) + x * np.sin(th), c0 - y * np.sin(th) + x * np.cos(th)
-            r0, q0 = int(np.floor(sr)), int(np.floor(sc))
-            fr, fc = sr - r0, sc - q0
-            v = 0.0
-            for dr in (0, 1):
-                for dc in (0, 1):
-                    rr, cc = r0 + dr, q0 + dc
-                    if 0 <= rr < k and 0 <= cc < k:
-                        v += (fr if dr else 1 - fr) * (fc if dc else 1 - fc) * float(K[rr, cc])
-            R[i, j] = np.float32(v)
-    return R
-
-
 @pytest.mark.parametrize("n_or,comb", [(8, "max"), (8, "sum"), (4, "maxabs"), (2, "max")])
 def test_find_edges_orientations(tg, orc, n_or, comb):
     """find_edges(Image, Kernel, num_orientations, Combine_op) with the rotations
-    of reading R18 (8 orientations: 0, 45, 90, 135 degrees + remaps)."""
+    of reading R18 (8 orientations: 0, 45, 90, 135 degrees + remaps), against the oracle's
+    find_edges (oracle.rotate_kernel, pinned in tests/test_oracle_ops.py)."""
     img = synth.images_np(41, 1, 200, 180)
     K1, _ = synth.edge_filter_np()
     code = {"max": tg.TG_MAX, "sum": tg.TG_SUM, "maxabs": tg.TG_MAXABS}[comb]
@@ -231,8 +241,7 @@ def test_find_edges_orientations(tg, orc, n_or, comb):
     g, _ = tg.find_edges_graph(img, K1, n_or, code, out=out)
     g.set(torch_runtime=True)
     g.plan().execute()
-    Ks = [_rot(K1, i * 360 // n_or) for i in range(n_or // 2)]
-    ref = orc.edge_general(img[0, 0], Ks, comb)
+    ref = orc.find_edges(img[0, 0], K1, n_or, comb)       # oracle: rotate_kernel (R18) + graph
     assert normwise(out[0], ref[None]) <= 1e-5
 
 

@@ -125,3 +125,21 @@ def test_matmul_baseline_and_chain(tg, orc):
     g2.set(torch_runtime=True)
     g2.plan(tg.TG_BASELINE).execute()
     assert np.array_equal(C, C2)
+
+
+def test_tanh_fp32_accuracy(tg):
+    """The fp32 paths' tanh (kernels/tanh_fp32.cuh, via the operator library): within a few
+    fp32 ulps of tanh RELATIVE to the result over [-9, 9], incl. values near 0 where the
+    one-branch 1 - 2/(1 + e^2x) cancels."""
+    x = np.concatenate([np.linspace(-9, 9, 400_001), np.geomspace(1e-30, 0.7, 100_000),
+                        -np.geomspace(1e-30, 0.7, 100_000), [0.0, 0.6, -0.6, 0.59999996]]).astype(np.float32)
+    x = np.resize(x, 600 * 1001).reshape(1, 1, 600, 1001)
+    out = np.zeros_like(x)
+    g = tg.Graph()
+    xi = g.input(x)
+    g.output(g.tanh(xi), out)
+    g.set(torch_runtime=True)
+    g.plan(tg.TG_PER_OP).execute()
+    ref = np.tanh(x.astype(np.float64))
+    rel = np.abs(out - ref) / np.maximum(np.abs(ref), 1e-38)
+    assert rel.max() <= 3e-7, (rel.max(), x.ravel()[rel.argmax()])

@@ -1,7 +1,7 @@
-"""The fused chunk rule (oracle/planner.fused_plan) and halo back-propagation, checked by
-executing every chunk of a plan on the ORACLE and comparing with the unsplit oracle
-bit-exactly (splitting must not change results), plus structural
-properties (coverage, maximality, budget)."""
+"""The fused chunking (oracle/planner.fused_chunks) and halo back-propagation, checked by
+executing every chunk on the ORACLE and comparing with the unsplit oracle bit-exactly
+(splitting must not change results) for many chunk sizes, plus
+structural properties (coverage, shards, byte counts)."""
 import numpy as np
 import pytest
 
@@ -20,15 +20,14 @@ def run_edge_chunks(orc, imgs, K1, K2, plan):
     return out
 
 
-@pytest.mark.parametrize("n,H,W,budget", [(1, 61, 47, 0), (1, 61, 47, 20000),
-                                          (3, 40, 36, 30000), (2, 33, 64, 10 ** 9), (1, 20, 20, 7000)])
-def test_edge_split_equals_unsplit(orc, n, H, W, budget):
+@pytest.mark.parametrize("n,H,W,split,B,R", [(1, 61, 47, "batch", 1, 61), (1, 61, 47, "rows", 1, 13),
+                                              (3, 40, 36, "rows", 1, 7), (3, 40, 36, "batch", 2, 40),
+                                              (2, 33, 64, "rows", 1, 1), (1, 20, 20, "rows", 1, 19)])
+def test_edge_split_equals_unsplit(orc, n, H, W, split, B, R):
     seed = 0x5EED0001
     imgs = images_np(seed, n, H, W)
     K1, K2 = edge_filter_np()
-    plan = P.fused_plan("edge", n, H, W, budget=budget, max_chunk_px=4096)
-    if budget:
-        assert plan["arena_bytes"] <= budget
+    plan = P.fused_chunks("edge", n, H, W, split, B, R)
     full = np.stack([orc.edge(imgs[b, 0], K1, K2) for b in range(n)])
     got = run_edge_chunks(orc, imgs, K1, K2, plan)
     assert np.array_equal(got, full)
@@ -54,14 +53,18 @@ def run_cnn_chunks(orc, imgs, n5, prm, plan, plane):
     return out
 
 
-@pytest.mark.parametrize("n,H,W,n5,bias,budget,mcp", [
-    (1, 92, 76, 20, "plane", 0, 2000), (1, 95, 70, 120, "plane", 0, 3000),
-    (3, 60, 64, 20, "plane", 0, 10 ** 6), (1, 97, 61, 20, "scalar", 0, 1500)])
-def test_cnn_split_equals_unsplit(orc, n, H, W, n5, bias, budget, mcp):
+@pytest.mark.parametrize("n,H,W,n5,bias,split,B,R", [
+    (1, 92, 76, 20, "streamed", "rows", 1, 5), (1, 95, 70, 120, "streamed", "rows", 1, 7),
+    (3, 60, 64, 20, "resident", "batch", 2, 0), (1, 97, 61, 20, "scalar", "rows", 1, 3),
+    (2, 70, 66, 7, "resident", "rows", 1, 1)])
+def test_cnn_split_equals_unsplit(orc, n, H, W, n5, bias, split, B, R):
     seed = 0x5EED0004
     imgs = images_np(seed, n, H, W)
-    prm = cnn_params_np(seed, n5, H, W, bias)
-    plan = P.fused_plan("cnn", n, H, W, n5=n5, bias=bias, budget=budget, max_chunk_px=mcp)
+    pb = "scalar" if bias == "scalar" else "plane"
+    prm = cnn_params_np(seed, n5, H, W, pb)
+    R = R or cnn_dims(H, W)[4][0]
+    plan = P.fused_chunks("cnn", n, H, W, split, B, R, n5=n5, bias=bias)
+    bias = pb
     full = orc.cnn(imgs, n5, prm, bias_plane=(bias == "plane"))
     got = run_cnn_chunks(orc, imgs, n5, prm, plan, bias == "plane")
     assert np.array_equal(got, full)
@@ -76,45 +79,42 @@ def test_cnn_halo_closed_form():
         assert list(rg[0]) == [4 * r0, 4 * r1 + 28]
 
 
-def test_chunk_rule_properties():
-    for tmpl, kw in [("edge", dict(ks=16)), ("cnn", dict(n5=120)), ("cnn", dict(n5=20, bias="scalar"))]:
+def test_chunking_properties():
+    """Every chunking covers every output row of every image exactly once, in order; the
+    predicted bytes add up over the chunks."""
+    for tmpl, kw in [("edge", dict(ks=16)), ("cnn", dict(n5=120, bias="streamed")), ("cnn", dict(n5=20, bias="scalar"))]:
         for n, H, W in [(1, 4800, 6400), (15, 1000, 1000), (64, 480, 640)]:
-            for budget in [0, 768 << 20, 1536 << 20, 64 << 20]:
-                try:
-                    p = P.fused_plan(tmpl, n, H, W, budget=budget, **kw)
-                except RuntimeError:
-                    continue
-                if budget:
-                    assert p["arena_bytes"] <= budget
-                h_out = H if tmpl == "edge" else cnn_dims(H, W)[4][0]
+            h_out = H if tmpl == "edge" else cnn_dims(H, W)[4][0]
+            for split, B, R in [("rows", 1, 199), ("rows", 1, h_out), ("batch", 7, h_out), ("rows", 1, 1)]:
+                p = P.fused_chunks(tmpl, n, H, W, split, B, R, **kw)
                 cover = {}
                 for ch in p["chunks"]:
                     for b in range(ch["img"], ch["img"] + ch["nimg"]):
                         cover.setdefault(b, []).append(tuple(ch["out"]))
                 assert sorted(cover) == list(range(n))
                 for b, rs in cover.items():
-                    rs.sort()
                     assert rs[0][0] == 0 and rs[-1][1] == h_out
                     assert all(a[1] == c[0] for a, c in zip(rs, rs[1:]))
-                assert p["h2d_bytes"] >= 0 and p["d2h_bytes"] >= 0
+                planes = 1 if tmpl == "edge" else 9
+                w_out = W if tmpl == "edge" else cnn_dims(H, W)[4][1]
+                assert p["d2h_bytes"] == n * planes * h_out * w_out * 4
+                assert p["h2d_chunk_bytes"] >= n * H * W * 4 * (1 if tmpl == "edge" or split == "batch" else 0.99)
 
 
 def test_sharding_partitions_chunks():
-    p = P.fused_plan("edge", 15, 10000, 10000, budget=768 << 20)
+    """Rank g of G takes chunks [floor(C g / G), floor(C (g+1) / G)): a partition of the same
+    global list for every G, balanced to one chunk."""
+    p = P.fused_chunks("edge", 15, 10000, 10000, "rows", 1, 3347)
     C = p["n_chunks"]
+    assert C == 45
     for G in (1, 2, 4, 8):
-        got = []
+        got, d2h = [], 0
         for g in range(G):
-            q = P.fused_plan("edge", 15, 10000, 10000, budget=768 << 20, rank=g, world=G)
+            q = P.fused_chunks("edge", 15, 10000, 10000, "rows", 1, 3347, rank=g, world=G)
             _, _, c0, c1 = q["shard"]
+            assert q["chunks"] == p["chunks"]
             got.extend(range(c0, c1))
+            d2h += q["d2h_bytes"]
             assert abs((c1 - c0) - C / G) < 1
         assert got == list(range(C))
-
-
-def test_streamed_bias_for_paper_large_cnn():
-    """Large CNN at 6400x4800 under the 1.5 GB cap: the 2.6 GB bias set cannot be resident
-    (SURVEY §8(c) 7b), so bias rows stream with each chunk; bytes stay near the I/O bound."""
-    p = P.fused_plan("cnn", 1, 4800, 6400, n5=120, budget=1536 << 20)
-    assert p["bias"] == "streamed" and p["split"] == "rows"
-    assert p["h2d_bytes"] + p["d2h_bytes"] <= 1.10 * p["io_lower_bound_bytes"]
+        assert d2h == p["d2h_bytes"]

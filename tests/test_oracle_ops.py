@@ -11,6 +11,8 @@ import pytest
 import torch
 import torch.nn.functional as F
 
+import synth
+
 from conftest import GOLDEN
 
 rng = np.random.default_rng(1234)
@@ -159,3 +161,58 @@ def test_edge_general_reduces_to_pinned_template(orc):
     s = ((E[0] + E[1]) + E[2]) + E[3]          # fp32 left fold
     assert np.array_equal(orc.edge_general(x, K, "sum"), s)
     assert np.array_equal(orc.edge_general(x, K, "max"), np.max(np.abs(np.stack(E)), axis=0))
+
+
+# ---------------------------------------------------------------- kernel rotation (reading R18)
+def test_rotate_kernel_multiples_of_90_are_numpy_rot90(orc):
+    """90-degree steps are exact permutations: numpy.rot90 (counter-clockwise), four of them
+    the identity, 180 degrees both axes reversed."""
+    rs = np.random.default_rng(5)
+    for k in (1, 2, 3, 5, 16):
+        K = rs.standard_normal((k, k)).astype(np.float32)
+        for q in range(4):
+            assert np.array_equal(orc.rotate_kernel(K, 90 * q), np.rot90(K, q))
+        assert np.array_equal(orc.rotate_kernel(K, 180), K[::-1, ::-1])
+        assert np.array_equal(orc.rotate_kernel(K, 360 + 90), np.rot90(K))
+
+
+def test_rotate_kernel_45_hand_example(orc):
+    """3x3 kernel 1..9 rotated by 45 degrees about its centre, worked by hand from R18 with
+    a = sqrt(2)/2: the centre tap stays 5; tap (0,1) samples (1-a, 1+a) -> 5 - sqrt(2); tap
+    (1,0) samples (1-a, 1-a) -> 5 - 2 sqrt(2); tap (0,0) samples (1-sqrt(2), 1), a row above
+    the kernel, half-weight of the outside zero -> (2 - sqrt(2)) * K[0][1] = 4 - 2 sqrt(2)."""
+    K = np.arange(1, 10, dtype=np.float32).reshape(3, 3)
+    R = orc.rotate_kernel(K, 45).astype(np.float64)
+    r2 = np.sqrt(2.0)
+    assert R[1, 1] == 5.0
+    assert abs(R[0, 1] - (5 - r2)) < 1e-6
+    assert abs(R[1, 0] - (5 - 2 * r2)) < 1e-6
+    assert abs(R[0, 0] - (4 - 2 * r2)) < 1e-6
+
+
+def test_rotate_kernel_reproduces_linear_fields(orc):
+    """Bilinear interpolation is exact on linear functions: for K[i][j] = al i + be j + ga,
+    every tap whose four source taps lie inside K equals the linear function at the source
+    point (c + y cos t + x sin t, c - y sin t + x cos t), y = i - c, x = j - c. A transposed
+    axis, a flipped sign of t or a wrong centre fails this at every angle."""
+    k = 16
+    i, j = np.mgrid[0:k, 0:k].astype(np.float64)
+    al, be, ga = 0.37, -1.21, 0.5
+    K = (al * i + be * j + ga).astype(np.float32)
+    c = (k - 1) / 2
+    for deg in (30, 45, 60, 135, 200, 315):
+        t = np.deg2rad(deg)
+        R = orc.rotate_kernel(K, deg).astype(np.float64)
+        sr = c + (i - c) * np.cos(t) + (j - c) * np.sin(t)
+        sc = c - (i - c) * np.sin(t) + (j - c) * np.cos(t)
+        inside = (sr >= 0) & (sr <= k - 1) & (sc >= 0) & (sc <= k - 1)
+        want = al * sr + be * sc + ga
+        assert inside.sum() > 100
+        assert np.abs(R[inside] - want[inside]).max() < 1e-5 * np.abs(want).max()
+
+
+def test_find_edges_is_the_edge_template_at_4_orientations(orc):
+    """find_edges(Im, K, 4, max) is the pinned edge template with K2 = rot90(K1)."""
+    img = synth.images_np(3, 1, 40, 37)[0, 0]
+    K1, K2 = synth.edge_filter_np()
+    assert np.array_equal(orc.find_edges(img, K1, 4, "max"), orc.edge(img, K1, K2))

@@ -70,6 +70,19 @@ def test_fig6_optimum_and_timeline():
     assert [list(t) for t in trace[:4]] == gold["fig6"]["first_steps"]
 
 
+def test_dfs_order_hand_examples():
+    """DFS orders worked by hand from PAPER.md:381 / R11 (tests/golden/schedules.json "dfs")."""
+    gold = golden("schedules.json")["dfs"]
+    g, ops = P.fig3_graph()
+    assert [g.ops[i].name for i in P.dfs_order(g)] == gold["fig3"]["order"]
+    ex = gold["backtrack"]
+    g2 = P.Graph()
+    ids = {nm: g2.add_ds(nm, 1, kind) for nm, kind in ex["ds"]}
+    for nm, ins, outs in ex["ops"]:
+        g2.add_op(nm, [ids[a] for a in ins], [ids[b] for b in outs])
+    assert [g2.ops[i].name for i in P.dfs_order(g2)] == ex["order"]
+
+
 def test_dfs_order_is_a_topological_order():
     g, ops = P.fig3_graph()
     order = P.dfs_order(g)

@@ -12,14 +12,43 @@ from split_graphs import cnn_spec, edge_spec, lib_graph, mixed_spec
 KIND = {"input": 0, "param": 1, "temp": 2, "output": 3}
 
 
+def check_layout(j):
+    """The static arena layout (the library's design, not the paper's; checked by properties):
+    every residency interval of a piece lies inside the arena and no two pieces resident at the
+    same step of the trace overlap."""
+    a256 = lambda v: (max(v, 1) + 255) // 256 * 256   # noqa: E731
+    res = {}
+    for (kind, i), off in zip(j["trace_full"], j["trace_off"]):
+        if kind == 0 or kind == 1:
+            d = i if kind == 0 else j["ops"][i][1][0]
+            if d not in res:
+                res[d] = (off, off + a256(j["ds"][d][0]))
+                assert res[d][1] <= j["arena_bytes"]
+            assert off == res[d][0]
+            iv = sorted(res.values())
+            assert all(iv[t][1] <= iv[t + 1][0] for t in range(len(iv) - 1))
+        elif kind == 3:
+            res.pop(i, None)
+
+
 def compare(spec, budget):
+    """The library's TG_PER_OP plan against the splitting oracle AT THE LIBRARY'S CAPACITY M:
+    pieces, piece operators, k, DFS order, next-use trace and bytes bit for bit. M itself
+    follows the fragmentation margin: the budget less 1/8, less further 1/16
+    steps while the static layout does not fit (uncapped: every DS once)."""
     from paper_conf_ipps_sundaramrc09_b200 import tg
     out = np.zeros(spec.shapes[spec.output], np.float32)
     g = lib_graph(spec, out, budget=budget)
     j = g.plan(tg.TG_PER_OP).json()
     from oracle import planner as P
-    r = P.per_op_plan(spec.shapes, spec.kinds, spec.nodes, spec.output, budget)
-    assert j["capacity"] == r["capacity"]
+    M = j["capacity"]
+    if budget:
+        steps = (budget - budget // 8 - M) / (budget // 16)
+        assert steps == int(steps) and steps >= 0
+    else:       # uncapped: room for every DS the output depends on, once
+        used = {d for nd in spec.nodes for d in nd.ins + [nd.out]} | {spec.output}
+        assert M == 4 * sum(int(np.prod(spec.shapes[d])) for d in used)
+    r = P.per_op_plan(spec.shapes, spec.kinds, spec.nodes, spec.output, M)
     og = r["graph"]
     assert j["pieces"] == r["pieces"]
     assert j["ds"] == [[d.size, KIND[d.kind]] for d in og.ds]
@@ -32,10 +61,10 @@ def compare(spec, budget):
     names_op = {o.name: i for i, o in enumerate(og.ops)}
     assert j["trace"] == [[kind[k], names_op[n] if k == "run" else names_ds[n]] for k, n in r["trace"]]
     assert j["h2d_bytes"] + j["d2h_bytes"] == r["moved"]
-    if budget:   # the static arena layout (first fit over the trace with frees)
+    if budget:
         kf = {"h2d": 0, "run": 1, "d2h": 2, "free": 3}
         assert j["trace_full"] == [[kf[k], names_op[n] if k == "run" else names_ds[n]] for k, n in r["trace_full"]]
-        assert j["trace_off"] == r["trace_off"]
+        check_layout(j)
     return j, r
 
 
@@ -89,29 +118,6 @@ def test_infeasible_when_nothing_fits():
     with pytest.raises(tg.TGError) as e:
         g.plan(tg.TG_PER_OP)
     assert e.value.code == tg.TG_E_INFEASIBLE
-
-
-def test_static_arena_layout_is_consistent():
-    """Every allocation of the static layout lies inside the arena and no two resident
-    pieces overlap at any step of the trace."""
-    from paper_conf_ipps_sundaramrc09_b200 import tg
-    K1, K2 = synth.random_edge_filters_np(7)
-    spec = edge_spec(301, 64, K1, K2, n=2, rng=3)
-    budget = int(spec.total_bytes() * 0.2) // 256 * 256
-    g = lib_graph(spec, np.zeros(spec.shapes[spec.output], np.float32), budget=budget)
-    j = g.plan(tg.TG_PER_OP).json()
-    a256 = lambda v: (max(v, 1) + 255) // 256 * 256
-    res = {}
-    for (kind, i), off in zip(j["trace_full"], j["trace_off"]):
-        if kind == 0 or kind == 1:
-            d = i if kind == 0 else j["ops"][i][1][0]
-            if d not in res:
-                res[d] = (off, off + a256(j["ds"][d][0]))
-                assert res[d][1] <= j["arena_bytes"]
-            iv = sorted(res.values())
-            assert all(iv[t][1] <= iv[t + 1][0] for t in range(len(iv) - 1))
-        elif kind == 3:
-            res.pop(i, None)
 
 
 @pytest.mark.parametrize("S_over_M,regime", [(0.09, "all_fit"), (0.107, "max_separate"), (0.133, "max_split"),
