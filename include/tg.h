@@ -161,7 +161,12 @@ tg_status tg_set_precision(tg_graph* g, int32_t prec);
  * (in-flight chunk slots, default 3, 1..8). */
 tg_status tg_set_chunking(tg_graph* g, int64_t max_chunk_px, int32_t depth);
 /* Multi-process sharding: this process executes chunk range [floor(C*rank/world),
- * floor(C*(rank+1)/world)) of the global chunk list (no collective). */
+ * floor(C*(rank+1)/world)) of the global chunk list (no collective). The chunk
+ * list is the same for every world size, so outputs are bit-identical across world sizes.
+ * The template input and output buffers are only read and written over the span of this
+ * shard's chunks (tg_plan_stats chunk_begin/chunk_end; the JSON plan lists each chunk's rows):
+ * a process may pass a base pointer whose other parts are not mapped, holding only its share
+ * of a global host input (only that span is page-locked). */
 tg_status tg_set_shard(tg_graph* g, int32_t rank, int32_t world);
 
 /* Runtime hooks (PyTorch-backed in the Python binding). alloc returns device memory on
@@ -228,7 +233,9 @@ tg_status tg_execute_on(tg_plan* plan, void* stream, int32_t blocking);
 
 /* Per-launch timing of the fused kernels measured with CUDA events on the compute stream
  * (enable before executing; tg_plan_timing_get synchronizes). Times are summed over all
- * executions since enabling. */
+ * executions since enabling. on = 1: kernels and every H2D/D2H copy (events on the copy
+ * streams make a copy engine finish one copy before starting the next, so streamed steps
+ * slow down); on = 2: kernels only (no events on the copy streams); 0: off. */
 typedef struct {
     int64_t launches;        /* kernel launches of the library                          */
     int64_t executions;
@@ -351,6 +358,13 @@ tg_status tg_sched_transfers(const tg_sched* s, const int32_t* order, uint64_t c
  * factorial: meant for graphs of ~12 operators or fewer); TG_E_INFEASIBLE if no order fits. */
 tg_status tg_sched_optimal(const tg_sched* s, uint64_t capacity, uint64_t max_orders, int32_t* order,
                            uint64_t* moved, uint64_t* n_orders, uint64_t* n_optimal);
+
+/* ------------------------------------------------------------------ measurement */
+/* Measured FP32 FFMA peak of `device` in TFLOP/s (2 flop per FMA lane): a probe kernel of
+ * independent paired-FMA (FFMA2) chains over every SM, best of a few launches of tens of ms,
+ * at the clocks the device runs at. The denominator of the ALU-bound rooflines (not part of
+ * the paper's method). Synchronizes the device; TG_E_CUDA on failure. */
+tg_status tg_probe_fp32_peak(int32_t device, double* tflops);
 
 const char* tg_last_error(void);
 /* Library version string, e.g. "tg 0.1 sm_100a". */

@@ -1,11 +1,14 @@
 // api.cpp -- the C ABI of include/tg.h: graph building, target parameters, plan handles.
 // Graph nodes follow the paper's operator graph (vertices are parallel
 // computations, edges data dependencies; footprints statically known).
+#include <cuda_runtime.h>
+
 #include <cmath>
 #include <cstring>
 #include <new>
 #include <string>
 
+#include "kernels/kernels.h"
 #include "tg_internal.h"
 
 namespace tg {
@@ -42,7 +45,16 @@ static tg_id add_ds(Graph& g, const int64_t d[4], DsKind kind) {
 extern "C" {
 
 const char* tg_last_error(void) { return g_last_error.c_str(); }
-const char* tg_version(void) { return "tg 0.1 sm_100a"; }
+const char* tg_version(void) { return "tg 0.2 sm_100a"; }
+
+tg_status tg_probe_fp32_peak(int32_t device, double* tflops) {
+    if (!tflops) return fail(TG_E_ARG, "tg_probe_fp32_peak: NULL out pointer");
+    TG_GUARD_BEGIN
+    cudaError_t e = probe_fp32_peak(device, tflops);
+    if (e != cudaSuccess) return fail(TG_E_CUDA, std::string("tg_probe_fp32_peak: ") + cudaGetErrorString(e));
+    return TG_OK;
+    TG_GUARD_END
+}
 
 tg_status tg_graph_create(tg_graph** g) {
     if (!g) return fail(TG_E_ARG, "tg_graph_create: NULL out pointer");
@@ -527,7 +539,7 @@ tg_status tg_plan_set_profiling(tg_plan* p, int32_t on) {
         exec_set_profiling_per_op(p, on != 0);
         return TG_OK;
     }
-    return exec_set_profiling(p, on != 0);
+    return exec_set_profiling(p, on);
     TG_GUARD_END
 }
 

@@ -15,6 +15,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <climits>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -59,6 +60,7 @@ struct tg_exec {
     std::vector<void*> registered;
     uint64_t registered_bytes = 0;
     bool profiling = false;
+    bool prof_copies = false;  // also time every copy (perturbs the copy engines)
     tg_timing timing{};
     std::vector<tg_trace_rec> trace;  // timeline collected from the profiling events
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
@@ -134,16 +136,33 @@ tg_status init_device(tg_plan* p, DevState& d) {
     return TG_OK;
 }
 
-// Register caller-owned pageable host buffers once, so async copies run at full speed.
+// Register caller-owned pageable host buffers once, so async copies run at full speed. Only the
+// span this process's shard touches is registered (tg_set_shard: a process may hold just its
+// part of a global input and output, the rest of the nominal [n][c][h][w] range unmapped).
 tg_status register_host(tg_plan* p, tg_exec* x) {
     const Graph& g = graph_of(p);
     const PlanCore& c = p->core;
-    if (c.device_io) return TG_OK;
+    if (c.device_io || c.c1 <= c.c0) return TG_OK;
+    const Template& t = c.t;
+    const Ds& X = g.ds[t.input];
+    const Ds& Y = g.ds[t.output];
+    // [lo, hi) in floats of the input rows and output rows of chunks [c0, c1)
+    const int64_t HW = t.H * t.W;
+    const int64_t out_img = t.kind == Tmpl::Edge ? HW : 9 * t.h[5] * t.w[5];
+    const int64_t out_plane = t.kind == Tmpl::Edge ? HW : t.h[5] * t.w[5];
+    const int64_t w_out = t.kind == Tmpl::Edge ? t.W : t.w[5];
+    const int64_t planes = t.kind == Tmpl::Edge ? 1 : 9;
+    int64_t xlo = INT64_MAX, xhi = 0, ylo = INT64_MAX, yhi = 0;
+    for (int64_t i = c.c0; i < c.c1; ++i) {
+        const Chunk& ch = c.chunks[i];
+        xlo = std::min(xlo, ch.img * HW + ch.in.a * t.W);
+        xhi = std::max(xhi, (ch.img + ch.nimg - 1) * HW + ch.in.b * t.W);
+        ylo = std::min(ylo, ch.img * out_img + ch.out.a * w_out);
+        yhi = std::max(yhi, (ch.img + ch.nimg - 1) * out_img + (planes - 1) * out_plane + ch.out.b * w_out);
+    }
     std::vector<std::pair<void*, size_t>> bufs;
-    const Ds& X = g.ds[c.t.input];
-    const Ds& Y = g.ds[c.t.output];
-    bufs.push_back({(void*)X.src, (size_t)X.numel() * 4});
-    bufs.push_back({(void*)Y.dst, (size_t)Y.numel() * 4});
+    bufs.push_back({(void*)(X.src + xlo), (size_t)(xhi - xlo) * 4});
+    bufs.push_back({(void*)(Y.dst + ylo), (size_t)(yhi - ylo) * 4});
     for (int id : c.param_ds) bufs.push_back({(void*)g.ds[id].src, (size_t)g.ds[id].numel() * 4});
     for (auto& b : bufs) {
         if (b.second < (1u << 20)) continue;  // small: pageable copies are fine
@@ -448,7 +467,7 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
     // resident in the arena for later ones (tg_plan_invalidate_params forces a re-upload)
     if (!d.params_resident) {
         ProfRec pr{10, nullptr, nullptr};
-        if (x->profiling) {
+        if (x->prof_copies) {
             pr.a = pool_event(d);
             pr.b = pool_event(d);
             cudaEventRecord(pr.a, S0);
@@ -466,7 +485,7 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
             CK(cudaMemcpyAsync(d.arena + c.k3tc_off, k3.data(), k3.size() * 2, cudaMemcpyHostToDevice, S0));
             CK(cudaMemcpyAsync(d.arena + c.k5tc_off, k5.data(), k5.size() * 2, cudaMemcpyHostToDevice, S0));
         }
-        if (x->profiling) {
+        if (x->prof_copies) {
             cudaEventRecord(pr.b, S0);
             d.prof.push_back(pr);
         }
@@ -481,14 +500,14 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
         if (!c.device_io) {
             if (d.seq >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
             ProfRec pr{10, nullptr, nullptr, d.c0 + k};
-            if (x->profiling) {
+            if (x->prof_copies) {
                 pr.a = pool_event(d);
                 pr.b = pool_event(d);
                 cudaEventRecord(pr.a, S0);
             }
             tg_status st = enqueue_h2d(p, d, ch, s);
             if (st != TG_OK) return st;
-            if (x->profiling) {
+            if (x->prof_copies) {
                 cudaEventRecord(pr.b, S0);
                 d.prof.push_back(pr);
             }
@@ -502,14 +521,14 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
         if (!c.device_io) {
             CK(cudaStreamWaitEvent(S2, d.ev_comp[s], 0));
             ProfRec pr{11, nullptr, nullptr, d.c0 + k};
-            if (x->profiling) {
+            if (x->prof_copies) {
                 pr.a = pool_event(d);
                 pr.b = pool_event(d);
                 cudaEventRecord(pr.a, S2);
             }
             st = enqueue_d2h(p, d, ch, s);
             if (st != TG_OK) return st;
-            if (x->profiling) {
+            if (x->prof_copies) {
                 cudaEventRecord(pr.b, S2);
                 d.prof.push_back(pr);
             }
@@ -617,9 +636,11 @@ tg_status exec_run(tg_plan* p, bool blocking, void* caller_stream, bool has_call
     return result;
 }
 
-tg_status exec_set_profiling(tg_plan* p, bool on) {
+tg_status exec_set_profiling(tg_plan* p, int level) {
     if (!p->exec) p->exec = new tg_exec();
+    const bool on = level != 0;
     p->exec->profiling = on;
+    p->exec->prof_copies = level == 1;
     if (on) {
         p->exec->timing = tg_timing{};
         p->exec->trace.clear();

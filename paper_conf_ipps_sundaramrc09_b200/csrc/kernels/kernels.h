@@ -25,6 +25,8 @@ struct EdgeArgs {
     int combine;            // 0 max over responses and remaps, 1 sum, 2 max |.|, 3 max
 };
 cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s);
+// measured FP32 FFMA peak (TFLOP/s, best of a few launches; probe.cu)
+cudaError_t probe_fp32_peak(int device, double* tflops);
 
 // CNN offload units (fp32 FFMA path). Row ranges are global level coordinates.
 struct CnnU1Args {          // C1(1->8, 5x5) + bias + tanh + S2 + tanh  -> T2

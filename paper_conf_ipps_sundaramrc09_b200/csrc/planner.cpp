@@ -393,12 +393,14 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     uint64_t pb = all_pb;
     SlotLayout slot;
     std::string bias_mode = base_bias;
-    // 1. batch mode
+    // 1. batch mode. Host I/O: at least 2 x depth chunks over each shard's share of the images
+    // (n_share = ceil(n / world)), so copies of some chunks overlap the kernels of others
+    const int64_t n_share = (n + g.world - 1) / g.world;
     int64_t bcap = 0;
     if (p.device_io)
         bcap = n;
     else if (H * W <= g.max_chunk_px)
-        bcap = std::min({n, g.max_chunk_px / (H * W), std::max<int64_t>(1, (n + 2 * depth - 1) / (2 * depth))});
+        bcap = std::min({n, g.max_chunk_px / (H * W), std::max<int64_t>(1, (n_share + 2 * depth - 1) / (2 * depth))});
     for (int64_t b = bcap; b >= 1; --b) {
         SlotLayout s = sz.slot(b, h_out, rows_of(t, 0, b, 0, h_out), false);
         if (fits(all_pb, s.bytes)) {
@@ -413,7 +415,13 @@ tg_status make_plan(const Graph& g, int32_t mode, PlanCore& p) {
     }
     // 2. row mode
     if (!have) {
-        const int64_t rcap = std::min<int64_t>(h_out, std::max<int64_t>(1, g.max_chunk_px / (W * in_per_out)));
+        // at most max_chunk_px input pixels per chunk, and (host I/O) at least 2 x depth chunks
+        // over each shard's images
+        int64_t rcap = std::min<int64_t>(h_out, std::max<int64_t>(1, g.max_chunk_px / (W * in_per_out)));
+        if (!p.device_io) {
+            const int64_t per_img = (2 * depth + n_share - 1) / n_share;  // chunks wanted per image
+            rcap = std::min<int64_t>(rcap, (h_out + per_img - 1) / per_img);
+        }
         struct Cand {
             uint64_t h2d;
             int64_t R;

@@ -126,6 +126,7 @@ _PROTOS = {
     "tg_execute": (c_i32, [vp]),
     "tg_execute_async": (c_i32, [vp]),
     "tg_execute_on": (c_i32, [vp, vp, c_i32]),
+    "tg_probe_fp32_peak": (c_i32, [c_i32, ctypes.POINTER(ctypes.c_double)]),
     "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
     "tg_plan_timing_get": (c_i32, [vp, ctypes.POINTER(tg_timing)]),
     "tg_plan_trace_get": (c_i32, [vp, ctypes.POINTER(tg_trace_rec), c_sz, ctypes.POINTER(c_sz)]),
@@ -335,8 +336,16 @@ def tg_execute_on(p, stream, blocking: bool = True) -> None:
     _ck(_lib.tg_execute_on(p, stream, 1 if blocking else 0))
 
 
-def tg_plan_set_profiling(p, on: bool) -> None:
-    _ck(_lib.tg_plan_set_profiling(p, 1 if on else 0))
+def tg_probe_fp32_peak(device: int = 0) -> float:
+    """Measured FP32 FFMA peak (TFLOP/s) of the device."""
+    v = ctypes.c_double(0.0)
+    _ck(_lib.tg_probe_fp32_peak(device, ctypes.byref(v)))
+    return v.value
+
+
+def tg_plan_set_profiling(p, on) -> None:
+    """on: 0 off, 1 (True) kernels and copies, 2 kernels only."""
+    _ck(_lib.tg_plan_set_profiling(p, int(on)))
 
 
 def tg_plan_timing_get(p) -> dict:
@@ -580,8 +589,9 @@ class Plan:
         else:
             (tg_execute if blocking else tg_execute_async)(self.h)
 
-    def profiling(self, on: bool = True) -> None:
-        tg_plan_set_profiling(self.h, on)
+    def profiling(self, on: bool = True, copies: bool = True) -> None:
+        """Per-launch CUDA-event timing; copies=False leaves the copy streams untouched."""
+        tg_plan_set_profiling(self.h, 0 if not on else (1 if copies else 2))
 
     def timing(self) -> dict:
         return tg_plan_timing_get(self.h)

@@ -9,7 +9,7 @@ import numpy as np
 import pytest
 
 import synth
-from gpu_util import need_gpu, normwise, pinned, torch
+from gpu_util import guard_runtime, need_gpu, normwise, pinned, torch
 
 pytestmark = pytest.mark.gpu
 
@@ -150,7 +150,7 @@ def test_cnn_delta_geometry(tg):
     assert np.abs(out[0] - exp).max() < 1e-6
 
 
-@pytest.mark.parametrize("prec", ["fp32", "fp32_tc"])
+@pytest.mark.parametrize("prec", ["fp32", "fp32_tc", "bf16_tc"])
 def test_large_cnn_paper_size_sampled_rows(tg, orc, prec):
     """Paper-literal configs[3]: large CNN on one 6400x4800 image (17.66e9-float Fig. 7
     footprint) under the 1.5 GB budget: bias rows stream; sampled output rows
@@ -161,7 +161,7 @@ def test_large_cnn_paper_size_sampled_rows(tg, orc, prec):
     prm = synth.cnn_params_np(seed, n5, H, W)
     h5, w5 = synth.cnn_dims(H, W)[4]
     out, p = run_cnn(tg, img, n5, prm, budget=1536 << 20,
-                     precision=tg.TG_FP32_TC if prec == "fp32_tc" else tg.TG_FP32)
+                     precision={"fp32": tg.TG_FP32, "fp32_tc": tg.TG_FP32_TC, "bf16_tc": tg.TG_BF16_TC}[prec])
     j = p.json()
     assert j["bias"] == "streamed" and j["arena_bytes"] <= 1536 << 20
     rows = {0, h5 - 1}
@@ -177,7 +177,7 @@ def test_large_cnn_paper_size_sampled_rows(tg, orc, prec):
         ref = orc.cnn(band, n5, bp)[0, :, 0]
         got = out[0, :, r]
         err = np.abs(got.astype(np.float64) - ref).max() / np.abs(ref).max()
-        assert err <= 1e-5, (r, err)
+        assert err <= (2e-2 if prec == "bf16_tc" else 1e-5), (r, err)
 
 
 # ------------------------------------------------------------------ tcgen05 bf16 path
@@ -387,3 +387,49 @@ def test_cnn_two_host_threads_tensor_core_operands(tg, orc, prec):
         p.execute()
         p.execute()
         assert np.array_equal(out, ref), rep
+
+
+@pytest.mark.parametrize("prec", ["fp32", "bf16_tc", "fp32_tc"])
+@pytest.mark.parametrize("mode", ["batch", "rows_streamed", "rows_resident", "scalar", "device"])
+def test_cnn_slot_layout_covers_every_buffer(tg, orc, prec, mode):
+    """The slot layout (the library's design; tests/test_plan_parity.py checks its sizes only by
+    properties) holds every buffer the kernels touch: with the arena between guard bands and
+    pre-filled with NaN bytes, every precision and chunking leaves the guards intact and matches
+    the oracle (an unfilled or overlapping buffer would show up as NaN or a wrong value)."""
+    P = {"fp32": tg.TG_FP32, "bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}[prec]
+    seed = 61
+    n, H, W, n5 = (7 if mode == "batch" else 3), 150, 172, 40
+    bias = "scalar" if mode == "scalar" else "plane"
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W, bias)
+    h5, w5 = synth.cnn_dims(H, W)[4]
+    budget = {"batch": 0, "rows_streamed": 1_200_000, "rows_resident": 2_200_000, "scalar": 600_000,
+              "device": 0}[mode]
+    bm = tg.TG_BIAS_PLANE if bias == "plane" else tg.TG_BIAS_SCALAR
+    if mode == "device":
+        x = torch.from_numpy(img).cuda()
+        out_t = torch.zeros((n, 9, h5, w5), dtype=torch.float32, device="cuda")
+        g, _ = tg.cnn_graph(x, n5, prm, out=out_t, bias_mode=bm, device=True)
+    else:
+        out = np.zeros((n, 9, h5, w5), np.float32)
+        g, _ = tg.cnn_graph(img, n5, prm, out=out, bias_mode=bm)
+    rt = guard_runtime(tg)
+    g.runtime = rt
+    tg.tg_set_runtime(g.h, rt.struct)
+    g.set(budget=budget, precision=P, max_chunk_px=(H * W * 2 if mode == "batch" else None))
+    p = g.plan()
+    j = p.json()
+    want_bias = {"batch": "resident", "rows_streamed": "streamed", "rows_resident": "resident",
+                 "scalar": "scalar", "device": "resident"}[mode]
+    assert j["bias"] == want_bias, j["bias"]
+    if mode.startswith("rows"):
+        assert j["split"] == "rows" and j["n_chunks"] > n
+    if mode == "batch":
+        assert j["split"] == "batch" and j["B"] > 1 and j["n_chunks"] > 1
+    p.execute()
+    p.execute()
+    got = out_t.cpu().numpy() if mode == "device" else out
+    assert rt.guards_intact()
+    ref = orc.cnn(img, n5, prm, bias_plane=(bias == "plane"))
+    assert np.isfinite(got).all()
+    assert normwise(got, ref) <= (2e-2 if prec == "bf16_tc" else 1e-5)

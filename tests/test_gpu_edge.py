@@ -10,7 +10,7 @@ import pytest
 
 import synth
 from conftest import GOLDEN
-from gpu_util import need_gpu, normwise, pinned, torch
+from gpu_util import guard_runtime, need_gpu, normwise, pinned, torch
 
 pytestmark = pytest.mark.gpu
 
@@ -302,3 +302,23 @@ def test_trace_respects_stream_dependencies(tg):
     for kind in ("h2d", "d2h", "edge"):
         iv = sorted((r["t0_ms"], r["t1_ms"]) for r in tr if r["kind"] == kind)
         assert all(a[1] <= b[0] + eps for a, b in zip(iv, iv[1:])), kind
+
+
+@pytest.mark.parametrize("budget,nf", [(0, 2), (300_000, 2), (120_000, 4), (90_000, 1)])
+def test_edge_slot_layout_covers_every_buffer(tg, orc, budget, nf):
+    """Slot-layout property on the GPU (see the CNN test of the same name): guard bands around a
+    NaN-filled arena stay intact and the output matches the oracle."""
+    img = synth.images_np(71, 2, 170, 236)
+    rs = np.random.default_rng(nf)
+    K = [(rs.standard_normal((16, 16)) / 16).astype(np.float32) for _ in range(nf)]
+    out = np.zeros_like(img)
+    g, _ = tg.edge_graph_general(img, K, "max", out=out)
+    rt = guard_runtime(tg)
+    g.runtime = rt
+    tg.tg_set_runtime(g.h, rt.struct)
+    g.set(budget=budget)
+    p = g.plan()
+    p.execute()
+    assert rt.guards_intact()
+    ref = np.stack([orc.edge_general(img[b, 0], K, "max") for b in range(2)])[:, None]
+    assert np.isfinite(out).all() and normwise(out, ref) <= 1e-5

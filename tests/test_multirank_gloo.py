@@ -65,7 +65,22 @@ def _worker(rank, world, port, q):
         # ---- timing reduction used by bench.py
         res["max"] = bench.max_over_ranks(float(rank + 1), world)
         res["min"] = bench.min_over_ranks(float(rank + 1), world)  # the host-link denominator
-        res["sum"] = bench.sum_over_ranks(1.0, world)
+        res["gather"] = bench.gather_objects({rank: rank * 10}, world)
+        # a rank may hold ONLY its share of the global input/output: the plan's shard touches a
+        # contiguous image span, and a base pointer offset into a smaller buffer plans the same
+        span = sorted({b for ch in plan["chunks"][c0:c1] for b in range(ch["img"], ch["img"] + ch["nimg"])})
+        part_in = np.ascontiguousarray(img[span[0]:span[-1] + 1])
+        gs = tg.Graph()
+        xs = tg.tg_input(gs.h, n, 1, H, W, part_in.ctypes.data - span[0] * H * W * 4)
+        k1 = gs.param(K1.reshape(1, 1, 16, 16))
+        k2 = gs.param(K2.reshape(1, 1, 16, 16))
+        e1 = gs.conv2d(xs, k1, -1, tg.TG_SAME)
+        e2 = gs.conv2d(xs, k2, -1, tg.TG_SAME)
+        e = gs.max_combine([e1, e2, gs.neg(e1), gs.neg(e2)])
+        part_out = np.zeros((span[-1] + 1 - span[0], 1, H, W), np.float32)
+        tg.tg_output(gs.h, e, part_out.ctypes.data - span[0] * H * W * 4)
+        gs.set(budget=60_000, shard=(rank, world))
+        res["span_plan_same"] = gs.plan().json()["chunks"] == plan["chunks"]
         q.put((rank, res))
         dist.destroy_process_group()
     except Exception as e:  # noqa: BLE001
@@ -91,4 +106,5 @@ def test_two_rank_sharding_gloo():
     assert ranges[0][0] == 0 and ranges[0][1] == ranges[1][0] and ranges[1][1] == C and C >= 4
     for r in range(world):
         assert results[r]["edge_exact"] and results[r]["edge_disjoint"] and results[r]["same_chunks"]
-        assert results[r]["max"] == 2.0 and results[r]["sum"] == 2.0 and results[r]["min"] == 1.0
+        assert results[r]["max"] == 2.0 and results[r]["min"] == 1.0
+        assert results[r]["gather"] == [{0: 0}, {1: 10}] and results[r]["span_plan_same"]

@@ -178,11 +178,15 @@ def test_plan_layout_properties(case):
     mcp = got["max_chunk_px"]
     h_out = H if tmpl == "edge" else synth.cnn_dims(H, W)[4][0]
     if got["split"] == "batch":
-        cap = n if got["device_io"] else min(n, mcp // (H * W), -(-n // (2 * depth)))
+        n_share = -(-n // kw.get("world", 1))
+        cap = n if got["device_io"] else min(n, mcp // (H * W), -(-n_share // (2 * depth)))
         assert got["chunk_cap"] == cap and 1 <= got["B"] <= cap
         at_cap = got["B"] == cap
     else:
         cap = min(h_out, max(1, mcp // (W * (1 if tmpl == "edge" else 4))))
+        if not got["device_io"]:       # >= 2 x depth chunks in all
+            per_img = -(-2 * depth // -(-n // kw.get("world", 1)))
+            cap = min(cap, -(-h_out // per_img))
         assert got["chunk_cap"] == cap and 1 <= got["R"] <= cap
         at_cap = got["R"] == cap
     if not at_cap:

@@ -1,0 +1,132 @@
+"""Kernel experiments without experiment hooks in the product sources: copy the package to
+_exp/<variant>/ (git-ignored), apply textual patches to one kernel source, build that copy, and time the
+CNN units of a workload through it (device-resident, per-unit CUDA events). Prints one JSON line
+per variant: {"variant", "unit_ms": {1: U1, 2: U2, 3: U3}, "value_mpx_s"}.
+
+  python tools/exp_kernel_variants.py --workload cnn3 --precision bf16_tc --variants base,no_epi,no_c5
+"""
+import argparse
+import json
+import os
+import shutil
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+PKG = "paper_conf_ipps_sundaramrc09_b200"
+
+# variant -> (kernel source, [(old, new), ...]); every `old` must occur in the source
+VARIANTS = {
+    "base": ("cnn_tc.cu", []),
+    # U3 bf16: the epilogue only does the barrier hand-offs (no TMEM loads, bias, tanh, stores)
+    "u3_no_epi": ("cnn_tc.cu", [
+        ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
+         "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
+        ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob")]),
+    # U3 bf16: no bias loads (bias 0), the rest of the epilogue as built
+    "u3_no_bias": ("cnn_tc.cu", [
+        ("            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = __ldg(p);",
+         "            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = 0.f;")]),
+    # U3 bf16: the MMA warp issues no C5 MMAs (commits still arrive)
+    "u3_no_c5": ("cnn_tc.cu", [
+        ("                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad, bd, idesc, ks > 0 ? 1u : 0u);",
+         "                            if (ks < 0) tc::mma_bf16(d_base + (uint32_t)(t * 128), ad, bd, idesc, ks > 0 ? 1u : 0u);")]),
+    # U3 bf16: no C6 MMAs
+    "u3_no_c6": ("cnn_tc.cu", [
+        ("                        tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL)",
+         "                        if (kk < 0) tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL)")]),
+    # U3 bf16: no slice copies (the MMAs read whatever the ring holds)
+    "u3_no_copy": ("cnn_tc.cu", [
+        ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
+         "            if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n            __syncwarp();\n            if (false)")]),
+}
+
+
+def build_variant(name, prebuilt=False):
+    src_file, patches = VARIANTS[name]
+    dst = os.path.join(ROOT, "_exp", name)   # git-ignored; travels to the GPU box with the snapshot
+    if prebuilt:
+        return dst
+    if os.path.exists(dst):
+        shutil.rmtree(dst)
+    os.makedirs(dst)
+    shutil.copytree(os.path.join(ROOT, PKG), os.path.join(dst, PKG),
+                    ignore=shutil.ignore_patterns("_build*", "libtg.so*", "__pycache__"))
+    shutil.copytree(os.path.join(ROOT, "include"), os.path.join(dst, "include"))
+    shutil.copytree(os.path.join(ROOT, "synth"), os.path.join(dst, "synth"))
+    path = os.path.join(dst, PKG, "csrc", "kernels", src_file)
+    s = open(path).read()
+    for old, new in patches:
+        assert old in s, (name, old[:80])
+        s = s.replace(old, new)
+    open(path, "w").write(s)
+    r = subprocess.run([sys.executable, os.path.join(dst, PKG, "build.py")], capture_output=True, text=True)
+    if r.returncode:
+        raise RuntimeError(r.stderr[-3000:])
+    shutil.rmtree(os.path.join(dst, PKG, "_build"), ignore_errors=True)   # keep the snapshot small
+    return dst
+
+
+TIMER = r'''
+import json, sys
+sys.path.insert(0, sys.argv[1])
+import torch, synth
+from paper_conf_ipps_sundaramrc09_b200 import tg
+wl, prec, steps = sys.argv[2], sys.argv[3], int(sys.argv[4])
+n, H, W = 64, 480, 640
+n5 = 20 if wl == "cnn3s" else 120
+if wl == "cnn4":
+    n, H, W = 1, 4800, 6400
+seed = synth.seed_for_config(3)
+torch.cuda.set_device(0)
+x = synth.images_torch(seed, n, H, W, "cuda:0")
+h5, w5 = synth.cnn_dims(H, W)[4]
+y = torch.empty((n, 9, h5, w5), dtype=torch.float32, device="cuda:0")
+prm = synth.cnn_params_np(seed, n5, H, W)
+g, _ = tg.cnn_graph(x, n5, prm, out=y, device=True)
+g.set(torch_runtime=True, precision={"fp32": 0, "bf16_tc": 1, "fp32_tc": 2}[prec])
+p = g.plan()
+for _ in range(3):
+    p.execute()
+p.profiling(True, copies=False)
+cs = p.compute_stream(0)
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record(cs)
+for _ in range(steps):
+    p.execute(blocking=False)
+e1.record(cs)
+torch.cuda.synchronize()
+t = p.timing()
+ms = e0.elapsed_time(e1) / steps
+print(json.dumps({"unit_ms": {u: t["kernel_ms"][u] / steps for u in (1, 2, 3)}, "step_ms": ms,
+                  "value_mpx_s": n * H * W / ms / 1e3, "checksum": float(y.double().abs().sum())}))
+'''
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="cnn3")
+    ap.add_argument("--precision", default="bf16_tc")
+    ap.add_argument("--variants", default="base")
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--build-only", action="store_true", help="build the variants here (no GPU needed)")
+    ap.add_argument("--prebuilt", action="store_true", help="run variants built earlier with --build-only")
+    args = ap.parse_args()
+    if args.build_only:
+        for v in args.variants.split(","):
+            build_variant(v)
+            print("built", v, flush=True)
+        return
+    for v in args.variants.split(","):
+        try:
+            d = build_variant(v, args.prebuilt)
+            r = subprocess.run([sys.executable, "-c", TIMER, d, args.workload, args.precision, str(args.steps)],
+                               capture_output=True, text=True, timeout=600)
+            out = json.loads(r.stdout.strip().splitlines()[-1]) if r.returncode == 0 else {"error": r.stderr[-800:]}
+        except Exception as e:  # noqa: BLE001
+            out = {"error": str(e)[-800:]}
+        print(json.dumps({"variant": v, "workload": args.workload, "precision": args.precision, **out}), flush=True)
+
+
+if __name__ == "__main__":
+    main()
