@@ -45,25 +45,31 @@ __device__ __forceinline__ float tanh_approx(float x) {
 constexpr int kTileM = 128;
 
 // ============================================================================ U2 (C3)
-// Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns [c0, c0+128): tile 0 = C3 row 2R,
-// tile 1 = row 2R+1 (M = 128 each, N = 32: 20 maps padded). Window: T2 rows [2R, 2R+6) x
-// cols [c0, c0+134), 8 channels per pixel (one 16-byte row each).
+// Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns [c0, c0+128): ONE M = 128 tile whose N
+// holds BOTH C3 rows: columns [0, 20) = row 2R, [24, 44) = row 2R+1 (N = 48). Window: T2 rows
+// [2R, 2R+6) x cols [c0, c0+134), 8 channels per pixel (one 16-byte row each).
+// Window row y feeds C3 row 2R with filter row y and row 2R+1 with filter row y - 1, so ONE
+// MMA per (window row, tap pair) serves both output rows: its B operand (one of 6 row variants)
+// holds filter row y in columns [0, 20) and filter row y - 1 in [24, 44) (zero where the filter
+// row does not exist). 6 rows x 3 tap pairs = 18 MMAs of N = 48 per segment instead of
+// 2 tiles x 15 of N = 32: the A operand -- the shared-memory read that bounds these small-N
+// MMAs -- is read 18 times instead of 30.
 // Warp-specialised and persistent (one CTA per SM, 10 warps; single-lane issue under elect.sync):
-//   warp 9               copy producer: the C3 B operand (15 K-steps) once per CTA by a bulk
+//   warp 9               copy producer: the C3 B operand (6 x 3 K-steps) once per CTA by a bulk
 //                        copy; per segment six 1-D bulk copies (TMA engine) of the window's T2
 //                        rows into one of U2_NA buffers, as soon as the buffer is free
-//   warp 8               MMA issuer: 2 tiles x 15 tcgen05.mma into one of 4 TMEM slots;
-//                        tcgen05.commit frees the window buffer and hands the slot to the
-//                        epilogue (copy issue -- ~150 cycles per bulk copy -- no longer
-//                        serialises with MMA issue)
+//   warp 8               MMA issuer: 18 tcgen05.mma into one of 4 TMEM slots; tcgen05.commit
+//                        frees the window buffer and hands the slot to the epilogue (copy issue
+//                        -- ~150 cycles per bulk copy -- does not serialise with MMA issue)
 //   warps 0-3 / 4-7      epilogue groups for even / odd segments: bias plane (prefetched one
 //                        segment ahead), tanh, the 2x2 subsample (rows in the same thread,
 //                        columns across neighbouring lanes), tanh -> T4 bf16 channel blocks
 constexpr int U2_WR = 6, U2_WP = kTileM + 6;  // +4 taps, +1 for the (4,5) tap pair, +1 spare
-constexpr int U2_N = 32;                      // 20 maps padded to 32
-constexpr int U2_KS = 15;                     // 5 rows x pairs (0,1) (2,3) (4,5)
+constexpr int U2_N = 48;                      // [0,20) row 2R, [24,44) row 2R+1, rest zero
+constexpr int U2_ROW1 = 24;                   // first column of C3 row 2R+1
+constexpr int U2_KS = 18;                     // 6 window rows x tap pairs (0,1) (2,3) (4,5)
 constexpr int U2_NA = 8;                      // window buffers
-constexpr int U2_NT = 4;                      // TMEM slots (2 per epilogue group)
+constexpr int U2_NT = 4;                      // TMEM slots (2 per epilogue group), 64 columns apart
 constexpr int kThreadsU2 = 10 * 32;
 
 struct U2P {
@@ -160,16 +166,13 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
             tc::fence_after_sync();
             const uint64_t abuf = adesc0 + (uint64_t)(buf * (U2_WR * U2_WP));
-            const uint32_t d0 = tmem + (uint32_t)(ts * 2 * U2_N);
+            const uint32_t d0 = tmem + (uint32_t)(ts * 64);
             if (tc::elect_one()) {
 #pragma unroll
-                for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
-#pragma unroll
-                    for (int ks = 0; ks < U2_KS; ++ks) {
-                        const int i = ks / 3, j = 2 * (ks % 3);
-                        tc::mma_bf16(d0 + (uint32_t)(t * U2_N), abuf + (uint64_t)((t + i) * U2_WP + j),
-                                     bdesc0 + (uint64_t)(ks * 2 * U2_N), idesc, ks > 0 ? 1u : 0u);
-                    }
+                for (int ks = 0; ks < U2_KS; ++ks) {  // window row y = ks / 3, tap pair (j, j+1)
+                    const int y = ks / 3, j = 2 * (ks % 3);
+                    tc::mma_bf16(d0, abuf + (uint64_t)(y * U2_WP + j), bdesc0 + (uint64_t)(ks * 2 * U2_N), idesc,
+                                 ks > 0 ? 1u : 0u);
                 }
             }
             __syncwarp();
@@ -210,10 +213,13 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             const int64_t C = c >> 1;               // T4 column
             tc::mbar_wait(&S.t_full[ts], (uint32_t)((k / U2_NT) & 1));
             tc::fence_after_sync();
-            float v0[32], v1[32];
-            tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 2 * U2_N), v0);
-            tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 2 * U2_N + U2_N), v1);
+            float va[32], vb[16], v1[20];
+            tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(ts * 64), va);       // columns [0, 32)
+            tc::tmem_ld16_async(tmem + lane_base + (uint32_t)(ts * 64 + 32), vb);  // columns [32, 48)
             tc::tmem_wait_ld();
+            const float* v0 = va;  // C3 row 2R: columns [0, 20)
+#pragma unroll
+            for (int co = 0; co < 20; ++co) v1[co] = co < 8 ? va[U2_ROW1 + co] : vb[U2_ROW1 + co - 32];
             tc::fence_before_sync();
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&S.t_empty[ts]);
@@ -582,17 +588,21 @@ bool set_smem_attr(const void* fn, size_t bytes, std::atomic<uint32_t>& flags) {
 
 }  // namespace
 
-// B operand of C3 for the 15 K-steps: [ks][half][n<32][8 ci]; half h of K-step (i, j-pair)
-// holds tap (i, j + h) (zero for j + h == 5), output maps >= 20 are zero.
+// B operand of C3 for the 18 K-steps (window row y, tap pair (j, j+1)): [ks][half][n<48][8 ci];
+// half h holds tap j + h (zero for j + h == 5); columns n < 20 = map n with filter row y (C3 row
+// 2R), 24 <= n < 44 = map n - 24 with filter row y - 1 (C3 row 2R+1), zero where the filter row
+// is outside 0..4 and in the padding columns.
 size_t cnn_k3_tc_bytes() { return (size_t)U2_KS * 2 * U2_N * 8 * 2; }
 void cnn_prepare_k3_tc(const float* k3, uint16_t* dst) {
     for (int ks = 0; ks < U2_KS; ++ks) {
-        const int i = ks / 3, j0 = 2 * (ks % 3);
+        const int y = ks / 3, j0 = 2 * (ks % 3);
         for (int h = 0; h < 2; ++h)
             for (int n = 0; n < U2_N; ++n)
                 for (int e = 0; e < 8; ++e) {
                     const int j = j0 + h;
-                    const float v = (n < 20 && j < 5) ? k3[(n * 8 + e) * 25 + i * 5 + j] : 0.f;
+                    const int t = n >= U2_ROW1 ? 1 : 0, map = n - t * U2_ROW1, i = y - t;
+                    const bool ok = map < 20 && j < 5 && i >= 0 && i < 5;
+                    const float v = ok ? k3[(map * 8 + e) * 25 + i * 5 + j] : 0.f;
                     dst[((ks * 2 + h) * U2_N + n) * 8 + e] = to_bf16(v);
                 }
     }

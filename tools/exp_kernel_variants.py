@@ -23,6 +23,13 @@ VARIANTS = {
         ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
          "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
         ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob")]),
+    # U3 bf16: epilogue hand-offs only AND the C5 MMAs at N = 64 instead of NP (half the B reads
+    # and half the math): tells a smem-operand-bound MMA phase from a compute-bound one
+    "u3_no_epi_n64": ("cnn_tc.cu", [
+        ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
+         "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
+        ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob"),
+        ("        const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);", "        const uint32_t idesc = tc::make_idesc_bf16(kTileM, 64);")]),
     # U3 bf16: no bias loads (bias 0), the rest of the epilogue as built
     "u3_no_bias": ("cnn_tc.cu", [
         ("            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = __ldg(p);",
@@ -43,6 +50,8 @@ VARIANTS = {
 
 
 def build_variant(name, prebuilt=False):
+    if name == "tree":             # the working tree as built in place
+        return ROOT
     src_file, patches = VARIANTS[name]
     dst = os.path.join(ROOT, "_exp", name)   # git-ignored; travels to the GPU box with the snapshot
     if prebuilt:
