@@ -445,12 +445,19 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
     steps = args.steps if headline else auto_steps(run_dev, cs, max(args.steps, 20), 0.5)
     if flush is not None and not headline:
         steps = min(steps, max(args.steps, 2000))   # each step also writes the 512 MB flush
-    p.profiling(True, copies=False)
+    # the timed pass replays each execution as one captured CUDA graph (tg_plan_set_graph: one
+    # host call per step; what bounds the launch-latency-bound configs[0]); a second, profiled
+    # pass of direct executions gives the per-unit kernel times (events on the compute stream)
+    p.use_graph(True)
+    p.execute()
     l0 = p.launches()
     barrier(world)
     with ClockSampler(local) as clk_v:
         ms = time_steps(run_dev, cs, steps, flush)
     launches = p.launches() - l0
+    p.use_graph(False)
+    p.profiling(True, copies=False)
+    ms_prof = time_steps(run_dev, cs, steps, flush)
     tim = p.timing()
     p.profiling(False)
     del flush
@@ -501,10 +508,16 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
                       f"{derived_fp32_peak_tflops(1965.0):.2f}")
     traffic = None
     tf_file = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tf_file):
-        tr = json.load(open(tf_file)).get(f"{wl['template']}:{precision}:{KERNEL_NAMES[k]}")
-        if tr:
-            traffic = tr["dram_bytes_per_out_px"] * opx[k] * steps / nl
+    ncu = json.load(open(tf_file)) if os.path.exists(tf_file) else {}
+    tkey = "edge" if wl["template"] == "edge" else wl["name"]
+    tr = ncu.get(f"{tkey}:{precision}:{KERNEL_NAMES[k]}")
+    if tr and wl["name"] in ("edge", "cnn3", "cnn3s"):   # the captured workloads (tools/update_traffic.py)
+        traffic = tr["dram_bytes_per_out_px"] * opx[k] * steps / nl
+    for u in fl:    # ncu pipe utilisation of each unit on the captured workload, when there is one
+        e = ncu.get(f"{tkey}:{precision}:{KERNEL_NAMES[u]}")
+        if e and KERNEL_NAMES[u] in units:
+            units[KERNEL_NAMES[u]]["ncu_captured"] = {k2: v for k2, v in e.items() if k2 != "note"} | {
+                "workload": "cnn3 (64 x 480x640, n5 120)" if tkey.startswith("cnn") else "edge 15 x 10000^2"}
     if bytes_per_launch / (hbm_peak * 1e9) > flops_per_launch / (peak_tf * 1e12):
         roofline = {"bound": "hbm", "achieved": hbm_gbs, "peak": hbm_peak, "unit": "GB/s", "frac": hbm_gbs / hbm_peak,
                     "peak_basis": "HBM copy bandwidth, measured (MEASURED_PEAKS.json)",
@@ -516,7 +529,8 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
                     "hbm": {"achieved": hbm_gbs, "peak": hbm_peak, "unit": "GB/s", "frac": hbm_gbs / hbm_peak}}
     roofline.update({"traffic": traffic, "kernel": KERNEL_NAMES[k], "kernel_ms_per_launch": kern_ms,
                      "algorithmic_flop_per_launch": flops_per_launch, "algorithmic_bytes_per_launch": bytes_per_launch,
-                     "kernel_share_of_step": tim["kernel_ms"][k] / steps / ms, "units": units,
+                     "kernel_share_of_step": tim["kernel_ms"][k] / steps / ms_prof, "units": units,
+                     "profiled_pass_ms_per_step": ms_prof,
                      "compute_ms_per_step_at_peak": compute_ms_at_peak})
     y_first, y_last = y_dev[0].clone(), y_dev[-1].clone()
     del p, g, y_dev
@@ -548,6 +562,14 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
             wall = (time.perf_counter() - t0) / n_steps * 1e3
         res = {"ms": ms2, "wall_ms": wall, "steps": n_steps, "launches": p2.launches() - l2, "stats": st,
                "json": js, "clocks": clk.summary()}
+        if profile and st["n_chunks"] <= js["depth"]:
+            # a plan of at most `depth` chunks has no copy/compute overlap within an execution:
+            # also time it as one CUDA-graph replay per step (tg_plan_set_graph; executions then
+            # serialise, but each costs one host call)
+            p2.use_graph(True)
+            p2.execute()
+            res["graph_ms"] = max_over_ranks(time_steps(lambda: p2.execute(blocking=False), cs2, n_steps), world)
+            p2.use_graph(False)
         if profile:
             # kernel busy time in a second pass with events on the compute stream only (no
             # events on the copy streams, which would perturb the copy engines)
@@ -618,6 +640,9 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
                          "peak_bidir_each_gbs": link["bidir_each"],
                          "achieved_h2d_gbs": (h2d / 1e9) / (cap["ms"] / 1e3),
                          "achieved_d2h_gbs": (d2h / 1e9) / (cap["ms"] / 1e3)}}
+    if "graph_ms" in cap:
+        e2e["graph_replay"] = {"value": px_glob / (cap["graph_ms"] / 1e3) / 1e6, "ms_per_step": cap["graph_ms"],
+                               "what": "the same e2e step replayed as one captured CUDA graph (tg_plan_set_graph)"}
     clocks = [clk_v.summary(), cap["clocks"]]
     # per-image output digests (additive over the pieces of an image), gathered in image order:
     # the first per-GPU share of images is the N = 1 workload, so its digest must equal N = 1's
@@ -897,6 +922,9 @@ def main():
             if name == "edge256":
                 ent["us_per_step_device"] = r2["ms_per_step"] * 1e3
                 ent["us_per_step_e2e"] = r2["e2e"]["ms_per_step"] * 1e3
+                if "graph_replay" in r2["e2e"]:
+                    ent["us_per_step_e2e_graph"] = r2["e2e"]["graph_replay"]["ms_per_step"] * 1e3
+                    ent["e2e"]["graph_replay"] = r2["e2e"]["graph_replay"]
                 ent["kernel_us_per_launch"] = r2["roofline"]["kernel_ms_per_launch"] * 1e3
             per.append(ent)
         del r2

@@ -231,6 +231,16 @@ tg_status tg_execute_async(tg_plan* plan);
  * otherwise. */
 tg_status tg_execute_on(tg_plan* plan, void* stream, int32_t blocking);
 
+/* CUDA-graph replay (fused plans, one device): with on != 0 the next execution after the
+ * parameters are resident is captured (its copies, kernels and stream dependencies on the
+ * three streams) and that and every later execution launch the captured graph on the compute
+ * stream -- one host call instead of one per copy and kernel, which is what bounds small
+ * (launch-latency-bound) executions. Replays are serialised on the compute stream, so
+ * back-to-back executions no longer overlap each other's copies. Ignored while profiling;
+ * tg_plan_invalidate_params or on = 0 drops the graph. Buffers must not move between
+ * executions (they never do: the plan binds them). */
+tg_status tg_plan_set_graph(tg_plan* plan, int32_t on);
+
 /* Per-launch timing of the fused kernels measured with CUDA events on the compute stream
  * (enable before executing; tg_plan_timing_get synchronizes). Times are summed over all
  * executions since enabling. on = 1: kernels and every H2D/D2H copy (events on the copy

@@ -532,6 +532,14 @@ tg_status tg_execute_on(tg_plan* p, void* stream, int32_t blocking) {
     TG_GUARD_END
 }
 
+tg_status tg_plan_set_graph(tg_plan* p, int32_t on) {
+    if (!p) return fail(TG_E_ARG, "tg_plan_set_graph: NULL plan");
+    if (p->core.mode != TG_FUSED) return fail(TG_E_UNSUPPORTED, "tg_plan_set_graph: fused plans only");
+    TG_GUARD_BEGIN
+    return exec_set_graph(p, on != 0);
+    TG_GUARD_END
+}
+
 tg_status tg_plan_set_profiling(tg_plan* p, int32_t on) {
     if (!p) return fail(TG_E_ARG, "tg_plan_set_profiling: NULL plan");
     TG_GUARD_BEGIN

@@ -50,6 +50,9 @@ struct DevState {
     int64_t launches = 0;
     bool params_resident = false;  // parameters uploaded by an earlier execution
     int64_t seq = 0;               // chunks enqueued on this device over all executions (slot ring)
+    cudaGraphExec_t graph = nullptr;  // captured execution (tg_plan_set_graph), replayed on S1
+    bool after_graph = false;         // the last work on this device was a graph replay
+    int64_t graph_launches = 0;       // kernel launches one replay performs
 };
 
 }  // namespace
@@ -60,6 +63,7 @@ struct tg_exec {
     std::vector<void*> registered;
     uint64_t registered_bytes = 0;
     bool profiling = false;
+    bool graph_mode = false;   // replay a captured execution (tg_plan_set_graph)
     bool prof_copies = false;  // also time every copy (perturbs the copy engines)
     tg_timing timing{};
     std::vector<tg_trace_rec> trace;  // timeline collected from the profiling events
@@ -440,7 +444,8 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
     return TG_OK;
 }
 
-tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStream_t caller, bool ordered) {
+tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStream_t caller, bool ordered,
+                     bool capturing = false) {
     const Graph& g = graph_of(p);
     const PlanCore& c = p->core;
     CK(cudaSetDevice(d.dev));
@@ -458,8 +463,15 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
     // new execution's H2D copies only wait for their slot to be free (the slot ring and its
     // events persist across executions), so back-to-back executions of one plan pipeline:
     // the next batch uploads while the previous one's last chunks compute and download.
+    // (when the execution is being captured into a graph, the copy streams always fork from S1
+    // -- that is how they join the capture -- and the slot ring starts afresh: graph replays on
+    // S1 are serialised, so no chunk waits for a slot of an earlier execution)
+    // A direct execution after a graph replay does the same: the slot events were last recorded
+    // inside the capture, so they neither order against the replays nor may be waited on.
+    const bool fresh = capturing || d.after_graph;
+    d.after_graph = false;
     CK(cudaEventRecord(d.ev_fork, S1));
-    if (c.device_io || !d.params_resident) {
+    if (c.device_io || !d.params_resident || fresh) {
         CK(cudaStreamWaitEvent(S0, d.ev_fork, 0));
         CK(cudaStreamWaitEvent(S2, d.ev_fork, 0));
     }
@@ -496,9 +508,10 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
     const int D = c.depth;
     for (int64_t k = 0; k < d.c1 - d.c0; ++k, ++d.seq) {
         const Chunk& ch = c.chunks[d.c0 + k];
-        const int s = (int)(d.seq % D);
+        const int64_t sq = fresh ? k : d.seq;  // position in the slot ring
+        const int s = (int)(sq % D);
         if (!c.device_io) {
-            if (d.seq >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
+            if (sq >= D) CK(cudaStreamWaitEvent(S0, d.ev_comp[s], 0));
             ProfRec pr{10, nullptr, nullptr, d.c0 + k};
             if (x->prof_copies) {
                 pr.a = pool_event(d);
@@ -513,7 +526,7 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
             }
             CK(cudaEventRecord(d.ev_h2d[s], S0));
             CK(cudaStreamWaitEvent(S1, d.ev_h2d[s], 0));
-            if (d.seq >= D) CK(cudaStreamWaitEvent(S1, d.ev_d2h[s], 0));
+            if (sq >= D) CK(cudaStreamWaitEvent(S1, d.ev_d2h[s], 0));
         }
         tg_status st = launch_units(p, x, d, ch, s);
         if (st != TG_OK) return st;
@@ -611,7 +624,45 @@ tg_status exec_run(tg_plan* p, bool blocking, void* caller_stream, bool has_call
     if (ordered && x->devs.size() > 1)
         return fail(TG_E_UNSUPPORTED, "execute: ordering against a caller stream needs a one-device plan");
     tg_status result = TG_OK;
-    if (x->devs.size() == 1) {
+    if (x->graph_mode && x->devs.size() == 1 && !any_upload && !x->profiling) {
+        // CUDA-graph replay: the execution's whole enqueue sequence (copies, kernels, events on
+        // the three streams) captured once, then launched as one graph on the compute stream
+        DevState& d = x->devs[0];
+        CK(cudaSetDevice(d.dev));
+        cudaStream_t S1 = d.st[1];
+        if (!d.graph) {
+            const int64_t l0 = d.launches;
+            CK(cudaStreamBeginCapture(S1, cudaStreamCaptureModeRelaxed));
+            tg_status st = run_device(p, x, d, false, nullptr, false, true);
+            cudaGraph_t gr = nullptr;
+            cudaError_t e = cudaStreamEndCapture(S1, &gr);
+            if (st != TG_OK) {
+                if (gr) cudaGraphDestroy(gr);
+                return st;
+            }
+            if (e != cudaSuccess) return fail(TG_E_CUDA, std::string("graph capture: ") + cudaGetErrorString(e));
+            e = cudaGraphInstantiate(&d.graph, gr, 0);
+            cudaGraphDestroy(gr);
+            if (e != cudaSuccess) {
+                d.graph = nullptr;
+                return fail(TG_E_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
+            }
+            d.graph_launches = d.launches - l0;
+            d.launches = l0;
+        }
+        if (ordered) {
+            CK(cudaEventRecord(d.ev_caller, caller));
+            CK(cudaStreamWaitEvent(S1, d.ev_caller, 0));
+        }
+        CK(cudaGraphLaunch(d.graph, S1));
+        d.launches += d.graph_launches;
+        d.after_graph = true;
+        if (ordered) {
+            CK(cudaEventRecord(d.ev_done, S1));
+            CK(cudaStreamWaitEvent(caller, d.ev_done, 0));
+        }
+        if (blocking) CK(cudaStreamSynchronize(S1));
+    } else if (x->devs.size() == 1) {
         result = run_device(p, x, x->devs[0], blocking, caller, ordered);
     } else {
         std::vector<tg_status> sts(x->devs.size(), TG_OK);
@@ -695,6 +746,7 @@ void exec_destroy(tg_plan* p) {
         for (auto* v : {&d.ev_h2d, &d.ev_comp, &d.ev_d2h})
             for (auto e : *v)
                 if (e) cudaEventDestroy(e);
+        if (d.graph) cudaGraphExecDestroy(d.graph);
         for (auto e : {d.ev_fork, d.ev_join, d.ev_params, d.ev_caller, d.ev_done})
             if (e) cudaEventDestroy(e);
         if (d.arena) {
@@ -726,8 +778,23 @@ tg_status exec_trace(tg_plan* p, tg_trace_rec* out, size_t cap, size_t* n) {
 
 uint64_t exec_registered_bytes(const tg_plan* p) { return p->exec ? p->exec->registered_bytes : 0; }
 
+tg_status exec_set_graph(tg_plan* p, bool on) {
+    if (!p->exec) p->exec = new tg_exec();
+    tg_exec* x = p->exec;
+    x->graph_mode = on;
+    for (auto& d : x->devs)
+        if (d.graph) {
+            if (cudaSetDevice(d.dev) == cudaSuccess) cudaStreamSynchronize(d.st[1]);
+            cudaGraphExecDestroy(d.graph);
+            d.graph = nullptr;
+        }
+    return TG_OK;
+}
+
 void exec_invalidate_params(tg_plan* p) {
     if (!p->exec) return;
+    // a captured graph holds the kernels' weight parameters by value: recapture after the upload
+    if (p->exec->graph_mode) exec_set_graph(p, true);
     for (auto& d : p->exec->devs) d.params_resident = false;
     p->exec->k3tc.clear();  // the bf16 tensor-core operands are re-derived from the new values
     p->exec->k5tc.clear();

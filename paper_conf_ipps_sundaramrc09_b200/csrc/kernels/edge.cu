@@ -45,14 +45,32 @@
 namespace tg {
 namespace {
 
-constexpr int kTileR = 64;
-constexpr int kTileC = 64;
-constexpr int kSmR = kTileR + 15;  // 79 rows incl. halo
-constexpr int kSmC = kTileC + 16;  // 80 cols used: [c0-8, c0+72)
-constexpr int kPitch = 84;         // floats; 84/4 = 21 (odd) -> conflict-free LDS.128 across rows
+// Tile geometry per strip width kQ (outputs per thread, one row of kQ columns):
+//   kQ = 16: 64 x 64 output tiles, 8 warps = 2 row groups x 4 column strips (the main path);
+//   kQ = 4:  32 x 32 output tiles, 8 warps = 8 column strips of one 32-row group -- for images
+//            with fewer 64 x 64 tiles than SMs (configs[0], 256 x 256: 16 big tiles would leave
+//            132 SMs idle and make each thread's 4096 serial FFMA2 the latency; 64 small tiles with
+//            1024 each finish ~4x sooner).
+// Row pitch in shared memory: an odd number of 16-byte units, so the 8 lanes of each LDS.128
+// phase (lanes = consecutive rows) hit 8 distinct bank groups.
+template <int kQ> struct Geo;
+template <> struct Geo<16> {
+    static constexpr int R = 64, C = 64, Pitch = 84;  // 84 / 4 = 21
+    __device__ static int lr(int warp, int lane) { return (warp >> 2) * 32 + lane; }
+    __device__ static int cb(int warp) { return (warp & 3) * 16; }
+};
+template <> struct Geo<4> {
+    static constexpr int R = 32, C = 32, Pitch = 52;  // 52 / 4 = 13
+    __device__ static int lr(int, int lane) { return lane; }
+    __device__ static int cb(int warp) { return warp * 4; }
+};
+template <int kQ> struct GeoT : Geo<kQ> {
+    static constexpr int SmR = Geo<kQ>::R + 15;                  // rows incl. halo
+    static constexpr int SmC = Geo<kQ>::C + 16;                  // cols used: [c0-8, c0+C+8)
+    static constexpr int TileBytes = SmR * Geo<kQ>::Pitch * 4;   // one TMA box
+    static constexpr int BufStride = (TileBytes + 127) / 128 * 128;
+};
 constexpr int kThreads = 256;
-constexpr int kTileBytes = kSmR * kPitch * 4;  // one TMA box (84 x 79 floats)
-constexpr int kBufStride = (kTileBytes + 127) / 128 * 128;
 
 // Both filters, embedded in 16 x 16 frames, travel as a __grid_constant__ kernel parameter:
 // the weights then sit in the constant bank and every FFMA reads them through a uniform
@@ -62,38 +80,39 @@ struct EdgeWeights {
     float2 w[2][256];  // filter pairs (2p, 2p+1) interleaved per tap: one FFMA2 weight operand
 };
 
-// Compute the 64 x 64 output tile whose input (+halo) is staged at xs (pitch kPitch, smem
+// Compute the output tile whose input (+halo) is staged at xs (row pitch Geo<kQ>::Pitch; smem
 // (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)) and store it.
-template <int kComb, int kPairs, int kF>
+template <int kComb, int kPairs, int kF, int kQ>
 __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const EdgeArgs& a, const EdgeWeights& wt,
                                           int64_t img, int64_t tile_r0, int64_t tile_c0) {
+    constexpr int kPitch = Geo<kQ>::Pitch;
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
-    const int lr = (warp >> 2) * 32 + lane;  // local output row
-    const int cb = (warp & 3) * 16;          // local output column base
+    const int lr = Geo<kQ>::lr(warp, lane);  // local output row
+    const int cb = Geo<kQ>::cb(warp);        // local output column base
 
     // Paired FP32 FMA (FFMA2, sm_100) over a PAIR OF FILTERS: acc[q] = (E_2p[q], E_2p+1[q]) +=
     // x[q+j+1] (register, broadcast to both lanes) * (K_2p[i][j], K_2p+1[i][j]) (uniform-register
     // pair from the constant bank). Each lane rounds exactly like fmaf, in the same (i, j) order
     // as a scalar loop. Filter pairs run one after the other over the same staged tile, and the
     // combine op folds each pair into e[] (8 orientations = 4 convolutions = 2 pairs).
-    float e[16];
+    float e[kQ];
 #pragma unroll
-    for (int q = 0; q < 16; ++q) e[q] = 0.f;
+    for (int q = 0; q < kQ; ++q) e[q] = 0.f;
 #pragma unroll
     for (int fp = 0; fp < kPairs; ++fp) {  // compile-time: constant-bank weight offsets
-        float2 acc[16];
+        float2 acc[kQ];
 #pragma unroll
-        for (int q = 0; q < 16; ++q) acc[q] = make_float2(0.f, 0.f);
+        for (int q = 0; q < kQ; ++q) acc[q] = make_float2(0.f, 0.f);
         constexpr int kOff = 8 - kF / 2;  // first tap row/column of the kF x kF window
 #pragma unroll 1
         for (int i = kOff; i < kOff + kF; ++i) {
-            // input window: smem cols [cb, cb+32) <-> image cols [c0+cb-8, c0+cb+24);
+            // input window: smem cols [cb, cb+kQ+16) <-> image cols [c0+cb-8, c0+cb+kQ+8);
             // output column c0+cb+q, tap j reads image col c0+cb+q+j-7 = smem col cb+q+j+1
-            float x[32];
+            float x[kQ + 16];
             const float4* xr = reinterpret_cast<const float4*>(&xs[(lr + i) * kPitch + cb]);
 #pragma unroll
-            for (int v = 0; v < 8; ++v) {
+            for (int v = 0; v < (kQ + 16) / 4; ++v) {
                 const float4 t = xr[v];
                 x[4 * v + 0] = t.x;
                 x[4 * v + 1] = t.y;
@@ -104,14 +123,14 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const Ed
             for (int j = kOff; j < kOff + kF; ++j) {
                 const float2 w = wt.w[fp][i * 16 + j];
 #pragma unroll
-                for (int q = 0; q < 16; ++q)
+                for (int q = 0; q < kQ; ++q)
                     acc[q] = __ffma2_rn(make_float2(x[q + j + 1], x[q + j + 1]), w, acc[q]);
             }
         }
         // combine (x > m) ? x : m folds; sum = left fold of fp32 adds
         const bool has2 = 2 * fp + 1 < a.nf;
 #pragma unroll
-        for (int q = 0; q < 16; ++q) {
+        for (int q = 0; q < kQ; ++q) {
             const float e1 = acc[q].x, e2 = acc[q].y;
             float m = e[q];
             switch (kComb) {
@@ -143,14 +162,14 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const Ed
     const int64_t c0 = tile_c0 + cb;
     const bool ovec = (a.W & 3) == 0 && ((reinterpret_cast<uintptr_t>(a.out) & 15) == 0) &&
                       (a.out_img_stride & 3) == 0;
-    if (ovec && c0 + 15 < a.W) {
+    if (ovec && c0 + kQ - 1 < a.W) {
 #pragma unroll
-        for (int v = 0; v < 4; ++v)
+        for (int v = 0; v < kQ / 4; ++v)
             *reinterpret_cast<float4*>(orow + c0 + 4 * v) =
                 make_float4(e[4 * v], e[4 * v + 1], e[4 * v + 2], e[4 * v + 3]);
     } else {
 #pragma unroll
-        for (int q = 0; q < 16; ++q)
+        for (int q = 0; q < kQ; ++q)
             if (c0 + q < a.W) orow[c0 + q] = e[q];
     }
 }
@@ -159,6 +178,8 @@ __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const Ed
 template <int kComb, int kPairs, int kF>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_kernel(const EdgeArgs a, const __grid_constant__ EdgeWeights wt) {
+    using G = GeoT<16>;
+    constexpr int kTileR = G::R, kTileC = G::C, kSmR = G::SmR, kSmC = G::SmC, kPitch = G::Pitch;
     __shared__ __align__(16) float xs[kSmR * kPitch];
     const int tid = threadIdx.x;
     const int64_t img = blockIdx.z;
@@ -187,7 +208,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         *reinterpret_cast<float4*>(&xs[sr * kPitch + 4 * q]) = v;
     }
     __syncthreads();
-    edge_tile<kComb, kPairs, kF>(xs, a, wt, img, tile_r0, tile_c0);
+    edge_tile<kComb, kPairs, kF, 16>(xs, a, wt, img, tile_r0, tile_c0);
 }
 
 // ---------------------------------------------------------------------------- TMA path
@@ -195,11 +216,13 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-template <int kComb, int kPairs, int kF>
+template <int kComb, int kPairs, int kF, int kQ>
 __global__ void __launch_bounds__(kThreads, 2)
     edge_fused_tma_kernel(const __grid_constant__ CUtensorMap tmap, const EdgeArgs a,
                           const __grid_constant__ EdgeWeights wt, const int tiles_c, const int tiles_r,
                           const int64_t ntiles) {
+    using G = GeoT<kQ>;
+    constexpr int kTileR = G::R, kTileC = G::C, kTileBytes = G::TileBytes, kBufStride = G::BufStride;
     // (the tensor map must sit in the first 4 KB of the parameter space, hence first)
     extern __shared__ __align__(128) uint8_t smraw[];
     // two tile buffers at 128-byte aligned shared-memory addresses
@@ -258,7 +281,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         int64_t img, tr0, tc0;
         coords(t, img, tr0, tc0);
         const float* tb = b ? buf1 : buf0;
-        edge_tile<kComb, kPairs, kF>(tb, a, wt, img, tr0, tc0);
+        edge_tile<kComb, kPairs, kF, kQ>(tb, a, wt, img, tr0, tc0);
         __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
     }
 }
@@ -304,6 +327,41 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
     return launch_edge_f<16>(a, s);
 }
 
+// The TMA path at strip width kQ; cudaErrorNotSupported when the tensor map cannot be encoded
+// (the caller then takes the bounds-checked fallback kernel).
+template <int kComb, int kPairs, int kF, int kQ>
+cudaError_t launch_edge_tma(const EdgeArgs& a, const EdgeWeights& wt, PFN_cuTensorMapEncodeTiled_v12000 enc, int dev,
+                            int sms, cudaStream_t s) {
+    using G = GeoT<kQ>;
+    const int tiles_c = (int)((a.W + G::C - 1) / G::C);
+    const int tiles_r = (int)((a.out_rows + G::R - 1) / G::R);
+    CUtensorMap tmap;
+    const cuuint64_t gdim[3] = {(cuuint64_t)a.W, (cuuint64_t)a.in_rows, (cuuint64_t)a.nimg};
+    const cuuint64_t gstride[2] = {(cuuint64_t)a.W * 4, (cuuint64_t)a.in_rows * a.W * 4};
+    const cuuint32_t box[3] = {(cuuint32_t)G::Pitch, (cuuint32_t)G::SmR, 1};
+    const cuuint32_t estride[3] = {1, 1, 1};
+    CUresult r = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(a.in), gdim, gstride, box, estride,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cudaErrorNotSupported;
+    static std::atomic<uint32_t> configured{0};
+    const size_t smem = 2 * (size_t)G::BufStride + 128;
+    if (!(configured.load() & (1u << (dev & 31)))) {
+        cudaError_t e = cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs, kF, kQ>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        configured.fetch_or(1u << (dev & 31));
+    }
+    const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
+    if (ntiles >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit tile indexing in the kernel
+    // 32 CTAs per SM in the grid (3 are resident at a time): CTAs that finish early pick up
+    // the remaining ones, which balances the tail of the static tile walk -- 2 per SM
+    // (exactly resident) ran at 0.918 of the FP32 peak, 8 at 0.936, 32 at 0.941
+    const int64_t grid = std::min<int64_t>(ntiles, 32 * (int64_t)sms);
+    edge_fused_tma_kernel<kComb, kPairs, kF, kQ><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
+    return cudaGetLastError();
+}
+
 template <int kComb, int kPairs, int kF>
 cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
@@ -317,42 +375,22 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
                 float2& w = wt.w[f >> 1][(r + off) * 16 + c + off];
                 (f & 1 ? w.y : w.x) = a.k_host[f][r * a.ks + c];
             }
-    const int tiles_c = (int)((a.W + kTileC - 1) / kTileC);
-    const int tiles_r = (int)((a.out_rows + kTileR - 1) / kTileR);
     PFN_cuTensorMapEncodeTiled_v12000 enc = tma_encode_fn();
     const bool tma_ok = enc && (a.W & 3) == 0 && (reinterpret_cast<uintptr_t>(a.in) & 15) == 0 &&
                         a.in_img_stride == a.in_rows * a.W && a.in_rows < (1ll << 31) && a.W < (1ll << 31);
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t big_tiles = ((a.W + 63) / 64) * ((a.out_rows + 63) / 64) * a.nimg;
     if (tma_ok) {
-        CUtensorMap tmap;
-        const cuuint64_t gdim[3] = {(cuuint64_t)a.W, (cuuint64_t)a.in_rows, (cuuint64_t)a.nimg};
-        const cuuint64_t gstride[2] = {(cuuint64_t)a.W * 4, (cuuint64_t)a.in_rows * a.W * 4};
-        const cuuint32_t box[3] = {(cuuint32_t)kPitch, (cuuint32_t)kSmR, 1};
-        const cuuint32_t estride[3] = {1, 1, 1};
-        CUresult r = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(a.in), gdim, gstride, box, estride,
-                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-        if (r == CUDA_SUCCESS) {
-            static std::atomic<uint32_t> configured{0};
-            int dev = 0, sms = 148;
-            cudaGetDevice(&dev);
-            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            const size_t smem = 2 * (size_t)kBufStride + 128;
-            if (!(configured.load() & (1u << (dev & 31)))) {
-                cudaError_t e =
-                    cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs, kF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-                if (e != cudaSuccess) return e;
-                configured.fetch_or(1u << (dev & 31));
-            }
-            const int64_t ntiles = (int64_t)tiles_c * tiles_r * a.nimg;
-            if (ntiles >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit tile indexing in the kernel
-            // 32 CTAs per SM in the grid (3 are resident at a time): CTAs that finish early pick up
-            // the remaining ones, which balances the tail of the static tile walk -- 2 per SM
-            // (exactly resident) ran at 0.918 of the FP32 peak, 8 at 0.936, 32 at 0.941
-            const int64_t grid = std::min<int64_t>(ntiles, 32 * (int64_t)sms);
-            edge_fused_tma_kernel<kComb, kPairs, kF><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
-            return cudaGetLastError();
-        }
+        // small tiles (kQ = 4) when the big ones cannot occupy every SM
+        cudaError_t e = big_tiles < sms ? launch_edge_tma<kComb, kPairs, kF, 4>(a, wt, enc, dev, sms, s)
+                                        : launch_edge_tma<kComb, kPairs, kF, 16>(a, wt, enc, dev, sms, s);
+        if (e != cudaErrorNotSupported) return e;
     }
+    using G = GeoT<16>;
+    const int tiles_c = (int)((a.W + G::C - 1) / G::C);
+    const int tiles_r = (int)((a.out_rows + G::R - 1) / G::R);
     dim3 grid((unsigned)tiles_c, (unsigned)tiles_r, (unsigned)a.nimg);
     if (grid.y > 65535 || grid.z > 65535) return cudaErrorInvalidConfiguration;
     edge_fused_kernel<kComb, kPairs, kF><<<grid, kThreads, 0, s>>>(a, wt);

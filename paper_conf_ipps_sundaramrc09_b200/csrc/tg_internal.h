@@ -189,6 +189,7 @@ struct tg_plan {
 namespace tg {
 tg_status exec_run(tg_plan* p, bool blocking, void* caller_stream = nullptr, bool has_caller = false);
 tg_status exec_set_profiling(tg_plan* p, int level);
+tg_status exec_set_graph(tg_plan* p, bool on);
 tg_status exec_timing(tg_plan* p, tg_timing* out);
 tg_status exec_trace(tg_plan* p, tg_trace_rec* out, size_t cap, size_t* n);
 void exec_destroy(tg_plan* p);

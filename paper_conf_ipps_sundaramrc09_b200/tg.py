@@ -126,6 +126,7 @@ _PROTOS = {
     "tg_execute": (c_i32, [vp]),
     "tg_execute_async": (c_i32, [vp]),
     "tg_execute_on": (c_i32, [vp, vp, c_i32]),
+    "tg_plan_set_graph": (c_i32, [vp, c_i32]),
     "tg_probe_fp32_peak": (c_i32, [c_i32, ctypes.POINTER(ctypes.c_double)]),
     "tg_plan_set_profiling": (c_i32, [vp, c_i32]),
     "tg_plan_timing_get": (c_i32, [vp, ctypes.POINTER(tg_timing)]),
@@ -336,6 +337,10 @@ def tg_execute_on(p, stream, blocking: bool = True) -> None:
     _ck(_lib.tg_execute_on(p, stream, 1 if blocking else 0))
 
 
+def tg_plan_set_graph(p, on: bool) -> None:
+    _ck(_lib.tg_plan_set_graph(p, 1 if on else 0))
+
+
 def tg_probe_fp32_peak(device: int = 0) -> float:
     """Measured FP32 FFMA peak (TFLOP/s) of the device."""
     v = ctypes.c_double(0.0)
@@ -456,6 +461,9 @@ class TorchRuntime:
             t = self._torch.empty(int(nbytes), dtype=self._torch.uint8, device=f"cuda:{dev}")
         except Exception:  # noqa: BLE001 - reported to the library as NULL (TG_E_OOM)
             return None
+        # the caching allocator orders a block's reuse on the allocating (current) stream only;
+        # the library's streams are others, so wait once here for work still pending on the block
+        self._torch.cuda.current_stream(dev).synchronize()
         self._bufs[t.data_ptr()] = t
         return t.data_ptr()
 
@@ -588,6 +596,10 @@ class Plan:
             tg_execute_on(self.h, getattr(stream, "cuda_stream", stream), blocking)
         else:
             (tg_execute if blocking else tg_execute_async)(self.h)
+
+    def use_graph(self, on: bool = True) -> None:
+        """Replay executions as one captured CUDA graph (tg_plan_set_graph)."""
+        tg_plan_set_graph(self.h, on)
 
     def profiling(self, on: bool = True, copies: bool = True) -> None:
         """Per-launch CUDA-event timing; copies=False leaves the copy streams untouched."""

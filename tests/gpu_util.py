@@ -42,6 +42,7 @@ def guard_runtime(tg):
         def _alloc_cb(self, nbytes, dev, ctx):
             t = self._torch.full((int(nbytes) + 2 * GUARD,), 0xA5, dtype=self._torch.uint8, device=f"cuda:{dev}")
             t[GUARD:GUARD + int(nbytes)] = 0xFF
+            self._torch.cuda.synchronize()     # the fill runs on torch's stream, the library on its own
             self.blocks.append((t, int(nbytes)))
             self._bufs[t.data_ptr() + GUARD] = t
             return t.data_ptr() + GUARD

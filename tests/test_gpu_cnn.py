@@ -433,3 +433,35 @@ def test_cnn_slot_layout_covers_every_buffer(tg, orc, prec, mode):
     ref = orc.cnn(img, n5, prm, bias_plane=(bias == "plane"))
     assert np.isfinite(got).all()
     assert normwise(got, ref) <= (2e-2 if prec == "bf16_tc" else 1e-5)
+
+
+@pytest.mark.parametrize("prec", ["fp32", "bf16_tc", "fp32_tc"])
+def test_cnn_graph_replay_and_new_parameters(tg, orc, prec):
+    """CUDA-graph replay of a streamed CNN plan (bias rows streamed, several chunks) equals the
+    direct execution; after tg_plan_invalidate_params with new weights the graph is recaptured
+    and follows them (the captured kernels hold the weights by value)."""
+    P = {"fp32": tg.TG_FP32, "bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}[prec]
+    seed = 77
+    n, H, W, n5 = 2, 150, 172, 40
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W)
+    h5, w5 = synth.cnn_dims(H, W)[4]
+    out = np.zeros((n, 9, h5, w5), np.float32)
+    g, _ = tg.cnn_graph(img, n5, prm, out=out)
+    g.set(torch_runtime=True, budget=1_200_000, precision=P)
+    p = g.plan()
+    assert p.json()["n_chunks"] > 2
+    p.execute()
+    direct = out.copy()
+    p.use_graph(True)
+    for rep in range(2):
+        out[:] = 0
+        p.execute()
+        assert np.array_equal(out, direct), rep
+    for k in (3, 6):                     # new C3 / C5 weights in the caller's parameter buffers
+        prm[k] *= np.float32(0.75)
+    p.invalidate_params()
+    p.execute()
+    p.execute()
+    ref = orc.cnn(img, n5, prm)
+    assert normwise(out, ref) <= (2e-2 if prec == "bf16_tc" else 1e-5)

@@ -322,3 +322,43 @@ def test_edge_slot_layout_covers_every_buffer(tg, orc, budget, nf):
     assert rt.guards_intact()
     ref = np.stack([orc.edge_general(img[b, 0], K, "max") for b in range(2)])[:, None]
     assert np.isfinite(out).all() and normwise(out, ref) <= 1e-5
+
+
+def test_graph_replay_equals_direct_execution(tg, orc):
+    """tg_plan_set_graph: executions replayed as one captured CUDA graph give the same bits as
+    direct executions, follow new input values in the bound buffers, and count their launches;
+    device-resident (configs[0]-sized) and host-streamed multi-chunk plans."""
+    img = synth.images_np(29, 2, 256, 256)
+    K1, K2 = synth.random_edge_filters_np(29)
+    ref = oracle_edge(orc, img, K1, K2)
+    x = torch.from_numpy(img).cuda()
+    y = torch.zeros_like(x)
+    g, _ = tg.edge_graph(x, K1, K2, out=y, device=True)
+    g.set(torch_runtime=True)
+    p = g.plan()
+    p.execute()
+    direct = y.clone()
+    p.use_graph(True)
+    for rep in range(3):
+        y.zero_()
+        l0 = p.launches()
+        p.execute()
+        assert p.launches() == l0 + 1
+        assert torch.equal(y, direct), rep
+    x.mul_(0.5)                                     # new values in the bound input buffer
+    p.execute()
+    assert normwise(y.cpu().numpy()[:, 0], oracle_edge(orc, img * np.float32(0.5), K1, K2)[:, 0]) <= 1e-5
+    assert normwise(direct.cpu().numpy()[:, 0], ref[:, 0]) <= 1e-5
+    # host-streamed, several chunks over a depth-2 ring
+    out = pinned((2, 1, 256, 256))
+    gh, _ = tg.edge_graph(pinned((2, 1, 256, 256)).copy_(torch.from_numpy(img)), K1, K2, out=out)
+    gh.set(torch_runtime=True, budget=300_000, depth=2)
+    ph = gh.plan()
+    assert ph.stats()["n_chunks"] >= 4
+    ph.execute()
+    want = out.clone()
+    ph.use_graph(True)
+    for rep in range(3):
+        out.zero_()
+        ph.execute()
+        assert torch.equal(out, want), rep
