@@ -362,3 +362,44 @@ def test_graph_replay_equals_direct_execution(tg, orc):
         out.zero_()
         ph.execute()
         assert torch.equal(out, want), rep
+
+
+def test_shard_holds_only_its_images(tg, orc):
+    """Multi-process sharding (tg_set_shard) as bench.py and tools/config5.py run it: each rank
+    pins host buffers for ITS images only and passes base pointers offset by the images before
+    them -- the library touches (and registers) nothing else. Every rank's rows equal the
+    one-process run bit for bit (the same global chunk list)."""
+    n, H, W = 6, 200, 256
+    img = synth.images_np(33, n, H, W)
+    K1, K2 = synth.random_edge_filters_np(33)
+    full = np.zeros_like(img)
+    g, _ = tg.edge_graph(img, K1, K2, out=full)
+    g.set(torch_runtime=True, budget=500_000)
+    g.plan().execute()
+    world = 3
+    for rank in range(world):
+        probe, _ = tg.edge_graph(img, K1, K2, out=np.zeros_like(img))
+        probe.set(budget=500_000, shard=(rank, world))
+        j = probe.plan().json()
+        mine = j["chunks"][j["shard"][2]:j["shard"][3]]
+        i0 = min(c["img"] for c in mine)
+        i1 = max(c["img"] + c["nimg"] for c in mine)
+        xs = pinned((i1 - i0, 1, H, W))
+        xs.copy_(torch.from_numpy(img[i0:i1]))
+        ys = pinned((i1 - i0, 1, H, W))
+        gs = tg.Graph()
+        x = tg.tg_input(gs.h, n, 1, H, W, xs.data_ptr() - i0 * H * W * 4)
+        k1 = gs.param(K1.reshape(1, 1, 16, 16))
+        k2 = gs.param(K2.reshape(1, 1, 16, 16))
+        e1 = gs.conv2d(x, k1, -1, tg.TG_SAME)
+        e2 = gs.conv2d(x, k2, -1, tg.TG_SAME)
+        tg.tg_output(gs.h, gs.max_combine([e1, e2, gs.neg(e1), gs.neg(e2)]), ys.data_ptr() - i0 * H * W * 4)
+        gs._keep += [xs, ys]
+        gs.set(torch_runtime=True, budget=500_000, shard=(rank, world))
+        p = gs.plan()
+        assert p.json()["chunks"] == j["chunks"]
+        p.execute()
+        for c in mine:
+            for b in range(c["img"], c["img"] + c["nimg"]):
+                r0, r1 = c["out"]
+                assert np.array_equal(ys[b - i0, 0, r0:r1].numpy(), full[b, 0, r0:r1]), (rank, b)

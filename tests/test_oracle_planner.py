@@ -120,3 +120,20 @@ def test_split_factors_8_orientations():
         g2 = P.edge_graph(1, S, orientations=8, kernel_floats=False)
         k = P.split_factors(g2, 1500)
         assert k["max"] == k_max and k["C1"] == k_cr and k["R1"] == k_cr
+
+
+def test_edge_graph_general_counts_by_hand():
+    """Operator / DS counts of the edge graph variants, counted by hand from PAPER.md:621-629:
+    max over nf responses and their remaps = nf convs + nf remaps + 1 max (Fig. 3 at nf = 2:
+    5 ops, 8 DS); sum = nf convs + 1 add, DS Im + nf kernels + nf responses + E; maxabs adds
+    one abs op and DS per response."""
+    for nf in (1, 2, 3, 4):
+        g = P.edge_graph_general(10, 12, 16, nf, "max")
+        assert (len(g.ops), len(g.ds)) == (2 * nf + 1, 1 + nf + 2 * nf + 1)
+        g = P.edge_graph_general(10, 12, 16, nf, "sum")
+        assert (len(g.ops), len(g.ds)) == (nf + 1, 1 + nf + nf + 1)
+        g = P.edge_graph_general(10, 12, 16, nf, "maxabs")
+        assert (len(g.ops), len(g.ds)) == (2 * nf + 1, 1 + nf + 2 * nf + 1)
+        assert g.io_lower_bound() == 2 * 10 * 12 + nf * 256
+    g = P.edge_graph_general(1000, 1000, 16, 2, "max")
+    assert (g.total_temp(), g.io_lower_bound(), g.baseline()) == (6_000_512, 2_000_512, 13_000_512)
