@@ -46,6 +46,23 @@ VARIANTS = {
     "u3_no_copy": ("cnn_tc.cu", [
         ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
          "            if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n            __syncwarp();\n            if (false)")]),
+    # U3 3xFP16 (TG_FP32_TC): no B-operand streaming (the ring stages arrive without copies)
+    "h3u3_no_bcopy": ("cnn_h3.cu", [
+        ("                        tc::mbar_expect_tx(&S.b_full[slot], stage_bytes);\n                        tc::bulk_g2s(S.b[slot], kb + (size_t)(ks / U3H_KST) * stage_bytes, stage_bytes, &S.b_full[slot]);",
+         "                        tc::mbar_arrive(&S.b_full[slot]);")]),
+    # U3 3xFP16: the epilogue only does the hand-offs
+    "h3u3_no_epi": ("cnn_h3.cu", [
+        ("#pragma unroll\n            for (int c = 0; c < NCH; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);",
+         "#pragma unroll\n            for (int c = 0; c < 0; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);"),
+        ("            if (cur.ok) {\n                float* ob = a.out + cur.img * a.out_img_stride", "            if (false) {\n                float* ob = a.out + cur.img * a.out_img_stride")]),
+    # U3 3xFP16: no MMAs (commits still arrive)
+    "h3u3_no_mma": ("cnn_h3.cu", [
+        ("                            tc::mma_bf16(d, a_hi, b_hi, idesc, ks > 0 ? 1u : 0u);\n                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);\n                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);",
+         "                            if (ks < 0) tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);")]),
+    # U3 3xFP16: two MMAs per K-step instead of three (hi.hi + hi.lo): the MMA-count sensitivity
+    "h3u3_2mma": ("cnn_h3.cu", [
+        ("                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);\n                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);",
+         "                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);")]),
 }
 
 
