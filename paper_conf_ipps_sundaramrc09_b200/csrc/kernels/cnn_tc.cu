@@ -568,242 +568,6 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
     if (warp == 0) tc::tmem_dealloc<512>(tmem);
 }
 
-// ============================================================================ U3, large nets: W5 in TMEM
-// For NP > 64 the MMAs above are bound by reading their A operand (the 128 x 16 slice tile) from
-// shared memory: ~78 cycles per MMA whatever N is. Here the operand roles are
-// swapped: C5 is D5[map][pos] = W5[map][k] X[k][pos] with A = W5 held in TENSOR memory for the
-// whole kernel (lanes = maps, 40 K-steps x 8 columns of bf16 pairs = 320 columns, loaded once per
-// CTA) and B = the slice pixels in shared memory -- the same slices and tap-shifted descriptors
-// as above, now N = 96 output positions (K-major 16-byte rows) -- so an MMA reads only its 3 KB B
-// tile. TMEM: D buffers at columns [0, 96) and [96, 192), W5 at [192, 512).
-// The epilogue works in two phases because D5 now has maps in lanes and positions in columns:
-//   phase 1 (warps 0-3, TMEM lane quadrants): D5 -> registers -> shared memory transposed,
-//            t5[position][map] (fp32, odd row pitch: both sides conflict-free);
-//   phase 2 (warps 4-9, thread = (position, half of the maps)): + bias plane (coalesced over
-//            positions), tanh, the 1x1 C6 as fp32 FMAs with weights in the constant bank; the two
-//            halves' partial sums meet in shared memory; + C6 bias -> output.
-// C6 thus runs in fp32 on T5 in fp32 (the NP <= 64 kernel rounds T5 to bf16 for its C6 MMA).
-constexpr int U3W_N = 96;              // output positions per tile (the MMA's N)
-constexpr int U3W_SPX = U3W_N + 8;     // pixels per slice block (102 used: +4 taps, +1 pair, +1)
-constexpr int U3W_NA = 6;              // slice buffers
-constexpr int U3W_WCOL = 2 * U3W_N;    // first TMEM column of W5
-constexpr int U3W_PITCH = 129;         // floats per t5 row (odd)
-constexpr int kU3WP1 = 4, kU3WP2 = 6;  // phase-1 / phase-2 warps
-constexpr int kThreadsU3W = (kU3WP1 + kU3WP2 + 2) * 32;
-
-struct U3WK6 {
-    float k6[U3_NMAX][12];  // [map][o] (9 used): C6 weights, read from the constant bank
-};
-
-struct U3WSmem {
-    uint4 a[U3W_NA][3][U3W_SPX];          // slice ring: [channel block][pixel] -> 8 bf16
-    float t5[2][U3W_N][U3W_PITCH];        // D5 of a tile, transposed: [buffer][position][map]
-    float red[2][U3W_N][9];               // phase 2: C6 partial sums of the upper map half
-    uint64_t a_full[U3W_NA], a_empty[U3W_NA], d_full[2], d_empty[2], t_full[2], t_empty[2];
-    uint32_t tmem;
-};
-
-// Phase 2 of one position over maps [M0, M0 + 64) ∩ [0, m1): + bias, tanh, the C6 dot products.
-// Fully unrolled so every C6 weight is an immediate constant-bank operand of its FFMA.
-template <int M0, bool kFull>
-__device__ __forceinline__ void u3w_c6_half(const float* __restrict__ t5, const float* __restrict__ pb, uint32_t bcs,
-                                            int m1, const U3WK6& k6w, float (&c6)[9]) {
-#pragma unroll
-    for (int j = 0; j < 64; ++j) {
-        const int m = M0 + j;
-        if (kFull || m < m1) {
-            const float t = tanh_approx(t5[m] + __ldg(pb + (size_t)m * bcs));
-#pragma unroll
-            for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[m][o], t, c6[o]);
-        }
-    }
-}
-
-__global__ void __launch_bounds__(kThreadsU3W, 1)
-    cnn_u3_tw_kernel(const CnnU3Args a, const __grid_constant__ U3WK6 k6w, const int64_t ntiles) {
-    extern __shared__ __align__(128) uint8_t smraw[];
-    U3WSmem& S = *reinterpret_cast<U3WSmem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int NP = a.n_pad;
-    const int64_t per_img = (a.out_rows * a.w4 + U3W_N - 1) / U3W_N;
-    const int64_t bplane = a.t4_rows * a.w4;                 // pixels per channel block of one image
-    const int64_t flat0 = (a.out_row0 - a.t4_row0) * a.w4;  // flat index of output row 0 in the T4 buffer
-
-    if (warp == 0) tc::tmem_alloc<512>(&S.tmem);
-    if (tid == 0) {
-        for (int i = 0; i < U3W_NA; ++i) {
-            tc::mbar_init(&S.a_full[i], 1);
-            tc::mbar_init(&S.a_empty[i], 1);
-        }
-        for (int i = 0; i < 2; ++i) {
-            tc::mbar_init(&S.d_full[i], 1);
-            tc::mbar_init(&S.d_empty[i], kU3WP1);
-            tc::mbar_init(&S.t_full[i], kU3WP1);
-            tc::mbar_init(&S.t_empty[i], kU3WP2);
-        }
-        tc::mbar_fence_init();
-    }
-    // slice buffers start zeroed: pixels a copy does not cover only ever hold finite values
-    for (int idx = tid; idx < U3W_NA * 3 * U3W_SPX; idx += kThreadsU3W) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
-    tc::fence_proxy_async();
-    tc::fence_before_sync();
-    __syncthreads();
-    tc::fence_after_sync();
-    const uint32_t tmem = S.tmem;
-    // W5 -> TMEM once: lane = map n (zero rows for n >= NP), column 8 ks + c = bf16 pair (2c, 2c+1)
-    // of K-step ks, i.e. half c / 4 of the [ks][half][n][8] operand prepared on the host
-    if (warp < kU3WP1) {
-        const int n = 32 * warp + lane;
-        const uint4* kw = reinterpret_cast<const uint4*>(a.k5_tc);
-        const uint32_t lane_base = (uint32_t)(32 * warp) << 16;
-        for (int ks2 = 0; ks2 < U3_KS; ks2 += 2) {
-            uint32_t r[16];
-#pragma unroll
-            for (int q = 0; q < 2; ++q)
-#pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    const uint4 v = n < NP ? kw[(size_t)((ks2 + q) * 2 + h) * NP + n] : make_uint4(0u, 0u, 0u, 0u);
-                    r[q * 8 + h * 4 + 0] = v.x;
-                    r[q * 8 + h * 4 + 1] = v.y;
-                    r[q * 8 + h * 4 + 2] = v.z;
-                    r[q * 8 + h * 4 + 3] = v.w;
-                }
-            tc::tmem_st16(tmem + lane_base + (uint32_t)(U3W_WCOL + ks2 * 8), r);
-        }
-        tc::tmem_wait_st();
-    }
-    tc::fence_before_sync();
-    __syncthreads();
-    tc::fence_after_sync();
-
-    const int64_t my = ntiles > blockIdx.x ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-    if (warp == kU3WP1 + kU3WP2 + 1) {
-        // ---------------------------------------------------------------- copy producer
-        const uint4* t4all = reinterpret_cast<const uint4*>(a.t4);
-        for (int64_t s = 0; s < my * 5; ++s) {
-            const int slot = (int)(s % U3W_NA);
-            if (s >= U3W_NA) tc::mbar_wait(&S.a_empty[slot], (uint32_t)(((s - U3W_NA) / U3W_NA) & 1));
-            const int64_t tile = blockIdx.x + (s / 5) * gridDim.x;
-            const int i = (int)(s % 5);
-            const int64_t img = (uint32_t)tile / (uint32_t)per_img;
-            const int64_t q0 = (tile - img * per_img) * U3W_N;
-            const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
-            const int64_t n = max((int64_t)0, min((int64_t)U3W_SPX, bplane - e));
-            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
-            __syncwarp();
-            if (n > 0 && lane < 3)  // one channel block per lane, in one warp instruction
-                tc::bulk_g2s(S.a[slot][lane], t4all + (img * 3 + lane) * bplane + e, (uint32_t)(n * 16), &S.a_full[slot]);
-            __syncwarp();
-        }
-    } else if (warp == kU3WP1 + kU3WP2) {
-        // ---------------------------------------------------------------- MMA issuer
-        const uint32_t idesc = tc::make_idesc_bf16(kTileM, U3W_N);
-        const uint32_t plane_bytes = (uint32_t)(U3W_SPX * 16);
-        int64_t s = 0;
-        for (int64_t k = 0; k < my; ++k) {
-            const int buf = (int)(k & 1);
-            if (k >= 2) {
-                tc::mbar_wait(&S.d_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
-                tc::fence_after_sync();
-            }
-            const uint32_t d = tmem + (uint32_t)(buf * U3W_N);
-            for (int i = 0; i < 5; ++i, ++s) {
-                const int slot = (int)(s % U3W_NA);
-                tc::mbar_wait(&S.a_full[slot], (uint32_t)((s / U3W_NA) & 1));
-                tc::fence_after_sync();
-                const uint32_t b_base = tc::smem_u32(S.a[slot][0]);
-                if (tc::elect_one()) {
-#pragma unroll
-                    for (int r8 = 0; r8 < 8; ++r8) {
-                        const int ks = i * 8 + r8;
-                        // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0 and 1); r8 >= 5: channels
-                        // 16-19 of taps (i, j) and (i, j+1), j = 2 (r8 - 5) (block 2, next pixel)
-                        const uint32_t b_addr = r8 < 5 ? b_base + (uint32_t)(r8 * 16)
-                                                       : b_base + 2 * plane_bytes + (uint32_t)(2 * (r8 - 5) * 16);
-                        const uint64_t bd = tc::make_desc(b_addr, r8 < 5 ? plane_bytes : 16u, 128);
-                        tc::mma_bf16_ts(d, tmem + (uint32_t)(U3W_WCOL + ks * 8), bd, idesc, ks > 0 ? 1u : 0u);
-                    }
-                    tc::commit(&S.a_empty[slot]);
-                    if (i == 4) tc::commit(&S.d_full[buf]);
-                }
-                __syncwarp();
-            }
-        }
-    } else if (warp < kU3WP1) {
-        // ---------------------------------------------------------------- phase 1: transpose
-        const uint32_t lane_base = (uint32_t)(32 * warp) << 16;
-        const int map = 32 * warp + lane;
-        for (int64_t k = 0; k < my; ++k) {
-            const int buf = (int)(k & 1);
-            tc::mbar_wait(&S.d_full[buf], (uint32_t)((k >> 1) & 1));
-            tc::fence_after_sync();
-            float v[U3W_N];
-#pragma unroll
-            for (int c = 0; c < U3W_N / 32; ++c)
-                tc::tmem_ld32_async(tmem + lane_base + (uint32_t)(buf * U3W_N + 32 * c),
-                                    *reinterpret_cast<float(*)[32]>(&v[32 * c]));
-            tc::tmem_wait_ld();
-            tc::fence_before_sync();
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&S.d_empty[buf]);  // the accumulator can be reused
-            if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
-#pragma unroll
-            for (int p = 0; p < U3W_N; ++p) S.t5[buf][p][map] = v[p];
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive(&S.t_full[buf]);
-        }
-    } else {
-        // ---------------------------------------------------------------- phase 2: bias, tanh, C6
-        const int p2 = tid - 32 * kU3WP1;        // 0 .. 32 kU3WP2 - 1
-        const int px = p2 % U3W_N, half = p2 / U3W_N;
-        const int m1 = min(64 * half + 64, a.n5);
-        const uint32_t bcs = a.b5_plane ? (uint32_t)(a.b5_rows * a.w5) : 1u;  // channel stride of the bias
-        const int w4 = (int)a.w4, w5 = (int)a.w5, orow_end = (int)(a.out_row0 + a.out_rows);
-        for (int64_t k = 0; k < my; ++k) {
-            const int buf = (int)(k & 1);
-            const int64_t tile = blockIdx.x + k * gridDim.x;
-            const int64_t img = (uint32_t)tile / (uint32_t)per_img;
-            const int qq = (int)(tile - img * per_img) * U3W_N + px;
-            const int r = qq / w4;
-            const int orow = (int)a.out_row0 + r, ocol = qq - r * w4;
-            const bool ok = orow < orow_end && ocol < w5;
-            const int orow_c = min(orow, orow_end - 1), ocol_c = min(ocol, w5 - 1);
-            const float* pb = a.b5_plane ? a.b5 + ((int64_t)(orow_c - a.b5_row0) * w5 + ocol_c) : a.b5;
-            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
-            float c6[9];
-#pragma unroll
-            for (int o = 0; o < 9; ++o) c6[o] = 0.f;
-            const float* t5 = S.t5[buf][px];
-            if (half == 0) {
-                if (m1 == 64) u3w_c6_half<0, true>(t5, pb, bcs, m1, k6w, c6);
-                else u3w_c6_half<0, false>(t5, pb, bcs, m1, k6w, c6);
-            } else {
-                if (m1 == 128) u3w_c6_half<64, true>(t5, pb, bcs, m1, k6w, c6);
-                else u3w_c6_half<64, false>(t5, pb, bcs, m1, k6w, c6);
-            }
-            if (half == 1) {
-#pragma unroll
-                for (int o = 0; o < 9; ++o) S.red[buf][px][o] = c6[o];
-            }
-            asm volatile("bar.sync 1, %0;\n" ::"n"(32 * kU3WP2) : "memory");
-            if (lane == 0) tc::mbar_arrive(&S.t_empty[buf]);  // t5[buf] read by every phase-2 warp
-            if (half == 0 && ok) {
-                float* ob = a.out + img * a.out_img_stride + (int64_t)(orow - a.out_row0) * w5 + ocol;
-#pragma unroll
-                for (int o = 0; o < 9; ++o) {
-                    const float b = a.b6_plane
-                                        ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (orow - a.b6_row0)) * w5 + ocol)
-                                        : __ldg(a.b6 + o);
-                    ob[o * a.out_plane_stride] = (c6[o] + S.red[buf][px][o]) + b;
-                }
-            }
-        }
-    }
-    tc::fence_before_sync();
-    __syncthreads();
-    if (warp == 0) tc::tmem_dealloc<512>(tmem);
-}
-
 uint16_t to_bf16(float f) {  // round to nearest even (host)
     uint32_t u;
     std::memcpy(&u, &f, 4);
@@ -888,30 +652,9 @@ cudaError_t launch_cnn_u2_tc(const CnnU2Args& a, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-// Large nets (NP > 64): the weights-in-TMEM kernel above.
-cudaError_t launch_cnn_u3_tw(const CnnU3Args& a, cudaStream_t s) {
-    static std::atomic<uint32_t> flags{0};
-    const size_t smem = sizeof(U3WSmem) + 128;
-    if (!set_smem_attr((const void*)cnn_u3_tw_kernel, smem, flags)) return cudaErrorInvalidValue;
-    if (a.b5_plane && (int64_t)a.n5 * a.b5_rows * a.w5 >= (1ll << 32)) return cudaErrorInvalidValue;
-    U3WK6 k6w{};
-    for (int m = 0; m < a.n5; ++m)
-        for (int o = 0; o < 9; ++o) k6w.k6[m][o] = a.k6_host[o * a.n5 + m];
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const int64_t per_img = (a.out_rows * a.w4 + U3W_N - 1) / U3W_N;
-    const int64_t ntiles = per_img * a.nimg;
-    if (ntiles >= (1ll << 32) || a.out_rows * a.w4 >= (1ll << 31)) return cudaErrorInvalidValue;
-    const unsigned grid = (unsigned)std::min<int64_t>(ntiles, sms);
-    cnn_u3_tw_kernel<<<grid, kThreadsU3W, smem, s>>>(a, k6w, ntiles);
-    return cudaGetLastError();
-}
-
 cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     if (a.out_rows <= 0 || a.nimg <= 0) return cudaSuccess;
     if (a.n_pad > U3_NMAX || a.n_pad % 16 || a.n5 > U3_NMAX) return cudaErrorInvalidValue;
-    if (a.n_pad > 64) return launch_cnn_u3_tw(a, s);
     const size_t smem = sizeof(U3Smem) + 128;
     const int nch = (a.n_pad + 31) / 32;
     const void* fns[4] = {(const void*)cnn_u3_tc_kernel<1>, (const void*)cnn_u3_tc_kernel<2>,

@@ -15,6 +15,11 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 PKG = "paper_conf_ipps_sundaramrc09_b200"
 
+VARIANTS_U3_NO_EPI = [
+    ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
+     "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
+    ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob")]
+
 # variant -> (kernel source, [(old, new), ...]); every `old` must occur in the source
 VARIANTS = {
     "base": ("cnn_tc.cu", []),
@@ -63,6 +68,10 @@ VARIANTS = {
     "h3u3_2mma": ("cnn_h3.cu", [
         ("                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);\n                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);",
          "                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);")]),
+    # U3 bf16: neither epilogue work nor slice copies (the MMA issue alone, plus C6)
+    "u3_mma_only": ("cnn_tc.cu", VARIANTS_U3_NO_EPI + [
+        ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
+         "            if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n            __syncwarp();\n            if (false)")]),
 }
 
 

@@ -1,0 +1,125 @@
+// umma_probe.cu -- measured cost of one tcgen05.mma (kind::f16, bf16 in, fp32 accumulate) as the
+// CNN units issue them: operands in shared memory, K-major, NO swizzle (8-row x 16-byte core
+// matrices), M = 128, N = 16 .. 256, back to back from one thread into one TMEM accumulator.
+// Also: A from TMEM (the "ts" form), and the same MMAs with the operands laid out with the 32-byte
+// swizzle (rows of one K-step = 32 bytes). Prints cycles per MMA (clock64 around a run of MMAs
+// whose completion is awaited through tcgen05.commit + mbarrier).
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -I paper_conf_ipps_sundaramrc09_b200/csrc/kernels \
+//        -o tools/micro/umma_probe tools/micro/umma_probe.cu && tools/micro/umma_probe
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "tc_sm100.cuh"
+
+using namespace tg;
+
+constexpr int kReps = 520;
+constexpr int kSmem = 200 * 1024;
+
+// layout: 0 = no swizzle (LBO = K-half distance, SBO = 128), 2 = 32-byte swizzle
+__device__ __forceinline__ uint64_t desc_sw(uint32_t addr, uint32_t lbo, uint32_t sbo, int swz) {
+    uint64_t d = tc::make_desc(addr, lbo, sbo);
+    if (swz == 32) d |= (uint64_t)6 << 61;  // layout type SWIZZLE_32B (sm_100 encoding: 6)
+    return d;
+}
+
+template <int N, bool kTs, int kSwz, int kShift = 0, int kLbo16 = 0, int kRot = 0, int kBRot = 0>
+__global__ void probe(long long* out) {
+    extern __shared__ __align__(1024) uint8_t sm[];
+    __shared__ uint64_t bar;
+    __shared__ uint32_t tm;
+    uint8_t* A = sm;                 // 128 rows x 16 K (4 KB) -- plus room
+    uint8_t* B = sm + 16384;         // N rows x 16 K (kBRot: 40 such blocks, one per K-step)
+    const int tid = threadIdx.x, warp = tid >> 5;
+    for (int i = tid; i < kSmem / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(sm)[i] = 0x3c003c00u;  // 1.0
+    if (warp == 0) tc::tmem_alloc<512>(&tm);
+    if (tid == 0) {
+        tc::mbar_init(&bar, 1);
+        tc::mbar_fence_init();
+    }
+    tc::fence_proxy_async();
+    tc::fence_before_sync();
+    __syncthreads();
+    tc::fence_after_sync();
+    if (warp == 0) {
+        const uint32_t idesc = tc::make_idesc_bf16(128, N);
+        const uint32_t a = tc::smem_u32(A), b = tc::smem_u32(B);
+        // no swizzle: K-half at LBO (A: 2048 B, B: N*16), 8-row groups at SBO = 128 B
+        // 32-byte swizzle: a row of one K-step is 32 contiguous bytes, 8-row atoms of 256 B
+        // kShift: A starts kShift 16-byte rows into its buffer (a tap-shifted implicit-GEMM window);
+        // kLbo16: the second K half is the NEXT row (LBO = 16 B, the tap-pair trick); kRot: the A
+        // start rotates over 8 shifts MMA by MMA (as the K-steps of one filter row do)
+        const uint64_t ad = kSwz ? desc_sw(a, 16, 256, kSwz)
+                                 : tc::make_desc(a + 16 * kShift, kLbo16 ? 16u : 2048u, 128);
+        const uint64_t bd = kSwz ? desc_sw(b, 16, 256, kSwz) : tc::make_desc(b, (uint32_t)(N * 16), 128);
+        long long t0 = 0, t1 = 0;
+        for (int pass = 0; pass < 2; ++pass) {
+            __syncwarp();
+            t0 = clock64();
+            if (tc::elect_one()) {
+                for (int r = 0; r < kReps; ++r) {
+                    if (kTs)
+                        tc::mma_bf16_ts(tm + 256, tm + 8 * (r & 7), bd, idesc, r > 0 ? 1u : 0u);
+                    else
+                        tc::mma_bf16(tm + 256, kRot ? ad + (uint64_t)(r & 7) : ad,
+                                     kBRot ? bd + (uint64_t)((r % 40) * 2 * N) : bd, idesc, r > 0 ? 1u : 0u);
+                }
+                tc::commit(&bar);
+            }
+            __syncwarp();
+            tc::mbar_wait(&bar, (uint32_t)pass);
+            t1 = clock64();
+        }
+        if (tid == 0) *out = (t1 - t0);
+    }
+    tc::fence_before_sync();
+    __syncthreads();
+    if (warp == 0) tc::tmem_dealloc<512>(tm);
+}
+
+template <int N, bool kTs, int kSwz, int kShift = 0, int kLbo16 = 0, int kRot = 0, int kBRot = 0>
+void run(const char* what) {
+    long long* d;
+    cudaMalloc(&d, sizeof(long long));
+    cudaFuncSetAttribute(probe<N, kTs, kSwz, kShift, kLbo16, kRot, kBRot>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
+    probe<N, kTs, kSwz, kShift, kLbo16, kRot, kBRot><<<1, 128, kSmem>>>(d);
+    cudaError_t e = cudaDeviceSynchronize();
+    long long h = 0;
+    cudaMemcpy(&h, d, sizeof h, cudaMemcpyDeviceToHost);
+    const double floor_cyc = 128.0 * N / 256.0;
+    printf("%-28s N=%3d  %7.1f cycles/MMA  (floor %5.1f)  %s\n", what, N, (double)h / kReps, floor_cyc,
+           e == cudaSuccess ? "" : cudaGetErrorString(e));
+    cudaFree(d);
+}
+
+int main() {
+    run<16, false, 0>("SS no-swizzle");
+    run<32, false, 0>("SS no-swizzle");
+    run<48, false, 0>("SS no-swizzle");
+    run<64, false, 0>("SS no-swizzle");
+    run<96, false, 0>("SS no-swizzle");
+    run<128, false, 0>("SS no-swizzle");
+    run<256, false, 0>("SS no-swizzle");
+    run<64, true, 0>("TS (A in TMEM) no-swizzle B");
+    run<96, true, 0>("TS (A in TMEM) no-swizzle B");
+    run<128, true, 0>("TS (A in TMEM) no-swizzle B");
+    run<256, true, 0>("TS (A in TMEM) no-swizzle B");
+    run<64, false, 32>("SS 32B-swizzle");
+    run<128, false, 32>("SS 32B-swizzle");
+    run<256, false, 32>("SS 32B-swizzle");
+    run<128, false, 0, 1>("SS A shifted 1 row");
+    run<128, false, 0, 3>("SS A shifted 3 rows");
+    run<128, false, 0, 8>("SS A shifted 8 rows");
+    run<128, false, 0, 0, 1>("SS A LBO=16 (next pixel)");
+    run<128, false, 0, 1, 1>("SS A shift 1, LBO=16");
+    run<128, false, 0, 0, 0, 1>("SS A rotating shifts");
+    run<32, false, 0, 1>("SS A shifted 1 row");
+    run<48, false, 0, 1>("SS A shifted 1 row");
+    run<48, false, 0, 0, 0, 1>("SS A rotating shifts");
+    run<128, false, 0, 0, 0, 1, 1>("SS A rot, B over 40 K-steps");
+    run<64, false, 0, 0, 0, 1, 1>("SS A rot, B over 40 K-steps");
+    run<48, false, 0, 0, 0, 1, 1>("SS A rot, B over 40 K-steps");
+    run<96, true, 0, 0, 0, 0, 1>("TS, B over 40 K-steps");
+    return 0;
+}
