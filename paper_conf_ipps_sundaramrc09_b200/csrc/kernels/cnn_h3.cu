@@ -176,20 +176,22 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
     } else if (warp == 8) {
         // ---------------------------------------------------------------- MMA issuer
-        tc::mbar_wait(&S.b_full, 0);
-        const uint32_t idesc64 = idesc_f16(kTileM, 2 * U2H_N), idesc32 = idesc_f16(kTileM, U2H_N);
-        // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding;
-        // A: the second K half is the next pixel (tap j+1, LBO = 16 B); B: LBO = one K half
-        const uint64_t a_desc0 = tc::make_desc(tc::smem_u32(S.a[0][0]), 16, 128);
-        const uint64_t b_desc0 = tc::make_desc(tc::smem_u32(S.b), 2 * U2H_N * 16, 128);
-        for (int64_t k = 0; k < my; ++k) {
-            const int buf = (int)(k % U2H_NA), ts = (int)(k % U2H_NT);
-            tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2H_NA) & 1));
-            if (k >= U2H_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2H_NT) / U2H_NT) & 1));
-            tc::fence_after_sync();
-            const uint64_t abuf = a_desc0 + (uint64_t)(buf * (2 * U2H_PLANE));
-            const uint32_t d0 = tmem + (uint32_t)(ts * 4 * U2H_N);
-            if (tc::elect_one()) {
+        // ONE elected lane runs the whole loop (warp-level hand-offs per segment left the tensor
+        // pipe idle, tools/micro/umma_probe.cu)
+        if (tc::elect_one()) {
+            tc::mbar_wait(&S.b_full, 0);
+            const uint32_t idesc64 = idesc_f16(kTileM, 2 * U2H_N), idesc32 = idesc_f16(kTileM, U2H_N);
+            // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding;
+            // A: the second K half is the next pixel (tap j+1, LBO = 16 B); B: LBO = one K half
+            const uint64_t a_desc0 = tc::make_desc(tc::smem_u32(S.a[0][0]), 16, 128);
+            const uint64_t b_desc0 = tc::make_desc(tc::smem_u32(S.b), 2 * U2H_N * 16, 128);
+            for (int64_t k = 0; k < my; ++k) {
+                const int buf = (int)(k % U2H_NA), ts = (int)(k % U2H_NT);
+                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2H_NA) & 1));
+                if (k >= U2H_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2H_NT) / U2H_NT) & 1));
+                tc::fence_after_sync();
+                const uint64_t abuf = a_desc0 + (uint64_t)(buf * (2 * U2H_PLANE));
+                const uint32_t d0 = tmem + (uint32_t)(ts * 4 * U2H_N);
 #pragma unroll
                 for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
 #pragma unroll
@@ -206,8 +208,8 @@ __global__ void __launch_bounds__(kThreads, 1)
                 tc::commit(&S.a_empty[buf]);
                 tc::commit(&S.t_full[ts]);
             }
-            __syncwarp();
         }
+        __syncwarp();
     } else {
         // ---------------------------------------------------------------- epilogue groups
         const int grp = warp >> 2, wq = warp & 3;
@@ -413,35 +415,37 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
     } else if (warp == kEpiWarps) {
         // ---------------------------------------------------------------- MMA issuer
-        const uint32_t idesc = idesc_f16(kTileM, NP), idesc2 = idesc_f16(kTileM, 2 * NP);
-        const uint32_t plane_bytes = (uint32_t)(U3H_SPX * 16), part_bytes = 3 * plane_bytes;
-        int64_t si = 0, gi = 0;
-        for (int64_t k = 0; k < my_bands; ++k) {
-            const int buf = (int)(k & 1);
-            if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
-            const uint32_t d_base = tmem + (uint32_t)(buf * 256);
-            uint32_t a_base = 0, b_base = 0;
-            int aslot = 0, bslot = 0;
-            for (int ks = 0; ks < U3H_KS; ++ks) {
-                if (ks % 8 == 0) {
-                    aslot = (int)(si % U3H_NA);
-                    tc::mbar_wait(&S.a_full[aslot], (uint32_t)((si / U3H_NA) & 1));
-                    a_base = tc::smem_u32(S.a[aslot][0][0]);
-                    ++si;
-                }
-                if (ks % U3H_KST == 0) {
-                    bslot = (int)(gi % U3H_BRING);
-                    tc::mbar_wait(&S.b_full[bslot], (uint32_t)((gi / U3H_BRING) & 1));
-                    b_base = tc::smem_u32(S.b[bslot]);
-                    ++gi;
-                }
-                tc::fence_after_sync();
-                const int r8 = ks % 8, u = ks % U3H_KST;
-                // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0, 1); r8 >= 5: channels 16-19 of
-                // taps (i, j) and (i, j+1), j = 2 (r8 - 5) (block 2, next pixel)
-                const uint32_t a_off = r8 < 5 ? (uint32_t)(r8 * 16) : 2 * plane_bytes + (uint32_t)(2 * (r8 - 5) * 16);
-                const uint32_t lbo = r8 < 5 ? plane_bytes : 16u;
-                if (tc::elect_one()) {
+        // ONE elected lane runs the whole loop: a warp-level hand-off after every K-step (6 MMAs)
+        // left the tensor pipe idle (tools/micro/umma_probe.cu)
+        if (tc::elect_one()) {
+            const uint32_t idesc = idesc_f16(kTileM, NP), idesc2 = idesc_f16(kTileM, 2 * NP);
+            const uint32_t plane_bytes = (uint32_t)(U3H_SPX * 16), part_bytes = 3 * plane_bytes;
+            int64_t si = 0, gi = 0;
+            for (int64_t k = 0; k < my_bands; ++k) {
+                const int buf = (int)(k & 1);
+                if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+                const uint32_t d_base = tmem + (uint32_t)(buf * 256);
+                uint32_t a_base = 0, b_base = 0;
+                int aslot = 0, bslot = 0;
+                for (int ks = 0; ks < U3H_KS; ++ks) {
+                    if (ks % 8 == 0) {
+                        aslot = (int)(si % U3H_NA);
+                        tc::mbar_wait(&S.a_full[aslot], (uint32_t)((si / U3H_NA) & 1));
+                        a_base = tc::smem_u32(S.a[aslot][0][0]);
+                        ++si;
+                    }
+                    if (ks % U3H_KST == 0) {
+                        bslot = (int)(gi % U3H_BRING);
+                        tc::mbar_wait(&S.b_full[bslot], (uint32_t)((gi / U3H_BRING) & 1));
+                        b_base = tc::smem_u32(S.b[bslot]);
+                        ++gi;
+                    }
+                    tc::fence_after_sync();
+                    const int r8 = ks % 8, u = ks % U3H_KST;
+                    // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0, 1); r8 >= 5: channels 16-19 of
+                    // taps (i, j) and (i, j+1), j = 2 (r8 - 5) (block 2, next pixel)
+                    const uint32_t a_off = r8 < 5 ? (uint32_t)(r8 * 16) : 2 * plane_bytes + (uint32_t)(2 * (r8 - 5) * 16);
+                    const uint32_t lbo = r8 < 5 ? plane_bytes : 16u;
 #pragma unroll
                     for (int t = 0; t < 2; ++t) {
                         const uint32_t ab = a_base + a_off + (uint32_t)(t * kTileM * 16);
@@ -466,9 +470,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                     if (r8 == 7) tc::commit(&S.a_empty[aslot]);
                     if (ks == U3H_KS - 1) tc::commit(&S.t_full[buf]);
                 }
-                __syncwarp();
             }
         }
+        __syncwarp();
     } else {
         // ---------------------------------------------------------------- epilogue warps
         // Thread = one output position of the band (tile t = warp / 4, TMEM lane group warp % 4),

@@ -153,35 +153,32 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
         }
     } else if (warp == 8) {
         // -------------------------------------------------------------------- MMA issuer
-        // (the whole warp runs the loop, so descriptors stay in uniform registers; one elected
-        // lane issues the MMAs and commits)
-        tc::mbar_wait(&S.b_full, 0);
-        const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
-        // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding
-        const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), U2_N * 16, 128);
-        const uint64_t adesc0 = tc::make_desc(tc::smem_u32(S.a[0]), 16, 128);  // 2nd K-half = next pixel
-        for (int64_t k = 0; k < my; ++k) {
-            const int buf = (int)(k % U2_NA), ts = (int)(k % U2_NT);
-            tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
-            if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
-            tc::fence_after_sync();
-            const uint64_t abuf = adesc0 + (uint64_t)(buf * (U2_WR * U2_WP));
-            const uint32_t d0 = tmem + (uint32_t)(ts * 64);
-            if (tc::elect_one()) {
+        // ONE elected lane runs the whole loop (barrier waits, MMAs, commits): warp-level
+        // hand-offs per segment left the tensor pipe idle (tools/micro/umma_probe.cu)
+        if (tc::elect_one()) {
+            tc::mbar_wait(&S.b_full, 0);
+            const uint32_t idesc = tc::make_idesc_bf16(kTileM, U2_N);
+            // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding
+            const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), U2_N * 16, 128);
+            const uint64_t adesc0 = tc::make_desc(tc::smem_u32(S.a[0]), 16, 128);  // 2nd K-half = next pixel
+            for (int64_t k = 0; k < my; ++k) {
+                const int buf = (int)(k % U2_NA), ts = (int)(k % U2_NT);
+                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
+                if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
+                tc::fence_after_sync();
+                const uint64_t abuf = adesc0 + (uint64_t)(buf * (U2_WR * U2_WP));
+                const uint32_t d0 = tmem + (uint32_t)(ts * 64);
 #pragma unroll
                 for (int ks = 0; ks < U2_KS; ++ks) {  // window row y = ks / 3, tap pair (j, j+1)
                     const int y = ks / 3, j = 2 * (ks % 3);
                     tc::mma_bf16(d0, abuf + (uint64_t)(y * U2_WP + j), bdesc0 + (uint64_t)(ks * 2 * U2_N), idesc,
                                  ks > 0 ? 1u : 0u);
                 }
-            }
-            __syncwarp();
-            if (tc::elect_one()) {
                 tc::commit(&S.a_empty[buf]);
                 tc::commit(&S.t_full[ts]);
             }
-            __syncwarp();
         }
+        __syncwarp();
     } else {
         // -------------------------------------------------------------------- epilogue groups
         const int grp = warp >> 2, wq = warp & 3;
@@ -379,71 +376,72 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), (uint32_t)(NP * 16), 128);
         const uint64_t b6desc0 = tc::make_desc(tc::smem_u32(S.b6), (uint32_t)(U3_C6N * 16), 128);
         const uint32_t plane_bytes = (uint32_t)(U3_SPX * 16);
-        // C6 of local band kb (its T5 is in TMEM): 2 tiles x NP/16 K-steps, A from TMEM
-        int64_t c6_next = 0;
-        auto issue_c6 = [&](int64_t kb) {
-            const uint32_t base = tmem + (uint32_t)((kb & 1) * 256);
-            if (tc::elect_one()) {
+        // ONE elected lane runs the whole issue loop: tcgen05.mma issue blocks once a few MMAs are
+        // queued, so warp-level hand-offs between slices (elect / __syncwarp, ~170 cycles per slice
+        // measured by tools/micro/umma_probe.cu) left the tensor pipe idle; a single lane's barrier
+        // waits cost less and the queue stays fed.
+        if (tc::elect_one()) {
+            // C6 of local band kb (its T5 is in TMEM): 2 tiles x NP/16 K-steps, A from TMEM
+            int64_t c6_next = 0;
+            auto issue_c6 = [&](int64_t kb) {
+                const uint32_t base = tmem + (uint32_t)((kb & 1) * 256);
                 for (int t = 0; t < 2; ++t)
                     for (int kk = 0; kk < NP / 16; ++kk)
                         tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL), base + (uint32_t)(t * 128 + kk * 8),
                                         b6desc0 + (uint64_t)(kk * 2 * U3_C6N), idesc6, kk > 0 ? 1u : 0u);
                 tc::commit(&S.c6_full[kb & 1]);
-            }
-            __syncwarp();
-        };
-        for (int64_t k = 0; k < my_bands; ++k) {
-            const int buf = (int)(k & 1);
-            if (k >= 2) {
-                // band k-2 shares this accumulator: its C6 must be issued before its epilogue
-                // can release the buffer
-                while (c6_next <= k - 2) {
-                    tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+            };
+            for (int64_t k = 0; k < my_bands; ++k) {
+                const int buf = (int)(k & 1);
+                if (k >= 2) {
+                    // band k-2 shares this accumulator: its C6 must be issued before its epilogue
+                    // can release the buffer
+                    while (c6_next <= k - 2) {
+                        tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                        tc::fence_after_sync();
+                        issue_c6(c6_next++);
+                    }
+                    tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
                     tc::fence_after_sync();
-                    issue_c6(c6_next++);
                 }
-                tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
-                tc::fence_after_sync();
-            }
-            const uint32_t d_base = tmem + (uint32_t)(buf * 256);
-            for (int i = 0; i < 5; ++i) {
-                const int64_t s = k * 5 + i;
-                const int slot = (int)(s % U3_NA);
-                tc::mbar_wait(&S.a_full[slot], (uint32_t)((s / U3_NA) & 1));
-                tc::fence_after_sync();
-                const uint32_t a_base = tc::smem_u32(S.a[slot][0]);
-                if (tc::elect_one()) {
+                const uint32_t d_base = tmem + (uint32_t)(buf * 256);
+                for (int i = 0; i < 5; ++i) {
+                    const int64_t s = k * 5 + i;
+                    const int slot = (int)(s % U3_NA);
+                    tc::mbar_wait(&S.a_full[slot], (uint32_t)((s / U3_NA) & 1));
+                    tc::fence_after_sync();
+                    // descriptors once per slice; the 16 MMAs add constant offsets (16-byte units)
+                    const uint32_t a_base = tc::smem_u32(S.a[slot][0]);
+                    const uint64_t ad_lo = tc::make_desc(a_base, plane_bytes, 128);            // blocks 0, 1
+                    const uint64_t ad_hi = tc::make_desc(a_base + 2 * plane_bytes, 16u, 128);  // block 2, next pixel
+                    const uint64_t bd_i = bdesc0 + (uint64_t)(i * 8 * 2 * NP);
 #pragma unroll
                     for (int r8 = 0; r8 < 8; ++r8) {
-                        const int ks = i * 8 + r8;
                         // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0 and 1); r8 >= 5: channels
                         // 16-19 of taps (i, j) and (i, j+1), j = 2(r8-5) (block 2, next pixel)
-                        const uint32_t a_addr = r8 < 5 ? a_base + (uint32_t)(r8 * 16)
-                                                       : a_base + 2 * plane_bytes + (uint32_t)(2 * (r8 - 5) * 16);
-                        const uint32_t lbo = r8 < 5 ? plane_bytes : 16u;
-                        const uint64_t bd = bdesc0 + (uint64_t)(ks * 2 * NP);  // start address in 16-B units
+                        const uint64_t ad = r8 < 5 ? ad_lo + (uint64_t)r8 : ad_hi + (uint64_t)(2 * (r8 - 5));
+                        const uint64_t bd = bd_i + (uint64_t)(r8 * 2 * NP);
 #pragma unroll
-                        for (int t = 0; t < 2; ++t) {
-                            const uint64_t ad = tc::make_desc(a_addr + (uint32_t)(t * kTileM * 16), lbo, 128);
-                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad, bd, idesc, ks > 0 ? 1u : 0u);
-                        }
+                        for (int t = 0; t < 2; ++t)
+                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,
+                                         (i | r8) > 0 ? 1u : 0u);
                     }
                     tc::commit(&S.a_empty[slot]);
                     if (i == 4) tc::commit(&S.t_full[buf]);
-                }
-                __syncwarp();
-                // the previous band's C6 as soon as its T5 is ready (between slices)
-                if (c6_next < k && tc::mbar_test(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1))) {
-                    tc::fence_after_sync();
-                    issue_c6(c6_next++);
+                    // the previous band's C6 as soon as its T5 is ready (between slices)
+                    if (c6_next < k && tc::mbar_test(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1))) {
+                        tc::fence_after_sync();
+                        issue_c6(c6_next++);
+                    }
                 }
             }
+            while (c6_next < my_bands) {
+                tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                tc::fence_after_sync();
+                issue_c6(c6_next++);
+            }
         }
-        while (c6_next < my_bands) {
-            tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
-            tc::fence_after_sync();
-            issue_c6(c6_next++);
-        }
+        __syncwarp();
     } else {
         // ---------------------------------------------------------------- epilogue groups
         // Two groups of 8 warps take alternate bands (group g: bands k = g, g+2, ..., always TMEM

@@ -41,8 +41,8 @@ VARIANTS = {
          "            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = 0.f;")]),
     # U3 bf16: the MMA warp issues no C5 MMAs (commits still arrive)
     "u3_no_c5": ("cnn_tc.cu", [
-        ("                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad, bd, idesc, ks > 0 ? 1u : 0u);",
-         "                            if (ks < 0) tc::mma_bf16(d_base + (uint32_t)(t * 128), ad, bd, idesc, ks > 0 ? 1u : 0u);")]),
+        ("                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,",
+         "                            if (r8 < 0) tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,")]),
     # U3 bf16: no C6 MMAs
     "u3_no_c6": ("cnn_tc.cu", [
         ("                        tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL)",

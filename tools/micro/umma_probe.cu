@@ -24,10 +24,11 @@ __device__ __forceinline__ uint64_t desc_sw(uint32_t addr, uint32_t lbo, uint32_
     return d;
 }
 
-template <int N, bool kTs, int kSwz, int kShift = 0, int kLbo16 = 0, int kRot = 0, int kBRot = 0>
+template <int N, bool kTs, int kSwz, int kShift = 0, int kLbo16 = 0, int kRot = 0, int kBRot = 0, int kAltD = 0,
+          int kCommit = 0, int kFence = 0>
 __global__ void probe(long long* out) {
     extern __shared__ __align__(1024) uint8_t sm[];
-    __shared__ uint64_t bar;
+    __shared__ uint64_t bar, dummy, done_bar;
     __shared__ uint32_t tm;
     uint8_t* A = sm;                 // 128 rows x 16 K (4 KB) -- plus room
     uint8_t* B = sm + 16384;         // N rows x 16 K (kBRot: 40 such blocks, one per K-step)
@@ -36,6 +37,9 @@ __global__ void probe(long long* out) {
     if (warp == 0) tc::tmem_alloc<512>(&tm);
     if (tid == 0) {
         tc::mbar_init(&bar, 1);
+        tc::mbar_init(&dummy, 1 << 20);   // never completes: a sink for the per-slice commits
+        tc::mbar_init(&done_bar, 1);
+        tc::mbar_arrive(&done_bar);       // phase 0 complete: waits on it return at once
         tc::mbar_fence_init();
     }
     tc::fence_proxy_async();
@@ -57,13 +61,29 @@ __global__ void probe(long long* out) {
         for (int pass = 0; pass < 2; ++pass) {
             __syncwarp();
             t0 = clock64();
-            if (tc::elect_one()) {
+            if (kFence) {   // the kernels' per-slice pattern: the whole warp waits on a (completed)
+                           // barrier, fences, re-elects a lane and issues 16 MMAs
+                for (int r0 = 0; r0 < kReps; r0 += 16) {
+                    if (kFence & 2) tc::mbar_wait(&done_bar, 0);
+                    if (kFence & 4) tc::fence_after_sync();
+                    if (tc::elect_one()) {
+                        for (int r = r0; r < r0 + 16 && r < kReps; ++r)
+                            tc::mma_bf16(tm + 128 * (r & 1), ad + (uint64_t)(r & 7), bd + (uint64_t)(((r >> 1) % 40) * 2 * N),
+                                         idesc, r > 1 ? 1u : 0u);
+                        tc::commit(&dummy);
+                    }
+                    __syncwarp();
+                }
+                if (tc::elect_one()) tc::commit(&bar);
+            } else if (tc::elect_one()) {
                 for (int r = 0; r < kReps; ++r) {
                     if (kTs)
                         tc::mma_bf16_ts(tm + 256, tm + 8 * (r & 7), bd, idesc, r > 0 ? 1u : 0u);
                     else
-                        tc::mma_bf16(tm + 256, kRot ? ad + (uint64_t)(r & 7) : ad,
-                                     kBRot ? bd + (uint64_t)((r % 40) * 2 * N) : bd, idesc, r > 0 ? 1u : 0u);
+                        tc::mma_bf16(kAltD ? tm + 128 * (r & 1) : tm + 256, kRot ? ad + (uint64_t)(r & 7) : ad,
+                                     kBRot ? bd + (uint64_t)(((r >> (kAltD ? 1 : 0)) % 40) * 2 * N) : bd, idesc,
+                                     r > (kAltD ? 1 : 0) ? 1u : 0u);
+                    if (kCommit && (r % kCommit) == kCommit - 1) tc::commit(&dummy);
                 }
                 tc::commit(&bar);
             }
@@ -71,24 +91,25 @@ __global__ void probe(long long* out) {
             tc::mbar_wait(&bar, (uint32_t)pass);
             t1 = clock64();
         }
-        if (tid == 0) *out = (t1 - t0);
+        if (tid == 0) out[blockIdx.x] = (t1 - t0);
     }
     tc::fence_before_sync();
     __syncthreads();
     if (warp == 0) tc::tmem_dealloc<512>(tm);
 }
 
-template <int N, bool kTs, int kSwz, int kShift = 0, int kLbo16 = 0, int kRot = 0, int kBRot = 0>
-void run(const char* what) {
+template <int N, bool kTs, int kSwz, int kShift = 0, int kLbo16 = 0, int kRot = 0, int kBRot = 0, int kAltD = 0,
+          int kCommit = 0, int kFence = 0>
+void run(const char* what, int grid = 1) {
     long long* d;
-    cudaMalloc(&d, sizeof(long long));
-    cudaFuncSetAttribute(probe<N, kTs, kSwz, kShift, kLbo16, kRot, kBRot>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
-    probe<N, kTs, kSwz, kShift, kLbo16, kRot, kBRot><<<1, 128, kSmem>>>(d);
+    cudaMalloc(&d, 256 * sizeof(long long));
+    cudaFuncSetAttribute(probe<N, kTs, kSwz, kShift, kLbo16, kRot, kBRot, kAltD, kCommit, kFence>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
+    probe<N, kTs, kSwz, kShift, kLbo16, kRot, kBRot, kAltD, kCommit, kFence><<<grid, 128, kSmem>>>(d);
     cudaError_t e = cudaDeviceSynchronize();
     long long h = 0;
     cudaMemcpy(&h, d, sizeof h, cudaMemcpyDeviceToHost);
     const double floor_cyc = 128.0 * N / 256.0;
-    printf("%-28s N=%3d  %7.1f cycles/MMA  (floor %5.1f)  %s\n", what, N, (double)h / kReps, floor_cyc,
+    printf("%-32s N=%3d grid %3d %7.1f cycles/MMA  (floor %5.1f)  %s\n", what, N, grid, (double)h / kReps, floor_cyc,
            e == cudaSuccess ? "" : cudaGetErrorString(e));
     cudaFree(d);
 }
@@ -121,5 +142,15 @@ int main() {
     run<64, false, 0, 0, 0, 1, 1>("SS A rot, B over 40 K-steps");
     run<48, false, 0, 0, 0, 1, 1>("SS A rot, B over 40 K-steps");
     run<96, true, 0, 0, 0, 0, 1>("TS, B over 40 K-steps");
+    run<128, false, 0, 0, 0, 1, 1, 1>("SS A rot, B rot, 2 accumulators");
+    run<128, false, 0, 0, 0, 1, 1, 1>("SS A rot, B rot, 2 accumulators", 148);
+    run<128, false, 0, 0, 0, 1, 1, 0>("SS A rot, B rot", 148);
+    run<128, false, 0, 0, 0, 1, 1, 1, 16>("SS 2 acc, commit every 16");
+    run<128, false, 0, 0, 0, 1, 1, 1, 4>("SS 2 acc, commit every 4");
+    run<128, false, 0, 0, 0, 1, 1, 1, 1>("SS 2 acc, commit every MMA");
+    run<128, false, 0, 0, 0, 1, 1, 1, 0, 1>("per-16: elect+syncwarp+commit");
+    run<128, false, 0, 0, 0, 1, 1, 1, 0, 3>("per-16: + mbar wait");
+    run<128, false, 0, 0, 0, 1, 1, 1, 0, 5>("per-16: + fence");
+    run<128, false, 0, 0, 0, 1, 1, 1, 0, 7>("per-16: + wait + fence");
     return 0;
 }
