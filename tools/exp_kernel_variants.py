@@ -72,6 +72,16 @@ VARIANTS = {
     "u3_mma_only": ("cnn_tc.cu", VARIANTS_U3_NO_EPI + [
         ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
          "            if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n            __syncwarp();\n            if (false)")]),
+    # U3 3xFP16: the epilogue computes as built but never loads TMEM (values from a register)
+    "h3u3_no_tmemld": ("cnn_h3.cu", [
+        ("                tc::tmem_ld32_async(tmem + lane_base + col, v);\n                if (kFuse) {",
+         "#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = __int_as_float(col + u) * 1e-30f;\n                if (false) {"),
+        ("                } else {\n                    tc::tmem_wait_ld();\n                }\n#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(",
+         "                } else {\n                }\n#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(")]),
+    # U3 3xFP16: the epilogue without the 9 C6 FMA chains per channel
+    "h3u3_no_c6": ("cnn_h3.cu", [
+        ("#pragma unroll\n                    for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], v[u], c6[o]);",
+         "                    c6[u % 9] += v[u];")]),
 }
 
 
