@@ -257,31 +257,39 @@ __global__ void __launch_bounds__(128, 3)
         }
         const int64_t R2 = r2_0 + ty;
         const bool row_ok = R2 < a.t2_row0 + a.t2_rows;
+        // bias, tanh, the 2x2 subsample, tanh -- per channel PAIR, the same pair the FFMA2
+        // accumulators hold, with paired FP32 arithmetic (each lane rounds like the scalar ops, so
+        // the bits equal a per-channel loop)
         float tv[2][8];
 #pragma unroll
-        for (int ch = 0; ch < 8; ++ch) {
-            float4 b4[2];
-            if (kPlane) {
+        for (int cp = 0; cp < 4; ++cp) {
+            float4 b4[2][2];  // [channel parity][C1 row]
 #pragma unroll
-                for (int ra = 0; ra < 2; ++ra)
-                    b4[ra] = *reinterpret_cast<const float4*>(&bs[(ch * U1T_BR + 2 * ty + ra) * U1T_BC + 4 * tx]);
-            } else {
-                const float bv = __ldg(a.b1 + ch);
-                b4[0] = b4[1] = make_float4(bv, bv, bv, bv);
+            for (int e = 0; e < 2; ++e) {
+                const int ch = 2 * cp + e;
+                if (kPlane) {
+#pragma unroll
+                    for (int ra = 0; ra < 2; ++ra)
+                        b4[e][ra] = *reinterpret_cast<const float4*>(&bs[(ch * U1T_BR + 2 * ty + ra) * U1T_BC + 4 * tx]);
+                } else {
+                    const float bv = __ldg(a.b1 + ch);
+                    b4[e][0] = b4[e][1] = make_float4(bv, bv, bv, bv);
+                }
             }
 #pragma unroll
             for (int q = 0; q < 2; ++q) {
-                float s = 0.f;
+                float2 s = make_float2(0.f, 0.f);
 #pragma unroll
                 for (int p = 0; p < 4; ++p) {
                     const int ra = p >> 1, cb = 2 * q + (p & 1);
-                    const float4 bb = b4[ra];
-                    const float bias = cb == 0 ? bb.x : cb == 1 ? bb.y : cb == 2 ? bb.z : bb.w;
-                    const float av = (ch & 1) ? acc[ch >> 1][ra][cb].y : acc[ch >> 1][ra][cb].x;
-                    const float th = kBf16 ? tanh_mufu(av + bias) : tanh_f(av + bias);
-                    s = fmaf(w.p2[ch][p], th, s);
+                    auto pick = [&](const float4& bb) { return cb == 0 ? bb.x : cb == 1 ? bb.y : cb == 2 ? bb.z : bb.w; };
+                    const float2 av = __fadd2_rn(acc[cp][ra][cb], make_float2(pick(b4[0][ra]), pick(b4[1][ra])));
+                    const float2 th = kBf16 ? make_float2(tanh_mufu(av.x), tanh_mufu(av.y)) : tanh_fp32x2(av);
+                    s = __ffma2_rn(make_float2(w.p2[2 * cp][p], w.p2[2 * cp + 1][p]), th, s);
                 }
-                tv[q][ch] = kBf16 ? tanh_mufu(s) : tanh_f(s);
+                const float2 t = kBf16 ? make_float2(tanh_mufu(s.x), tanh_mufu(s.y)) : tanh_fp32x2(s);
+                tv[q][2 * cp] = t.x;
+                tv[q][2 * cp + 1] = t.y;
             }
         }
         __syncthreads();  // stage b is free for the prefetch issued in iteration k+1
