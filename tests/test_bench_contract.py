@@ -41,3 +41,24 @@ def test_recorded_line_has_the_contract_keys():
     for t in j["per_template"]:
         if t.get("verified") is not None:
             assert t["verified"]["ok"], t["template"]
+
+
+@pytest.mark.skipif(not os.path.exists(LINE) or "r02" not in LINE, reason="no round-2 bench line")
+def test_recorded_line_covers_every_config_and_measures_its_denominators():
+    """Round-2 contract additions: a line per BASELINE config, each verified against
+    the oracle in the run; the FP32 peak and the host link measured in the run; per-image output
+    digests; overlap and bytes computed like for like; the streamed roofline of SURVEY §8(d)."""
+    j = json.loads(open(LINE).read().strip().splitlines()[-1])
+    cfgs = {j["config"]["baseline_config"]} | {t["baseline_config"] for t in j["per_template"]}
+    assert {"configs[0]", "configs[1]", "configs[2]", "configs[3](a)", "configs[3](b)"} <= cfgs
+    assert j["verified"]["ok"] and all(t["verified"]["ok"] for t in j["per_template"])
+    mp = j["measured_peaks"]
+    assert 60 < mp["fp32_tflops"] <= mp["fp32_unit_count_tflops_at_1965"] * 1.01
+    assert j["roofline"]["peak"] == mp["fp32_tflops"]
+    assert set(mp["host_link_gbs"]) == {"h2d", "d2h", "bidir_each"}
+    assert j["checksum"]["digest_all"] == j["checksum"]["digest_first_share"]   # N = 1
+    e = j["e2e"]
+    assert 1.0 <= e["bytes_vs_lower_bound"] < 1.1
+    assert e["streamed_roofline"]["bound"] in ("link", "compute") and e["streamed_roofline"]["frac"] > 0.5
+    assert "uncapped" in e and e["uncapped"]["value"] > 0
+    assert j["clocks"]["samples"] >= 5

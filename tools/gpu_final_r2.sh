@@ -13,3 +13,7 @@ t0=$(date +%s); timeout 1500 python bench.py --steps 20 --warmup 5 > gpurun_out/
 t0=$(date +%s); timeout 900 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err; echo "ref rc=$? $(( $(date +%s) - t0 )) s"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"edge" --csv --log-file gpurun_out/launches_bench_edge256.csv python bench.py --template edge256 --steps 20 --warmup 3 --no-cpu --no-verify --per-template none > /dev/null 2>&1; echo "ncu edge256 rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_bf16_full -f python tools/prof_cnn.py 120 bf16 > gpurun_out/ncu_cnn_bf16.log 2>&1; echo "cnn bf16 rc=$?"
+for pr in fp32tc fp32; do
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_${pr}_full -f python tools/prof_cnn.py 120 $pr > gpurun_out/ncu_cnn_$pr.log 2>&1; echo "cnn $pr rc=$?"
+done
+TG_BENCH_DIST_BACKEND=gloo timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --no-verify --per-template edge256:fp32,cnn4:bf16_tc,cnn26:bf16_tc > gpurun_out/bench_2rank.json 2> gpurun_out/bench_2rank.err; echo "2rank rc=$?"
