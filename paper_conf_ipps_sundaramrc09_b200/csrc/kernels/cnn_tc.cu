@@ -161,15 +161,27 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding
             const uint64_t bdesc0 = tc::make_desc(tc::smem_u32(S.b), U2_N * 16, 128);
             const uint64_t adesc0 = tc::make_desc(tc::smem_u32(S.a[0]), 16, 128);  // 2nd K-half = next pixel
+            // the barriers of the NEXT segment are probed (mbarrier.test_wait) before the last MMAs
+            // of the current one: a barrier access waits ~150 cycles for the shared-memory port the
+            // MMA operand reads saturate, and overlaps the queued MMAs this way instead of stalling
+            // the issue between segments (blocking waits only after a failed probe;
+            // tools/micro/umma_probe.cu)
+            bool a_ready = false, t_ready = false;
             for (int64_t k = 0; k < my; ++k) {
                 const int buf = (int)(k % U2_NA), ts = (int)(k % U2_NT);
-                tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
-                if (k >= U2_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
+                if (!a_ready) tc::mbar_wait(&S.a_full[buf], (uint32_t)((k / U2_NA) & 1));
+                if (k >= U2_NT && !t_ready) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2_NT) / U2_NT) & 1));
                 tc::fence_after_sync();
                 const uint64_t abuf = adesc0 + (uint64_t)(buf * (U2_WR * U2_WP));
                 const uint32_t d0 = tmem + (uint32_t)(ts * 64);
+                const int64_t kn = k + 1;
 #pragma unroll
                 for (int ks = 0; ks < U2_KS; ++ks) {  // window row y = ks / 3, tap pair (j, j+1)
+                    if (ks == U2_KS - 4) {
+                        a_ready = kn < my && tc::mbar_test(&S.a_full[kn % U2_NA], (uint32_t)((kn / U2_NA) & 1));
+                        t_ready = kn >= U2_NT && kn < my &&
+                                  tc::mbar_test(&S.t_empty[kn % U2_NT], (uint32_t)(((kn - U2_NT) / U2_NT) & 1));
+                    }
                     const int y = ks / 3, j = 2 * (ks % 3);
                     tc::mma_bf16(d0, abuf + (uint64_t)(y * U2_WP + j), bdesc0 + (uint64_t)(ks * 2 * U2_N), idesc,
                                  ks > 0 ? 1u : 0u);
@@ -391,6 +403,13 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                                         b6desc0 + (uint64_t)(kk * 2 * U3_C6N), idesc6, kk > 0 ? 1u : 0u);
                 tc::commit(&S.c6_full[kb & 1]);
             };
+            // The barrier probes for the NEXT slice (and for a pending C6) are issued before the
+            // last MMAs of the current slice (mbarrier.test_wait, non-blocking): a barrier access
+            // waits ~150 cycles for the shared-memory port the MMAs' operand reads saturate, and
+            // so overlaps the queued MMAs instead of stalling the issue between slices (a blocking
+            // wait only follows when a probe failed; tools/micro/umma_probe.cu).
+            bool a_ready = false, t5_ready = false;
+            const int64_t total_s = my_bands * 5;
             for (int64_t k = 0; k < my_bands; ++k) {
                 const int buf = (int)(k & 1);
                 if (k >= 2) {
@@ -400,6 +419,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                         tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
                         tc::fence_after_sync();
                         issue_c6(c6_next++);
+                        t5_ready = false;
                     }
                     tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
                     tc::fence_after_sync();
@@ -408,7 +428,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                 for (int i = 0; i < 5; ++i) {
                     const int64_t s = k * 5 + i;
                     const int slot = (int)(s % U3_NA);
-                    tc::mbar_wait(&S.a_full[slot], (uint32_t)((s / U3_NA) & 1));
+                    if (!a_ready) tc::mbar_wait(&S.a_full[slot], (uint32_t)((s / U3_NA) & 1));
                     tc::fence_after_sync();
                     // descriptors once per slice; the 16 MMAs add constant offsets (16-byte units)
                     const uint32_t a_base = tc::smem_u32(S.a[slot][0]);
@@ -417,6 +437,12 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                     const uint64_t bd_i = bdesc0 + (uint64_t)(i * 8 * 2 * NP);
 #pragma unroll
                     for (int r8 = 0; r8 < 8; ++r8) {
+                        if (r8 == 6) {
+                            a_ready = s + 1 < total_s &&
+                                      tc::mbar_test(&S.a_full[(s + 1) % U3_NA], (uint32_t)(((s + 1) / U3_NA) & 1));
+                            if (c6_next < k && !t5_ready)
+                                t5_ready = tc::mbar_test(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                        }
                         // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0 and 1); r8 >= 5: channels
                         // 16-19 of taps (i, j) and (i, j+1), j = 2(r8-5) (block 2, next pixel)
                         const uint64_t ad = r8 < 5 ? ad_lo + (uint64_t)r8 : ad_hi + (uint64_t)(2 * (r8 - 5));
@@ -429,9 +455,10 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                     tc::commit(&S.a_empty[slot]);
                     if (i == 4) tc::commit(&S.t_full[buf]);
                     // the previous band's C6 as soon as its T5 is ready (between slices)
-                    if (c6_next < k && tc::mbar_test(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1))) {
+                    if (t5_ready) {
                         tc::fence_after_sync();
                         issue_c6(c6_next++);
+                        t5_ready = false;
                     }
                 }
             }

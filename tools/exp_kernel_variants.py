@@ -20,6 +20,17 @@ VARIANTS_U3_NO_EPI = [
      "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
     ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob")]
 
+
+U3_NO_C5 = [("                            tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,",
+             "                            if (r8 < 0) tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,")]
+U3_NO_BIAS = [("            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = __ldg(p);",
+               "            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = 0.f;")]
+U3_NO_TANH = [("for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[0][u]);", "for (int u = 0; u < 16; ++u) v[u] = v[u] + bv[0][u];"),
+              ("for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[1][u]);", "for (int u = 0; u < 16; ++u) v[u] = v[u] + bv[1][u];")]
+U3_NO_TMEMLD = [("                    tc::tmem_ld16_async(region + (uint32_t)(16 * c), v);\n                    tc::tmem_wait_ld();",
+                 "#pragma unroll\n                    for (int u = 0; u < 16; ++u) v[u] = __int_as_float(region + u) * 1e-30f;")]
+U3_NO_TMEMST = [("                    tc::tmem_st8(region + (uint32_t)(8 * c), r);", "                    if (r[0] == 12345u) tc::tmem_st8(region + (uint32_t)(8 * c), r);")]
+
 # variant -> (kernel source, [(old, new), ...]); every `old` must occur in the source
 VARIANTS = {
     "base": ("cnn_tc.cu", []),
@@ -68,6 +79,21 @@ VARIANTS = {
     "h3u3_2mma": ("cnn_h3.cu", [
         ("                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);\n                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);",
          "                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);")]),
+    # U3 bf16 epilogue decomposition: no C5 MMAs, then each epilogue step removed in turn
+    "u3e": ("cnn_tc.cu", U3_NO_C5),
+    "u3e_no_bias": ("cnn_tc.cu", U3_NO_C5 + U3_NO_BIAS),
+    "u3e_no_tanh": ("cnn_tc.cu", U3_NO_C5 + U3_NO_TANH),
+    "u3e_no_tmemld": ("cnn_tc.cu", U3_NO_C5 + U3_NO_TMEMLD),
+    "u3e_no_tmemst": ("cnn_tc.cu", U3_NO_C5 + U3_NO_TMEMST),
+    "u3e_no_bias_tanh": ("cnn_tc.cu", U3_NO_C5 + U3_NO_BIAS + U3_NO_TANH),
+    "u3e_bare": ("cnn_tc.cu", U3_NO_C5 + U3_NO_BIAS + U3_NO_TANH + U3_NO_TMEMLD + U3_NO_TMEMST),
+    "u3_mma_only_no_c6": ("cnn_tc.cu", VARIANTS_U3_NO_EPI + [
+        ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
+         "            if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n            __syncwarp();\n            if (false)"),
+        ("                        tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL)",
+         "                        if (kk < 0) tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL)")]),
+    # U3 bf16: copies but no epilogue work (the MMA + copy pipeline alone)
+    "u3_no_epi_work": ("cnn_tc.cu", VARIANTS_U3_NO_EPI),
     # U3 bf16: neither epilogue work nor slice copies (the MMA issue alone, plus C6)
     "u3_mma_only": ("cnn_tc.cu", VARIANTS_U3_NO_EPI + [
         ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
