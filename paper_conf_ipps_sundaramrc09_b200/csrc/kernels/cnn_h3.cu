@@ -19,9 +19,12 @@
 // The implicit GEMMs are those of the bf16 kernels (cnn_tc.cu): U2 pairs taps (j, j+1) in one
 // K = 16 step (15 K-steps per tile), U3 runs 8 K-steps per filter row (taps 0-4 over blocks 0-1,
 // then block 2 of tap pairs), 40 per tile.
-//   U2: N = 20 maps is A-read bound, so A_hi is read ONCE for both of its products:
-//       A_hi x [B_hi | B_lo] (N = 64) and A_lo x B_hi (N = 32) accumulated onto the cross-term
-//       columns; the epilogue adds the two 32-column halves.
+//   U2: as the bf16 U2, ONE M = 128 tile per segment serves both C3 rows (window row y feeds row
+//       2R with filter row y and row 2R+1 with filter row y - 1: N = 48, 18 K-steps of 6 window
+//       rows x 3 tap pairs), and A_hi is read ONCE for both of its products: A_hi x [B_hi | B_lo]
+//       (N = 96) and A_lo x B_hi (N = 48) accumulated onto the hi.hi columns; the epilogue adds
+//       the two 48-column halves. (Earlier: two tiles of 15 K-steps at N = 64 + 32, 2640 vs 1800
+//       shared-memory operand cycles per segment.)
 //   U3: three MMAs per K-step into one accumulator (N = n5 padded to 16), or for NP <= 64 the
 //       same read-once fusion as U2; the B operand (40 K-steps x 2 parts, up to 320 KB) streams
 //       through a ring of 32 KB stages.
@@ -85,13 +88,14 @@ float from_f16(uint16_t u) {
 }
 
 // ============================================================================ U2 (C3)
-// Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns: tile t = C3 row 2R + t. Window: T2
-// rows [2R, 2R+6) x cols [c0, c0+134) of both parts, [part][row][col] -> 8 fp16 channels.
+// Segment = T4 row R (C3 rows 2R, 2R+1) x 128 C3 columns, one M = 128 tile. Window: T2 rows
+// [2R, 2R+6) x cols [c0, c0+134) of both parts, [part][row][col] -> 8 fp16 channels.
 constexpr int U2H_WR = 6, U2H_WP = kTileM + 6;
-constexpr int U2H_N = 32;                  // 20 maps padded; B rows per K half = 2 x U2H_N
-constexpr int U2H_KS = 15;                 // 5 rows x tap pairs (0,1) (2,3) (4,5)
+constexpr int U2H_N = 48;                  // [0,20) row 2R, [24,44) row 2R+1; B rows per K half = 2 x U2H_N
+constexpr int U2H_ROW1 = 24;               // first column of C3 row 2R+1
+constexpr int U2H_KS = 18;                 // 6 window rows x tap pairs (0,1) (2,3) (4,5)
 constexpr int U2H_NA = 6;                  // window buffers
-constexpr int U2H_NT = 4;                  // TMEM slots (128 columns each)
+constexpr int U2H_NT = 4;                  // TMEM slots (128 columns apart, 2 x U2H_N used)
 constexpr int U2H_PLANE = U2H_WR * U2H_WP;
 constexpr int kThreads = 10 * 32;
 
@@ -101,7 +105,7 @@ struct U2HP {
 
 struct U2HSmem {
     uint4 a[U2H_NA][2][U2H_PLANE];           // [buf][part][row*WP + col] -> 8 fp16
-    uint4 b[U2H_KS * 2 * 2 * U2H_N];         // [ks][half][row < 64: hi maps, then lo] -> 8 fp16
+    uint4 b[U2H_KS * 2 * 2 * U2H_N];         // [ks][half][row < 96: hi columns, then lo] -> 8 fp16
     uint64_t b_full, a_full[U2H_NA], a_empty[U2H_NA], t_full[U2H_NT], t_empty[U2H_NT];
     uint32_t tmem;
 };
@@ -180,7 +184,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         // pipe idle, tools/micro/umma_probe.cu)
         if (tc::elect_one()) {
             tc::mbar_wait(&S.b_full, 0);
-            const uint32_t idesc64 = idesc_f16(kTileM, 2 * U2H_N), idesc32 = idesc_f16(kTileM, U2H_N);
+            const uint32_t idesc2n = idesc_f16(kTileM, 2 * U2H_N), idesc1n = idesc_f16(kTileM, U2H_N);
             // descriptors: the start address is the low 14 bits (16-byte units), advanced by adding;
             // A: the second K half is the next pixel (tap j+1, LBO = 16 B); B: LBO = one K half
             const uint64_t a_desc0 = tc::make_desc(tc::smem_u32(S.a[0][0]), 16, 128);
@@ -191,19 +195,16 @@ __global__ void __launch_bounds__(kThreads, 1)
                 if (k >= U2H_NT) tc::mbar_wait(&S.t_empty[ts], (uint32_t)(((k - U2H_NT) / U2H_NT) & 1));
                 tc::fence_after_sync();
                 const uint64_t abuf = a_desc0 + (uint64_t)(buf * (2 * U2H_PLANE));
-                const uint32_t d0 = tmem + (uint32_t)(ts * 4 * U2H_N);
+                const uint32_t d = tmem + (uint32_t)(ts * 128);
 #pragma unroll
-                for (int t = 0; t < 2; ++t) {  // tile t = C3 row 2R + t
-#pragma unroll
-                    for (int ks = 0; ks < U2H_KS; ++ks) {
-                        const int i = ks / 3, j = 2 * (ks % 3);
-                        const uint64_t a_hi = abuf + (uint64_t)((t + i) * U2H_WP + j);
-                        const uint64_t a_lo = a_hi + (uint64_t)U2H_PLANE;
-                        const uint64_t b_ks = b_desc0 + (uint64_t)(ks * 2 * 2 * U2H_N);  // rows 0..31 = B_hi
-                        const uint32_t d = d0 + (uint32_t)(t * 2 * U2H_N);
-                        tc::mma_bf16(d, a_hi, b_ks, idesc64, ks > 0 ? 1u : 0u);
-                        tc::mma_bf16(d + U2H_N, a_lo, b_ks, idesc32, 1u);
-                    }
+                for (int ks = 0; ks < U2H_KS; ++ks) {  // window row y = ks / 3, tap pair (j, j+1)
+                    const int y = ks / 3, j = 2 * (ks % 3);
+                    const uint64_t a_hi = abuf + (uint64_t)(y * U2H_WP + j);
+                    const uint64_t a_lo = a_hi + (uint64_t)U2H_PLANE;
+                    const uint64_t b_ks = b_desc0 + (uint64_t)(ks * 2 * 2 * U2H_N);  // rows 0..47 = B_hi
+                    // hi.hi -> [0, 48), hi.lo -> [48, 96); lo.hi accumulates onto hi.hi
+                    tc::mma_bf16(d, a_hi, b_ks, idesc2n, ks > 0 ? 1u : 0u);
+                    tc::mma_bf16(d, a_lo, b_ks, idesc1n, 1u);
                 }
                 tc::commit(&S.a_empty[buf]);
                 tc::commit(&S.t_full[ts]);
@@ -240,29 +241,23 @@ __global__ void __launch_bounds__(kThreads, 1)
             tc::fence_after_sync();
             float v0[20], v1[20];
             {
-                // per tile: columns [0, 32) hi.hi and [32, 64) hi.lo + lo.hi, 20 maps used
-                const uint32_t tb = tmem + lane_base + (uint32_t)(ts * 4 * U2H_N);
-                float p[16], q[16];
-                tc::tmem_ld16_async(tb, p);
-                tc::tmem_ld16_async(tb + U2H_N, q);
+                // columns [0, 48) hi.hi + lo.hi, [48, 96) hi.lo; C3 row 2R at column co, row 2R+1
+                // at U2H_ROW1 + co (20 maps each)
+                const uint32_t tb = tmem + lane_base + (uint32_t)(ts * 128);
+                float p[32], q[32];
+                tc::tmem_ld32_async(tb, p);           // [0, 32)
+                tc::tmem_ld32_async(tb + U2H_N, q);   // [48, 80)
                 tc::tmem_wait_ld();
 #pragma unroll
-                for (int co = 0; co < 16; ++co) v0[co] = (p[co] + q[co]) * a.w_unscale;
-                tc::tmem_ld16_async(tb + 16, p);
-                tc::tmem_ld16_async(tb + U2H_N + 16, q);
+                for (int co = 0; co < 20; ++co) v0[co] = (p[co] + q[co]) * a.w_unscale;
+#pragma unroll
+                for (int co = 0; co < 8; ++co) v1[co] = (p[U2H_ROW1 + co] + q[U2H_ROW1 + co]) * a.w_unscale;
+                float p2[16], q2[16];
+                tc::tmem_ld16_async(tb + 32, p2);           // [32, 48)
+                tc::tmem_ld16_async(tb + U2H_N + 32, q2);   // [80, 96)
                 tc::tmem_wait_ld();
 #pragma unroll
-                for (int co = 16; co < 20; ++co) v0[co] = (p[co - 16] + q[co - 16]) * a.w_unscale;
-                tc::tmem_ld16_async(tb + 2 * U2H_N, p);
-                tc::tmem_ld16_async(tb + 3 * U2H_N, q);
-                tc::tmem_wait_ld();
-#pragma unroll
-                for (int co = 0; co < 16; ++co) v1[co] = (p[co] + q[co]) * a.w_unscale;
-                tc::tmem_ld16_async(tb + 2 * U2H_N + 16, p);
-                tc::tmem_ld16_async(tb + 3 * U2H_N + 16, q);
-                tc::tmem_wait_ld();
-#pragma unroll
-                for (int co = 16; co < 20; ++co) v1[co] = (p[co - 16] + q[co - 16]) * a.w_unscale;
+                for (int co = 8; co < 20; ++co) v1[co] = (p2[U2H_ROW1 + co - 32] + q2[U2H_ROW1 + co - 32]) * a.w_unscale;
             }
             tc::fence_before_sync();
             __syncwarp();
@@ -573,9 +568,10 @@ __global__ void __launch_bounds__(kThreads, 1)
 
 }  // namespace
 
-// B operand of the 3xFP16 C3: [ks < 15][half][row < 64][8] fp16, K-step ks = filter row
-// i = ks / 3, taps j0 = 2 (ks % 3) + half (tap 5 = zero); row n < 32: hi of map n, row 32 + n:
-// lo of map n, of w * 2^8 with w = K3[n][e][i][j]; maps 20..31 zero.
+// B operand of the 3xFP16 C3: [ks < 18][half][row < 96][8] fp16, K-step ks = window row y = ks / 3,
+// taps j = 2 (ks % 3) + half (tap 5 = zero); column n < 48 as the bf16 C3 (cnn_prepare_k3_tc: n < 20
+// = map n with filter row y, 24 <= n < 44 = map n - 24 with filter row y - 1, zero where the filter
+// row is outside 0..4) holds the hi part, row 48 + n the lo part, of w * scale.
 size_t cnn_k3_h3_bytes() { return (size_t)U2H_KS * 2 * 2 * U2H_N * 8 * 2; }
 float cnn_h3_act_scale() { return kActScale; }
 float cnn_h3_weight_scale(const float* w, size_t n) {
@@ -590,12 +586,14 @@ float cnn_h3_weight_scale(const float* w, size_t n) {
 void cnn_prepare_k3_h3(const float* k3, float scale, uint16_t* dst) {
     std::memset(dst, 0, cnn_k3_h3_bytes());
     for (int ks = 0; ks < U2H_KS; ++ks) {
-        const int i = ks / 3, j0 = 2 * (ks % 3);
+        const int y = ks / 3, j0 = 2 * (ks % 3);
         for (int h = 0; h < 2; ++h)
-            for (int n = 0; n < 20; ++n)
+            for (int n = 0; n < U2H_N; ++n)
                 for (int e = 0; e < 8; ++e) {
                     const int j = j0 + h;
-                    const float w = j < 5 ? k3[(n * 8 + e) * 25 + i * 5 + j] * scale : 0.f;
+                    const int t = n >= U2H_ROW1 ? 1 : 0, map = n - t * U2H_ROW1, i = y - t;
+                    const bool ok = map < 20 && j < 5 && i >= 0 && i < 5;
+                    const float w = ok ? k3[(map * 8 + e) * 25 + i * 5 + j] * scale : 0.f;
                     const uint16_t hi = to_f16(w);
                     dst[(((size_t)ks * 2 + h) * 2 * U2H_N + n) * 8 + e] = hi;
                     dst[(((size_t)ks * 2 + h) * 2 * U2H_N + U2H_N + n) * 8 + e] = to_f16(w - from_f16(hi));
