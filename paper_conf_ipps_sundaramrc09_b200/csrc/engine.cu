@@ -468,10 +468,14 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
     // S1 are serialised, so no chunk waits for a slot of an earlier execution)
     // A direct execution after a graph replay does the same: the slot events were last recorded
     // inside the capture, so they neither order against the replays nor may be waited on.
+    // A device-resident plan moves no data on the copy streams (only a parameter upload on S0), so
+    // it forks them only for that upload and never joins them: its captured graph is then just the
+    // kernels on S1 (configs[0]: fewer graph nodes, less launch overhead per step).
     const bool fresh = capturing || d.after_graph;
     d.after_graph = false;
-    CK(cudaEventRecord(d.ev_fork, S1));
-    if (c.device_io || !d.params_resident || fresh) {
+    const bool fork = c.device_io ? !d.params_resident : (!d.params_resident || fresh);
+    if (fork) {
+        CK(cudaEventRecord(d.ev_fork, S1));
         CK(cudaStreamWaitEvent(S0, d.ev_fork, 0));
         CK(cudaStreamWaitEvent(S2, d.ev_fork, 0));
     }
@@ -549,8 +553,12 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
         }
     }
     // join: the compute stream waits for the last D2H, so it marks the end of everything
-    CK(cudaEventRecord(d.ev_join, S2));
-    CK(cudaStreamWaitEvent(S1, d.ev_join, 0));
+    // (device-resident I/O: nothing ran on the copy streams but a parameter upload, which S1
+    // already waited for through ev_params)
+    if (!c.device_io) {
+        CK(cudaEventRecord(d.ev_join, S2));
+        CK(cudaStreamWaitEvent(S1, d.ev_join, 0));
+    }
     if (ordered) {
         CK(cudaEventRecord(d.ev_done, S1));
         CK(cudaStreamWaitEvent(caller, d.ev_done, 0));

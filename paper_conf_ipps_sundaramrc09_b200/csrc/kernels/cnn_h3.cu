@@ -17,8 +17,8 @@
 //   T2 [part][rows][w2][8 ch]          part 0 = hi, 1 = lo (16 B per pixel per part)
 //   T4 [part][block][rows][w4][8 ch]   blocks: channels 0-7, 8-15, 16-19 + 4 zeros
 // The implicit GEMMs are those of the bf16 kernels (cnn_tc.cu): U2 pairs taps (j, j+1) in one
-// K = 16 step (15 K-steps per tile), U3 runs 8 K-steps per filter row (taps 0-4 over blocks 0-1,
-// then block 2 of tap pairs), 40 per tile.
+// K = 16 step (18 K-steps per segment: 6 window rows x 3 tap pairs, both C3 rows in N), U3 runs
+// 8 K-steps per filter row (taps 0-4 over blocks 0-1, then block 2 of tap pairs), 40 per tile.
 //   U2: as the bf16 U2, ONE M = 128 tile per segment serves both C3 rows (window row y feeds row
 //       2R with filter row y and row 2R+1 with filter row y - 1: N = 48, 18 K-steps of 6 window
 //       rows x 3 tap pairs), and A_hi is read ONCE for both of its products: A_hi x [B_hi | B_lo]

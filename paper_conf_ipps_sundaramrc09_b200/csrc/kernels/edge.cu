@@ -45,32 +45,39 @@
 namespace tg {
 namespace {
 
-// Tile geometry per strip width kQ (outputs per thread, one row of kQ columns):
-//   kQ = 16: 64 x 64 output tiles, 8 warps = 2 row groups x 4 column strips (the main path);
-//   kQ = 4:  32 x 32 output tiles, 8 warps = 8 column strips of one 32-row group -- for images
-//            with fewer 64 x 64 tiles than SMs (configs[0], 256 x 256: 16 big tiles would leave
-//            132 SMs idle and make each thread's 4096 serial FFMA2 the latency; 64 small tiles with
-//            1024 each finish ~4x sooner).
+// Tile geometries kG (Q = outputs per thread, one row of Q columns):
+//   kG = 16: 64 x 64 output tiles, 8 warps = 2 row groups x 4 column strips, Q = 16 (the main path);
+//   kG = 4:  32 x 32 output tiles, 8 warps = 8 column strips of one 32-row group, Q = 4 -- for images
+//            with fewer 64 x 64 tiles than SMs (16 big tiles of a 256 x 256 image would leave 132
+//            SMs idle and make each thread's 4096 serial FFMA2 the latency);
+//   kG = 5:  16 x 32 output tiles, 4 warps (lanes 0-15 / 16-31 = two column strips of the same 16
+//            rows), Q = 4 -- when even the 32 x 32 tiles are fewer than the SMs (configs[0]: 128
+//            tiles of 16 x 32 on 148 SMs, one warp per SM sub-partition, instead of 64 of 32 x 32).
 // Row pitch in shared memory: an odd number of 16-byte units, so the 8 lanes of each LDS.128
 // phase (lanes = consecutive rows) hit 8 distinct bank groups.
-template <int kQ> struct Geo;
+template <int kG> struct Geo;
 template <> struct Geo<16> {
-    static constexpr int R = 64, C = 64, Pitch = 84;  // 84 / 4 = 21
+    static constexpr int R = 64, C = 64, Pitch = 84, Q = 16, Threads = 256;  // 84 / 4 = 21
     __device__ static int lr(int warp, int lane) { return (warp >> 2) * 32 + lane; }
-    __device__ static int cb(int warp) { return (warp & 3) * 16; }
+    __device__ static int cb(int warp, int) { return (warp & 3) * 16; }
 };
 template <> struct Geo<4> {
-    static constexpr int R = 32, C = 32, Pitch = 52;  // 52 / 4 = 13
+    static constexpr int R = 32, C = 32, Pitch = 52, Q = 4, Threads = 256;  // 52 / 4 = 13
     __device__ static int lr(int, int lane) { return lane; }
-    __device__ static int cb(int warp) { return warp * 4; }
+    __device__ static int cb(int warp, int) { return warp * 4; }
 };
-template <int kQ> struct GeoT : Geo<kQ> {
-    static constexpr int SmR = Geo<kQ>::R + 15;                  // rows incl. halo
-    static constexpr int SmC = Geo<kQ>::C + 16;                  // cols used: [c0-8, c0+C+8)
-    static constexpr int TileBytes = SmR * Geo<kQ>::Pitch * 4;   // one TMA box
+template <> struct Geo<5> {
+    static constexpr int R = 16, C = 32, Pitch = 52, Q = 4, Threads = 128;  // 52 / 4 = 13
+    __device__ static int lr(int, int lane) { return lane & 15; }
+    __device__ static int cb(int warp, int lane) { return (2 * warp + (lane >> 4)) * 4; }
+};
+template <int kG> struct GeoT : Geo<kG> {
+    static constexpr int SmR = Geo<kG>::R + 15;                  // rows incl. halo
+    static constexpr int SmC = Geo<kG>::C + 16;                  // cols used: [c0-8, c0+C+8)
+    static constexpr int TileBytes = SmR * Geo<kG>::Pitch * 4;   // one TMA box
     static constexpr int BufStride = (TileBytes + 127) / 128 * 128;
 };
-constexpr int kThreads = 256;
+constexpr int kThreads = 256;  // the fallback kernel (geometry 16)
 
 // Both filters, embedded in 16 x 16 frames, travel as a __grid_constant__ kernel parameter:
 // the weights then sit in the constant bank and every FFMA reads them through a uniform
@@ -82,14 +89,14 @@ struct EdgeWeights {
 
 // Compute the output tile whose input (+halo) is staged at xs (row pitch Geo<kQ>::Pitch; smem
 // (sr, sc) <-> image (tile_r0 - 7 + sr, tile_c0 - 8 + sc)) and store it.
-template <int kComb, int kPairs, int kF, int kQ>
+template <int kComb, int kPairs, int kF, int kG>
 __device__ __forceinline__ void edge_tile(const float* __restrict__ xs, const EdgeArgs& a, const EdgeWeights& wt,
                                           int64_t img, int64_t tile_r0, int64_t tile_c0) {
-    constexpr int kPitch = Geo<kQ>::Pitch;
+    constexpr int kPitch = Geo<kG>::Pitch, kQ = Geo<kG>::Q;
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
-    const int lr = Geo<kQ>::lr(warp, lane);  // local output row
-    const int cb = Geo<kQ>::cb(warp);        // local output column base
+    const int lr = Geo<kG>::lr(warp, lane);     // local output row
+    const int cb = Geo<kG>::cb(warp, lane);     // local output column base
 
     // Paired FP32 FMA (FFMA2, sm_100) over a PAIR OF FILTERS: acc[q] = (E_2p[q], E_2p+1[q]) +=
     // x[q+j+1] (register, broadcast to both lanes) * (K_2p[i][j], K_2p+1[i][j]) (uniform-register
@@ -216,12 +223,12 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-template <int kComb, int kPairs, int kF, int kQ>
-__global__ void __launch_bounds__(kThreads, 2)
+template <int kComb, int kPairs, int kF, int kG>
+__global__ void __launch_bounds__(Geo<kG>::Threads, 2)
     edge_fused_tma_kernel(const __grid_constant__ CUtensorMap tmap, const EdgeArgs a,
                           const __grid_constant__ EdgeWeights wt, const int tiles_c, const int tiles_r,
                           const int64_t ntiles) {
-    using G = GeoT<kQ>;
+    using G = GeoT<kG>;
     constexpr int kTileR = G::R, kTileC = G::C, kTileBytes = G::TileBytes, kBufStride = G::BufStride;
     // (the tensor map must sit in the first 4 KB of the parameter space, hence first)
     extern __shared__ __align__(128) uint8_t smraw[];
@@ -281,7 +288,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         int64_t img, tr0, tc0;
         coords(t, img, tr0, tc0);
         const float* tb = b ? buf1 : buf0;
-        edge_tile<kComb, kPairs, kF, kQ>(tb, a, wt, img, tr0, tc0);
+        edge_tile<kComb, kPairs, kF, kG>(tb, a, wt, img, tr0, tc0);
         __syncthreads();  // buffer b is free for the prefetch issued in iteration k+1
     }
 }
@@ -327,12 +334,12 @@ cudaError_t launch_edge(const EdgeArgs& a, cudaStream_t s) {
     return launch_edge_f<16>(a, s);
 }
 
-// The TMA path at strip width kQ; cudaErrorNotSupported when the tensor map cannot be encoded
+// The TMA path in tile geometry kG; cudaErrorNotSupported when the tensor map cannot be encoded
 // (the caller then takes the bounds-checked fallback kernel).
-template <int kComb, int kPairs, int kF, int kQ>
+template <int kComb, int kPairs, int kF, int kG>
 cudaError_t launch_edge_tma(const EdgeArgs& a, const EdgeWeights& wt, PFN_cuTensorMapEncodeTiled_v12000 enc, int dev,
                             int sms, cudaStream_t s) {
-    using G = GeoT<kQ>;
+    using G = GeoT<kG>;
     const int tiles_c = (int)((a.W + G::C - 1) / G::C);
     const int tiles_r = (int)((a.out_rows + G::R - 1) / G::R);
     CUtensorMap tmap;
@@ -347,7 +354,7 @@ cudaError_t launch_edge_tma(const EdgeArgs& a, const EdgeWeights& wt, PFN_cuTens
     static std::atomic<uint32_t> configured{0};
     const size_t smem = 2 * (size_t)G::BufStride + 128;
     if (!(configured.load() & (1u << (dev & 31)))) {
-        cudaError_t e = cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs, kF, kQ>,
+        cudaError_t e = cudaFuncSetAttribute(edge_fused_tma_kernel<kComb, kPairs, kF, kG>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         configured.fetch_or(1u << (dev & 31));
@@ -358,7 +365,7 @@ cudaError_t launch_edge_tma(const EdgeArgs& a, const EdgeWeights& wt, PFN_cuTens
     // the remaining ones, which balances the tail of the static tile walk -- 2 per SM
     // (exactly resident) ran at 0.918 of the FP32 peak, 8 at 0.936, 32 at 0.941
     const int64_t grid = std::min<int64_t>(ntiles, 32 * (int64_t)sms);
-    edge_fused_tma_kernel<kComb, kPairs, kF, kQ><<<(unsigned)grid, kThreads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
+    edge_fused_tma_kernel<kComb, kPairs, kF, kG><<<(unsigned)grid, G::Threads, smem, s>>>(tmap, a, wt, tiles_c, tiles_r, ntiles);
     return cudaGetLastError();
 }
 
@@ -382,10 +389,12 @@ cudaError_t launch_edge_t(const EdgeArgs& a, cudaStream_t s) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int64_t big_tiles = ((a.W + 63) / 64) * ((a.out_rows + 63) / 64) * a.nimg;
+    const int64_t mid_tiles = ((a.W + 31) / 32) * ((a.out_rows + 31) / 32) * a.nimg;
     if (tma_ok) {
-        // small tiles (kQ = 4) when the big ones cannot occupy every SM
-        cudaError_t e = big_tiles < sms ? launch_edge_tma<kComb, kPairs, kF, 4>(a, wt, enc, dev, sms, s)
-                                        : launch_edge_tma<kComb, kPairs, kF, 16>(a, wt, enc, dev, sms, s);
+        // smaller tiles when the big ones cannot occupy every SM
+        cudaError_t e = big_tiles >= sms   ? launch_edge_tma<kComb, kPairs, kF, 16>(a, wt, enc, dev, sms, s)
+                        : mid_tiles >= sms ? launch_edge_tma<kComb, kPairs, kF, 4>(a, wt, enc, dev, sms, s)
+                                           : launch_edge_tma<kComb, kPairs, kF, 5>(a, wt, enc, dev, sms, s);
         if (e != cudaErrorNotSupported) return e;
     }
     using G = GeoT<16>;

@@ -4,6 +4,7 @@
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/micro/pipe_probe tools/micro/pipe_probe.cu
 #include <cstdio>
 #include <cstdint>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 constexpr int kIters = 4096;
@@ -21,7 +22,10 @@ __global__ void probe(long long* cyc, float* sink) {
         for (int j = 0; j < 8; ++j) {
             if (kOp == 0) asm volatile("tanh.approx.f32 %0, %0;" : "+f"(v[j]));
             if (kOp == 1) asm volatile("ex2.approx.ftz.f32 %0, %0;" : "+f"(v[j]));
-            if (kOp == 2) asm volatile("rcp.approx.ftz.f32 %0, %0;" : "+f"(v[j]));
+            if (kOp == 2) {  // rcp chain with a dependency the compiler cannot fold
+                asm volatile("rcp.approx.ftz.f32 %0, %0;" : "+f"(v[j]));
+                v[j] += 1.0f;
+            }
             if (kOp == 3) {  // pack two floats to bf16x2, feed the bits back as a float
                 uint32_t r;
                 asm volatile("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(v[j]), "f"(v[(j + 1) & 7]));
@@ -33,6 +37,15 @@ __global__ void probe(long long* cyc, float* sink) {
                 x = __ffma2_rn(x, x, x);
                 v[j] = x.x; v[(j + 4) & 7] = x.y;
             }
+            if (kOp == 7) {  // HFMA2: two fp16 FMAs per lane
+                __half2 h = __floats2half2_rn(v[j], v[(j + 4) & 7]);
+                asm volatile("fma.rn.f16x2 %0, %0, %0, %0;" : "+r"(*reinterpret_cast<uint32_t*>(&h)));
+                const float2 f = __half22float2(h);
+                v[j] = f.x;
+            }
+            if (kOp == 8) {  // HFMA2 chain kept in half2 registers (the conversion outside the loop)
+                asm volatile("fma.rn.f16x2 %0, %0, %0, %0;" : "+r"(u[j]));
+            }
             if (kOp == 6) {  // integer bf16 rounding + pack (alu/fma pipes): the F2FP alternative
                 const uint32_t a0 = __float_as_uint(v[j]), a1 = __float_as_uint(v[(j + 1) & 7]);
                 const uint32_t r0 = a0 + 0x7fffu + ((a0 >> 16) & 1u), r1 = a1 + 0x7fffu + ((a1 >> 16) & 1u);
@@ -43,7 +56,7 @@ __global__ void probe(long long* cyc, float* sink) {
     const long long t1 = clock64();
     float s = 0.f;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) s += v[j];
+    for (int j = 0; j < 8; ++j) s += v[j] + __uint_as_float(u[j]);
     if (s == 1.2345f) sink[threadIdx.x] = s;
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
@@ -73,5 +86,6 @@ int main() {
     run<4>("FFMA", 1);
     run<5>("FFMA2 (lanes)", 2);
     run<6>("int bf16 round+pack (values packed)", 2);
+    run<8>("HFMA2 (lanes x 2)", 2);
     return 0;
 }
