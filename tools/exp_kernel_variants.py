@@ -104,6 +104,10 @@ VARIANTS = {
          "#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = __int_as_float(col + u) * 1e-30f;\n                if (false) {"),
         ("                } else {\n                    tc::tmem_wait_ld();\n                }\n#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(",
          "                } else {\n                }\n#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(")]),
+    # U3 3xFP16: no bias-plane loads (bias 0)
+    "h3u3_no_bias": ("cnn_h3.cu", [
+        ("                for (int u = 0; u < 32; ++u, p += bcs) bv[u] = __ldg(p);\n            } else {",
+         "                for (int u = 0; u < 32; ++u, p += bcs) bv[u] = 0.f;\n            } else {")]),
     # U3 3xFP16: the epilogue without the 9 C6 FMA chains per channel
     "h3u3_no_c6": ("cnn_h3.cu", [
         ("#pragma unroll\n                    for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], v[u], c6[o]);",
