@@ -390,6 +390,12 @@ def time_steps(fn, stream, steps, flush=None):
     return sum(a.elapsed_time(b) for a, b in evs) / steps
 
 
+def repeats_summary(values, steps_each):
+    """Five repeats of a timed measurement: the values, their median and best."""
+    return {"n": len(values), "steps_each": steps_each, "values": values,
+            "median": statistics.median(values), "best": max(values)}
+
+
 def auto_steps(fn, stream, floor_steps, min_s):
     """Enough steps for a timed region of at least min_s seconds (clock evidence, stability)."""
     import torch
@@ -466,9 +472,17 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
     ms_prof = time_steps(run_dev, cs, steps, flush)
     tim = p.timing()
     p.profiling(False)
+    px_all = sum(gather_objects(px, world))
+    # SURVEY §8(d) "five repeats: median and best": 5 more graph-replay runs of steps / 5 steps each
+    p.use_graph(True)
+    p.execute()   # (re-)capture the graph outside the timed repeats
+    rep_each = max(1, steps // 5)
+    value_repeats = repeats_summary([px_all / (max_over_ranks(time_steps(run_dev, cs, rep_each, flush), world) / 1e3)
+                                     / 1e6 for _ in range(5)], rep_each)
+    p.use_graph(False)
     del flush
     ms_max = max_over_ranks(ms, world)
-    value = sum(gather_objects(px, world)) / (ms_max / 1e3) / 1e6
+    value = px_all / (ms_max / 1e3) / 1e6
 
     # ---- roofline of the dominant kernel and of every unit
     peaks = measured_peaks()
@@ -568,6 +582,12 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
             wall = (time.perf_counter() - t0) / n_steps * 1e3
         res = {"ms": ms2, "wall_ms": wall, "steps": n_steps, "launches": p2.launches() - l2, "stats": st,
                "json": js, "clocks": clk.summary()}
+        if profile:   # SURVEY §8(d) "five repeats: median and best": 5 more timed runs of n_steps / 5 steps
+            each = max(1, n_steps // 5)
+            p2.execute()
+            res["repeats_ms"] = [max_over_ranks(time_steps(lambda: p2.execute(blocking=False), cs2, each), world)
+                                 for _ in range(5)]
+            res["repeat_steps"] = each
         if profile and st["n_chunks"] <= js["depth"]:
             # a plan of at most `depth` chunks has no copy/compute overlap within an execution:
             # also time it as one CUDA-graph replay per step (tg_plan_set_graph; executions then
@@ -646,6 +666,8 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
                          "peak_bidir_each_gbs": link["bidir_each"],
                          "achieved_h2d_gbs": (h2d / 1e9) / (cap["ms"] / 1e3),
                          "achieved_d2h_gbs": (d2h / 1e9) / (cap["ms"] / 1e3)}}
+    if "repeats_ms" in cap:
+        e2e["repeats"] = repeats_summary([px_glob / (r / 1e3) / 1e6 for r in cap["repeats_ms"]], cap["repeat_steps"])
     if "graph_ms" in cap:
         e2e["graph_replay"] = {"value": px_glob / (cap["graph_ms"] / 1e3) / 1e6, "ms_per_step": cap["graph_ms"],
                                "what": "the same e2e step replayed as one captured CUDA graph (tg_plan_set_graph)"}
@@ -699,7 +721,8 @@ def run_line(args, ctx, wl_name: str, precision: str, headline: bool) -> dict:
                                                               else ": L2 flushed (512 MB write) before every "
                                                                    "device-resident timed step")}
     config = config_of(wl, precision, world) | l2
-    return {"value": value, "ms_per_step": ms_max, "steps": steps, "clocks": merge_clocks(*clocks),
+    return {"value": value, "value_repeats": value_repeats, "ms_per_step": ms_max, "steps": steps,
+            "clocks": merge_clocks(*clocks),
             "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "config": config, "checksum": checksum,
             "verified": verified, "y_host": y_host if (headline and rank == 0) else None}
 
@@ -890,6 +913,7 @@ def main():
                 "dtype": {"fp32": "f32", "bf16_tc": "bf16 (fp32 accumulate)",
                           "fp32_tc": "f32 (3xFP16 tensor cores, fp32 accumulate)"}[args.precision],
                 "data": "synthetic (counter-based generator synth/, 8-bit levels k/255)",
+                "value_repeats": res["value_repeats"],
                 "config": res["config"], "roofline": res["roofline"], "e2e": res["e2e"], "clocks": res["clocks"],
                 "gpu_launches": res["gpu_launches"], "checksum": res["checksum"], "verified": res["verified"],
                 "measured_peaks": {"fp32_tflops": fp32_peak, "fp32_probe_clocks": ctx["fp32_probe_clocks"],
@@ -914,10 +938,11 @@ def main():
         if rank == 0:
             ent = {"template": name, "baseline_config": r2["config"]["baseline_config"], "precision": pr,
                    "steps": r2["steps"], "workload": r2["config"]["workload"], "value": r2["value"],
+                   "value_repeats": r2["value_repeats"],
                    "unit": "Mpixels/s", "ms_per_step": r2["ms_per_step"],
                    "e2e": {k: r2["e2e"].get(k) for k in ("value", "ms_per_step", "steps", "h2d_bytes_per_step",
                                                          "d2h_bytes_per_step", "bytes_vs_lower_bound", "overlap",
-                                                         "chunks", "split", "bias", "uncapped")}
+                                                         "chunks", "split", "bias", "uncapped", "repeats")}
                    | {"streamed_roofline_frac": r2["e2e"]["streamed_roofline"]["frac"],
                       "link_ms": r2["e2e"]["streamed_roofline"]["link_ms"],
                       "streamed_roofline_bound": r2["e2e"]["streamed_roofline"]["bound"]},
