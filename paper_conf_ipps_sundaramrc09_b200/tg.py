@@ -495,7 +495,8 @@ class Graph:
         self.device_io = False
 
     def __del__(self):
-        if getattr(self, "h", None):
+        # (at interpreter exit the module's functions may already be torn down)
+        if getattr(self, "h", None) and callable(tg_graph_destroy):
             tg_graph_destroy(self.h)
             self.h = None
 
@@ -572,7 +573,7 @@ class Plan:
         self.h = h
 
     def __del__(self):
-        if getattr(self, "h", None):
+        if getattr(self, "h", None) and callable(tg_plan_destroy):
             tg_plan_destroy(self.h)
             self.h = None
 

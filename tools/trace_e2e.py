@@ -24,13 +24,12 @@ ap.add_argument("--tag", default="")
 ap.add_argument("--n", type=int, default=None, help="override the number of images")
 a = ap.parse_args()
 torch.cuda.set_device(0)
-wl = bench.workload(a.template, 0)
+wl = bench.workload(a.template)
 n, H, W = a.n or wl["n"], wl["H"], wl["W"]
+params = bench.params_of(wl)
 if wl["template"] == "edge":
-    params = [synth.edge_filter_np()[0]]
     out_shape = (n, 1, H, W)
 else:
-    params = synth.cnn_params_np(wl["seed"], wl["n5"], H, W)
     out_shape = (n, 9) + tuple(synth.cnn_dims(H, W)[4])
 if a.device:
     x = synth.images_torch(wl["seed"], n, H, W, "cuda")
@@ -39,10 +38,11 @@ else:
     x = torch.empty((n, 1, H, W), dtype=torch.float32).pin_memory()
     x.copy_(synth.images_torch(wl["seed"], n, H, W, "cuda").cpu())
     y = torch.empty(out_shape, dtype=torch.float32).pin_memory()
-g = bench.build_graph(tg, wl, x, y, a.device, params)
-g.set(budget=0 if a.device else wl["budget"], torch_runtime=True,
-      precision={"fp32": tg.TG_FP32, "fp32_tc": tg.TG_FP32_TC, "bf16_tc": tg.TG_BF16_TC}[a.precision],
-      max_chunk_px=a.max_chunk_px, depth=a.depth)
+g = bench.make_graph(tg, wl, n, x.data_ptr(), y.data_ptr(), a.device, params,
+                     budget=0 if a.device else wl["budget"],
+                     prec={"fp32": tg.TG_FP32, "fp32_tc": tg.TG_FP32_TC, "bf16_tc": tg.TG_BF16_TC}[a.precision],
+                     chunking={"max_chunk_px": a.max_chunk_px, "depth": a.depth})
+g._keep += [x, y]
 p = g.plan()
 for _ in range(3):
     p.execute()
