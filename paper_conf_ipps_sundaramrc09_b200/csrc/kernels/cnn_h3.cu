@@ -415,56 +415,62 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (tc::elect_one()) {
             const uint32_t idesc = idesc_f16(kTileM, NP), idesc2 = idesc_f16(kTileM, 2 * NP);
             const uint32_t plane_bytes = (uint32_t)(U3H_SPX * 16), part_bytes = 3 * plane_bytes;
+            // Descriptors are built once per slice / B stage and advanced by constant offsets (the
+            // start address is the descriptor's low field, in 16-byte units): with the K-step loop
+            // unrolled per stage, the issuing thread spends a few uniform adds per MMA instead of
+            // rebuilding four descriptors per tile and K-step (which left it barely ahead of the pipe)
+            static_assert(U3H_KST == 4 && 8 % U3H_KST == 0, "two B stages per slice");
+            const uint64_t b_step = (uint64_t)(2 * 2 * NP);       // one K-step of B, 16-byte units
+            const uint64_t b_part = (uint64_t)(2 * NP);           // B_lo after B_hi (NP > 64 layout)
+            const uint64_t a_part = (uint64_t)(part_bytes >> 4);  // A_lo after A_hi
             int64_t si = 0, gi = 0;
             for (int64_t k = 0; k < my_bands; ++k) {
                 const int buf = (int)(k & 1);
                 if (k >= 2) tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
                 const uint32_t d_base = tmem + (uint32_t)(buf * 256);
-                uint32_t a_base = 0, b_base = 0;
-                int aslot = 0, bslot = 0;
-                for (int ks = 0; ks < U3H_KS; ++ks) {
-                    if (ks % 8 == 0) {
-                        aslot = (int)(si % U3H_NA);
-                        tc::mbar_wait(&S.a_full[aslot], (uint32_t)((si / U3H_NA) & 1));
-                        a_base = tc::smem_u32(S.a[aslot][0][0]);
-                        ++si;
-                    }
-                    if (ks % U3H_KST == 0) {
-                        bslot = (int)(gi % U3H_BRING);
-                        tc::mbar_wait(&S.b_full[bslot], (uint32_t)((gi / U3H_BRING) & 1));
-                        b_base = tc::smem_u32(S.b[bslot]);
-                        ++gi;
-                    }
-                    tc::fence_after_sync();
-                    const int r8 = ks % 8, u = ks % U3H_KST;
-                    // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0, 1); r8 >= 5: channels 16-19 of
-                    // taps (i, j) and (i, j+1), j = 2 (r8 - 5) (block 2, next pixel)
-                    const uint32_t a_off = r8 < 5 ? (uint32_t)(r8 * 16) : 2 * plane_bytes + (uint32_t)(2 * (r8 - 5) * 16);
-                    const uint32_t lbo = r8 < 5 ? plane_bytes : 16u;
+                for (int i = 0; i < 5; ++i) {
+                    const int aslot = (int)(si % U3H_NA);
+                    tc::mbar_wait(&S.a_full[aslot], (uint32_t)((si / U3H_NA) & 1));
+                    ++si;
+                    const uint32_t a_base = tc::smem_u32(S.a[aslot][0][0]);
+                    // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0, 1; LBO = one block plane);
+                    // r8 >= 5: channels 16-19 of taps (i, j), (i, j+1), j = 2 (r8 - 5) (block 2, next pixel)
+                    const uint64_t ad_lo = tc::make_desc(a_base, plane_bytes, 128);
+                    const uint64_t ad_hi = tc::make_desc(a_base + 2 * plane_bytes, 16u, 128);
 #pragma unroll
-                    for (int t = 0; t < 2; ++t) {
-                        const uint32_t ab = a_base + a_off + (uint32_t)(t * kTileM * 16);
-                        const uint64_t a_hi = tc::make_desc(ab, lbo, 128);
-                        const uint64_t a_lo = tc::make_desc(ab + part_bytes, lbo, 128);
-                        const uint32_t bb = b_base + (uint32_t)(u * 2 * 2 * NP * 16);
-                        if (kFuse) {  // A_hi read once: [B_hi | B_lo] at N = 2 NP, then A_lo x B_hi
-                            const uint64_t b_ks = tc::make_desc(bb, (uint32_t)(2 * NP * 16), 128);
-                            const uint32_t d = d_base + (uint32_t)(t * 2 * NP);
-                            tc::mma_bf16(d, a_hi, b_ks, idesc2, ks > 0 ? 1u : 0u);
-                            tc::mma_bf16(d + (uint32_t)NP, a_lo, b_ks, idesc, 1u);
-                        } else {
-                            const uint64_t b_hi = tc::make_desc(bb, (uint32_t)(NP * 16), 128);
-                            const uint64_t b_lo = tc::make_desc(bb + (uint32_t)(2 * NP * 16), (uint32_t)(NP * 16), 128);
-                            const uint32_t d = d_base + (uint32_t)(t * NP);
-                            tc::mma_bf16(d, a_hi, b_hi, idesc, ks > 0 ? 1u : 0u);
-                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);
-                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);
+                    for (int hs = 0; hs < 2; ++hs) {
+                        const int bslot = (int)(gi % U3H_BRING);
+                        tc::mbar_wait(&S.b_full[bslot], (uint32_t)((gi / U3H_BRING) & 1));
+                        ++gi;
+                        tc::fence_after_sync();
+                        const uint64_t bd0 = kFuse ? tc::make_desc(tc::smem_u32(S.b[bslot]), (uint32_t)(2 * NP * 16), 128)
+                                                   : tc::make_desc(tc::smem_u32(S.b[bslot]), (uint32_t)(NP * 16), 128);
+#pragma unroll
+                        for (int u = 0; u < U3H_KST; ++u) {
+                            const int r8 = 4 * hs + u;
+                            const uint64_t ad = r8 < 5 ? ad_lo + (uint64_t)r8 : ad_hi + (uint64_t)(2 * (r8 - 5));
+                            const uint64_t bd = bd0 + (uint64_t)u * b_step;
+                            const uint32_t acc0 = (i | r8) > 0 ? 1u : 0u;
+#pragma unroll
+                            for (int t = 0; t < 2; ++t) {
+                                const uint64_t a_hi = ad + (uint64_t)(t * kTileM), a_lo = a_hi + a_part;
+                                if (kFuse) {  // A_hi read once: [B_hi | B_lo] at N = 2 NP, then A_lo x B_hi
+                                    const uint32_t d = d_base + (uint32_t)(t * 2 * NP);
+                                    tc::mma_bf16(d, a_hi, bd, idesc2, acc0);
+                                    tc::mma_bf16(d + (uint32_t)NP, a_lo, bd, idesc, 1u);
+                                } else {
+                                    const uint32_t d = d_base + (uint32_t)(t * NP);
+                                    tc::mma_bf16(d, a_hi, bd, idesc, acc0);
+                                    tc::mma_bf16(d, a_hi, bd + b_part, idesc, 1u);
+                                    tc::mma_bf16(d, a_lo, bd, idesc, 1u);
+                                }
+                            }
                         }
+                        tc::commit(&S.b_empty[bslot]);
                     }
-                    if (u == U3H_KST - 1) tc::commit(&S.b_empty[bslot]);
-                    if (r8 == 7) tc::commit(&S.a_empty[aslot]);
-                    if (ks == U3H_KS - 1) tc::commit(&S.t_full[buf]);
+                    tc::commit(&S.a_empty[aslot]);
                 }
+                tc::commit(&S.t_full[buf]);
             }
         }
         __syncwarp();

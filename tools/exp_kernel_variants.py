@@ -31,6 +31,17 @@ U3_NO_TMEMLD = [("                    tc::tmem_ld16_async(region + (uint32_t)(16
                  "#pragma unroll\n                    for (int u = 0; u < 16; ++u) v[u] = __int_as_float(region + u) * 1e-30f;")]
 U3_NO_TMEMST = [("                    tc::tmem_st8(region + (uint32_t)(8 * c), r);", "                    if (r[0] == 12345u) tc::tmem_st8(region + (uint32_t)(8 * c), r);")]
 
+H3U3_NO_EPI = [
+    ("#pragma unroll\n            for (int c = 0; c < NCH; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);",
+     "#pragma unroll\n            for (int c = 0; c < 0; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);"),
+    ("            if (cur.ok) {\n                float* ob = a.out + cur.img * a.out_img_stride", "            if (false) {\n                float* ob = a.out + cur.img * a.out_img_stride")]
+H3U3_NO_BCOPY = [
+    ("                        tc::mbar_expect_tx(&S.b_full[slot], stage_bytes);\n                        tc::bulk_g2s(S.b[slot], kb + (size_t)(ks / U3H_KST) * stage_bytes, stage_bytes, &S.b_full[slot]);",
+     "                        tc::mbar_arrive(&S.b_full[slot]);")]
+H3U3_NO_ACOPY = [
+    ("                    if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(6 * n * 16));\n                    __syncwarp();\n                    if (n > 0 && lane < 6) {",
+     "                    if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n                    __syncwarp();\n                    if (false) {")]
+
 # variant -> (kernel source, [(old, new), ...]); every `old` must occur in the source
 VARIANTS = {
     "base": ("cnn_tc.cu", []),
@@ -104,6 +115,9 @@ VARIANTS = {
          "#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = __int_as_float(col + u) * 1e-30f;\n                if (false) {"),
         ("                } else {\n                    tc::tmem_wait_ld();\n                }\n#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(",
          "                } else {\n                }\n#pragma unroll\n                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(")]),
+    # U3 3xFP16: the MMA issue loop alone (no epilogue work, no copies: every wait finds its barrier done)
+    "h3u3_mma_only": ("cnn_h3.cu", H3U3_NO_EPI + H3U3_NO_BCOPY + H3U3_NO_ACOPY),
+    "h3u3_no_epi_no_bcopy": ("cnn_h3.cu", H3U3_NO_EPI + H3U3_NO_BCOPY),
     # U3 3xFP16: no bias-plane loads (bias 0)
     "h3u3_no_bias": ("cnn_h3.cu", [
         ("                for (int u = 0; u < 32; ++u, p += bcs) bv[u] = __ldg(p);\n            } else {",
