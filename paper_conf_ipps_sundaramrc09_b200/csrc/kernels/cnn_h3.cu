@@ -539,7 +539,13 @@ __global__ void __launch_bounds__(kThreads, 1)
                     tc::tmem_wait_ld();
                 }
 #pragma unroll
-                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], a.w_unscale, bv[u]));
+                for (int u = 0; u < 32; u += 2) {
+                    const float2 x = __ffma2_rn(make_float2(v[u], v[u + 1]), make_float2(a.w_unscale, a.w_unscale),
+                                                make_float2(bv[u], bv[u + 1]));
+                    const float2 y = tanh_fp32x2(x);
+                    v[u] = y.x;
+                    v[u + 1] = y.y;
+                }
                 if (c + 1 < NCH)
                     load_bias(cur.pb, c + 1);
                 else if (has_next)

@@ -31,6 +31,9 @@ U3_NO_TMEMLD = [("                    tc::tmem_ld16_async(region + (uint32_t)(16
                  "#pragma unroll\n                    for (int u = 0; u < 16; ++u) v[u] = __int_as_float(region + u) * 1e-30f;")]
 U3_NO_TMEMST = [("                    tc::tmem_st8(region + (uint32_t)(8 * c), r);", "                    if (r[0] == 12345u) tc::tmem_st8(region + (uint32_t)(8 * c), r);")]
 
+H3U3_NO_MMA = [
+    ("                                    tc::mma_bf16(d, a_hi, bd, idesc, acc0);\n                                    tc::mma_bf16(d, a_hi, bd + b_part, idesc, 1u);\n                                    tc::mma_bf16(d, a_lo, bd, idesc, 1u);",
+     "                                    if (acc0 > 7u) tc::mma_bf16(d, a_lo, bd, idesc, 1u);")]
 H3U3_NO_EPI = [
     ("#pragma unroll\n            for (int c = 0; c < NCH; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);",
      "#pragma unroll\n            for (int c = 0; c < 0; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);"),
@@ -83,13 +86,30 @@ VARIANTS = {
          "#pragma unroll\n            for (int c = 0; c < 0; ++c) {\n                float v[32];\n                const uint32_t col = (uint32_t)(buf * 256 + t * (kFuse ? 2 * NP : NP) + 32 * c);"),
         ("            if (cur.ok) {\n                float* ob = a.out + cur.img * a.out_img_stride", "            if (false) {\n                float* ob = a.out + cur.img * a.out_img_stride")]),
     # U3 3xFP16: no MMAs (commits still arrive)
-    "h3u3_no_mma": ("cnn_h3.cu", [
-        ("                            tc::mma_bf16(d, a_hi, b_hi, idesc, ks > 0 ? 1u : 0u);\n                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);\n                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);",
-         "                            if (ks < 0) tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);")]),
+    "h3u3_no_mma": ("cnn_h3.cu", H3U3_NO_MMA),
     # U3 3xFP16: two MMAs per K-step instead of three (hi.hi + hi.lo): the MMA-count sensitivity
     "h3u3_2mma": ("cnn_h3.cu", [
-        ("                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);\n                            tc::mma_bf16(d, a_lo, b_hi, idesc, 1u);",
-         "                            tc::mma_bf16(d, a_hi, b_lo, idesc, 1u);")]),
+        ("                                    tc::mma_bf16(d, a_hi, bd + b_part, idesc, 1u);\n                                    tc::mma_bf16(d, a_lo, bd, idesc, 1u);",
+         "                                    tc::mma_bf16(d, a_hi, bd + b_part, idesc, 1u);")]),
+    # U3 3xFP16: the scalar tanh (A/B against the paired tanh_fp32x2 of the tree)
+    "h3u3_tanh_scalar": ("cnn_h3.cu", [
+        ("""                for (int u = 0; u < 32; u += 2) {
+                    const float2 x = __ffma2_rn(make_float2(v[u], v[u + 1]), make_float2(a.w_unscale, a.w_unscale),
+                                                make_float2(bv[u], bv[u + 1]));
+                    const float2 y = tanh_fp32x2(x);
+                    v[u] = y.x;
+                    v[u + 1] = y.y;
+                }""", """                for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], a.w_unscale, bv[u]));""")]),
+    # U3 3xFP16 epilogue decomposition (no MMAs; then one epilogue step removed at a time)
+    "h3e_no_c6": ("cnn_h3.cu", H3U3_NO_MMA + [
+        ("#pragma unroll\n                    for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], v[u], c6[o]);",
+         "                    c6[u % 9] += v[u];")]),
+    "h3e_no_bias": ("cnn_h3.cu", H3U3_NO_MMA + [
+        ("                for (int u = 0; u < 32; ++u, p += bcs) bv[u] = __ldg(p);\n            } else {",
+         "                for (int u = 0; u < 32; ++u, p += bcs) bv[u] = 0.f;\n            } else {")]),
+    "h3e_no_tanh": ("cnn_h3.cu", H3U3_NO_MMA + [
+        ("for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], a.w_unscale, bv[u]));",
+         "for (int u = 0; u < 32; ++u) v[u] = fmaf(v[u], a.w_unscale, bv[u]);")]),
     # U3 bf16 epilogue decomposition: no C5 MMAs, then each epilogue step removed in turn
     "u3e": ("cnn_tc.cu", U3_NO_C5),
     "u3e_no_bias": ("cnn_tc.cu", U3_NO_C5 + U3_NO_BIAS),
