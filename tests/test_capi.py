@@ -47,6 +47,19 @@ def test_errors_are_reported():
     assert e.value.code == tg.TG_E_STATE
 
 
+def test_cnn_n5_range_is_checked():
+    """tg_cnn takes 1 <= n5 <= 128 (include/tg.h; the tensor-core U3 holds n5 padded to 16 maps in
+    one 128-column accumulator): outside that range the graph call fails with TG_E_ARG."""
+    from paper_conf_ipps_sundaramrc09_b200 import tg
+    for n5 in (0, 129):
+        g = tg.Graph()
+        x = g.input(np.zeros((1, 1, 64, 64), np.float32))
+        prm = [g.param(np.zeros((1, 1, 1, 1), np.float32)) for _ in range(10)]
+        with pytest.raises(tg.TGError) as e:
+            g.cnn(x, n5, prm)
+        assert e.value.code == tg.TG_E_ARG and "n5" in str(e.value)
+
+
 def test_unsupported_graph_and_infeasible_budget():
     from paper_conf_ipps_sundaramrc09_b200 import tg
     img = np.zeros((1, 1, 64, 64), np.float32)

@@ -180,6 +180,23 @@ def test_large_cnn_paper_size_sampled_rows(tg, orc, prec):
         assert err <= (2e-2 if prec == "bf16_tc" else 1e-5), (r, err)
 
 
+@pytest.mark.parametrize("prec", ["fp32", "bf16_tc", "fp32_tc"])
+@pytest.mark.parametrize("n5", [1, 16, 128])
+def test_cnn_n5_boundaries(tg, orc, n5, prec):
+    """The smallest C5 width, exactly one 16-map chunk (no padding, one TMEM chunk, the degenerate
+    one-buffer bias ring) and the largest (128 = the whole accumulator, no padding): every precision
+    path against the oracle, two images spanning several U3 bands."""
+    seed = synth.seed_for_config(3) + n5
+    n, H, W = 2, 100, 130
+    img = synth.images_np(seed, n, H, W)
+    prm = synth.cnn_params_np(seed, n5, H, W, "plane")
+    code = {"fp32": tg.TG_FP32, "bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}[prec]
+    out, p = run_cnn(tg, img, n5, prm, "plane", precision=code)
+    assert p.json()["precision"] == prec
+    err = normwise(out, orc.cnn(img, n5, prm, bias_plane=True))
+    assert err <= (2e-2 if prec == "bf16_tc" else 1e-5), err
+
+
 # ------------------------------------------------------------------ tcgen05 bf16 path
 @pytest.mark.parametrize("n,H,W,n5,bias", [(2, 92, 100, 20, "plane"), (1, 120, 160, 120, "plane"),
                                           (2, 480, 640, 120, "plane"), (1, 480, 640, 20, "scalar"),

@@ -63,6 +63,19 @@ def test_edge_parity(tg, orc, n, H, W, ks):
     assert np.all(out >= 0)
 
 
+def test_edge_tile_geometry_invariance(tg, orc):
+    """K1 picks its tile geometry from the work size (64x64 tiles of 8 warps; 32x32 when those are
+    fewer than the SMs; 16x32 of 4 warps when even those are -- kernels/edge.cu): one 256x256 image
+    alone (16x32 tiles), in a batch of 4 (32x32) and in a batch of 10 (64x64) gives the SAME bits,
+    since every output pixel is the same FFMA sequence in the same order, and matches the oracle."""
+    seed = synth.seed_for_config(1) + 5
+    K1, K2 = synth.random_edge_filters_np(seed, 16)
+    batch = synth.images_np(seed, 10, 256, 256)
+    outs = [run_edge(tg, np.ascontiguousarray(batch[:n]), K1, K2)[0][0] for n in (1, 4, 10)]
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
+    assert normwise(outs[0][None], oracle_edge(orc, batch[:1], K1, K2)[0]) <= 1e-5
+
+
 def test_find_edges_rotation(tg, orc):
     """find_edges(Image, Kernel, 4, MAX) (PAPER.md:623) with K2 = rot90(K1) derived in the
     library equals the oracle's template on the synthetic oriented filter."""

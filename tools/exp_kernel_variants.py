@@ -45,6 +45,10 @@ H3U3_NO_ACOPY = [
     ("                    if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(6 * n * 16));\n                    __syncwarp();\n                    if (n > 0 && lane < 6) {",
      "                    if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n                    __syncwarp();\n                    if (false) {")]
 
+U2_NO_COPY = [("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(rows * cols * 16));\n            __syncwarp();\n            if (lane < rows) {",
+               "            if (lane == 0) tc::mbar_arrive(&S.a_full[buf]);\n            __syncwarp();\n            if (false) {")]
+U2_NO_EPI = [("            const bool out_ok = !(lane & 1) && C < a.w4;", "            const bool out_ok = false; if (k >= 0) continue;")]
+
 # variant -> (kernel source, [(old, new), ...]); every `old` must occur in the source
 VARIANTS = {
     "base": ("cnn_tc.cu", []),
@@ -91,6 +95,10 @@ VARIANTS = {
     "h3u3_2mma": ("cnn_h3.cu", [
         ("                                    tc::mma_bf16(d, a_hi, bd + b_part, idesc, 1u);\n                                    tc::mma_bf16(d, a_lo, bd, idesc, 1u);",
          "                                    tc::mma_bf16(d, a_hi, bd + b_part, idesc, 1u);")]),
+    # U2 bf16 decomposition
+    "u2_no_copy": ("cnn_tc.cu", U2_NO_COPY),
+    "u2_no_epi": ("cnn_tc.cu", U2_NO_EPI),
+    "u2_mma_only": ("cnn_tc.cu", U2_NO_COPY + U2_NO_EPI),
     # U3 3xFP16: the scalar tanh (A/B against the paired tanh_fp32x2 of the tree)
     "h3u3_tanh_scalar": ("cnn_h3.cu", [
         ("""                for (int u = 0; u < 32; u += 2) {
