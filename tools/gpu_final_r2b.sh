@@ -1,0 +1,22 @@
+#!/bin/bash
+# Round-2 closing evidence: GPU tests, smoke, sanitizers, the default bench line, the reference arm,
+# launch lists, ncu full captures of the CNN units (three precisions) and K1, the 2-rank functional
+# run, and the paper's Fig. 2 / Fig. 8 / Table 2 re-runs
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/sanitizer
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
+timeout 1200 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -2 gpurun_out/pytest_gpu.log
+timeout 600 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -8 gpurun_out/smoke.log
+for tool in memcheck racecheck synccheck; do
+  timeout 900 compute-sanitizer --tool $tool --print-limit 10 python __graft_entry__.py smoke > gpurun_out/sanitizer/$tool.log 2>&1
+  echo "$tool rc=$?"; grep -E "ERROR SUMMARY|RACECHECK SUMMARY|SYNCCHECK" gpurun_out/sanitizer/$tool.log | tail -2
+done
+t0=$(date +%s); timeout 1500 python bench.py --steps 20 --warmup 5 > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err; echo "bench rc=$? $(( $(date +%s) - t0 )) s"
+t0=$(date +%s); timeout 900 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err; echo "ref rc=$? $(( $(date +%s) - t0 )) s"
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"edge" --csv --log-file gpurun_out/launches_bench_edge256.csv python bench.py --template edge256 --steps 20 --warmup 3 --no-cpu --no-verify --per-template none > /dev/null 2>&1; echo "ncu edge256 rc=$?"
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"cnn" --csv --log-file gpurun_out/launches_bench_cnn3_bf16_tc.csv python bench.py --template cnn3 --precision bf16_tc --steps 5 --warmup 3 --no-cpu --no-verify --per-template none > /dev/null 2>&1; echo "ncu cnn3 launches rc=$?"
+for pr in bf16 fp32tc fp32; do
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:cnn -s 3 -c 3 -o gpurun_out/cnn_${pr}_full -f python tools/prof_cnn.py 120 $pr > gpurun_out/ncu_cnn_$pr.log 2>&1; echo "cnn $pr rc=$?"
+done
+TG_BENCH_DIST_BACKEND=gloo timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --no-verify --per-template edge256:fp32,cnn4:bf16_tc,cnn26:bf16_tc > gpurun_out/bench_2rank.json 2> gpurun_out/bench_2rank.err; echo "2rank rc=$?"
+timeout 1200 python tools/paper_fig2_fig8.py > gpurun_out/paper_fig2_fig8_b200.jsonl 2> gpurun_out/fig28.err; echo "fig2/8 rc=$?"
+timeout 1200 python tools/paper_table2.py > gpurun_out/paper_table2_b200.jsonl 2> gpurun_out/table2.err; echo "table2 rc=$?"
