@@ -70,6 +70,7 @@ struct tg_exec {
     std::vector<uint16_t> k3tc, k5tc;  // host copies of the bf16 tensor-core B operands
     std::vector<uint16_t> k3h3, k5h3;  // host copies of the 3xFP16 B operands (TG_FP32_TC)
     float k3_scale = 1.f, k5_scale = 1.f;  // their power-of-two weight scales
+    std::vector<float> b5q4;  // C5 bias planes channel-quad interleaved [n5/4][h5][w5][4] (b5_quads)
 };
 
 namespace {
@@ -189,6 +190,16 @@ tg_status register_host(tg_plan* p, tg_exec* x) {
         x->registered_bytes += b.second;
     }
     return TG_OK;
+}
+
+// The tensor-core U3 kernels read the resident C5 bias planes channel-quad interleaved,
+// [n5/4][h5][w5][4]: a warp's 32 consecutive positions load 4 channels each with one 128-bit load
+// (512 contiguous bytes), 4 loads per 16 channels instead of 16 scalar ones, with the same L1
+// wavefronts. Same bytes as the plane layout, so the plan (offsets, budget) is
+// unchanged; it needs n5 % 4 == 0 (the paper's 20 and 120; other n5 keep the planes).
+inline bool b5_quads(const PlanCore& c) {
+    return c.t.kind == Tmpl::Cnn && c.bias == "resident" && c.param_off[7] != UINT64_MAX && c.t.n5 % 4 == 0 &&
+           (c.precision == TG_BF16_TC || c.precision == TG_FP32_TC);
 }
 
 inline char* slot_base(const PlanCore& c, DevState& d, int s) {
@@ -405,6 +416,7 @@ tg_status launch_units(tg_plan* p, tg_exec* x, DevState& d, const Chunk& ch, int
         a.k5 = param(6);
         a.k6 = param(8);
         a.b5_plane = a.b6_plane = plane;
+        a.b5_q4 = b5_quads(c) ? 1 : 0;
         if (strm) {
             a.b5 = (const float*)(base + c.slot.b5);
             a.b6 = (const float*)(base + c.slot.b6);
@@ -491,7 +503,8 @@ tg_status run_device(tg_plan* p, tg_exec* x, DevState& d, bool blocking, cudaStr
         for (size_t i = 0; i < c.param_ds.size(); ++i) {
             if (c.param_off[i] == UINT64_MAX) continue;
             const Ds& P = g.ds[c.param_ds[i]];
-            CK(cudaMemcpyAsync(d.arena + c.param_off[i], P.src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
+            const float* src = (i == 7 && b5_quads(c)) ? x->b5q4.data() : P.src;
+            CK(cudaMemcpyAsync(d.arena + c.param_off[i], src, (size_t)P.numel() * 4, cudaMemcpyHostToDevice, S0));
         }
         if (c.k5tc_off != UINT64_MAX) {
             // tensor-core B operands (bf16, or fp16-split for TG_FP32_TC), prepared on the host
@@ -574,6 +587,13 @@ void prepare_tc_operands(tg_plan* p, tg_exec* x) {
     const Graph& g = graph_of(p);
     const PlanCore& c = p->core;
     if (c.k5tc_off == UINT64_MAX) return;
+    if (b5_quads(c) && x->b5q4.empty()) {  // [n5][hw] -> [n5/4][hw][4]
+        const float* src = g.ds[c.t.prm[7]].src;
+        const int64_t n5 = c.t.n5, hw = c.t.h[5] * c.t.w[5];
+        x->b5q4.resize((size_t)(n5 * hw));
+        for (int64_t ch = 0; ch < n5; ++ch)
+            for (int64_t q = 0; q < hw; ++q) x->b5q4[((ch >> 2) * hw + q) * 4 + (ch & 3)] = src[ch * hw + q];
+    }
     const Ds& K3 = g.ds[c.t.prm[3]];
     const Ds& K5 = g.ds[c.t.prm[6]];
     if (c.precision == TG_FP32_TC && x->k5h3.empty()) {
@@ -808,6 +828,7 @@ void exec_invalidate_params(tg_plan* p) {
     p->exec->k5tc.clear();
     p->exec->k5h3.clear();
     p->exec->k3h3.clear();
+    p->exec->b5q4.clear();
 }
 
 }  // namespace tg

@@ -498,11 +498,24 @@ __global__ void __launch_bounds__(kThreads, 1)
             q.ocol = qq - r * w4;
             q.ok = q.orow < orow_end && q.ocol < w5;
             const int orow_c = min(q.orow, orow_end - 1), ocol_c = min(q.ocol, w5 - 1);
-            q.pb = a.b5_plane ? a.b5 + ((int64_t)(orow_c - a.b5_row0) * w5 + ocol_c) : a.b5;
+            const int64_t pix = (int64_t)(orow_c - a.b5_row0) * w5 + ocol_c;
+            q.pb = a.b5_plane ? a.b5 + (a.b5_q4 ? 4 * pix : pix) : a.b5;
             return q;
         };
         float bv[32];
         auto load_bias = [&](const float* pb, int c) {
+            if (a.b5_q4) {  // channel-quad bias: 8 x 128-bit loads (n5 % 4 == 0)
+                const float4* p4 = reinterpret_cast<const float4*>(pb) + (size_t)(8 * c) * bcs;
+#pragma unroll
+                for (int u = 0; u < 8; ++u) {
+                    const float4 f = (32 * c + 4 * u < a.n5) ? __ldg(p4 + (size_t)u * bcs) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    bv[4 * u] = f.x;
+                    bv[4 * u + 1] = f.y;
+                    bv[4 * u + 2] = f.z;
+                    bv[4 * u + 3] = f.w;
+                }
+                return;
+            }
             const float* p = pb + (size_t)(32 * c) * bcs;
             if (c < NCH - 1) {
 #pragma unroll
@@ -521,9 +534,9 @@ __global__ void __launch_bounds__(kThreads, 1)
             const float* nxt_pb = pos_of(has_next ? band + gridDim.x : band).pb;
             tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
             tc::fence_after_sync();
-            float c6[9];
+            float2 c6[5];  // C6 maps (2j, 2j+1) as pairs for FFMA2; map 9 is padding (weight 0)
 #pragma unroll
-            for (int o = 0; o < 9; ++o) c6[o] = 0.f;
+            for (int o = 0; o < 5; ++o) c6[o] = make_float2(0.f, 0.f);
 #pragma unroll
             for (int c = 0; c < NCH; ++c) {
                 float v[32];
@@ -554,7 +567,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                 for (int u = 0; u < 32; ++u) {
                     const int ch = 32 * c + u;
 #pragma unroll
-                    for (int o = 0; o < 9; ++o) c6[o] = fmaf(k6w.k6[ch][o], v[u], c6[o]);
+                    for (int o = 0; o < 5; ++o)
+                        c6[o] = __ffma2_rn(make_float2(k6w.k6[ch][2 * o], k6w.k6[ch][2 * o + 1]), make_float2(v[u], v[u]),
+                                           c6[o]);
                 }
             }
             tc::fence_before_sync();
@@ -567,7 +582,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                     const float b = a.b6_plane
                                         ? __ldg(a.b6 + ((int64_t)o * a.b6_rows + (cur.orow - a.b6_row0)) * w5 + cur.ocol)
                                         : __ldg(a.b6 + o);
-                    ob[o * a.out_plane_stride] = c6[o] + b;
+                    ob[o * a.out_plane_stride] = ((o & 1) ? c6[o >> 1].y : c6[o >> 1].x) + b;
                 }
             }
             if (has_next) cur = pos_of(band + gridDim.x);

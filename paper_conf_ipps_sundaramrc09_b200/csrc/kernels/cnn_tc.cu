@@ -311,7 +311,10 @@ struct U3Smem {
     uint32_t tmem;
 };
 
-template <int NCH>  // TMEM chunks of 32 columns: NP = n5 padded to 16, NCH = ceil(NP / 32)
+// NCH: TMEM chunks of 32 columns (NP = n5 padded to 16, NCH = ceil(NP / 32)); Q4: the C5 bias
+// planes are channel-quad interleaved (CnnU3Args::b5_q4), a compile-time choice so the plane-layout
+// drain carries no branch
+template <int NCH, bool Q4>
 __global__ void __launch_bounds__(kThreadsU3, 1)
     cnn_u3_tc_kernel(const CnnU3Args a, const __grid_constant__ U3P pw, const int64_t nbands) {
     extern __shared__ __align__(128) uint8_t smraw[];
@@ -501,7 +504,8 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             // positions past the chunk's last row / the row's last column compute on clamped
             // (in-bounds) bias addresses and are not stored: the drain stays branch-free
             const int orow_c = min(q.orow, orow_end - 1), ocol_c = min(q.ocol, w5 - 1);
-            q.pb = a.b5_plane ? a.b5 + ((int64_t)(orow_c - a.b5_row0) * w5 + ocol_c) : a.b5;
+            const int64_t pix = (int64_t)(orow_c - a.b5_row0) * w5 + ocol_c;
+            q.pb = a.b5_plane ? a.b5 + (Q4 ? 4 * pix : pix) : a.b5;
             return q;
         };
         // bias ring of 2 chunk buffers loaded 2 chunks ahead (nc is even or 1 ... the ring index
@@ -509,6 +513,18 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         // one buffer loaded one chunk ahead)
         float bv[2][16];
         auto load_bias = [&](const float* pb, int c, int r) {
+            if (Q4) {                   // channel quads: 4 x 128-bit loads (n5 % 4 == 0)
+                const float4* p4 = reinterpret_cast<const float4*>(pb) + (size_t)(4 * c) * bcs;
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const float4 f = (16 * c + 4 * u < a.n5) ? __ldg(p4 + (size_t)u * bcs) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    bv[r][4 * u] = f.x;
+                    bv[r][4 * u + 1] = f.y;
+                    bv[r][4 * u + 2] = f.z;
+                    bv[r][4 * u + 3] = f.w;
+                }
+                return;
+            }
             const float* p = pb + (size_t)(16 * c) * bcs;
             if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)
 #pragma unroll
@@ -547,6 +563,9 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
 #pragma unroll
                         for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[1][u]);
                     }
+                    uint32_t r[8];
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) r[u] = tc::pack_bf16(v[2 * u], v[2 * u + 1]);
                     // refill the consumed buffer with the chunk `ring` steps ahead
                     const int cn = c + ring;
                     if (rb == 0) {
@@ -557,9 +576,6 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                         else if (has_next) load_bias(nxt_pb, cn - nc, 1);
                     }
                     // T5 chunk c -> TMEM columns [8c, 8c+8) (already drained), bf16 pairs
-                    uint32_t r[8];
-#pragma unroll
-                    for (int u = 0; u < 8; ++u) r[u] = tc::pack_bf16(v[2 * u], v[2 * u + 1]);
                     tc::tmem_st8(region + (uint32_t)(8 * c), r);
                 }
             }
@@ -682,10 +698,13 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     if (a.n_pad > U3_NMAX || a.n_pad % 16 || a.n5 > U3_NMAX) return cudaErrorInvalidValue;
     const size_t smem = sizeof(U3Smem) + 128;
     const int nch = (a.n_pad + 31) / 32;
-    const void* fns[4] = {(const void*)cnn_u3_tc_kernel<1>, (const void*)cnn_u3_tc_kernel<2>,
-                          (const void*)cnn_u3_tc_kernel<3>, (const void*)cnn_u3_tc_kernel<4>};
-    static std::atomic<uint32_t> flag_n[4];
-    if (!set_smem_attr(fns[nch - 1], smem, flag_n[nch - 1])) return cudaErrorInvalidValue;
+    const bool q4 = a.b5_plane && a.b5_q4;
+    const void* fns[2][4] = {{(const void*)cnn_u3_tc_kernel<1, false>, (const void*)cnn_u3_tc_kernel<2, false>,
+                              (const void*)cnn_u3_tc_kernel<3, false>, (const void*)cnn_u3_tc_kernel<4, false>},
+                             {(const void*)cnn_u3_tc_kernel<1, true>, (const void*)cnn_u3_tc_kernel<2, true>,
+                              (const void*)cnn_u3_tc_kernel<3, true>, (const void*)cnn_u3_tc_kernel<4, true>}};
+    static std::atomic<uint32_t> flag_n[2][4];
+    if (!set_smem_attr(fns[q4][nch - 1], smem, flag_n[q4][nch - 1])) return cudaErrorInvalidValue;
     const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
     // the epilogue addresses bias channels with 32-bit offsets
     if (a.b5_plane && (int64_t)a.n5 * a.b5_rows * a.w5 >= (1ll << 32)) return cudaErrorInvalidValue;
@@ -705,13 +724,8 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     const int64_t nbands = per_img * a.nimg;
     if (nbands >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit band indexing in the kernel
     const unsigned grid = (unsigned)std::min<int64_t>(nbands, sms);
-    switch (nch) {
-        case 1: cnn_u3_tc_kernel<1><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
-        case 2: cnn_u3_tc_kernel<2><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
-        case 3: cnn_u3_tc_kernel<3><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
-        default: cnn_u3_tc_kernel<4><<<grid, kThreadsU3, smem, s>>>(a, pw, nbands); break;
-    }
-    return cudaGetLastError();
+    void* args[] = {(void*)&a, (void*)&pw, (void*)&nbands};
+    return cudaLaunchKernel(fns[q4][nch - 1], dim3(grid), dim3(kThreadsU3), args, smem, s);
 }
 
 }  // namespace tg

@@ -60,6 +60,7 @@ struct CnnU3Args {          // C5(20->n5, 5x5) + bias + tanh + C6(n5->9, 1x1) + 
     const float* t4; int64_t t4_img_stride; int64_t t4_row0, t4_rows; int64_t w4;
     const float* k5;        // [n5][20][25]
     const float* b5; int64_t b5_row0, b5_rows; int b5_plane;      // plane [n5][b5_rows][w5]
+    int b5_q4;              // tensor-core paths: b5 is channel-quad interleaved [n5/4][b5_rows][w5][4]
     const float* k6;        // [9][n5]
     const float* b6; int64_t b6_row0, b6_rows; int b6_plane;      // plane [9][b6_rows][w5]
     float* out; int64_t out_img_stride; int64_t out_plane_stride; int64_t out_row0, out_rows; int64_t w5;

@@ -289,18 +289,19 @@ def test_cnn_config3_full_batch_sampled(tg, orc, n5, prec):
         assert normwise(out[b:b + 1], ref) <= tol, b
 
 
-@pytest.mark.parametrize("prec", ["fp32", "bf16_tc"])
+@pytest.mark.parametrize("prec", ["fp32", "bf16_tc", "fp32_tc"])
 def test_cnn_invalidate_params(tg, orc, prec):
     """Parameters stay resident in the arena after the first execution; after the caller
     changes them in place, tg_plan_invalidate_params makes the next execution re-upload them
-    (and re-derive the bf16 tensor-core operands). Without it the old values are used."""
+    (and re-derive the tensor-core operands and the channel-quad bias planes). Without it the old
+    values are used."""
     seed = 77
     n, H, W, n5 = 2, 100, 120, 20
     img = synth.images_np(seed, n, H, W)
     prm = synth.cnn_params_np(seed, n5, H, W)
     out = np.zeros((n, 9) + synth.cnn_dims(H, W)[4], np.float32)
     g, _ = tg.cnn_graph(img, n5, prm, out=out)
-    g.set(torch_runtime=True, precision=tg.TG_BF16_TC if prec == "bf16_tc" else tg.TG_FP32)
+    g.set(torch_runtime=True, precision={"fp32": tg.TG_FP32, "bf16_tc": tg.TG_BF16_TC, "fp32_tc": tg.TG_FP32_TC}[prec])
     p = g.plan()
     p.execute()
     first = out.copy()

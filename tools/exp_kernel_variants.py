@@ -52,6 +52,9 @@ U2_NO_EPI = [("            const bool out_ok = !(lane & 1) && C < a.w4;", "     
 # variant -> (kernel source, [(old, new), ...]); every `old` must occur in the source
 VARIANTS = {
     "base": ("cnn_tc.cu", []),
+    # U3 (both tensor-core paths): the C5 bias planes in the plane layout (no channel-quad loads)
+    "no_q4": ("../engine.cu", [("    return c.t.kind == Tmpl::Cnn && c.bias == \"resident\" && c.param_off[7] != UINT64_MAX",
+                                "    return false && c.t.kind == Tmpl::Cnn && c.bias == \"resident\" && c.param_off[7] != UINT64_MAX")]),
     # U3 bf16: the epilogue only does the barrier hand-offs (no TMEM loads, bias, tanh, stores)
     "u3_no_epi": ("cnn_tc.cu", [
         ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
@@ -160,6 +163,18 @@ VARIANTS = {
 def build_variant(name, prebuilt=False):
     if name == "tree":             # the working tree as built in place
         return ROOT
+    if name == "head":             # the last commit's sources (same-box A/B against the working tree)
+        dst = os.path.join(ROOT, "_exp", name)
+        if prebuilt:
+            return dst
+        shutil.rmtree(dst, ignore_errors=True)
+        os.makedirs(dst)
+        subprocess.run(f"git -C {ROOT} archive HEAD {PKG} include synth | tar -x -C {dst}", shell=True, check=True)
+        r = subprocess.run([sys.executable, os.path.join(dst, PKG, "build.py")], capture_output=True, text=True)
+        if r.returncode:
+            raise RuntimeError(r.stderr[-3000:])
+        shutil.rmtree(os.path.join(dst, PKG, "_build"), ignore_errors=True)
+        return dst
     src_file, patches = VARIANTS[name]
     dst = os.path.join(ROOT, "_exp", name)   # git-ignored; travels to the GPU box with the snapshot
     if prebuilt:
