@@ -265,38 +265,44 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
 }
 
 // ============================================================================ U3 (C5 + C6)
-// Band = 256 consecutive output positions in the FLATTENED (row, col) index of the chunk with
-// pitch w4 (two M=128 tiles; the w4 - w5 = 4 positions past each row's end are computed and
-// dropped). For any width, filter row i of a band reads one contiguous run of T4: flat pixels
-// [q0 + i*w4, q0 + i*w4 + 262) -- the band's "slice" i (+4 taps, +1 for the (4,5) tap pair,
-// +1 spare).
+// Band = U3_BT x 128 consecutive output positions in the FLATTENED (row, col) index of the chunk
+// with pitch w4 (U3_BT M=128 tiles; the w4 - w5 = 4 positions past each row's end are computed
+// and dropped). For any width, filter row i of a band reads one contiguous run of T4: flat pixels
+// [q0 + i*w4, q0 + i*w4 + 128 U3_BT + 6) -- the band's "slice" i (+4 taps, +1 for the (4,5) tap
+// pair, +1 spare).
 // Both layers run on the tensor cores:
 //   C5  D5[px][n] = sum_k A5[px][k] B5[k][n]  (A5: the slices in smem, B5: resident in smem)
 //   C6  D6[px][o] = sum_n T5[px][n] B6[n][o]  with T5 = tanh(D5 + bias plane) written back by
 //       the epilogue into the drained TMEM columns as bf16 pairs, and the MMA reading its A
 //       operand straight from TMEM (M = 128 lanes, K = NP channels, N = 16: 9 maps padded)
-// TMEM (512 columns): accumulator buffer b in {0,1}, tile t: 128-column region at 256b + 128t
-// holding D5 in [0, NP), then T5 in [0, NP/2) and D6 in [64, 80).
-// Warp-specialised and persistent (one CTA per SM, 10 warps; single-lane issue under elect.sync):
-//   warp 9               copy producer: the whole C5 B operand (40 K-steps x NP maps, up to
+// TMEM (512 columns): U3_NB accumulator buffers; buffer b, tile t: the 128-column region at
+// 128 (U3_BT b + t), holding D5 in [0, NP), then T5 in [0, NP/2) and D6 in [64, 80).
+// Warp-specialised and persistent (one CTA per SM, 18 warps; single-lane issue under elect.sync):
+//   warp 17              copy producer: the whole C5 B operand (40 K-steps x NP maps, up to
 //                        160 KB) ONCE per CTA (it stays resident), then the slices through a ring
 //                        of U3_NA buffers (three 1-D bulk copies each, one per channel block)
-//   warp 8               MMA issuer: per slice 8 K-steps x 2 tiles of tcgen05.mma; after the 5th
-//                        slice the accumulator goes to the epilogue. The C6 MMAs of the previous
-//                        band are slotted in between slices as soon as its T5 is in TMEM.
-//   warps 0-7            epilogue: TMEM -> registers, + bias plane, tanh -> bf16 T5 -> TMEM;
-//                        then D6 -> registers, + C6 bias -> output (fp32)
-// so the epilogue of band k overlaps the C5 MMAs of band k+1. (Earlier versions re-streamed
-// B5 for every band, and computed C6 as 9 x n5 FFMA per position on the CUDA cores.)
+//   warp 16              MMA issuer: per slice 8 K-steps x U3_BT tiles of tcgen05.mma; after the
+//                        5th slice the accumulator goes to the epilogue. The C6 MMAs of earlier
+//                        bands are slotted in between slices as soon as their T5 is in TMEM.
+//   warps 0-15           U3_NB epilogue groups; group g owns buffer g and takes bands k = g mod
+//                        U3_NB: TMEM -> registers, + bias plane, tanh -> bf16 T5 -> TMEM; then
+//                        D6 -> registers, + C6 bias -> output (fp32)
+// so the MMAs run up to U3_NB - 1 bands ahead of the epilogue. With one tile per band (U3_BT = 1,
+// four buffers) a band's epilogue latency -- drain, C6 round trip, D6 -- may take three MMA band
+// times; with two tiles per band (two buffers) it had one, and the MMAs waited for it (DESIGN.md
+// §5.3). (Earlier versions re-streamed B5 for every band, and computed C6 as 9 x n5 FFMA per
+// position on the CUDA cores.)
 constexpr int U3_KS = 40;
 constexpr int U3_NMAX = 128;
-constexpr int U3_SPX = 2 * kTileM + 8;  // pixels per slice buffer (262 used)
-constexpr int U3_NA = 4;                // slice buffers
+constexpr int U3_BT = 2;                // M = 128 tiles per band
+constexpr int U3_NB = 4 / U3_BT;        // TMEM accumulator buffers (512 columns, 128 per tile)
+constexpr int U3_SPX = U3_BT * kTileM + 8;  // pixels per slice buffer (U3_BT * 128 + 6 used)
+constexpr int U3_NA = 8 / U3_BT;        // slice buffers
 constexpr int U3_C6K = U3_NMAX / 16;    // C6 K-steps (max)
 constexpr int U3_C6N = 16;              // C6 N: 9 maps padded
 constexpr int U3_C6COL = 64;            // D6 column within a tile region
-constexpr int kEpiGroups = 2;                 // epilogue groups, alternating bands
-constexpr int kEpiWarps = 8 * kEpiGroups;
+constexpr int kEpiGroups = U3_NB;             // epilogue groups: group g takes bands k = g mod U3_NB
+constexpr int kEpiWarps = 4 * U3_BT * kEpiGroups;
 constexpr int kThreadsU3 = (kEpiWarps + 2) * 32;
 
 struct U3P {
@@ -307,21 +313,21 @@ struct U3Smem {
     uint4 b[U3_KS * 2 * U3_NMAX];     // resident C5 B operand: [ks][half][n] -> 8 bf16
     uint4 b6[U3_C6K * 2 * U3_C6N];    // C6 B operand
     uint4 a[U3_NA][3][U3_SPX];        // slice ring: [channel block][pixel] -> 8 bf16
-    uint64_t b_full, a_full[U3_NA], a_empty[U3_NA], t_full[2], t_empty[2], t5_full[2], c6_full[2];
+    uint64_t b_full, a_full[U3_NA], a_empty[U3_NA], t_full[U3_NB], t_empty[U3_NB], t5_full[U3_NB], c6_full[U3_NB];
     uint32_t tmem;
 };
 
-// NCH: TMEM chunks of 32 columns (NP = n5 padded to 16, NCH = ceil(NP / 32)); Q4: the C5 bias
-// planes are channel-quad interleaved (CnnU3Args::b5_q4), a compile-time choice so the plane-layout
-// drain carries no branch
-template <int NCH, bool Q4>
+// NCH: TMEM chunks of 32 columns (NP = n5 padded to 16, NCH = ceil(NP / 32)); BQ: the C5 bias
+// layout (CnnU3Args::b5_q4: 0 planes, 1 channel quads), a compile-time choice so the drain carries
+// no branch
+template <int NCH, int BQ>
 __global__ void __launch_bounds__(kThreadsU3, 1)
     cnn_u3_tc_kernel(const CnnU3Args a, const __grid_constant__ U3P pw, const int64_t nbands) {
     extern __shared__ __align__(128) uint8_t smraw[];
     U3Smem& S = *reinterpret_cast<U3Smem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int NP = a.n_pad;
-    const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
+    const int64_t per_img = (a.out_rows * a.w4 + U3_BT * kTileM - 1) / (U3_BT * kTileM);
     const int64_t bplane = a.t4_rows * a.w4;                 // pixels per channel block of one image
     const int64_t flat0 = (a.out_row0 - a.t4_row0) * a.w4;  // flat index of output row 0 in the T4 buffer
 
@@ -332,10 +338,10 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             tc::mbar_init(&S.a_full[i], 1);
             tc::mbar_init(&S.a_empty[i], 1);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < U3_NB; ++i) {
             tc::mbar_init(&S.t_full[i], 1);
-            tc::mbar_init(&S.t_empty[i], 8);   // the 8 warps of the group that owns buffer i
-            tc::mbar_init(&S.t5_full[i], 8);
+            tc::mbar_init(&S.t_empty[i], 4 * U3_BT);   // the warps of the group that owns buffer i
+            tc::mbar_init(&S.t5_full[i], 4 * U3_BT);
             tc::mbar_init(&S.c6_full[i], 1);
         }
         tc::mbar_fence_init();
@@ -373,7 +379,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             const int64_t band = blockIdx.x + (s / 5) * gridDim.x;
             const int i = (int)(s % 5);
             const int64_t img = (uint32_t)band / (uint32_t)per_img;
-            const int64_t q0 = (band - img * per_img) * 2 * kTileM;
+            const int64_t q0 = (band - img * per_img) * U3_BT * kTileM;
             const int64_t e = flat0 + q0 + (int64_t)i * a.w4;
             const int64_t n = max((int64_t)0, min((int64_t)U3_SPX, bplane - e));
             if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));
@@ -399,12 +405,12 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             // C6 of local band kb (its T5 is in TMEM): 2 tiles x NP/16 K-steps, A from TMEM
             int64_t c6_next = 0;
             auto issue_c6 = [&](int64_t kb) {
-                const uint32_t base = tmem + (uint32_t)((kb & 1) * 256);
-                for (int t = 0; t < 2; ++t)
+                const uint32_t base = tmem + (uint32_t)((kb % U3_NB) * U3_BT * 128);
+                for (int t = 0; t < U3_BT; ++t)
                     for (int kk = 0; kk < NP / 16; ++kk)
                         tc::mma_bf16_ts(base + (uint32_t)(t * 128 + U3_C6COL), base + (uint32_t)(t * 128 + kk * 8),
                                         b6desc0 + (uint64_t)(kk * 2 * U3_C6N), idesc6, kk > 0 ? 1u : 0u);
-                tc::commit(&S.c6_full[kb & 1]);
+                tc::commit(&S.c6_full[kb % U3_NB]);
             };
             // The barrier probes for the NEXT slice (and for a pending C6) are issued before the
             // last MMAs of the current slice (mbarrier.test_wait, non-blocking): a barrier access
@@ -414,20 +420,20 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             bool a_ready = false, t5_ready = false;
             const int64_t total_s = my_bands * 5;
             for (int64_t k = 0; k < my_bands; ++k) {
-                const int buf = (int)(k & 1);
-                if (k >= 2) {
-                    // band k-2 shares this accumulator: its C6 must be issued before its epilogue
+                const int buf = (int)(k % U3_NB);
+                if (k >= U3_NB) {
+                    // band k-NB shares this accumulator: its C6 must be issued before its epilogue
                     // can release the buffer
-                    while (c6_next <= k - 2) {
-                        tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                    while (c6_next <= k - U3_NB) {
+                        tc::mbar_wait(&S.t5_full[c6_next % U3_NB], (uint32_t)((c6_next / U3_NB) & 1));
                         tc::fence_after_sync();
                         issue_c6(c6_next++);
                         t5_ready = false;
                     }
-                    tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - 2) >> 1) & 1));
+                    tc::mbar_wait(&S.t_empty[buf], (uint32_t)(((k - U3_NB) / U3_NB) & 1));
                     tc::fence_after_sync();
                 }
-                const uint32_t d_base = tmem + (uint32_t)(buf * 256);
+                const uint32_t d_base = tmem + (uint32_t)(buf * U3_BT * 128);
                 for (int i = 0; i < 5; ++i) {
                     const int64_t s = k * 5 + i;
                     const int slot = (int)(s % U3_NA);
@@ -444,14 +450,14 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                             a_ready = s + 1 < total_s &&
                                       tc::mbar_test(&S.a_full[(s + 1) % U3_NA], (uint32_t)(((s + 1) / U3_NA) & 1));
                             if (c6_next < k && !t5_ready)
-                                t5_ready = tc::mbar_test(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                                t5_ready = tc::mbar_test(&S.t5_full[c6_next % U3_NB], (uint32_t)((c6_next / U3_NB) & 1));
                         }
                         // r8 < 5: channels 0-15 of tap (i, r8) (blocks 0 and 1); r8 >= 5: channels
                         // 16-19 of taps (i, j) and (i, j+1), j = 2(r8-5) (block 2, next pixel)
                         const uint64_t ad = r8 < 5 ? ad_lo + (uint64_t)r8 : ad_hi + (uint64_t)(2 * (r8 - 5));
                         const uint64_t bd = bd_i + (uint64_t)(r8 * 2 * NP);
 #pragma unroll
-                        for (int t = 0; t < 2; ++t)
+                        for (int t = 0; t < U3_BT; ++t)
                             tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,
                                          (i | r8) > 0 ? 1u : 0u);
                     }
@@ -466,7 +472,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                 }
             }
             while (c6_next < my_bands) {
-                tc::mbar_wait(&S.t5_full[c6_next & 1], (uint32_t)((c6_next >> 1) & 1));
+                tc::mbar_wait(&S.t5_full[c6_next % U3_NB], (uint32_t)((c6_next / U3_NB) & 1));
                 tc::fence_after_sync();
                 issue_c6(c6_next++);
             }
@@ -479,8 +485,8 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         // Thread = one output position of the band (tile t, TMEM lane group warp % 4), all NP
         // channels in chunks of 16 TMEM columns. Bias-plane values are loaded RING chunks ahead
         // (across band boundaries), so their L2 latency hides behind the chunk compute.
-        const int grp = warp >> 3;
-        const int t = (warp >> 2) & 1;  // tile
+        const int grp = warp / (4 * U3_BT);
+        const int t = (warp >> 2) % U3_BT;  // tile
         const uint32_t lane_base = (uint32_t)(32 * (warp & 3)) << 16;
         const int m = t * kTileM + 32 * (warp & 3) + lane;
         constexpr int NC = 2 * NCH;     // 16-column chunks (NP = 16 NC or 16 NC - 16)
@@ -495,7 +501,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         auto pos_of = [&](int64_t band) {
             Pos q;
             const int64_t img = (uint32_t)band / (uint32_t)per_img;
-            const int qq = (int)(band - img * per_img) * 2 * kTileM + m;
+            const int qq = (int)(band - img * per_img) * U3_BT * kTileM + m;
             q.img = (int)img;
             const int r = qq / w4;
             q.orow = (int)a.out_row0 + r;
@@ -505,7 +511,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             // (in-bounds) bias addresses and are not stored: the drain stays branch-free
             const int orow_c = min(q.orow, orow_end - 1), ocol_c = min(q.ocol, w5 - 1);
             const int64_t pix = (int64_t)(orow_c - a.b5_row0) * w5 + ocol_c;
-            q.pb = a.b5_plane ? a.b5 + (Q4 ? 4 * pix : pix) : a.b5;
+            q.pb = a.b5_plane ? a.b5 + (BQ == 1 ? 4 * pix : pix) : a.b5;
             return q;
         };
         // bias ring of 2 chunk buffers loaded 2 chunks ahead (nc is even or 1 ... the ring index
@@ -513,7 +519,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         // one buffer loaded one chunk ahead)
         float bv[2][16];
         auto load_bias = [&](const float* pb, int c, int r) {
-            if (Q4) {                   // channel quads: 4 x 128-bit loads (n5 % 4 == 0)
+            if (BQ == 1) {              // channel quads: 4 x 128-bit loads (n5 % 4 == 0)
                 const float4* p4 = reinterpret_cast<const float4*>(pb) + (size_t)(4 * c) * bcs;
 #pragma unroll
                 for (int u = 0; u < 4; ++u) {
@@ -543,11 +549,11 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         }
         int64_t k = grp;
         for (int64_t band = first; band < nbands; band += kEpiGroups * gridDim.x, k += kEpiGroups) {
-            const int buf = (int)(k & 1);
-            const uint32_t region = tmem + lane_base + (uint32_t)(buf * 256 + t * 128);
+            const int buf = (int)(k % U3_NB);
+            const uint32_t region = tmem + lane_base + (uint32_t)((buf * U3_BT + t) * 128);
             const bool has_next = band + kEpiGroups * gridDim.x < nbands;
             const float* nxt_pb = pos_of(has_next ? band + kEpiGroups * gridDim.x : band).pb;
-            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));
+            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));
             tc::fence_after_sync();
 #pragma unroll
             for (int c = 0; c < NC; ++c) {
@@ -584,7 +590,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&S.t5_full[buf]);  // T5 ready for the C6 MMA
             float d6[16];
-            tc::mbar_wait(&S.c6_full[buf], (uint32_t)((k >> 1) & 1));
+            tc::mbar_wait(&S.c6_full[buf], (uint32_t)((k / U3_NB) & 1));
             tc::fence_after_sync();
             tc::tmem_ld16_async(region + (uint32_t)U3_C6COL, d6);
             tc::tmem_wait_ld();
@@ -698,14 +704,14 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     if (a.n_pad > U3_NMAX || a.n_pad % 16 || a.n5 > U3_NMAX) return cudaErrorInvalidValue;
     const size_t smem = sizeof(U3Smem) + 128;
     const int nch = (a.n_pad + 31) / 32;
-    const bool q4 = a.b5_plane && a.b5_q4;
-    const void* fns[2][4] = {{(const void*)cnn_u3_tc_kernel<1, false>, (const void*)cnn_u3_tc_kernel<2, false>,
-                              (const void*)cnn_u3_tc_kernel<3, false>, (const void*)cnn_u3_tc_kernel<4, false>},
-                             {(const void*)cnn_u3_tc_kernel<1, true>, (const void*)cnn_u3_tc_kernel<2, true>,
-                              (const void*)cnn_u3_tc_kernel<3, true>, (const void*)cnn_u3_tc_kernel<4, true>}};
+    const int q4 = a.b5_plane && a.b5_q4 ? 1 : 0;
+    const void* fns[2][4] = {{(const void*)cnn_u3_tc_kernel<1, 0>, (const void*)cnn_u3_tc_kernel<2, 0>,
+                              (const void*)cnn_u3_tc_kernel<3, 0>, (const void*)cnn_u3_tc_kernel<4, 0>},
+                             {(const void*)cnn_u3_tc_kernel<1, 1>, (const void*)cnn_u3_tc_kernel<2, 1>,
+                              (const void*)cnn_u3_tc_kernel<3, 1>, (const void*)cnn_u3_tc_kernel<4, 1>}};
     static std::atomic<uint32_t> flag_n[2][4];
     if (!set_smem_attr(fns[q4][nch - 1], smem, flag_n[q4][nch - 1])) return cudaErrorInvalidValue;
-    const int64_t per_img = (a.out_rows * a.w4 + 2 * kTileM - 1) / (2 * kTileM);
+    const int64_t per_img = (a.out_rows * a.w4 + U3_BT * kTileM - 1) / (U3_BT * kTileM);
     // the epilogue addresses bias channels with 32-bit offsets
     if (a.b5_plane && (int64_t)a.n5 * a.b5_rows * a.w5 >= (1ll << 32)) return cudaErrorInvalidValue;
     // C6 B operand: bf16 [ks][half][o][8 ch], value K6[o][16 ks + 8 half + e] (zero padding)

@@ -16,8 +16,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 PKG = "paper_conf_ipps_sundaramrc09_b200"
 
 VARIANTS_U3_NO_EPI = [
-    ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
-     "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
+    ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
+     "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
     ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob")]
 
 
@@ -25,6 +25,8 @@ U3_NO_C5 = [("                            tc::mma_bf16(d_base + (uint32_t)(t * 1
              "                            if (r8 < 0) tc::mma_bf16(d_base + (uint32_t)(t * 128), ad + (uint64_t)(t * kTileM), bd, idesc,")]
 U3_NO_BIAS = [("            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = __ldg(p);",
                "            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = 0.f;")]
+U3_NO_BIAS_Q4 = [("                    const float4 f = (16 * c + 4 * u < a.n5) ? __ldg(p4 + (size_t)u * bcs) : make_float4(0.f, 0.f, 0.f, 0.f);",
+                   "                    const float4 f = make_float4(0.f, 0.f, 0.f, 0.f);")]
 U3_NO_TANH = [("for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[0][u]);", "for (int u = 0; u < 16; ++u) v[u] = v[u] + bv[0][u];"),
               ("for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[1][u]);", "for (int u = 0; u < 16; ++u) v[u] = v[u] + bv[1][u];")]
 U3_NO_TMEMLD = [("                    tc::tmem_ld16_async(region + (uint32_t)(16 * c), v);\n                    tc::tmem_wait_ld();",
@@ -57,15 +59,23 @@ VARIANTS = {
                                 "    return false && c.t.kind == Tmpl::Cnn && c.bias == \"resident\" && c.param_off[7] != UINT64_MAX")]),
     # U3 bf16: the epilogue only does the barrier hand-offs (no TMEM loads, bias, tanh, stores)
     "u3_no_epi": ("cnn_tc.cu", [
-        ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
-         "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
+        ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
+         "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
         ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob")]),
     # U3 bf16: epilogue hand-offs only AND the C5 MMAs at N = 64 instead of NP (half the B reads
     # and half the math): tells a smem-operand-bound MMA phase from a compute-bound one
     "u3_no_epi_n64": ("cnn_tc.cu", [
-        ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
-         "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k >> 1) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
+        ("            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < nc) {",
+         "            tc::mbar_wait(&S.t_full[buf], (uint32_t)((k / U3_NB) & 1));\n            tc::fence_after_sync();\n#pragma unroll\n            for (int c = 0; c < NC; ++c) {\n                if (c < 0) {"),
         ("            if (cur.ok) {\n                float* ob", "            if (false) {\n                float* ob"),
+        ("        const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);", "        const uint32_t idesc = tc::make_idesc_bf16(kTileM, 64);")]),
+    # U3 bf16: the C5 MMAs at N = 64 with the full epilogue (wrong values; timing only): half the B
+    # operand's shared-memory reads -- does the MMAs' port traffic slow the epilogue?
+    "u3_n64": ("cnn_tc.cu", [
+        ("        const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);", "        const uint32_t idesc = tc::make_idesc_bf16(kTileM, 64);")]),
+    "u3_n64_mma_only": ("cnn_tc.cu", VARIANTS_U3_NO_EPI + [
+        ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[slot], (uint32_t)(3 * n * 16));\n            __syncwarp();\n            if (n > 0 && lane < 3)",
+         "            if (lane == 0) tc::mbar_arrive(&S.a_full[slot]);\n            __syncwarp();\n            if (false)"),
         ("        const uint32_t idesc = tc::make_idesc_bf16(kTileM, NP);", "        const uint32_t idesc = tc::make_idesc_bf16(kTileM, 64);")]),
     # U3 bf16: no bias loads (bias 0), the rest of the epilogue as built
     "u3_no_bias": ("cnn_tc.cu", [
@@ -121,6 +131,12 @@ VARIANTS = {
     "h3e_no_tanh": ("cnn_h3.cu", H3U3_NO_MMA + [
         ("for (int u = 0; u < 32; ++u) v[u] = tanh_acc(fmaf(v[u], a.w_unscale, bv[u]));",
          "for (int u = 0; u < 32; ++u) v[u] = fmaf(v[u], a.w_unscale, bv[u]);")]),
+    # U3 bf16 with the MMAs: each epilogue step removed in turn (what the combination costs)
+    "u3_no_tanh": ("cnn_tc.cu", U3_NO_TANH),
+    "u3_no_tmemld": ("cnn_tc.cu", U3_NO_TMEMLD),
+    "u3_no_tmemst": ("cnn_tc.cu", U3_NO_TMEMST),
+    "u3_no_bias_q4": ("cnn_tc.cu", U3_NO_BIAS_Q4),
+    "u3_one_tile_bands": ("cnn_tc.cu", [("constexpr int U3_BT = 2;", "constexpr int U3_BT = 1;")]),
     # U3 bf16 epilogue decomposition: no C5 MMAs, then each epilogue step removed in turn
     "u3e": ("cnn_tc.cu", U3_NO_C5),
     "u3e_no_bias": ("cnn_tc.cu", U3_NO_C5 + U3_NO_BIAS),
@@ -175,7 +191,8 @@ def build_variant(name, prebuilt=False):
             raise RuntimeError(r.stderr[-3000:])
         shutil.rmtree(os.path.join(dst, PKG, "_build"), ignore_errors=True)
         return dst
-    src_file, patches = VARIANTS[name]
+    spec = VARIANTS[name]
+    files = spec if isinstance(spec, list) else [spec]   # [(kernel source, patches), ...]
     dst = os.path.join(ROOT, "_exp", name)   # git-ignored; travels to the GPU box with the snapshot
     if prebuilt:
         return dst
@@ -186,12 +203,13 @@ def build_variant(name, prebuilt=False):
                     ignore=shutil.ignore_patterns("_build*", "libtg.so*", "__pycache__"))
     shutil.copytree(os.path.join(ROOT, "include"), os.path.join(dst, "include"))
     shutil.copytree(os.path.join(ROOT, "synth"), os.path.join(dst, "synth"))
-    path = os.path.join(dst, PKG, "csrc", "kernels", src_file)
-    s = open(path).read()
-    for old, new in patches:
-        assert old in s, (name, old[:80])
-        s = s.replace(old, new)
-    open(path, "w").write(s)
+    for src_file, patches in files:
+        path = os.path.join(dst, PKG, "csrc", "kernels", src_file)
+        s = open(path).read()
+        for old, new in patches:
+            assert old in s, (name, old[:80])
+            s = s.replace(old, new)
+        open(path, "w").write(s)
     r = subprocess.run([sys.executable, os.path.join(dst, PKG, "build.py")], capture_output=True, text=True)
     if r.returncode:
         raise RuntimeError(r.stderr[-3000:])
