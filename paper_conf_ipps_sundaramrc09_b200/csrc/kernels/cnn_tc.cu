@@ -519,7 +519,7 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
         // one buffer loaded one chunk ahead)
         float bv[2][16];
         auto load_bias = [&](const float* pb, int c, int r) {
-            if (BQ == 1) {              // channel quads: 4 x 128-bit loads (n5 % 4 == 0)
+            if (BQ == 1) {              // channel quads (or a scalar bias): 4 x 128-bit loads
                 const float4* p4 = reinterpret_cast<const float4*>(pb) + (size_t)(4 * c) * bcs;
 #pragma unroll
                 for (int u = 0; u < 4; ++u) {
@@ -540,7 +540,10 @@ __global__ void __launch_bounds__(kThreadsU3, 1)
                 for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = (16 * c + u < a.n5) ? __ldg(p) : 0.f;
             }
         };
-        const int ring = (nc % 2 == 0) ? 2 : 1;
+        // channel quads: one chunk ahead (a ring of two loaded two chunks ahead -- 32 registers
+        // instead of 16 at the 96-register budget of 576 threads -- measured 2-3 % slower, DESIGN.md
+        // §5.3); scalar loads (planes): two chunks ahead (one spills)
+        const int ring = (BQ == 1 || nc % 2) ? 1 : 2;
         const int64_t first = blockIdx.x + (int64_t)grp * gridDim.x;
         Pos cur = pos_of(first);
         if (first < nbands) {
@@ -704,7 +707,8 @@ cudaError_t launch_cnn_u3_tc(const CnnU3Args& a, cudaStream_t s) {
     if (a.n_pad > U3_NMAX || a.n_pad % 16 || a.n5 > U3_NMAX) return cudaErrorInvalidValue;
     const size_t smem = sizeof(U3Smem) + 128;
     const int nch = (a.n_pad + 31) / 32;
-    const int q4 = a.b5_plane && a.b5_q4 ? 1 : 0;
+    // a scalar bias ([n5], 16-byte aligned in the arena) is read like one position of channel quads
+    const int q4 = (a.b5_plane ? a.b5_q4 != 0 : a.n5 % 4 == 0) ? 1 : 0;
     const void* fns[2][4] = {{(const void*)cnn_u3_tc_kernel<1, 0>, (const void*)cnn_u3_tc_kernel<2, 0>,
                               (const void*)cnn_u3_tc_kernel<3, 0>, (const void*)cnn_u3_tc_kernel<4, 0>},
                              {(const void*)cnn_u3_tc_kernel<1, 1>, (const void*)cnn_u3_tc_kernel<2, 1>,

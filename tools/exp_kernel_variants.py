@@ -136,6 +136,8 @@ VARIANTS = {
     "u3_no_tmemld": ("cnn_tc.cu", U3_NO_TMEMLD),
     "u3_no_tmemst": ("cnn_tc.cu", U3_NO_TMEMST),
     "u3_no_bias_q4": ("cnn_tc.cu", U3_NO_BIAS_Q4),
+    # U3 bf16: the bias ring of two chunk buffers loaded two chunks ahead (as before the end of round 2)
+    "u3_bias_ring2": ("cnn_tc.cu", [("        const int ring = (BQ == 1 || nc % 2) ? 1 : 2;", "        const int ring = (nc % 2 == 0) ? 2 : 1;")]),
     "u3_one_tile_bands": ("cnn_tc.cu", [("constexpr int U3_BT = 2;", "constexpr int U3_BT = 1;")]),
     # U3 bf16 epilogue decomposition: no C5 MMAs, then each epilogue step removed in turn
     "u3e": ("cnn_tc.cu", U3_NO_C5),
@@ -232,8 +234,9 @@ torch.cuda.set_device(0)
 x = synth.images_torch(seed, n, H, W, "cuda:0")
 h5, w5 = synth.cnn_dims(H, W)[4]
 y = torch.empty((n, 9, h5, w5), dtype=torch.float32, device="cuda:0")
-prm = synth.cnn_params_np(seed, n5, H, W)
-g, _ = tg.cnn_graph(x, n5, prm, out=y, device=True)
+scalar = wl == "cnn3b"   # scalar C-layer biases (TG_BIAS_SCALAR)
+prm = synth.cnn_params_np(seed, n5, H, W, "scalar" if scalar else "plane")
+g, _ = tg.cnn_graph(x, n5, prm, out=y, device=True, bias_mode=tg.TG_BIAS_SCALAR if scalar else tg.TG_BIAS_PLANE)
 g.set(torch_runtime=True, precision={"fp32": 0, "bf16_tc": 1, "fp32_tc": 2}[prec])
 p = g.plan()
 for _ in range(3):
