@@ -263,19 +263,27 @@ __global__ void __launch_bounds__(kThreads, 1)
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&S.t_empty[ts]);
             const bool out_ok = !(lane & 1) && C < a.w4;
+            // the two C3 rows' tanh as one pair (tanh_fp32x2: paired FP32 arithmetic, bit-identical
+            // to the scalar form), then the S4 tanh of channels (co, co+1) as one pair
             float tv[24];
 #pragma unroll
-            for (int co = 0; co < 20; ++co) {
-                const float t0 = tanh_acc(v0[co] + b0v[co]);
-                const float t1 = tanh_acc(v1[co] + b1v[co]);
-                const float t01 = __shfl_down_sync(0xffffffffu, t0, 1);  // column c+1
-                const float t11 = __shfl_down_sync(0xffffffffu, t1, 1);
-                float s4 = 0.f;
-                s4 = fmaf(pw.p4[co][0], t0, s4);
-                s4 = fmaf(pw.p4[co][1], t01, s4);
-                s4 = fmaf(pw.p4[co][2], t1, s4);
-                s4 = fmaf(pw.p4[co][3], t11, s4);
-                tv[co] = tanh_acc(s4) * kActScale;
+            for (int co = 0; co < 20; co += 2) {
+                float s4[2];
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    const float2 t = tanh_fp32x2(__fadd2_rn(make_float2(v0[co + e], v1[co + e]),
+                                                            make_float2(b0v[co + e], b1v[co + e])));
+                    const float t01 = __shfl_down_sync(0xffffffffu, t.x, 1);  // column c+1
+                    const float t11 = __shfl_down_sync(0xffffffffu, t.y, 1);
+                    float s = 0.f;
+                    s = fmaf(pw.p4[co + e][0], t.x, s);
+                    s = fmaf(pw.p4[co + e][1], t01, s);
+                    s = fmaf(pw.p4[co + e][2], t.y, s);
+                    s4[e] = fmaf(pw.p4[co + e][3], t11, s);
+                }
+                const float2 t4 = tanh_fp32x2(make_float2(s4[0], s4[1]));
+                tv[co] = t4.x * kActScale;
+                tv[co + 1] = t4.y * kActScale;
             }
 #pragma unroll
             for (int co = 20; co < 24; ++co) tv[co] = 0.f;

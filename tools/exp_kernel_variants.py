@@ -27,6 +27,8 @@ U3_NO_BIAS = [("            if (16 * c + 16 <= a.n5) {  // a full chunk of real 
                "            if (16 * c + 16 <= a.n5) {  // a full chunk of real channels (uniform)\n#pragma unroll\n                for (int u = 0; u < 16; ++u, p += bcs) bv[r][u] = 0.f;")]
 U3_NO_BIAS_Q4 = [("                    const float4 f = (16 * c + 4 * u < a.n5) ? __ldg(p4 + (size_t)u * bcs) : make_float4(0.f, 0.f, 0.f, 0.f);",
                    "                    const float4 f = make_float4(0.f, 0.f, 0.f, 0.f);")]
+H3U2_NO_EPI = [("            const bool out_ok = !(lane & 1) && C < a.w4;\n            // the two C3 rows",
+                "            const bool out_ok = false; if (k >= 0) continue;\n            // the two C3 rows")]
 U3_NO_TANH = [("for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[0][u]);", "for (int u = 0; u < 16; ++u) v[u] = v[u] + bv[0][u];"),
               ("for (int u = 0; u < 16; ++u) v[u] = tanh_approx(v[u] + bv[1][u]);", "for (int u = 0; u < 16; ++u) v[u] = v[u] + bv[1][u];")]
 U3_NO_TMEMLD = [("                    tc::tmem_ld16_async(region + (uint32_t)(16 * c), v);\n                    tc::tmem_wait_ld();",
@@ -138,6 +140,11 @@ VARIANTS = {
     "u3_no_bias_q4": ("cnn_tc.cu", U3_NO_BIAS_Q4),
     # U3 bf16: the bias ring of two chunk buffers loaded two chunks ahead (as before the end of round 2)
     "u3_bias_ring2": ("cnn_tc.cu", [("        const int ring = (BQ == 1 || nc % 2) ? 1 : 2;", "        const int ring = (nc % 2 == 0) ? 2 : 1;")]),
+    # U2 3xFP16 decomposition: epilogue hand-offs only; and also no window copies (MMAs alone)
+    "h3u2_no_epi": ("cnn_h3.cu", H3U2_NO_EPI),
+    "h3u2_mma_only": ("cnn_h3.cu", H3U2_NO_EPI + [
+        ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(2 * rows * cols * 16));\n            __syncwarp();\n            if (lane < 2 * rows) {",
+         "            if (lane == 0) tc::mbar_arrive(&S.a_full[buf]);\n            __syncwarp();\n            if (false) {")]),
     "u3_one_tile_bands": ("cnn_tc.cu", [("constexpr int U3_BT = 2;", "constexpr int U3_BT = 1;")]),
     # U3 bf16 epilogue decomposition: no C5 MMAs, then each epilogue step removed in turn
     "u3e": ("cnn_tc.cu", U3_NO_C5),
