@@ -98,6 +98,8 @@ constexpr int U2H_NA = 6;                  // window buffers
 constexpr int U2H_NT = 4;                  // TMEM slots (128 columns apart, 2 x U2H_N used)
 constexpr int U2H_PLANE = U2H_WR * U2H_WP;
 constexpr int kThreads = 10 * 32;
+constexpr int U2H_G = 3;                    // U2 epilogue groups (4 warps each), taking segments in turn
+constexpr int kThreadsU2H = (4 * U2H_G + 2) * 32;
 
 struct U2HP {
     float p4[20][4];  // S4 weights (constant bank)
@@ -110,7 +112,7 @@ struct U2HSmem {
     uint32_t tmem;
 };
 
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kThreadsU2H, 1)
     cnn_u2_h3_kernel(const CnnU2Args a, const __grid_constant__ U2HP pw, const int64_t nseg) {
     extern __shared__ __align__(128) uint8_t smraw[];
     U2HSmem& S = *reinterpret_cast<U2HSmem*>(smraw + ((128 - (tc::smem_u32(smraw) & 127)) & 127));
@@ -142,7 +144,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     // windows start zeroed: pixels a copy does not cover (beyond the image) only ever hold
     // finite T2 values; they feed C3 columns that are not stored
-    for (int idx = tid; idx < U2H_NA * 2 * U2H_PLANE; idx += kThreads) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
+    for (int idx = tid; idx < U2H_NA * 2 * U2H_PLANE; idx += kThreadsU2H) (&S.a[0][0][0])[idx] = make_uint4(0u, 0u, 0u, 0u);
     tc::fence_proxy_async();
     tc::fence_before_sync();
     __syncthreads();
@@ -150,7 +152,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint32_t tmem = S.tmem;
     const int64_t my = nseg > blockIdx.x ? (nseg - 1 - blockIdx.x) / gridDim.x + 1 : 0;
 
-    if (warp == 9) {
+    if (warp == 4 * U2H_G + 1) {
         // ---------------------------------------------------------------- copy producer
         const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
         const int64_t tplane = a.t2_rows * a.w2;  // pixels per part plane of one image's T2
@@ -178,7 +180,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             __syncwarp();
         }
-    } else if (warp == 8) {
+    } else if (warp == 4 * U2H_G) {
         // ---------------------------------------------------------------- MMA issuer
         // ONE elected lane runs the whole loop (warp-level hand-offs per segment left the tensor
         // pipe idle, tools/micro/umma_probe.cu)
@@ -231,7 +233,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
         };
         if (grp < my) load_bias(grp);
-        for (int64_t k = grp; k < my; k += 2) {
+        for (int64_t k = grp; k < my; k += U2H_G) {
             const int ts = (int)(k % U2H_NT);
             int64_t img, R, c0;
             seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
@@ -287,7 +289,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
 #pragma unroll
             for (int co = 20; co < 24; ++co) tv[co] = 0.f;
-            if (k + 2 < my) load_bias(k + 2);
+            if (k + U2H_G < my) load_bias(k + U2H_G);
             if (out_ok) {
                 uint4* t4 = reinterpret_cast<uint4*>(a.t4) + img * 6 * bplane + (R - a.t4_row0) * a.w4 + C;
 #pragma unroll
@@ -685,7 +687,7 @@ cudaError_t launch_cnn_u2_h3(const CnnU2Args& a, cudaStream_t s) {
     const int64_t nseg = a.t4_rows * ((a.w3 + kTileM - 1) / kTileM) * a.nimg;
     if (nseg >= (1ll << 32)) return cudaErrorInvalidValue;  // 32-bit segment indexing in the kernel
     const unsigned grid = (unsigned)std::min<int64_t>(nseg, sms);
-    cnn_u2_h3_kernel<<<grid, kThreads, smem, s>>>(a, pw, nseg);
+    cnn_u2_h3_kernel<<<grid, kThreadsU2H, smem, s>>>(a, pw, nseg);
     return cudaGetLastError();
 }
 

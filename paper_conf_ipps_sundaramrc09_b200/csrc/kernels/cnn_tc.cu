@@ -54,23 +54,28 @@ constexpr int kTileM = 128;
 // row does not exist). 6 rows x 3 tap pairs = 18 MMAs of N = 48 per segment instead of
 // 2 tiles x 15 of N = 32: the A operand -- the shared-memory read that bounds these small-N
 // MMAs -- is read 18 times instead of 30.
-// Warp-specialised and persistent (one CTA per SM, 10 warps; single-lane issue under elect.sync):
-//   warp 9               copy producer: the C3 B operand (6 x 3 K-steps) once per CTA by a bulk
+// Warp-specialised and persistent (one CTA per SM, 4 U2_G + 2 warps; single-lane issue under
+// elect.sync):
+//   warp 4 U2_G + 1      copy producer: the C3 B operand (6 x 3 K-steps) once per CTA by a bulk
 //                        copy; per segment six 1-D bulk copies (TMA engine) of the window's T2
 //                        rows into one of U2_NA buffers, as soon as the buffer is free
-//   warp 8               MMA issuer: 18 tcgen05.mma into one of 4 TMEM slots; tcgen05.commit
+//   warp 4 U2_G          MMA issuer: 18 tcgen05.mma into one of U2_NT TMEM slots; tcgen05.commit
 //                        frees the window buffer and hands the slot to the epilogue (copy issue
 //                        -- ~150 cycles per bulk copy -- does not serialise with MMA issue)
-//   warps 0-3 / 4-7      epilogue groups for even / odd segments: bias plane (prefetched one
-//                        segment ahead), tanh, the 2x2 subsample (rows in the same thread,
-//                        columns across neighbouring lanes), tanh -> T4 bf16 channel blocks
+//   warps 0 .. 4 U2_G-1  U2_G epilogue groups of 4 warps taking segments in turn: bias plane
+//                        (prefetched one segment of the group ahead), tanh, the 2x2 subsample
+//                        (rows in the same thread, columns across neighbouring lanes), tanh -> T4
+//                        bf16 channel blocks. Three groups rather than two: U2 0.193 -> 0.159 ms
+//                        on the single 6400x4800 image (bias planes from HBM), +1 % on cnn3
 constexpr int U2_WR = 6, U2_WP = kTileM + 6;  // +4 taps, +1 for the (4,5) tap pair, +1 spare
 constexpr int U2_N = 48;                      // [0,20) row 2R, [24,44) row 2R+1, rest zero
 constexpr int U2_ROW1 = 24;                   // first column of C3 row 2R+1
 constexpr int U2_KS = 18;                     // 6 window rows x tap pairs (0,1) (2,3) (4,5)
 constexpr int U2_NA = 8;                      // window buffers
-constexpr int U2_NT = 4;                      // TMEM slots (2 per epilogue group), 64 columns apart
-constexpr int kThreadsU2 = 10 * 32;
+constexpr int U2_G = 3;                       // epilogue groups (4 warps each), taking segments in turn
+constexpr int U2_NT = 4;                      // TMEM slots, 64 columns apart
+constexpr int U2_TCOLS = U2_NT * 64;          // TMEM columns allocated (a power of two)
+constexpr int kThreadsU2 = (4 * U2_G + 2) * 32;
 
 struct U2P {
     float p4[20][4];  // S4 weights (constant bank)
@@ -100,7 +105,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
         c0 = (int64_t)(rem - rr * spr_u) * kTileM;
     };
 
-    if (warp == 0) tc::tmem_alloc<256>(&S.tmem);
+    if (warp == 0) tc::tmem_alloc<U2_TCOLS>(&S.tmem);
     if (tid == 0) {
         tc::mbar_init(&S.b_full, 1);
         for (int i = 0; i < U2_NA; ++i) {
@@ -123,7 +128,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
     const uint32_t tmem = S.tmem;
     const int64_t my = nseg > blockIdx.x ? (nseg - 1 - blockIdx.x) / gridDim.x + 1 : 0;
 
-    if (warp == 9) {
+    if (warp == 4 * U2_G + 1) {
         // -------------------------------------------------------------------- copy producer
         // (the whole warp runs the loop; the window rows are issued by one lane each)
         const uint4* t2all = reinterpret_cast<const uint4*>(a.t2);
@@ -151,7 +156,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             }
             __syncwarp();
         }
-    } else if (warp == 8) {
+    } else if (warp == 4 * U2_G) {
         // -------------------------------------------------------------------- MMA issuer
         // ONE elected lane runs the whole loop (barrier waits, MMAs, commits): warp-level
         // hand-offs per segment left the tensor pipe idle (tools/micro/umma_probe.cu)
@@ -214,7 +219,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
             }
         };
         if (grp < my) load_bias(grp);
-        for (int64_t k = grp; k < my; k += 2) {
+        for (int64_t k = grp; k < my; k += U2_G) {
             const int ts = (int)(k % U2_NT);
             int64_t img, R, c0;
             seg_coords(blockIdx.x + k * gridDim.x, img, R, c0);
@@ -247,7 +252,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
                 s4 = fmaf(pw.p4[co][3], t11, s4);
                 tv[co] = tanh_approx(s4);
             }
-            if (k + 2 < my) load_bias(k + 2);
+            if (k + U2_G < my) load_bias(k + U2_G);
             if (out_ok) {
                 // T4 as bf16 channel blocks [3][rows][w4][8] (U3's tensor-core operand rows)
                 uint4* t4 = reinterpret_cast<uint4*>(a.t4) + img * 3 * bplane + (R - a.t4_row0) * a.w4 + C;
@@ -261,7 +266,7 @@ __global__ void __launch_bounds__(kThreadsU2, 1)
     }
     tc::fence_before_sync();
     __syncthreads();
-    if (warp == 0) tc::tmem_dealloc<256>(tmem);
+    if (warp == 0) tc::tmem_dealloc<U2_TCOLS>(tmem);
 }
 
 // ============================================================================ U3 (C5 + C6)

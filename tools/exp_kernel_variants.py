@@ -146,9 +146,9 @@ VARIANTS = {
         ("            if (lane == 0) tc::mbar_expect_tx(&S.a_full[buf], (uint32_t)(2 * rows * cols * 16));\n            __syncwarp();\n            if (lane < 2 * rows) {",
          "            if (lane == 0) tc::mbar_arrive(&S.a_full[buf]);\n            __syncwarp();\n            if (false) {")]),
     # U2 bf16: three epilogue groups (14 warps, 128 registers) and / or 8 TMEM slots
-    "u2_g3": ("cnn_tc.cu", [("constexpr int U2_G = 2;", "constexpr int U2_G = 3;")]),
-    "u2_g3_nt8": ("cnn_tc.cu", [("constexpr int U2_G = 2;", "constexpr int U2_G = 3;"), ("constexpr int U2_NT = 4;", "constexpr int U2_NT = 8;")]),
     "u2_nt8": ("cnn_tc.cu", [("constexpr int U2_NT = 4;", "constexpr int U2_NT = 8;")]),
+    "h3u2_g2": ("cnn_h3.cu", [("constexpr int U2H_G = 3;", "constexpr int U2H_G = 2;")]),
+    "u2_g2": ("cnn_tc.cu", [("constexpr int U2_G = 3;", "constexpr int U2_G = 2;")]),
     "u3_one_tile_bands": ("cnn_tc.cu", [("constexpr int U3_BT = 2;", "constexpr int U3_BT = 1;")]),
     # U3 bf16 epilogue decomposition: no C5 MMAs, then each epilogue step removed in turn
     "u3e": ("cnn_tc.cu", U3_NO_C5),
