@@ -202,7 +202,7 @@ def test_cnn_n5_boundaries(tg, orc, n5, prec):
                                           (2, 480, 640, 120, "plane"), (1, 480, 640, 20, "scalar"),
                                           (1, 97, 1003, 120, "plane"), (1, 61, 67, 7, "plane"),
                                           (1, 140, 1400, 33, "scalar"), (2, 100, 300, 80, "plane"),
-                                          (1, 60, 1500, 60, "plane")])
+                                          (1, 60, 1500, 60, "plane"), (1, 200, 260, 120, "scalar")])
 def test_cnn_bf16_tc_parity(tg, orc, n, H, W, n5, bias):
     """C3, C5 on tcgen05 (bf16 operands, fp32 accumulation): normwise <= 2e-2 (north_star);
     covers the flattened (narrow) and column-window (wide) band modes of U3."""
