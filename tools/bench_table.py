@@ -39,10 +39,11 @@ def main(path):
         frac, bound = (sr["frac"], sr["bound"]) if sr else (e["streamed_roofline_frac"], e["streamed_roofline_bound"])
         r = t["roofline"]
         v = t["verified"]
+        verr = f"{v['max_normwise_err']:.1e}" if v else "n/a (N > 1)"
         cfg = t["baseline_config"].replace("configs", "")
         out.append(f"| {DESC[t['template']]}, {t['precision']} | {cfg} | {t['value']:,.0f} | {e['value']:,.0f} | "
                    f"{frac:.2f} ({bound}) | {e['bytes_vs_lower_bound']:.4f} | "
-                   f"{SHORT.get(r['kernel'], r['kernel'])} {r['frac']:.2f} ({r['bound']}) | {v['max_normwise_err']:.1e} |")
+                   f"{SHORT.get(r['kernel'], r['kernel'])} {r['frac']:.2f} ({r['bound']}) | {verr} |")
         if e.get("uncapped"):
             unc.append(f"{DESC[t['template']].split(',')[0]} {t['precision']} {e['uncapped']['value']:,.0f}")
     link = j["measured_peaks"]["host_link_gbs"]
@@ -59,9 +60,11 @@ def main(path):
         out.append(f"configs[0] (256²): {small['us_per_step_device']:.1f} µs per device step (graph replay), "
                    f"{small['us_per_step_e2e']:.1f} µs end to end.")
     c = j["checksum"]
-    cb = j["cpu_baseline"]
-    out.append(f"Output digest {c['digest_all']}; CPU oracle ({cb['cores']} host cores): {cb['value']:.1f} Mpx/s "
-               f"({cb['sample']}); clocks {j['clocks'].get('sm_mhz')} MHz, reasons {j['clocks'].get('reasons')}.")
+    cb = j.get("cpu_baseline")  # rank 0 at N = 1 only
+    first = f" (first share {c['digest_first_share']})" if "digest_first_share" in c else ""
+    oracle = f"; CPU oracle ({cb['cores']} host cores): {cb['value']:.1f} Mpx/s ({cb['sample']})" if cb else ""
+    out.append(f"N = {j['n_gpus']}: output digest {c['digest_all']}{first}{oracle}; clocks {j['clocks'].get('sm_mhz')} "
+               f"MHz, reasons {j['clocks'].get('reasons')}.")
     print("\n".join(out))
 
 
